@@ -1,0 +1,230 @@
+"""CPU ORACLE — test infrastructure only.
+
+ctypes wrapper around ``oracle/liboracle.so`` (plain C, see ``oracle/oracle.h``).  Only
+``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline / ``--impl
+reference`` leg may import this module.  It never imports the CUDA path; inputs arrive
+as plain numpy arrays (or any object with the ReyesScene attributes) produced by
+``paper_conf_micro_zhengozsyc17_b200/inputs.py``.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+
+
+def build(force: bool = False) -> str:
+    """Compile the C oracle (make -C oracle)."""
+    if force or not os.path.exists(_LIB_PATH) or any(
+            os.path.getmtime(os.path.join(_HERE, f)) > os.path.getmtime(_LIB_PATH)
+            for f in os.listdir(_HERE) if f.endswith((".c", ".h"))):
+        subprocess.run(["make", "-s", "-C", _HERE], check=True)
+    return _LIB_PATH
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        _lib = C.CDLL(_LIB_PATH)
+        _declare(_lib)
+    return _lib
+
+
+MAX_STAGES = 8
+P = C.c_void_p
+
+
+class Stats(C.Structure):
+    _fields_ = [("deq", C.c_uint64 * MAX_STAGES), ("enq", C.c_uint64 * MAX_STAGES)]
+
+
+class TraceRec(C.Structure):
+    _fields_ = [("id", C.c_uint64), ("stage", C.c_uint32), ("pad", C.c_uint32)]
+
+
+TRACE_DTYPE = np.dtype([("id", "<u8"), ("stage", "<u4"), ("pad", "<u4")])
+
+
+class ReyesSceneC(C.Structure):
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_frames", C.c_int32),
+                ("patches_per_frame", C.c_int32), ("max_depth", C.c_int32), ("pad0", C.c_int32),
+                ("t_dice", C.c_float), ("near_w", C.c_float), ("M", P), ("albedo", P),
+                ("L", C.c_float * 4)]
+
+
+class ReyesOutC(C.Structure):
+    _fields_ = [("key", P), ("s", P), ("colour", P),
+                ("n_bound", C.c_uint64), ("n_split", C.c_uint64), ("n_dice", C.c_uint64),
+                ("n_shade", C.c_uint64), ("n_culled", C.c_uint64),
+                ("depth_hist", C.c_uint64 * 16), ("culled_depth_hist", C.c_uint64 * 16),
+                ("leaf_ids", P), ("leaf_cap", C.c_size_t), ("n_leaves", C.c_size_t),
+                ("leaf_grids", P),
+                ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t)]
+
+
+def _declare(L):
+    L.orc_toy_definition.argtypes = [P, C.c_size_t, C.c_int32, P, P]
+    L.orc_toy_pipeline.argtypes = [P, C.c_size_t, C.c_int32, P, P, P]
+    L.orc_collatz_definition.argtypes = [P, C.c_size_t, P]
+    L.orc_collatz_pipeline.argtypes = [P, C.c_size_t, C.c_uint32, P, P, P]
+    L.orc_reyes_definition.argtypes = [P, P, C.c_size_t, P]
+    L.orc_reyes_pipeline.argtypes = [P, P, C.c_size_t, P]
+    L.orc_reyes_bound.argtypes = [P, P, P]
+    L.orc_reyes_split.argtypes = [P, C.c_int, P, P]
+    L.orc_reyes_dice.argtypes = [P, P, P]
+    L.orc_reyes_project.argtypes = [P, P, P]
+    L.orc_reyes_shade_factor.argtypes = [P, P]
+    L.orc_reyes_shade_factor.restype = C.c_float
+
+
+def _ptr(a: np.ndarray):
+    assert a.flags["C_CONTIGUOUS"]
+    return a.ctypes.data_as(C.c_void_p)
+
+
+# ------------------------------------------------------------------ toy / collatz
+def toy_definition(seeds: np.ndarray, threshold: int):
+    seeds = np.ascontiguousarray(seeds, np.int32)
+    out = np.zeros_like(seeds)
+    passes = C.c_uint64(0)
+    rc = lib().orc_toy_definition(_ptr(seeds), seeds.size, threshold, _ptr(out), C.byref(passes))
+    assert rc == 0
+    return out, passes.value
+
+
+def toy_pipeline(seeds: np.ndarray, threshold: int):
+    seeds = np.ascontiguousarray(seeds, np.int32)
+    out = np.zeros_like(seeds)
+    n_out = C.c_size_t(0)
+    st = Stats()
+    rc = lib().orc_toy_pipeline(_ptr(seeds), seeds.size, threshold, _ptr(out), C.byref(n_out), C.byref(st))
+    assert rc == 0
+    return out[: n_out.value], list(st.deq[:3]), list(st.enq[:3])
+
+
+def collatz_definition(seeds: np.ndarray):
+    seeds = np.ascontiguousarray(seeds)
+    out = np.zeros(seeds.size, np.uint32)
+    assert lib().orc_collatz_definition(_ptr(seeds), seeds.size, _ptr(out)) == 0
+    return out
+
+
+def collatz_pipeline(seeds: np.ndarray, max_steps: int = 1000):
+    seeds = np.ascontiguousarray(seeds)
+    out = np.zeros(seeds.size, np.uint32)
+    seen = np.zeros(seeds.size, np.uint32)
+    st = Stats()
+    rc = lib().orc_collatz_pipeline(_ptr(seeds), seeds.size, max_steps, _ptr(out), _ptr(seen), C.byref(st))
+    return rc, out, seen, list(st.deq[:2]), list(st.enq[:2])
+
+
+# ------------------------------------------------------------------ Reyes
+class _SceneHolder:
+    """Keeps the numpy arrays referenced by the C struct alive."""
+
+    def __init__(self, scene):
+        self.M = np.ascontiguousarray(scene.M, np.float32).reshape(-1)
+        self.albedo = np.ascontiguousarray(scene.albedo, np.float32).reshape(-1)
+        s = ReyesSceneC()
+        s.W, s.H, s.n_frames = scene.W, scene.H, scene.n_frames
+        s.patches_per_frame = scene.patches_per_frame
+        s.max_depth = scene.max_depth
+        s.t_dice, s.near_w = scene.t_dice, scene.near_w
+        s.M, s.albedo = self.M.ctypes.data, self.albedo.ctypes.data
+        for i in range(4):
+            s.L[i] = float(np.float32(scene.light[i]))
+        self.c = s
+
+
+def _reyes_run(fn, scene, seeds=None, leaf_cap=0, want_grids=False, trace_cap=0):
+    seeds = np.ascontiguousarray(scene.seeds if seeds is None else seeds)
+    h = _SceneHolder(scene)
+    npix = scene.n_frames * scene.W * scene.H
+    key = np.empty(npix, np.uint64)
+    s = np.empty(npix, np.float32)
+    colour = np.empty((npix, 4), np.float32)
+    o = ReyesOutC()
+    o.key, o.s, o.colour = key.ctypes.data, s.ctypes.data, colour.ctypes.data
+    leaf_ids = np.zeros(max(leaf_cap, 1), np.uint64)
+    grids = np.zeros((max(leaf_cap, 1) if want_grids else 1, 6, 81), np.float32)
+    if leaf_cap:
+        o.leaf_ids, o.leaf_cap = leaf_ids.ctypes.data, leaf_cap
+        if want_grids:
+            o.leaf_grids = grids.ctypes.data
+    trace = np.zeros(max(trace_cap, 1), TRACE_DTYPE)
+    if trace_cap:
+        o.trace, o.trace_cap = trace.ctypes.data, trace_cap
+    rc = fn(C.byref(h.c), _ptr(seeds), seeds.size, C.byref(o))
+    assert rc == 0, rc
+    shp = (scene.n_frames, scene.H, scene.W)
+    res = dict(key=key.reshape(shp), s=s.reshape(shp), colour=colour.reshape(shp + (4,)),
+               n_bound=o.n_bound, n_split=o.n_split, n_dice=o.n_dice, n_shade=o.n_shade,
+               n_culled=o.n_culled, depth_hist=list(o.depth_hist),
+               culled_depth_hist=list(o.culled_depth_hist), n_leaves=o.n_leaves)
+    if leaf_cap:
+        assert o.n_leaves <= leaf_cap, "leaf_cap too small"
+        res["leaf_ids"] = leaf_ids[: o.n_leaves].copy()
+        if want_grids:
+            res["leaf_grids"] = grids[: o.n_leaves].copy()
+    if trace_cap:
+        assert o.trace_n <= trace_cap, "trace_cap too small"
+        res["trace"] = trace[: o.trace_n].copy()
+    return res
+
+
+def reyes_definition(scene, seeds=None, leaf_cap=0, want_grids=False):
+    return _reyes_run(lib().orc_reyes_definition, scene, seeds, leaf_cap, want_grids)
+
+
+def reyes_pipeline(scene, seeds=None, leaf_cap=0, trace_cap=0):
+    return _reyes_run(lib().orc_reyes_pipeline, scene, seeds, leaf_cap, False, trace_cap)
+
+
+def reyes_bound(scene, patch_item):
+    h = _SceneHolder(scene)
+    it = np.ascontiguousarray(patch_item).reshape(1)
+    d = C.c_int(0)
+    cls = lib().orc_reyes_bound(C.byref(h.c), _ptr(it), C.byref(d))
+    return cls, d.value
+
+
+def reyes_split(patch_item, direction: int):
+    it = np.ascontiguousarray(patch_item).reshape(1)
+    left = np.zeros(1, it.dtype)
+    right = np.zeros(1, it.dtype)
+    lib().orc_reyes_split(_ptr(it), direction, _ptr(left), _ptr(right))
+    return left[0], right[0]
+
+
+def reyes_dice(scene, patch_item):
+    h = _SceneHolder(scene)
+    it = np.ascontiguousarray(patch_item).reshape(1)
+    g = np.zeros((6, 81), np.float32)
+    lib().orc_reyes_dice(C.byref(h.c), _ptr(it), _ptr(g))
+    return g
+
+
+def reyes_project(M16: np.ndarray, p4: np.ndarray):
+    M = np.ascontiguousarray(M16, np.float32).reshape(16)
+    p = np.ascontiguousarray(p4, np.float32).reshape(4)
+    c = np.zeros(4, np.float32)
+    lib().orc_reyes_project(_ptr(M), _ptr(p), _ptr(c))
+    return c
+
+
+def reyes_shade_factor(n3, L4):
+    n = np.ascontiguousarray(n3, np.float32).reshape(3)
+    L = np.ascontiguousarray(L4, np.float32).reshape(4)
+    return float(lib().orc_reyes_shade_factor(_ptr(n), _ptr(L)))
+
+
+REYES_CULL, REYES_SPLIT, REYES_DICE = 0, 1, 2

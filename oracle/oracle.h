@@ -1,0 +1,115 @@
+/* oracle.h — CPU ORACLE. TEST INFRASTRUCTURE ONLY.
+ *
+ * Plain, slow, single-threaded C99 implementation of what the VersaPipe hot path
+ * computes (PAPER.md = /root/reference/PAPER.md; "L<n>" = its line numbers).  Only
+ * tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference leg
+ * may load this library.  It shares NO code, header, table or constant with the CUDA
+ * path in paper_conf_micro_zhengozsyc17_b200/csrc; the two meet only at the seeded
+ * input byte layouts produced by paper_conf_micro_zhengozsyc17_b200/inputs.py.
+ *
+ * Built with gcc -O2 -ffp-contract=off (no FMA contraction, no fast-math, SSE float),
+ * SURVEY §8(c-G) rule 2.
+ *
+ * Two layers per workload (SURVEY §8(c) "Structure"):
+ *   1. a *definition* oracle written as the textbook loop/recursion, and
+ *   2. the *pipeline* oracle: the generic sequential fixpoint engine below, which
+ *      runs each stage's per-item operation over FIFO work queues until every queue is
+ *      empty -- the paper's producer/consumer pipeline (L5 §1 "A task of a previous
+ *      stage fetches input data from its queue, executes this stage, and finally puts
+ *      output data into the queue of the next stage, which is repeated until all stages
+ *      finish") executed sequentially.
+ */
+#ifndef VP_ORACLE_H
+#define VP_ORACLE_H
+#include <stddef.h>
+#include <stdint.h>
+
+#define ORC_MAX_STAGES 8
+
+/* ---------------- generic fixpoint engine (fixpoint.c) ---------------- */
+typedef struct orc_fifo {
+  uint8_t* data;
+  size_t stride, head, tail, cap; /* items [head, tail) are queued */
+} orc_fifo;
+
+typedef struct orc_trace_rec { uint64_t id; uint32_t stage, pad; } orc_trace_rec;
+
+struct orc_engine;
+typedef void (*orc_exec_fn)(struct orc_engine* e, int stage, const void* item);
+
+typedef struct orc_engine {
+  int n_stages;
+  orc_fifo q[ORC_MAX_STAGES];
+  orc_exec_fn exec;
+  void* user;
+  uint64_t deq[ORC_MAX_STAGES]; /* items executed per stage                  */
+  uint64_t enq[ORC_MAX_STAGES]; /* items pushed per stage (seeds included)   */
+  uint64_t max_depth_seen[ORC_MAX_STAGES];
+  /* optional trace of (stage, item id) per executed task */
+  orc_trace_rec* trace;
+  size_t trace_cap, trace_n;
+  int error;
+} orc_engine;
+
+void orc_engine_init(orc_engine* e, int n_stages, const size_t* strides, orc_exec_fn exec, void* user);
+void orc_engine_free(orc_engine* e);
+void orc_push(orc_engine* e, int stage, const void* item);   /* insertIntoQueue / enqueue<S>() */
+void orc_record(orc_engine* e, int stage, uint64_t id);        /* trace hook, called by exec fns */
+int  orc_run(orc_engine* e);                                   /* fixpoint; returns 0 or error   */
+
+/* ---------------- toy pipeline, Fig. 9 (toy.c) ---------------- */
+typedef struct orc_stats { uint64_t deq[ORC_MAX_STAGES], enq[ORC_MAX_STAGES]; } orc_stats;
+int orc_toy_definition(const int32_t* in, size_t n, int32_t threshold, int32_t* out, uint64_t* s1_passes);
+int orc_toy_pipeline(const int32_t* in, size_t n, int32_t threshold, int32_t* out, size_t* n_out,
+                     orc_stats* st);
+
+/* ---------------- Collatz queue stress (collatz.c) ---------------- */
+typedef struct orc_collatz_item { uint32_t id, steps; uint64_t v; } orc_collatz_item;
+int orc_collatz_definition(const orc_collatz_item* in, size_t n, uint32_t* steps_out);
+int orc_collatz_pipeline(const orc_collatz_item* in, size_t n, uint32_t max_steps, uint32_t* steps_out,
+                         uint32_t* seen, orc_stats* st);
+
+/* ---------------- Reyes (reyes.c) ---------------- */
+typedef struct orc_patch {
+  float cp[16][4]; /* P[a][b] at cp[4a+b], a = u index, b = v index; (x,y,z,1) */
+  uint32_t id;     /* frame << 12 | patch                                      */
+  uint32_t path;   /* bit d: 0 = left, 1 = right child taken at depth d        */
+  uint32_t dirs;   /* bit d: split direction at depth d (0 = u, 1 = v)         */
+  uint32_t depth;
+} orc_patch;
+
+typedef struct orc_reyes_scene {
+  int32_t W, H, n_frames, patches_per_frame, max_depth, pad0;
+  float t_dice, near_w;
+  const float* M;      /* [n_frames][16] row-major                 */
+  const float* albedo; /* [patches_per_frame][4]                   */
+  float L[4];
+} orc_reyes_scene;
+
+typedef struct orc_reyes_out {
+  uint64_t* key;   /* [n_frames*H*W], UINT64_MAX = uncovered                     */
+  float* s;        /* [n_frames*H*W] shade factor of the winning micropolygon    */
+  float* colour;   /* [n_frames*H*W*4] resolved colour (rgb, alpha = coverage)   */
+  /* counts */
+  uint64_t n_bound, n_split, n_dice, n_shade, n_culled;
+  uint64_t depth_hist[16];        /* leaves (diced) per depth                     */
+  uint64_t culled_depth_hist[16]; /* culled nodes per depth                       */
+  /* optional: leaf node ids (id << 12 | depth << 8 | path) and their grids */
+  uint64_t* leaf_ids; size_t leaf_cap, n_leaves;
+  float* leaf_grids;  /* [leaf_cap][6][81]: x, y, z, sx, sy, zs (SoA per leaf)        */
+  /* optional per-stage trace (pipeline oracle only) */
+  orc_trace_rec* trace; size_t trace_cap, trace_n;
+} orc_reyes_out;
+
+enum { ORC_REYES_CULL = 0, ORC_REYES_SPLIT = 1, ORC_REYES_DICE = 2 };
+
+int orc_reyes_definition(const orc_reyes_scene* sc, const orc_patch* seeds, size_t n, orc_reyes_out* out);
+int orc_reyes_pipeline(const orc_reyes_scene* sc, const orc_patch* seeds, size_t n, orc_reyes_out* out);
+/* exposed pieces, so tests can pin them individually against independent math */
+int  orc_reyes_bound(const orc_reyes_scene* sc, const orc_patch* p, int* split_dir);
+void orc_reyes_split(const orc_patch* p, int dir, orc_patch* left, orc_patch* right);
+void orc_reyes_dice(const orc_reyes_scene* sc, const orc_patch* p, float grid[6][81]);
+void orc_reyes_project(const float M[16], const float p[4], float c[4]);
+float orc_reyes_shade_factor(const float n[3], const float L[4]);
+
+#endif

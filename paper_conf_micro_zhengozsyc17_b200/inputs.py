@@ -1,0 +1,216 @@
+"""Seeded synthetic input generators shared by the CUDA path and the CPU oracle.
+
+This module holds NO arithmetic of the method (no projection, no bound/split/dice/
+shade, no queueing).  It only draws seeded random numbers and lays them out in the
+byte layouts both sides consume (DESIGN.md §3 "Input recipes").  Camera matrices are
+scene *inputs* (computed in float64 with trigonometry, then rounded to float32),
+exactly as SURVEY §8(d) "Common protocol" prescribes: anything needing sin/cos is
+computed on the host and stored as float data.
+
+Random numbers: SplitMix64 (Steele, Lea, Flood 2014), floats from the top 24 bits:
+``(x >> 40) * 2**-24``.  Seed convention: ``0x56500000 + 256*config + rep``.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+
+import numpy as np
+
+GOLDEN = np.uint64(0x9E3779B97F4A7C15)
+
+
+def seed_for(config: int, rep: int = 0) -> int:
+    return 0x56500000 + 256 * config + rep
+
+
+def splitmix64(seed: int, n: int) -> np.ndarray:
+    """n successive SplitMix64 outputs for a generator started at ``seed``."""
+    with np.errstate(over="ignore"):
+        i = np.arange(1, n + 1, dtype=np.uint64)
+        z = np.uint64(seed & 0xFFFFFFFFFFFFFFFF) + i * GOLDEN
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    return z
+
+
+def uniform01(seed: int, n: int) -> np.ndarray:
+    """float64 values in [0,1) with 24 random bits each (exactly representable in f32)."""
+    return (splitmix64(seed, n) >> np.uint64(40)).astype(np.float64) * (2.0 ** -24)
+
+
+# ----------------------------------------------------------------------------------------
+# Toy pipeline (Fig. 9) and the Collatz queue-stress pipeline (SURVEY c-0b)
+# ----------------------------------------------------------------------------------------
+TOY_THRESHOLD = 1 << 20
+
+
+def toy_seeds(n: int, seed: int = seed_for(0), threshold: int = TOY_THRESHOLD) -> np.ndarray:
+    """int32 items in [1, threshold)."""
+    x = splitmix64(seed, n)
+    return (np.uint64(1) + x % np.uint64(threshold - 1)).astype(np.int32)
+
+
+COLLATZ_DTYPE = np.dtype([("id", "<u4"), ("steps", "<u4"), ("v", "<u8")])  # 16 B
+
+
+def collatz_seeds(n: int, seed: int = seed_for(0, 1), vmax: int = 1 << 16) -> np.ndarray:
+    x = splitmix64(seed, n)
+    a = np.zeros(n, dtype=COLLATZ_DTYPE)
+    a["id"] = np.arange(n, dtype=np.uint32)
+    a["v"] = np.uint64(1) + x % np.uint64(vmax - 1)
+    return a
+
+
+# ----------------------------------------------------------------------------------------
+# Reyes (Fig. 1; L55; BASELINE configs 1 and 5)
+# ----------------------------------------------------------------------------------------
+# Patch item, 272 B (Table 2): float4 cp[16] (object space, w = 1), then
+# u32 id = frame << 12 | patch, u32 path, u32 dirs, u32 depth.
+PATCH_DTYPE = np.dtype([("cp", "<f4", (16, 4)), ("id", "<u4"), ("path", "<u4"),
+                        ("dirs", "<u4"), ("depth", "<u4")])
+assert PATCH_DTYPE.itemsize == 272
+
+
+@dataclass
+class ReyesScene:
+    """Everything a Reyes run reads besides the seed patches."""
+    W: int
+    H: int
+    n_frames: int
+    patches_per_frame: int
+    M: np.ndarray            # [n_frames, 16] float32, row-major clip = M . p
+    albedo: np.ndarray       # [patches_per_frame, 4] float32 (rgb, 0)
+    light: np.ndarray        # [4] float32 unit vector (x, y, z, 0)
+    seeds: np.ndarray        # PATCH_DTYPE [n_frames * patches_per_frame], frame-major
+    max_depth: int = 8
+    t_dice: float = 8.0
+    near_w: float = 1e-3
+    extra: dict = field(default_factory=dict)
+
+
+def look_at_perspective(eye, target=(0.0, 0.0, 0.0), up=(0.0, 0.0, 1.0), fovy_deg=50.0,
+                        aspect=1.0, near=0.1, far=100.0) -> np.ndarray:
+    """float64 4x4 view-projection, D3D-style depth (z/w in [0,1] between near and far)."""
+    eye = np.asarray(eye, np.float64)
+    f = np.asarray(target, np.float64) - eye
+    f /= np.linalg.norm(f)
+    r = np.cross(f, np.asarray(up, np.float64))
+    r /= np.linalg.norm(r)
+    u = np.cross(r, f)
+    V = np.eye(4)
+    V[0, :3], V[1, :3], V[2, :3] = r, u, f
+    V[:3, 3] = -V[:3, :3] @ eye
+    t = 1.0 / math.tan(math.radians(fovy_deg) / 2)
+    P = np.zeros((4, 4))
+    P[0, 0] = t / aspect
+    P[1, 1] = t
+    P[2, 2] = far / (far - near)
+    P[2, 3] = -near * far / (far - near)
+    P[3, 2] = 1.0
+    return P @ V
+
+
+def heightfield_lattice(n_patch_side: int, seed: int, z_amp: float) -> np.ndarray:
+    """(3n+1)^2 control lattice over [-1,1]^2, z ~ U(-z_amp, z_amp). float32 [(3n+1),(3n+1),4]."""
+    m = 3 * n_patch_side + 1
+    g = np.zeros((m, m, 4), np.float32)
+    coords = -1.0 + 2.0 * np.arange(m) / (m - 1)
+    g[:, :, 0] = coords[:, None]
+    g[:, :, 1] = coords[None, :]
+    g[:, :, 2] = (-z_amp + 2 * z_amp * uniform01(seed, m * m)).reshape(m, m)
+    g[:, :, 3] = 1.0
+    return g
+
+
+def lattice_patches(lat: np.ndarray, n_patch_side: int) -> np.ndarray:
+    """16 control points per patch: P[a][b] = lattice[3pi+a][3pj+b] (a = u index, b = v)."""
+    n = n_patch_side * n_patch_side
+    cps = np.zeros((n, 16, 4), np.float32)
+    for pi in range(n_patch_side):
+        for pj in range(n_patch_side):
+            cps[pi * n_patch_side + pj] = lat[3 * pi:3 * pi + 4, 3 * pj:3 * pj + 4].reshape(16, 4)
+    return cps
+
+
+def make_patch_items(cps: np.ndarray, n_frames: int) -> np.ndarray:
+    n = cps.shape[0]
+    items = np.zeros(n_frames * n, PATCH_DTYPE)
+    for f in range(n_frames):
+        sl = slice(f * n, (f + 1) * n)
+        items["cp"][sl] = cps
+        items["id"][sl] = (np.uint32(f) << np.uint32(12)) | np.arange(n, dtype=np.uint32)
+    return items
+
+
+def default_light() -> np.ndarray:
+    L = np.array([0.3, -0.5, 0.8])
+    L /= np.linalg.norm(L)
+    return np.array([L[0], L[1], L[2], 0.0], np.float32)
+
+
+def reyes_config1(seed: int = seed_for(1), W: int = 256, H: int = 256, n_side: int = 4,
+                  max_depth: int = 8) -> ReyesScene:
+    """BASELINE config 1: 16 bicubic Bezier patches, 256x256, max split depth 8.
+
+    4x4 patches tile a height field over [-1,1]^2 (13x13 lattice, z ~ U(-0.25,0.25));
+    camera eye (0,-1.6,1.2) -> origin, up +z, fovy 50 deg, near 0.1.
+    """
+    lat = heightfield_lattice(n_side, seed, 0.25)
+    cps = lattice_patches(lat, n_side)
+    M = look_at_perspective((0.0, -1.6, 1.2), aspect=W / H).astype(np.float32).reshape(1, 16)
+    alb = np.zeros((n_side * n_side, 4), np.float32)
+    alb[:, :3] = uniform01(seed + 1, n_side * n_side * 3).reshape(-1, 3)
+    return ReyesScene(W=W, H=H, n_frames=1, patches_per_frame=n_side * n_side, M=M, albedo=alb,
+                      light=default_light(), seeds=make_patch_items(cps, 1), max_depth=max_depth)
+
+
+def reyes_frame_camera(f: int, n_frames_orbit: int = 512, W: int = 256, H: int = 256) -> np.ndarray:
+    """Per-frame orbit camera of config 5: angle 2*pi*f/512, distance 1.3+1.2*(1+cos(2*pi*f/64))/2."""
+    th = 2 * math.pi * f / n_frames_orbit
+    d = 1.3 + 1.2 * (1 + math.cos(2 * math.pi * f / 64)) / 2
+    eye = (0.8 * d * math.sin(th), -0.8 * d * math.cos(th), 0.6 * d)
+    return look_at_perspective(eye, aspect=W / H).astype(np.float32).reshape(16)
+
+
+def reyes_config5(n_frames: int = 512, n_side: int = 64, frame0: int = 0, seed: int = seed_for(5),
+                  W: int = 256, H: int = 256, z_amp: float = 0.05, max_depth: int = 8) -> ReyesScene:
+    """BASELINE config 5: a batch of frames x 4096 patches (64x64 patch height field,
+    193x193 lattice) with a per-frame orbit camera.  ``frame0`` selects a shard
+    [frame0, frame0 + n_frames) of the 512-frame orbit (multi-GPU sharding)."""
+    lat = heightfield_lattice(n_side, seed, z_amp)
+    cps = lattice_patches(lat, n_side)
+    M = np.stack([reyes_frame_camera(frame0 + f, 512, W, H) for f in range(n_frames)])
+    alb = np.zeros((n_side * n_side, 4), np.float32)
+    alb[:, :3] = uniform01(seed + 1, n_side * n_side * 3).reshape(-1, 3)
+    items = make_patch_items(cps, n_frames)
+    # ids carry the LOCAL frame index (frame buffers are per shard)
+    return ReyesScene(W=W, H=H, n_frames=n_frames, patches_per_frame=n_side * n_side, M=M,
+                      albedo=alb, light=default_light(), seeds=items, max_depth=max_depth,
+                      extra={"frame0": frame0})
+
+
+def reyes_planar(S_px: float, W: int = 64, H: int = 64, x0: float = 8.0, y0: float = 8.0,
+                 max_depth: int = 8, albedo=(0.5, 0.25, 0.75)) -> ReyesScene:
+    """Closed-form special case (SURVEY c-1 pin 4): a planar patch parallel to the image
+    plane, control points on a uniform grid, orthographic M that maps object (x, y) to
+    NDC so that the patch spans [x0, x0+S] x [y0, y0+S] pixels (dyadic coordinates)."""
+    cps = np.zeros((1, 16, 4), np.float32)
+    for a in range(4):
+        for b in range(4):
+            cps[0, 4 * a + b] = (a, b, 0.0, 1.0)  # x = a, y = b in [0,3]
+    # object x in [0,3] -> screen x0 + S*x/3 : sx = (ndc*0.5+0.5)*W, ndc = 2*sx/W - 1
+    sx_scale = S_px / 3.0
+    M = np.zeros((4, 4))
+    M[0, 0] = 2.0 * sx_scale / W
+    M[0, 3] = 2.0 * x0 / W - 1.0
+    M[1, 1] = 2.0 * sx_scale / H
+    M[1, 3] = 2.0 * y0 / H - 1.0
+    M[2, 3] = 0.5
+    M[3, 3] = 1.0
+    alb = np.zeros((1, 4), np.float32)
+    alb[0, :3] = albedo
+    return ReyesScene(W=W, H=H, n_frames=1, patches_per_frame=1, M=M.astype(np.float32).reshape(1, 16),
+                      albedo=alb, light=np.array([0.0, 0.0, 1.0, 0.0], np.float32),
+                      seeds=make_patch_items(cps, 1), max_depth=max_depth)
