@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""bench.py — VersaPipe Reyes batch (BASELINE config 5) on 1..8 B200s.
+
+One "step" = one pass of the whole hot path (every §8(a) row: seed claim, Bound,
+recursive Split, Dice, Shade with per-stage queues, the configured execution model,
+the resolve sink) over this rank's shard of the 512-frame x 4096-patch batch.
+Frames are sharded over ranks (no data-path collective); NCCL is used only for the
+timing reduction and the post-run output gather (timed separately).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl vp|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...
+
+Prints ONE JSON line on rank 0.  --impl reference times the CPU oracle (the
+reference arm for this paper-only tier) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+TOTAL_FRAMES = 512
+PATCH_SIDE = 64                      # 4096 patches per frame
+MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
+
+# Algorithmic fp32 operations per task (counted from the stage
+# definitions, excluding per-point constant Bernstein tables and integer coverage work):
+FLOP_DICE = 81 * (16 * 7 + 28 + 9)   # 16-term tensor sum (w, 3 mul+add), M.p, screen = 12069
+FLOP_SHADE = 64 * 41                 # edges, cross, |n|, n.L, sqrt/div, shade, zq, Q8 snap = 2624
+FLOP_BOUND = 16 * (28 + 9) + 40      # 16 projections + split metric = 632
+FLOP_SPLIT = 3 * 4 * 12              # de Casteljau, 3 coords x 4 curves = 144
+
+
+def env_int(k, d):
+    try:
+        return int(os.environ.get(k, d))
+    except ValueError:
+        return d
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="vp", choices=["vp", "reference"])
+    ap.add_argument("--frames", type=int, default=TOTAL_FRAMES)
+    ap.add_argument("--model", default="hybrid", help="hybrid|megakernel|kbk|coarse|fine")
+    ap.add_argument("--split", type=int, default=0, help="SMs for the [Bound,Split] group (hybrid)")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-baselines", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args()
+
+
+def peaks():
+    try:
+        return json.load(open(MEASURED))
+    except Exception:
+        return {}
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, gpu_index):
+        self.p = None
+        self.path = os.path.join(ROOT, "gpurun_out", f"clocks_rank{gpu_index}.csv")
+        try:
+            os.makedirs(os.path.dirname(self.path), exist_ok=True)
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(
+                ["nvidia-smi", "-i", str(gpu_index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        self.f.close()
+        rows = [r.split(",") for r in open(self.path).read().strip().splitlines() if r.count(",") >= 6]
+        sm = [float(r[0]) for r in rows if r[0].strip().replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].strip().replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if "Active" in r[3 + i] and "Not" not in r[3 + i]})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(rows)}
+
+
+def hybrid_binding(vp, nsm, split):
+    s = split or max(8, nsm // 4)
+    return vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, s), (2, 3, vp.GROUP_RTC, s, nsm)], nsm)
+
+
+def configure(vp, rp, model, nsm, split):
+    if model == "hybrid":
+        rp.configure(vp.HYBRID, hybrid_binding(vp, nsm, split))
+    else:
+        rp.configure({"megakernel": vp.MEGAKERNEL, "kbk": vp.KBK, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+
+
+def time_steps(torch, rp, steps, stream):
+    """K steps bracketed by events on the launching stream; returns (ms total, last stats)."""
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    st = None
+    kms = []
+    for _ in range(steps):
+        st = rp.run(stream)
+        kms.append(st["kernel_ms"])
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    return ev0.elapsed_time(ev1), st, kms
+
+
+def cpu_oracle_sample(frames_total, seconds, frame0=0):
+    """The CPU oracle as it stands (single-threaded C per frame), frames spread over the
+    host cores with a process pool; returns (frames/s, items/s, cores, sample text)."""
+    import multiprocessing as mp
+    t0 = time.perf_counter()
+    _oracle_frame(frame0)  # one frame first, to size the sample
+    one = time.perf_counter() - t0
+    cores = os.cpu_count() or 1
+    n = int(max(cores, min(frames_total, seconds * cores / max(one, 1e-3))))
+    n = max(1, min(n, frames_total))
+    t0 = time.perf_counter()
+    with mp.get_context("fork").Pool(cores) as pool:
+        res = pool.map(_oracle_frame, [(frame0 + f) % TOTAL_FRAMES for f in range(n)])
+    dt = time.perf_counter() - t0
+    items = sum(r for r in res)
+    return n / dt, items / dt, cores, f"{n} of {frames_total} frames (config 5, 4096 patches each), oracle per frame on {cores} processes, {dt:.1f} s"
+
+
+def _oracle_frame(f):
+    import oracle
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    sc = inputs.reyes_config5(n_frames=1, n_side=PATCH_SIDE, frame0=f)
+    r = oracle.reyes_pipeline(sc)
+    return r["n_bound"] + r["n_split"] + r["n_dice"] + r["n_shade"]
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle, rank 0 only (other ranks exit without work)."""
+    if rank != 0:
+        return
+    import oracle
+    oracle.build()
+    vals, items = [], []
+    for _ in range(args.warmup):
+        _oracle_frame(0)
+    info = None
+    for _ in range(args.steps):
+        fps, ips, cores, sample = cpu_oracle_sample(args.frames, max(1.0, args.cpu_seconds / max(args.steps, 1)))
+        vals.append(fps)
+        items.append(ips)
+        info = (cores, sample)
+    v = float(np.median(vals))
+    line = {"impl": "reference", "metric": "frames/sec", "value": v, "unit": "frames/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * args.frames / v,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic", "items_per_sec": float(np.median(items)),
+            "config": {"workload": "reyes_batch_config5", "frames": args.frames, "patches_per_frame": 4096,
+                       "image": "256x256", "max_depth": 8},
+            "cpu_baseline": {"value": v, "unit": "frames/s", "cores": info[0], "kind": "oracle", "sample": info[1]},
+            "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = env_int("RANK", 0), env_int("WORLD_SIZE", 1), env_int("LOCAL_RANK", 0)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_micro_zhengozsyc17_b200 import build as vpbuild
+    vpbuild.build()
+    from paper_conf_micro_zhengozsyc17_b200 import inputs, vp
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    nsm, cc = vp.device_info(local)
+    # ---- shard: rank r renders frames [r*F/P, (r+1)*F/P) of the orbit
+    f0 = rank * args.frames // world
+    f1 = (rank + 1) * args.frames // world
+    scene = inputs.reyes_config5(n_frames=f1 - f0, n_side=PATCH_SIDE, frame0=f0)
+    rp = ReyesPipeline(scene, device=local)
+    configure(vp, rp, args.model, nsm, args.split)
+    stream = torch.cuda.current_stream()
+    for _ in range(max(args.warmup, 3) if args.warmup >= 3 else args.warmup):
+        rp.run(stream)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    # ---- timed region: inputs resident in HBM (seeds 4096 x 272 B per frame > L2)
+    barrier()
+    clk = Clocks(local)
+    t_ms, st, kms = time_steps(torch, rp, args.steps, stream)
+    barrier()
+    clocks = clk.stop()
+    t = torch.tensor([t_ms], dtype=torch.float64, device="cuda")
+    items_local = sum(st["dequeued"][:4])
+    cnt = torch.tensor([items_local, f1 - f0], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(cnt, op=dist.ReduceOp.SUM)
+    t_ms = float(t.item())
+    items_all, frames_all = float(cnt[0].item()), float(cnt[1].item())
+    ms_per_step = t_ms / args.steps
+    fps = frames_all * args.steps / (t_ms / 1e3)
+    ips = items_all * args.steps / (t_ms / 1e3)
+
+    # ---- dominant kernel (largest event time among the persistent kernels of the step)
+    nk = st["num_kernels"]
+    kmean = np.mean(np.array(kms), axis=0) if nk else np.array([ms_per_step])
+    dom = int(np.argmax(kmean)) if nk else 0
+    lo, hi, _ = st["kernels"][dom] if nk else (0, 3, 0)
+    d = st["dequeued"]
+    per_stage_flop = [FLOP_BOUND, FLOP_SPLIT, FLOP_DICE, FLOP_SHADE]
+    dom_flop = sum(d[s] * per_stage_flop[s] for s in range(lo, hi + 1))
+    pk = peaks()
+    sm_max = pk.get("sm_max_mhz", 1965.0)
+    # fp32 non-FMA issue peak: 148 SMs x 128 lanes x 1 op/clk (FMA contraction is disabled
+    # for bit-exactness), at clocks.max.sm
+    alu_peak = nsm * 128 * sm_max * 1e6 / 1e12
+    achieved = dom_flop / (kmean[dom] / 1e3) / 1e12
+    roofline = {"bound": "alu", "achieved": achieved, "peak": alu_peak, "unit": "TFLOP/s",
+                "frac": achieved / alu_peak, "traffic": None,
+                "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if args.model == 'hybrid' and lo == 2 else 'MEGA'}>",
+                "peak_source": "derived: SMs x 128 fp32 lanes x clocks.max.sm (MEASURED_PEAKS sm_max_mhz), non-FMA",
+                "kernel_ms": float(kmean[dom]), "kernel_share_of_step": float(kmean[dom] / ms_per_step)}
+    hbm = pk.get("hbm_gbs", 6548.5)
+    # HBM bytes per step that must move: seeds read + fb clear/CAS/resolve + colour write
+    npix = scene.n_frames * scene.W * scene.H
+    bytes_step = scene.seeds.nbytes + npix * (16 + 16 + 16 + 16)
+
+    # ---- baselines on the same shard: KBK (one launch per stage per wave) + megakernel
+    extra = {}
+    if not args.no_baselines:
+        for name in ("kbk", "megakernel"):
+            if name == args.model:
+                continue
+            configure(vp, rp, name, nsm, args.split)
+            rp.run(stream)
+            bt, bst, _ = time_steps(torch, rp, max(1, min(args.steps, 3)), stream)
+            bt_t = torch.tensor([bt], dtype=torch.float64, device="cuda")
+            if world > 1:
+                dist.all_reduce(bt_t, op=dist.ReduceOp.MAX)
+            extra[name] = {"ms_per_step": float(bt_t.item()) / max(1, min(args.steps, 3)),
+                           "launches_per_step": int(bst["kbk_launches"])}
+        configure(vp, rp, args.model, nsm, args.split)
+
+    # ---- e2e through the public API with HOST buffers: H2D seeds + run + D2H colours
+    e2e = None
+    if not args.no_e2e:
+        host_seeds = torch.from_numpy(scene.seeds.view(np.uint8).reshape(-1).copy()).pin_memory()
+        host_out = torch.empty(rp.colour.shape, dtype=torch.float32).pin_memory()
+        e_steps = max(1, min(args.steps, 5))
+        for _ in range(2):
+            rp.p.insert(0, host_seeds.numpy(), n=scene.seeds.size, replace=True, stream=stream)
+            rp.run(stream)
+            host_out.copy_(rp.colour, non_blocking=True)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(e_steps):
+            rp.p.insert(0, host_seeds.numpy(), n=scene.seeds.size, replace=True, stream=stream)
+            rp.run(stream)
+            host_out.copy_(rp.colour, non_blocking=True)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        et = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e = {"value": frames_all * e_steps / (float(et.item()) / 1e3), "unit": "frames/s",
+               "h2d_bytes_per_step": int(host_seeds.numel()) * world,
+               "d2h_bytes_per_step": int(host_out.numel() * 4) * world}
+        # restore device-resident seeds
+        rp.p.insert(0, rp.seeds_dev, n=scene.seeds.size, replace=True)
+
+    # ---- NCCL output gather (config 5), timed separately
+    gather_ms = None
+    if world > 1 and (f1 - f0) * world == args.frames:
+        out = torch.empty((args.frames,) + tuple(rp.colour.shape[1:]), dtype=torch.float32, device="cuda")
+        barrier()
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(stream)
+        dist.all_gather_into_tensor(out, rp.colour)
+        g1.record(stream)
+        torch.cuda.synchronize()
+        gt = torch.tensor([g0.elapsed_time(g1)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(gt, op=dist.ReduceOp.MAX)
+        gather_ms = float(gt.item())
+
+    cpu = None
+    if rank == 0 and world == 1:
+        try:
+            cfps, cips, cores, sample = cpu_oracle_sample(args.frames, args.cpu_seconds)
+            cpu = {"value": cfps, "unit": "frames/s", "cores": cores, "kind": "oracle", "sample": sample,
+                   "items_per_sec": cips}
+        except Exception as ex:  # the oracle is a reported baseline only
+            cpu = {"value": None, "unit": "frames/s", "cores": os.cpu_count(), "kind": "oracle",
+                   "sample": f"failed: {ex}"}
+
+    launches = 3 + nk + int(st["kbk_launches"])   # run-init, fb clear, resolve + kernels + waves
+    line = {
+        "metric": "frames/sec", "value": fps, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": "reyes_batch_config5", "frames": args.frames, "frames_per_gpu": f1 - f0,
+                   "patches_per_frame": 4096, "image": "256x256", "max_depth": 8, "model": args.model,
+                   "parallelism": f"frames sharded over {world} GPU(s)",
+                   "l2": "inputs larger than L2 (seeds %.0f MB/GPU, frame buffers %.0f MB/GPU)" % (
+                       scene.seeds.nbytes / 1e6, npix * 32 / 1e6)},
+        "items_per_sec": ips, "items_per_step": items_all,
+        "stage_counts": [int(x) for x in d[:4]],
+        "roofline": roofline,
+        "hbm": {"min_bytes_per_step": bytes_step * world, "achieved_gbs": bytes_step * world / (ms_per_step / 1e3) / 1e9,
+                "pct_of_measured": 100.0 * bytes_step * world / (ms_per_step / 1e3) / 1e9 / hbm,
+                "note": "ALU/latency-bound workload (SURVEY §8(d) d5); % HBM reported, not the bound"},
+        "speedup_vs_kbk": (extra["kbk"]["ms_per_step"] / ms_per_step) if "kbk" in extra else None,
+        "baselines": extra, "e2e": e2e, "gather_ms": gather_ms, "clocks": clocks, "gpu_launches": launches * args.steps,
+        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs",
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,258 @@
+/* vp.h — C ABI of libvp.so, a B200 (sm_100a) implementation of the VersaPipe pipeline
+ * runtime (Zheng, Oh, Zhai, Shen, Yi, Chen; MICRO-50 2017).
+ *
+ * Citations "L<n>" are line numbers of the paper text.  The calls follow
+ * the paper's programming model: "users only need to write the operations for each
+ * pipeline stage. VersaPipe will then automatically assemble the stages into a hybrid
+ * execution model and configure it" (L3 abstract; L13 §3; L37 §6).
+ *
+ * Conventions
+ *  - Every call returns vp_status (VP_OK == 0).  No C++ exception crosses the ABI.
+ *  - Out-parameters come last.  Handles are opaque and NOT thread-safe (one per host thread).
+ *  - Call order is enforced: create -> stage_register (all stages) -> insert ->
+ *    configure | autotune -> run (repeatable) -> destroy.  Violations: VP_ERR_INVALID.
+ *  - Device pointers are CUDA device addresses on the pipeline's device.  "Borrowed"
+ *    pointers must stay valid until vp_pipeline_destroy; "copied" data is copied
+ *    before the call returns.
+ *  - On any error the detailed message is available from vp_last_error(p).
+ */
+#ifndef VP_H
+#define VP_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum vp_status {
+  VP_OK = 0,
+  VP_ERR_INVALID = 1,        /* bad argument or call order                                  */
+  VP_ERR_UNSUPPORTED = 2,    /* e.g. RTC on a recursive / latched group (L11: RTC suits     */
+                             /* "regular pipeline programs (without recursion or global     */
+                             /* synchronizations)")                                         */
+  VP_ERR_CUDA = 3,           /* CUDA runtime error; text in vp_last_error                   */
+  VP_ERR_OOM = 4,
+  VP_ERR_QUEUE_OVERFLOW = 5, /* a producer found its target ring full for > 200 ms          */
+  VP_ERR_TIMEOUT = 6,        /* device watchdog (vp_pipeline_desc.watchdog_ms) or tuner cap */
+  VP_ERR_BINDING = 7,        /* strict binding requested and a quota was not reached        */
+  VP_ERR_FANOUT = 8          /* a stage emitted more items than its declared fan-out        */
+} vp_status;
+
+/* Execution models, §4: RTC, KBK, Megakernel (§4.1), coarse and fine
+ * pipeline (§4.2.2), hybrid (§4.2.3). */
+typedef enum vp_model {
+  VP_RTC = 0,
+  VP_KBK = 1,
+  VP_MEGAKERNEL = 2,
+  VP_COARSE = 3,
+  VP_FINE = 4,
+  VP_HYBRID = 5
+} vp_model;
+
+/* Per-group models inside VP_HYBRID (the auto-tuner explores "RTC, KBK, Megakernel,
+ * and fine pipeline" per group, L45).  Groups are coarse-pipelined with each other. */
+typedef enum vp_group_model {
+  VP_GROUP_RTC = 0,
+  VP_GROUP_KBK = 1,
+  VP_GROUP_MEGA = 2,
+  VP_GROUP_FINE = 3
+} vp_group_model;
+
+/* Built-in stage functions compiled into libvp.so (BaseStage::execute, L37).  A pipeline
+ * registers the stages of ONE workload family, in this order.  User-defined families
+ * use the C++ template layer (csrc/vp_runtime.cuh) and are instantiated at build time. */
+typedef enum vp_stage_kind {
+  VP_KIND_INVALID = 0,
+  /* Fig. 9 toy (L37): S1 v*=2, recursive until >= threshold; S2 v+1; S3 sink */
+  VP_TOY_S1 = 1, VP_TOY_S2 = 2, VP_TOY_S3 = 3,
+  /* Collatz queue stress (not in the paper): step (recursive), sink */
+  VP_COLLATZ_STEP = 10, VP_COLLATZ_SINK = 11,
+  /* Reyes (Fig. 1, L3; L55): Bound, Split (recursive via Bound), Dice, Shade */
+  VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23
+} vp_stage_kind;
+
+#define VP_MAX_STAGES 8
+#define VP_MAX_SM 256
+
+/* vp_pipeline_desc.flags */
+#define VP_FLAG_TRACE 0x1u          /* record (stage, item id, smid) of every task           */
+#define VP_FLAG_QUEUE_DEPTH 0x2u    /* track max ring depth per stage (one extra read/flush) */
+#define VP_FLAG_STRICT_BINDING 0x4u /* vp_run fails with VP_ERR_BINDING on quota shortfall   */
+#define VP_FLAG_TIMERS 0x8u         /* in-kernel %globaltimer accumulators per stage/kernel  */
+
+typedef struct vp_pipeline_desc {
+  int max_stages;                 /* <= VP_MAX_STAGES                                      */
+  uint32_t flags;                 /* VP_FLAG_*                                             */
+  int64_t default_queue_capacity; /* ring slots per stage (rounded up to a power of 2);    */
+                                  /* 0 = the family's default                              */
+  int watchdog_ms;                /* device watchdog per vp_run; 0 = 30000                 */
+  int64_t trace_capacity;         /* records, with VP_FLAG_TRACE                           */
+} vp_pipeline_desc;
+
+typedef struct vp_stage_desc {
+  const char* name;        /* informational, copied                                         */
+  int kind;                /* vp_stage_kind                                                 */
+  int item_bytes;          /* DataItemType size (L37); must equal the kind's item size      */
+  int threads_per_item;    /* threadNum (L37); 0 = the kind's default; informational for    */
+                           /* built-ins, whose execute() is written for a fixed mapping     */
+  int64_t queue_capacity;  /* ring slots; 0 = pipeline default                              */
+  const void* params;      /* HOST pointer to the family's parameter struct (vp_*_params),  */
+                           /* copied; the device pointers inside it are BORROWED.  Stages   */
+                           /* of one family may repeat it or pass NULL after the first.     */
+  size_t params_bytes;     /* sizeof(the vp_*_params struct)                                */
+} vp_stage_desc;
+
+/* SM binding / grouping configuration {g, s, b} (L41; Fig. 10 L43). */
+typedef struct vp_sm_binding {
+  int num_groups;
+  int group_of_stage[VP_MAX_STAGES];   /* groups are contiguous stage ranges (L45)           */
+  int group_model[VP_MAX_STAGES];      /* vp_group_model, per group                          */
+  uint32_t group_sm_mask[VP_MAX_STAGES][VP_MAX_SM / 32]; /* s_flag(group, sm), Fig. 5       */
+  int blocks_per_sm[VP_MAX_STAGES];    /* per stage (fine groups) / per group first stage     */
+                                       /* (mega/RTC groups); 0 = as many as fit              */
+  int batch[VP_MAX_STAGES];            /* items per claim per stage; 0 = default             */
+} vp_sm_binding;
+
+typedef struct vp_config {
+  int model;                 /* vp_model                                                   */
+  int has_binding;
+  vp_sm_binding binding;
+  int batch;                 /* global items-per-claim override, 0 = per-stage defaults    */
+} vp_config;
+
+typedef struct vp_run_stats {
+  double device_ms;                         /* CUDA events around the run on the stream   */
+  uint64_t dequeued[VP_MAX_STAGES];         /* tasks executed per stage                   */
+  uint64_t enqueued[VP_MAX_STAGES];         /* items pushed per stage, seeds included     */
+  uint64_t max_depth[VP_MAX_STAGES];        /* with VP_FLAG_QUEUE_DEPTH                   */
+  int num_kernels;                          /* persistent kernels launched                */
+  int kernel_lo[16], kernel_hi[16];         /* stage range of each persistent kernel      */
+  int kernel_quota[16];                     /* requested blocks/SM (0 = fill)             */
+  double kernel_ms[16];                     /* CUDA-event duration of each persistent     */
+                                            /* kernel on its own stream                   */
+  uint32_t blocks_on_sm[16][VP_MAX_SM];     /* blocks that ran the prologue on each SM    */
+  uint64_t admitted[16];                    /* blocks that stayed (check_sm/check_sm_blk) */
+  uint64_t fallback_admits;                 /* progress-guarantee admissions              */
+  uint64_t kbk_launches;                    /* wave launches (KBK / RTC)                   */
+  uint64_t trace_records;                   /* with VP_FLAG_TRACE                          */
+  int abort_reason;                         /* 0 none, 1 timeout, 2 overflow, 3 fan-out   */
+  int num_sms;
+  /* VP_FLAG_TIMERS: block-time (ns, summed over blocks) spent executing each stage     */
+  /* (stage-in + execute), publishing its outputs (queue overhead, §8.5), and idle per  */
+  /* persistent kernel (no claimable item)                                              */
+  uint64_t stage_exec_ns[VP_MAX_STAGES];
+  uint64_t stage_flush_ns[VP_MAX_STAGES];
+  uint64_t kernel_idle_ns[16];
+} vp_run_stats;
+
+typedef struct vp_autotune_opts {
+  double time_budget_s;      /* total tuning wall time; 0 = 60 s                           */
+  int sm_granularity;        /* SM split step; 0 = 4 (L45 pruning, B200 has 148 SMs)       */
+  int batch_choices[4];      /* candidate items-per-claim multipliers; 0-terminated        */
+  uint32_t models_allowed;   /* bitmask of 1 << vp_group_model; 0 = all                    */
+  int max_candidates;        /* 0 = 400                                                    */
+  int repeats;               /* timed runs per candidate (min taken); 0 = 1                */
+} vp_autotune_opts;
+
+typedef struct vp_tune_report {
+  int candidates_total;      /* after pruning                                              */
+  int candidates_run;
+  int candidates_timed_out;  /* stopped by timeoutexec (Fig. 10)                           */
+  double best_ms;
+  double baseline_kbk_ms;
+  double baseline_mega_ms;
+  int max_blocks_per_sm[VP_MAX_STAGES];  /* profiling component (L13, L45)                */
+  int regs_per_thread[VP_MAX_STAGES];
+  int smem_per_block[VP_MAX_STAGES];
+} vp_tune_report;
+
+/* ---------------- family parameter structs (device pointers are BORROWED) ------------ */
+typedef struct vp_toy_params {
+  int32_t threshold;         /* THRESHOLD of Fig. 9                                        */
+  int32_t pad;
+  int32_t* out;              /* sink output values, capacity >= #seeds                     */
+  unsigned long long* n_out; /* device counter, reset by every vp_run                      */
+} vp_toy_params;
+
+typedef struct vp_collatz_params {
+  uint32_t* steps_out;       /* [n ids] stopping time per id                               */
+  uint32_t* seen;            /* [n ids] times each id reached the sink (reset by vp_run)  */
+  uint32_t n_ids;
+  uint32_t max_steps;        /* recursion guard                                            */
+} vp_collatz_params;
+
+typedef struct vp_reyes_params {
+  int32_t W, H, n_frames, patches_per_frame, max_depth, pad0;
+  float t_dice, near_w;
+  const float* M;            /* [n_frames][16] view-projection, row-major                  */
+  const float* albedo;       /* [patches_per_frame][4]                                     */
+  float L[4];                /* light direction                                            */
+  void* fb;                  /* [n_frames*H*W] 16-B records {u64 key, f32 s, u32 pad},     */
+                             /* reset by vp_run; key = UINT64_MAX when uncovered           */
+  float* colour;             /* [n_frames*H*W][4] resolved colour, written by vp_run       */
+} vp_reyes_params;
+
+/* ---------------- calls ---------------- */
+const char* vp_status_string(vp_status s);
+const char* vp_last_error(void* p);
+
+/* Create an empty pipeline on CUDA device `device` (Fig. 2 framework object). */
+vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out);
+vp_status vp_pipeline_destroy(void* p);
+
+/* Register the next stage (class Stage_k : public BaseStage, L37).  Stage ids are dense,
+ * assigned in registration order; the kinds must be one family in its canonical order. */
+vp_status vp_stage_register(void* p, const vp_stage_desc* s, int* stage_id);
+
+/* VersaPipe::insertIntoQueue(initItems, n) (L37).  Items are COPIED (host or device
+ * memory per flags) and snapshotted: every vp_run re-seeds from them.  flags:
+ *   VP_INSERT_DEVICE  items is a device pointer
+ *   VP_INSERT_REPLACE drop previously inserted items of this stage first            */
+#define VP_INSERT_DEVICE 0x1
+#define VP_INSERT_REPLACE 0x2
+vp_status vp_insert(void* p, int stage_id, const void* items, size_t n, int flags);
+/* Stream-ordered variant (the copy is enqueued on `cuda_stream`). */
+vp_status vp_insert_async(void* p, int stage_id, const void* items, size_t n, int flags, void* cuda_stream);
+
+/* Choose the execution model and SM / block binding (optional step of §6; L37).
+ * binding == NULL: defaults (all SMs; coarse: equal SM split; fine: equal block split).
+ * batch: items per claim for every stage (0 = per-stage defaults / binding->batch). */
+vp_status vp_configure(void* p, int model, const vp_sm_binding* binding, int batch);
+vp_status vp_configure_config(void* p, const vp_config* c);
+vp_status vp_get_config(void* p, vp_config* out);
+
+/* Run the pipeline to completion on `cuda_stream` (NULL = legacy default stream), then
+ * return.  stats may be NULL. */
+vp_status vp_run(void* p, void* cuda_stream, vp_run_stats* stats);
+
+/* Device watchdog for subsequent runs, in milliseconds (> 0).  The auto-tuner's
+ * timeoutexec(mintime, config) (Fig. 10) uses the same mechanism. */
+vp_status vp_set_timeout(void* p, double ms);
+
+/* Offline auto-tuner (L41–L45, Fig. 10): profile, enumerate pruned {g, s, b}, run each
+ * candidate under timeoutexec(mintime), keep and apply the fastest.  best/report may be NULL. */
+vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best, vp_tune_report* report);
+
+/* Profiling component (L13, L45): max resident blocks per SM of each single-stage kernel. */
+vp_status vp_profile(void* p, int* max_blocks_per_sm, int* regs_per_thread, int* smem_per_block);
+
+/* Library-owned / borrowed outputs of the family (sink results). index 0 = primary. */
+vp_status vp_get_output(void* p, int index, void** dev_ptr, size_t* bytes);
+
+/* The task trace of the last run (VP_FLAG_TRACE): library-owned device array of
+ * {u64 item id, u32 stage, u32 smid} records, valid until the next vp_run. */
+vp_status vp_get_trace(void* p, void** dev_ptr, size_t* n_records);
+
+vp_status vp_config_to_string(const vp_config* c, char* buf, size_t buf_len);
+vp_status vp_config_from_string(const char* s, vp_config* out);
+
+/* Device properties the binding layer needs (no torch types cross the ABI). */
+vp_status vp_device_info(int device, int* num_sms, int* cc_major, int* cc_minor);
+/* Minimal CUDA plumbing for bindings without their own CUDA runtime. kind: 0 H2D, 1 D2H, 2 D2D */
+vp_status vp_memcpy(void* dst, const void* src, size_t bytes, int kind, void* cuda_stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,506 @@
+// fam_reyes.cu — Reyes rendering as VersaPipe stages (Fig. 1: Primitives ->
+// Bound -> diceable? -> Split (back to Bound) | Dice -> Shade -> Image; L55; Table 2 272-B
+// item).  The paper gives no formulas; the arithmetic follows DESIGN.md §2 readings
+// R-R1..R-R12.  Compiled with -fmad=false: every float operation is a
+// separately rounded IEEE op in the written order, so results are bit-identical to the
+// CPU oracle.
+//
+// Thread mapping (threadNum, L37): Bound 16 threads/patch (one per control point),
+// Split 16 (one per output control point), Dice 32 (one warp per patch, 81 grid points),
+// Shade 64 (one per micropolygon).
+#include <math.h>
+
+#include <limits.h>
+
+#include <algorithm>
+
+#include "../../include/vp.h"
+#include "vp_family.cuh"
+
+namespace vp {
+
+#ifndef VP_REYES_MINB
+#define VP_REYES_MINB 3
+#endif
+
+struct RPatch {           // 272 B
+  float4 cp[16];          // P[a][b] at cp[4a+b]; a = u index, b = v index
+  uint32_t id, path, dirs, depth;
+};
+static_assert(sizeof(RPatch) == 272, "patch item is 272 B (Table 2)");
+
+constexpr int kG = 8, kNG = 9, kNP = 81;
+struct RGrid {            // Dice -> Shade item: header + SoA grid (x,y,z object; sx,sy,zs screen)
+  uint32_t id, path, depth, dirs;
+  float g[6][kNP];
+  uint32_t pad[2];
+};
+static_assert(sizeof(RGrid) == 1968, "grid item stride");
+
+struct __align__(16) FbRec {
+  unsigned long long key;
+  float s;
+  uint32_t pad;
+};
+
+__device__ __forceinline__ float4 project(const float* __restrict__ M, float x, float y, float z, float w) {
+  float c[4];
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    float acc = __ldg(M + 4 * r + 0) * x;
+    acc = acc + __ldg(M + 4 * r + 1) * y;
+    acc = acc + __ldg(M + 4 * r + 2) * z;
+    acc = acc + __ldg(M + 4 * r + 3) * w;
+    c[r] = acc;
+  }
+  return make_float4(c[0], c[1], c[2], c[3]);
+}
+
+__device__ __forceinline__ void screen(const vp_reyes_params& p, float4 c, float& sx, float& sy, float& zs) {
+  float nx = c.x / c.w;
+  float ny = c.y / c.w;
+  sx = (nx * 0.5f + 0.5f) * (float)p.W;
+  sy = (ny * 0.5f + 0.5f) * (float)p.H;
+  zs = c.z / c.w;
+}
+
+__device__ __forceinline__ float red16_max(float v) {
+#pragma unroll
+  for (int o = 8; o >= 1; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o, 16));
+  return v;
+}
+__device__ __forceinline__ float red16_min(float v) {
+#pragma unroll
+  for (int o = 8; o >= 1; o >>= 1) v = fminf(v, __shfl_xor_sync(0xffffffffu, v, o, 16));
+  return v;
+}
+
+__device__ __forceinline__ void bernstein(float t, float B[4]) {
+  float s = 1.0f - t;
+  B[0] = (s * s) * s;
+  B[1] = ((3.0f * t) * s) * s;
+  B[2] = ((3.0f * t) * t) * s;
+  B[3] = (t * t) * t;
+}
+
+__device__ __forceinline__ uint32_t zkey(float z) {
+  uint32_t b = __float_as_uint(z);
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+
+template <class I>
+__device__ __forceinline__ I edge(I ax, I ay, I bx, I by, I px, I py) {
+  return (bx - ax) * (py - ay) - (by - ay) * (px - ax);
+}
+// top-left-style ownership of boundary points (reading R-R9)
+template <class I>
+__device__ __forceinline__ bool owns(I ax, I ay, I bx, I by) {
+  I dx = bx - ax, dy = by - ay;
+  return dy > 0 || (dy == 0 && dx < 0);
+}
+__device__ __forceinline__ long long fdiv256(long long a) { return a >> 8; }  // floor(a / 256)
+
+// 128-bit compare-and-swap (sm_90+): atomically keep the minimum key with its shade factor.
+__device__ __forceinline__ void fb_min(FbRec* rec, unsigned long long key, float s) {
+  unsigned long long* a = (unsigned long long*)rec;
+  // first attempt assumes the cleared record {UINT64_MAX, 0}: one L2 round trip for a
+  // first touch; otherwise the failed CAS returns the current record
+  unsigned long long cur_k = ~0ull, cur_s = 0ull;
+  const unsigned long long new_s = (unsigned long long)__float_as_uint(s);
+  while (key < cur_k) {
+    unsigned long long ok, os;
+    asm volatile(
+        "{\n\t.reg .b128 c, n, o;\n\t"
+        "mov.b128 c, {%2, %3};\n\t"
+        "mov.b128 n, {%4, %5};\n\t"
+        "atom.global.relaxed.gpu.cas.b128 o, [%6], c, n;\n\t"
+        "mov.b128 {%0, %1}, o;\n\t}"
+        : "=l"(ok), "=l"(os)
+        : "l"(cur_k), "l"(cur_s), "l"(key), "l"(new_s), "l"(a)
+        : "memory");
+    if (ok == cur_k && os == cur_s) return;
+    cur_k = ok;
+    cur_s = os;
+  }
+}
+
+// Pixel-centre loop of one positively oriented triangle, coordinates relative to an
+// origin inside its bounding box (exact in I: int32 when the box is < 2^14 Q8 units).
+template <class I>
+__device__ __forceinline__ void cover(const vp_reyes_params& p, FbRec* fb, I ax, I ay, I bx, I by, I cx, I cy,
+                                      long long ox, long long oy, long long px0, long long px1, long long py0,
+                                      long long py1, unsigned long long key, float s) {
+  const bool o0 = owns(ax, ay, bx, by), o1 = owns(bx, by, cx, cy), o2 = owns(cx, cy, ax, ay);
+  for (long long py = py0; py <= py1; ++py) {
+    const I Y = (I)(py * 256 + 128 - oy);
+    for (long long px = px0; px <= px1; ++px) {
+      const I X = (I)(px * 256 + 128 - ox);
+      I w0 = edge(ax, ay, bx, by, X, Y), w1 = edge(bx, by, cx, cy, X, Y), w2 = edge(cx, cy, ax, ay, X, Y);
+      bool in = (w0 > 0 || (w0 == 0 && o0)) && (w1 > 0 || (w1 == 0 && o1)) && (w2 > 0 || (w2 == 0 && o2));
+      if (in) fb_min(fb + (size_t)py * p.W + px, key, s);
+    }
+  }
+}
+
+__device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, long long ay, long long bx, long long by,
+                           long long cx, long long cy, unsigned long long key, float s) {
+  long long xmin = min(ax, min(bx, cx)), xmax = max(ax, max(bx, cx));
+  long long ymin = min(ay, min(by, cy)), ymax = max(ay, max(by, cy));
+  long long px0 = -fdiv256(-(xmin - 128)), px1 = fdiv256(xmax - 128);
+  long long py0 = -fdiv256(-(ymin - 128)), py1 = fdiv256(ymax - 128);
+  if (px0 < 0) px0 = 0;
+  if (py0 < 0) py0 = 0;
+  if (px1 > p.W - 1) px1 = p.W - 1;
+  if (py1 > p.H - 1) py1 = p.H - 1;
+  if (px0 > px1 || py0 > py1) return;  // no pixel centre inside the box
+  if (xmax - xmin < (1ll << 14) && ymax - ymin < (1ll << 14)) {
+    // every |difference| < 2^14 -> products < 2^28: int32 is exact
+    int Ax = (int)(ax - xmin), Ay = (int)(ay - ymin), Bx = (int)(bx - xmin), By = (int)(by - ymin);
+    int Cx = (int)(cx - xmin), Cy = (int)(cy - ymin);
+    int area = edge(Ax, Ay, Bx, By, Cx, Cy);
+    if (area == 0) return;
+    if (area < 0) cover<int>(p, fb, Ax, Ay, Cx, Cy, Bx, By, xmin, ymin, px0, px1, py0, py1, key, s);
+    else cover<int>(p, fb, Ax, Ay, Bx, By, Cx, Cy, xmin, ymin, px0, px1, py0, py1, key, s);
+  } else {
+    long long area = edge(ax, ay, bx, by, cx, cy);
+    if (area == 0) return;
+    if (area < 0) cover<long long>(p, fb, ax, ay, cx, cy, bx, by, 0, 0, px0, px1, py0, py1, key, s);
+    else cover<long long>(p, fb, ax, ay, bx, by, cx, cy, 0, 0, px0, px1, py0, py1, key, s);
+  }
+}
+
+struct ReyesF {
+  static constexpr int S = 4;
+  static constexpr int BOUND = 0, SPLIT = 1, DICE = 2, SHADE = 3;
+  static constexpr int kinds[S] = {VP_REYES_BOUND, VP_REYES_SPLIT, VP_REYES_DICE, VP_REYES_SHADE};
+  using Params = vp_reyes_params;
+  static constexpr int stride(int s) { return s == SHADE ? (int)sizeof(RGrid) : (int)sizeof(RPatch); }
+  static constexpr int threads_per_item(int s) { return s == BOUND ? 16 : s == SPLIT ? 16 : s == DICE ? 32 : 64; }
+  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 32 : 8; }
+  static constexpr int default_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 8 : 4; }
+  static constexpr int fanout(int s, int t) {
+    return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
+  }
+  static constexpr bool uses_latches(int, int) { return false; }
+  static constexpr int scratch_bytes(int, int) { return 0; }
+  static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
+  // register budget: kernels containing Shade are held to 3 resident blocks per SM
+  static constexpr int min_blocks(int lo, int hi, bool) { return hi == SHADE ? VP_REYES_MINB : 1; }
+
+  template <int s>
+  static __device__ unsigned long long item_id(const uint8_t* it) {
+    // node id = (id << 12) | (depth << 8) | path  (frame, patch, depth, path)
+    if constexpr (s == SHADE) {
+      const RGrid* g = (const RGrid*)it;
+      return ((unsigned long long)g->id << 12) | ((unsigned long long)(g->depth & 15u) << 8) | (g->path & 0xFFu);
+    } else {
+      const RPatch* q = (const RPatch*)it;
+      return ((unsigned long long)q->id << 12) | ((unsigned long long)(q->depth & 15u) << 8) | (q->path & 0xFFu);
+    }
+  }
+
+  template <int s, class Ctx>
+  static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
+    if constexpr (s == BOUND) bound(ctx, items, n);
+    else if constexpr (s == SPLIT) split(ctx, items, n);
+    else if constexpr (s == DICE) dice(ctx, items, n);
+    else shade(ctx, items, n);
+  }
+
+  // -------------------------------------------------------------- Bound (16 thr/patch)
+  template <class Ctx>
+  static __device__ void bound(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    const int lane = threadIdx.x & 15;
+    for (int r0 = 0; r0 < n; r0 += kThreads / 16) {
+      const int k = r0 + (threadIdx.x >> 4);
+      const bool valid = k < n;
+      const RPatch* P = (const RPatch*)(items + (size_t)(valid ? k : 0) * sizeof(RPatch));
+      const uint32_t id = P->id, depth = P->depth;
+      uint32_t frame = id >> 12;
+      if (frame >= (uint32_t)p.n_frames) frame = 0;
+      const float* M = p.M + 16 * (size_t)frame;
+      const float4 q = P->cp[lane];
+      float4 c = project(M, q.x, q.y, q.z, q.w);
+      const bool behind = !(c.w > p.near_w);
+      const unsigned bal = __ballot_sync(0xffffffffu, behind);
+      const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
+      float sx, sy, zs;
+      screen(p, c, sx, sy, zs);
+      // screen-space split metric (reading R-R5)
+      float sx12 = __shfl_sync(0xffffffffu, sx, (lane & 3) + 12, 16), sy12 = __shfl_sync(0xffffffffu, sy, (lane & 3) + 12, 16);
+      float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
+      float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
+      float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
+      // object-space metric (near-plane straddle, R-R4)
+      float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16), oy12 = __shfl_sync(0xffffffffu, q.y, (lane & 3) + 12, 16),
+            oz12 = __shfl_sync(0xffffffffu, q.z, (lane & 3) + 12, 16);
+      float ox3 = __shfl_down_sync(0xffffffffu, q.x, 3, 16), oy3 = __shfl_down_sync(0xffffffffu, q.y, 3, 16),
+            oz3 = __shfl_down_sync(0xffffffffu, q.z, 3, 16);
+      float olu = 0.0f, olv = 0.0f;
+      if (lane < 4) {
+        olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
+        olu = olu + fabsf(oz12 - q.z);
+      }
+      if ((lane & 3) == 0) {
+        olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
+        olv = olv + fabsf(oz3 - q.z);
+      }
+      float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
+      lu = red16_max(lu);
+      lv = red16_max(lv);
+      olu = red16_max(olu);
+      olv = red16_max(olv);
+      int cls;  // 0 cull, 1 split, 2 dice
+      int dir = 0;
+      if (nbehind == 16) {
+        cls = 0;
+      } else if (nbehind > 0) {
+        cls = ((int)depth >= p.max_depth) ? 0 : 1;
+        dir = (olu >= olv) ? 0 : 1;
+      } else if (xmax < 0.0f || xmin >= (float)p.W || ymax < 0.0f || ymin >= (float)p.H) {
+        cls = 0;
+      } else {
+        float bw = xmax - xmin, bh = ymax - ymin;
+        float ext = bw > bh ? bw : bh;
+        if ((int)depth >= p.max_depth || ext <= p.t_dice) cls = 2;
+        else {
+          cls = 1;
+          dir = (lu >= lv) ? 0 : 1;
+        }
+      }
+      if (!valid) cls = 0;
+      int slot = -1;
+      if (lane == 0 && cls == 1) slot = ctx.template reserve<SPLIT>();
+      if (lane == 0 && cls == 2) slot = ctx.template reserve<DICE>();
+      slot = __shfl_sync(0xffffffffu, slot, 0, 16);
+      if (cls != 0 && slot >= 0) {
+        RPatch* out = (RPatch*)(cls == 1 ? ctx.template out_ptr<SPLIT>(slot) : ctx.template out_ptr<DICE>(slot));
+        out->cp[lane] = q;
+        if (lane == 0) {
+          out->id = id;
+          out->path = P->path;
+          out->dirs = (cls == 1) ? ((P->dirs & ~(1u << depth)) | ((uint32_t)dir << depth)) : P->dirs;
+          out->depth = depth;
+        }
+      }
+    }
+  }
+
+  // -------------------------------------------------------------- Split (16 thr/patch)
+  template <class Ctx>
+  static __device__ void split(Ctx& ctx, const uint8_t* items, int n) {
+    const int lane = threadIdx.x & 15;
+    const int line = lane >> 2, t = lane & 3;
+    for (int r0 = 0; r0 < n; r0 += kThreads / 16) {
+      const int k = r0 + (threadIdx.x >> 4);
+      const bool valid = k < n;
+      const RPatch* P = (const RPatch*)(items + (size_t)(valid ? k : 0) * sizeof(RPatch));
+      const uint32_t depth = P->depth;
+      const int dir = (int)((P->dirs >> depth) & 1u);
+      // control point u of this thread's curve: (u, line) for a u-split, (line, u) for v
+      const int base = dir == 0 ? line : 4 * line, step = dir == 0 ? 4 : 1;
+      const int my = base + step * t;
+      float4 a = P->cp[base], b = P->cp[base + step], c = P->cp[base + 2 * step], d = P->cp[base + 3 * step];
+      float4 L, R;
+      // de Casteljau at t = 1/2 (reading R-R6), per component, exactly this order
+#define VP_CASTELJAU(comp)                                                   \
+  {                                                                          \
+    float ab = (a.comp + b.comp) * 0.5f, bc = (b.comp + c.comp) * 0.5f;      \
+    float cd = (c.comp + d.comp) * 0.5f;                                     \
+    float abc = (ab + bc) * 0.5f, bcd = (bc + cd) * 0.5f;                    \
+    float m = (abc + bcd) * 0.5f;                                            \
+    L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
+    R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
+  }
+      VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+#undef VP_CASTELJAU
+      int slot = -1;
+      if (lane == 0 && valid) slot = ctx.template reserve<BOUND>(2);
+      slot = __shfl_sync(0xffffffffu, slot, 0, 16);
+      if (valid && slot >= 0) {
+        RPatch* l = (RPatch*)ctx.template out_ptr<BOUND>(slot);
+        RPatch* r = (RPatch*)ctx.template out_ptr<BOUND>(slot + 1);
+        l->cp[my] = L;
+        r->cp[my] = R;
+        if (lane == 0) {
+          l->id = r->id = P->id;
+          l->dirs = r->dirs = (P->dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
+          l->depth = r->depth = depth + 1;
+          l->path = P->path & ~(1u << depth);
+          r->path = P->path | (1u << depth);
+        }
+      }
+    }
+  }
+
+  // -------------------------------------------------------------- Dice (warp/patch)
+  template <class Ctx>
+  static __device__ void dice(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    const int lane = threadIdx.x & 31;
+    for (int r0 = 0; r0 < n; r0 += kThreads / 32) {
+      const int k = r0 + (threadIdx.x >> 5);
+      if (k >= n) break;  // warp-uniform
+      const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
+      uint32_t frame = P->id >> 12;
+      if (frame >= (uint32_t)p.n_frames) frame = 0;
+      const float* M = p.M + 16 * (size_t)frame;
+      int slot = 0;
+      if (lane == 0) slot = ctx.template reserve<SHADE>();
+      slot = __shfl_sync(0xffffffffu, slot, 0);
+      if (slot < 0) continue;
+      RGrid* out = (RGrid*)ctx.template out_ptr<SHADE>(slot);
+      for (int g = lane; g < kNP; g += 32) {
+        const int i = g / kNG, j = g - i * kNG;
+        float Bu[4], Bv[4];
+        bernstein((float)i * 0.125f, Bu);
+        bernstein((float)j * 0.125f, Bv);
+        float x = 0.0f, y = 0.0f, z = 0.0f;
+#pragma unroll
+        for (int a = 0; a < 4; ++a)
+#pragma unroll
+          for (int b = 0; b < 4; ++b) {
+            const float w = Bu[a] * Bv[b];
+            const float4 cp = P->cp[4 * a + b];
+            x = x + w * cp.x;
+            y = y + w * cp.y;
+            z = z + w * cp.z;
+          }
+        float4 c = project(M, x, y, z, 1.0f);
+        float sx, sy, zs;
+        screen(p, c, sx, sy, zs);
+        out->g[0][g] = x;
+        out->g[1][g] = y;
+        out->g[2][g] = z;
+        // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
+        const float X = sx * 256.0f, Y = sy * 256.0f;
+        const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
+        out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
+        out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
+        out->g[5][g] = zs;
+      }
+      if (lane == 0) {
+        out->id = P->id;
+        out->path = P->path;
+        out->depth = P->depth;
+        out->dirs = P->dirs;
+      }
+    }
+  }
+
+  // -------------------------------------------------------------- Shade (64 thr/grid)
+  template <class Ctx>
+  static __device__ void shade(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    const int q = threadIdx.x & 63;
+    const int i = q >> 3, j = q & 7;
+    for (int r0 = 0; r0 < n; r0 += kThreads / 64) {
+      const int k = r0 + (threadIdx.x >> 6);
+      if (k >= n) break;  // uniform per pair of warps
+      const RGrid* Gd = (const RGrid*)(items + (size_t)k * sizeof(RGrid));
+      const uint32_t frame = Gd->id >> 12, patch = Gd->id & 0xFFFu;
+      if (frame >= (uint32_t)p.n_frames) continue;
+      const int g00 = i * kNG + j, g10 = (i + 1) * kNG + j, g01 = i * kNG + j + 1, g11 = (i + 1) * kNG + j + 1;
+      float e1[3], e2[3];
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        e1[c] = Gd->g[c][g10] - Gd->g[c][g00];
+        e2[c] = Gd->g[c][g01] - Gd->g[c][g00];
+      }
+      float nx = e1[1] * e2[2] - e1[2] * e2[1];
+      float ny = e1[2] * e2[0] - e1[0] * e2[2];
+      float nz = e1[0] * e2[1] - e1[1] * e2[0];
+      float nn = nx * nx + ny * ny;
+      nn = nn + nz * nz;
+      float s;
+      if (nn == 0.0f) {
+        s = 0.1f;
+      } else {
+        float d = nx * p.L[0] + ny * p.L[1];
+        d = d + nz * p.L[2];
+        float t = d / sqrtf(nn);
+        if (!(t > 0.0f)) t = 0.0f;
+        s = 0.1f + 0.9f * t;
+      }
+      const float zq = ((Gd->g[5][g00] + Gd->g[5][g10]) + (Gd->g[5][g11] + Gd->g[5][g01])) * 0.25f;
+      const uint32_t mp = (patch << 18) | ((Gd->path & 0xFFu) << 10) | ((Gd->depth & 0xFu) << 6) | (uint32_t)q;
+      const unsigned long long key = ((unsigned long long)zkey(zq) << 32) | mp;
+      const int gi[4] = {g00, g10, g11, g01};
+      long long vx[4], vy[4];
+      bool ok = true;
+#pragma unroll
+      for (int v = 0; v < 4; ++v) {
+        const int X = __float_as_int(Gd->g[3][gi[v]]), Y = __float_as_int(Gd->g[4][gi[v]]);
+        if (X == INT_MIN || Y == INT_MIN) ok = false;
+        vx[v] = X;
+        vy[v] = Y;
+      }
+      if (!ok) continue;
+      FbRec* fb = (FbRec*)p.fb + (size_t)frame * p.W * p.H;
+      raster_tri(p, fb, vx[0], vy[0], vx[1], vy[1], vx[2], vy[2], key, s);
+      raster_tri(p, fb, vx[0], vy[0], vx[2], vy[2], vx[3], vy[3], key, s);
+    }
+  }
+
+  // -------------------------------------------------------------- sinks
+  static cudaError_t init_run(const Params& p, cudaStream_t st);
+  static cudaError_t finalize(const Params& p, cudaStream_t st);
+  static bool output(const Params& p, int idx, void** ptr, size_t* bytes) {
+    size_t npix = (size_t)p.n_frames * p.W * p.H;
+    if (idx == 0) { *ptr = p.fb; *bytes = npix * sizeof(FbRec); return true; }
+    if (idx == 1) { *ptr = p.colour; *bytes = npix * 16; return true; }
+    return false;
+  }
+  static const char* validate(const Params& p) {
+    if (p.W <= 0 || p.H <= 0 || p.W > 32768 || p.H > 32768) return "vp_reyes_params: bad W/H";
+    if (p.n_frames <= 0 || p.n_frames > (1 << 20)) return "vp_reyes_params: bad n_frames";
+    if (p.patches_per_frame <= 0 || p.patches_per_frame > 4096) return "vp_reyes_params: patches_per_frame must be in [1, 4096]";
+    if (p.max_depth < 0 || p.max_depth > 8) return "vp_reyes_params: max_depth must be in [0, 8] (8-bit path)";
+    if (!p.M || !p.albedo || !p.fb || !p.colour) return "vp_reyes_params: M, albedo, fb, colour are required device pointers";
+    if (((uintptr_t)p.fb & 15) || ((uintptr_t)p.colour & 15)) return "vp_reyes_params: fb and colour must be 16-B aligned";
+    return nullptr;
+  }
+};
+
+__global__ void k_reyes_clear(FbRec* fb, size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    FbRec r;
+    r.key = ~0ull;
+    r.s = 0.0f;
+    r.pad = 0;
+    fb[i] = r;
+  }
+}
+// Resolve (sink): colour = albedo[patch of the winning micropolygon] * s (reading R-R11).
+__global__ void k_reyes_resolve(const FbRec* __restrict__ fb, float4* __restrict__ colour, const float* __restrict__ albedo,
+                                size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    FbRec r = fb[i];
+    float4 c = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (r.key != ~0ull) {
+      uint32_t patch = (uint32_t)(r.key >> 18) & 0xFFFu;
+      const float* a = albedo + 4 * (size_t)patch;
+      c = make_float4(a[0] * r.s, a[1] * r.s, a[2] * r.s, 1.0f);
+    }
+    colour[i] = c;
+  }
+}
+
+cudaError_t ReyesF::init_run(const Params& p, cudaStream_t st) {
+  size_t n = (size_t)p.n_frames * p.W * p.H;
+  k_reyes_clear<<<(int)std::min<size_t>((n + 255) / 256, 148 * 16), 256, 0, st>>>((FbRec*)p.fb, n);
+  return cudaGetLastError();
+}
+cudaError_t ReyesF::finalize(const Params& p, cudaStream_t st) {
+  size_t n = (size_t)p.n_frames * p.W * p.H;
+  k_reyes_resolve<<<(int)std::min<size_t>((n + 255) / 256, 148 * 16), 256, 0, st>>>((const FbRec*)p.fb, (float4*)p.colour, p.albedo, n);
+  return cudaGetLastError();
+}
+
+const FamilyOps* family_reyes() {
+  static FamilyImpl<ReyesF> f("reyes");
+  return &f;
+}
+
+}  // namespace vp

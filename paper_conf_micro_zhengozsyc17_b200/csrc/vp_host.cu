@@ -1,0 +1,951 @@
+// vp_host.cu — the C ABI of libvp.so (include/vp.h): pipeline assembly, the
+// high-level control of PAPER.md §5 (L27: "puts stages into different kernels and do
+// SM assignment for them ... we put each kernel into a separate CUDA stream"), the
+// KBK host loop (L13 Fig. 3b), the profiling component and the offline auto-tuner
+// (L41–L45, Fig. 10).
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "../../include/vp.h"
+#include "vp_family.cuh"
+
+using namespace vp;
+
+namespace {
+
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr};
+void init_families() {
+  if (!all_families[0]) {
+    all_families[0] = family_toy();
+    all_families[1] = family_collatz();
+    all_families[2] = family_reyes();
+  }
+}
+const FamilyOps* family_of_kind(int kind, int* pos) {
+  init_families();
+  for (const FamilyOps* f : all_families)
+    for (int s = 0; s < f->S; ++s)
+      if (f->kinds[s] == kind) {
+        *pos = s;
+        return f;
+      }
+  return nullptr;
+}
+
+// ---------------------------------------------------------------- device helpers
+__global__ void k_init_seq(unsigned long long* seq, unsigned long long cap, unsigned long long start) {
+  for (unsigned long long i = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; i < cap;
+       i += (unsigned long long)gridDim.x * blockDim.x) {
+    // slot (start + i) & mask is free for ticket start + i
+    unsigned long long t = start + i;
+    seq[t & (cap - 1)] = t;
+  }
+}
+
+struct RunInit {
+  long long pending;
+  unsigned long long watchdog_ns;
+  unsigned long long seeds[kMaxStages];
+};
+
+__global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
+  int t = threadIdx.x;
+  for (int i = t; i < kMaxKernels * kMaxSM; i += blockDim.x) blk[i] = 0;
+  if (t < kMaxStages) {
+    c->seed_head[t].v = 0;
+    c->deq[t] = 0;
+    c->enq[t] = ri.seeds[t];
+    c->max_depth[t] = 0;
+    c->exec_ns[t] = 0;
+    c->flush_ns[t] = 0;
+  }
+  if (t < kMaxKernels) c->idle_ns[t] = 0;
+  if (t < kMaxKernels) {
+    c->arrivals[t].v = 0;
+    c->admitted[t].v = 0;
+  }
+  if (t == 0) {
+    c->pending.v = (unsigned long long)ri.pending;
+    c->abort.v = 0;
+    c->trace_n.v = 0;
+    c->fallback_admits = 0;
+    c->deadline.v = globaltimer() + ri.watchdog_ns;
+  }
+}
+
+__global__ void k_reset_queues(Ctrl* c) {
+  int t = threadIdx.x;
+  if (t < kMaxStages) {
+    c->tail[t].v = 0;
+    c->head[t].v = 0;
+    c->count[t].v = 0;
+  }
+}
+
+// ---------------------------------------------------------------- pipeline object
+struct StageRec {
+  vp_stage_desc d;
+  std::string name;
+  int cap_log2 = 0;
+  uint8_t* slots = nullptr;
+  unsigned long long* seq = nullptr;
+  uint8_t* seeds = nullptr;
+  size_t seed_cap = 0;  // items
+  size_t n_seeds = 0;
+};
+
+struct KernelPlan {
+  int lo, hi;
+  bool rtc;
+  int quota;
+  uint32_t mask[kMaskWords];
+  int grid;
+  bool coop;
+  int kslot;
+};
+
+struct Plan {
+  int model = -1;
+  std::vector<KernelPlan> kernels;     // persistent kernels
+  std::vector<int> kbk_stages;         // stages driven by the host wave loop
+  bool wave_rtc = false;               // standalone RTC: waves of the [0,S-1] RTC kernel
+  int batch[kMaxStages] = {};
+  vp_config cfg{};
+};
+
+}  // namespace
+
+struct vp_pipeline_s {
+  int device = 0;
+  int num_sms = 0;
+  vp_pipeline_desc desc{};
+  const FamilyOps* fam = nullptr;
+  std::vector<uint8_t> params;
+  std::vector<StageRec> st;
+  bool queues_ready = false;
+  bool configured = false;
+  bool dirty_queues = false;  // after an aborted run: reset rings before the next one
+  Plan plan;
+  Ctrl* ctrl = nullptr;
+  uint32_t* blk = nullptr;
+  TraceRec* trace = nullptr;
+  Ctrl* h_ctrl = nullptr;     // pinned readback
+  uint32_t* h_blk = nullptr;
+  volatile uint32_t* h_arrive = nullptr;  // mapped pinned: per-kernel dispatch-complete flags
+  uint32_t* d_arrive = nullptr;
+  uint32_t epoch = 0;
+  cudaStream_t streams[kMaxKernels] = {};
+  cudaEvent_t ev_fork = nullptr, ev_start = nullptr, ev_end = nullptr, ev_join[kMaxKernels] = {};
+  cudaEvent_t ev_kbeg[kMaxKernels] = {};
+  std::string err;
+  int kernel_occ_cache[kMaxStages][kMaxStages][2] = {};
+  double timeout_ms = 30000;
+};
+
+namespace {
+
+vp_status fail(vp_pipeline_s* p, vp_status s, const char* fmt, ...) {
+  if (p) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    p->err = buf;
+  }
+  return s;
+}
+#define CUDA_TRY(p, x)                                                                        \
+  do {                                                                                        \
+    cudaError_t e_ = (x);                                                                     \
+    if (e_ != cudaSuccess) {                                                                  \
+      return fail((p), e_ == cudaErrorMemoryAllocation ? VP_ERR_OOM : VP_ERR_CUDA, "%s: %s (%s:%d)", #x, \
+                  cudaGetErrorString(e_), __FILE__, __LINE__);                                \
+    }                                                                                         \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    cudaGetDevice(&prev);
+    if (prev != d) cudaSetDevice(d);
+  }
+  ~DeviceGuard() {
+    int cur;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+int occupancy(vp_pipeline_s* p, int lo, int hi, bool rtc) {
+  int& c = p->kernel_occ_cache[lo][hi][rtc ? 1 : 0];
+  if (c) return c;
+  const void* fn = p->fam->kernel(lo, hi, rtc);
+  if (!fn) return 0;
+  size_t sm = p->fam->smem(lo, hi, rtc);
+  if (sm > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+  int occ = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kThreads, sm) != cudaSuccess) occ = 0;
+  c = occ;
+  return occ;
+}
+
+void mask_all(uint32_t* m, int nsm) {
+  memset(m, 0, sizeof(uint32_t) * kMaskWords);
+  for (int i = 0; i < nsm; ++i) m[i >> 5] |= 1u << (i & 31);
+}
+void mask_range(uint32_t* m, int a, int b) {
+  memset(m, 0, sizeof(uint32_t) * kMaskWords);
+  for (int i = a; i < b; ++i) m[i >> 5] |= 1u << (i & 31);
+}
+int mask_count(const uint32_t* m, int nsm) {
+  int c = 0;
+  for (int i = 0; i < nsm; ++i) c += (m[i >> 5] >> (i & 31)) & 1u;
+  return c;
+}
+
+vp_status ensure_queues(vp_pipeline_s* p) {
+  if (p->queues_ready) return VP_OK;
+  for (size_t s = 0; s < p->st.size(); ++s) {
+    StageRec& r = p->st[s];
+    size_t cap = 1ull << r.cap_log2;
+    CUDA_TRY(p, cudaMalloc(&r.slots, cap * (size_t)p->fam->stride((int)s)));
+    CUDA_TRY(p, cudaMalloc(&r.seq, cap * sizeof(unsigned long long)));
+    k_init_seq<<<256, 256>>>(r.seq, cap, 0);
+    CUDA_TRY(p, cudaGetLastError());
+  }
+  CUDA_TRY(p, cudaDeviceSynchronize());
+  p->queues_ready = true;
+  return VP_OK;
+}
+
+vp_status reset_queues(vp_pipeline_s* p, cudaStream_t st) {
+  k_reset_queues<<<1, 32, 0, st>>>(p->ctrl);
+  for (size_t s = 0; s < p->st.size(); ++s) {
+    size_t cap = 1ull << p->st[s].cap_log2;
+    k_init_seq<<<256, 256, 0, st>>>(p->st[s].seq, cap, 0);
+  }
+  CUDA_TRY(p, cudaGetLastError());
+  p->dirty_queues = false;
+  return VP_OK;
+}
+
+Common make_common(vp_pipeline_s* p) {
+  Common c;
+  memset(&c, 0, sizeof(c));
+  for (size_t s = 0; s < p->st.size(); ++s) {
+    const StageRec& r = p->st[s];
+    c.q[s].slots = r.slots;
+    c.q[s].seq = r.seq;
+    c.q[s].seeds = r.seeds;
+    c.q[s].n_seeds = (long long)r.n_seeds;
+    c.q[s].cap_log2 = (uint32_t)r.cap_log2;
+    c.q[s].stride = (uint32_t)p->fam->stride((int)s);
+  }
+  c.ctrl = p->ctrl;
+  c.blk = p->blk;
+  c.trace = p->trace;
+  c.trace_cap = (p->desc.flags & VP_FLAG_TRACE) ? (unsigned long long)p->desc.trace_capacity : 0ull;
+  c.flags = ((p->desc.flags & VP_FLAG_TRACE) ? FLAG_TRACE : 0u) | ((p->desc.flags & VP_FLAG_QUEUE_DEPTH) ? FLAG_DEPTH : 0u) |
+            ((p->desc.flags & VP_FLAG_TIMERS) ? FLAG_TIMERS : 0u);
+  c.n_stages = (int)p->st.size();
+  c.host_arrive = p->d_arrive;
+  c.epoch = p->epoch;
+  return c;
+}
+
+// Per-block SM resources of a kernel (register allocation per warp in units of 256,
+// static + dynamic + 1 KB reserved shared memory).
+struct KRes {
+  int regs, smem, threads;
+};
+KRes kernel_res(vp_pipeline_s* p, int lo, int hi, bool rtc) {
+  KRes r{0, 0, kThreads};
+  cudaFuncAttributes at;
+  if (cudaFuncGetAttributes(&at, p->fam->kernel(lo, hi, rtc)) != cudaSuccess) return KRes{1 << 30, 1 << 30, kThreads};
+  int per_warp = ((at.numRegs * 32 + 255) / 256) * 256;
+  r.regs = per_warp * (kThreads / 32);
+  r.smem = (int)(at.sharedSizeBytes + p->fam->smem(lo, hi, rtc)) + 1024;
+  return r;
+}
+bool fits_sm(vp_pipeline_s* p, const KRes* res, const int* q, int n) {
+  cudaDeviceProp prop;
+  cudaGetDeviceProperties(&prop, p->device);
+  long long regs = 0, smem = 0, thr = 0, blocks = 0;
+  for (int i = 0; i < n; ++i) {
+    regs += (long long)q[i] * res[i].regs;
+    smem += (long long)q[i] * res[i].smem;
+    thr += (long long)q[i] * res[i].threads;
+    blocks += q[i];
+  }
+  return regs <= prop.regsPerMultiprocessor && smem <= (long long)prop.sharedMemPerMultiprocessor &&
+         thr <= prop.maxThreadsPerMultiProcessor && blocks <= prop.maxBlocksPerMultiProcessor;
+}
+// Block quotas for the single-stage kernels of a fine group [lo,hi] sharing each SM:
+// requested quotas are checked for co-residency; missing ones are filled greedily
+// (one block each, then round-robin while the SM still fits them all).
+vp_status fine_quotas(vp_pipeline_s* p, int lo, int hi, const int* req, int* q) {
+  const int n = hi - lo + 1;
+  KRes res[kMaxStages];
+  int qq[kMaxStages];
+  bool fixed[kMaxStages];
+  for (int i = 0; i < n; ++i) {
+    res[i] = kernel_res(p, lo + i, lo + i, false);
+    fixed[i] = req && req[lo + i] > 0;
+    qq[i] = fixed[i] ? req[lo + i] : 1;
+  }
+  if (!fits_sm(p, res, qq, n))
+    return fail(p, VP_ERR_INVALID, "fine group [%d,%d]: block quotas do not fit one SM (registers/smem/threads)", lo, hi);
+  for (bool grew = true; grew;) {
+    grew = false;
+    for (int i = 0; i < n; ++i) {
+      if (fixed[i]) continue;
+      qq[i]++;
+      if (fits_sm(p, res, qq, n)) grew = true;
+      else qq[i]--;
+    }
+  }
+  for (int i = 0; i < n; ++i) q[lo + i] = qq[i];
+  return VP_OK;
+}
+
+vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int batch, Plan& out) {
+  const int S = (int)p->st.size();
+  const int N = p->num_sms;
+  Plan pl;
+  pl.model = model;
+  for (int s = 0; s < S; ++s) {
+    int bs = p->fam->default_batch(s);
+    if (b && b->batch[s] > 0) bs = b->batch[s];
+    if (batch > 0) bs = batch;
+    if (bs > p->fam->max_batch(s)) bs = p->fam->max_batch(s);
+    if (bs < 1) return fail(p, VP_ERR_INVALID, "batch for stage %d must be >= 1", s);
+    pl.batch[s] = bs;
+  }
+  auto add_kernel = [&](int lo, int hi, bool rtc, int quota, const uint32_t* mask, bool coop) -> vp_status {
+    int occ = occupancy(p, lo, hi, rtc);
+    if (occ <= 0) return fail(p, VP_ERR_UNSUPPORTED, "kernel [%d,%d]%s cannot be resident (occupancy 0)", lo, hi, rtc ? " RTC" : "");
+    if (quota > occ) return fail(p, VP_ERR_INVALID, "infeasible block quota %d > %d resident blocks/SM for stages [%d,%d]", quota, occ, lo, hi);
+    KernelPlan k;
+    k.lo = lo;
+    k.hi = hi;
+    k.rtc = rtc;
+    k.quota = quota;
+    memcpy(k.mask, mask, sizeof(k.mask));
+    k.coop = coop;
+    int per = quota > 0 ? quota : occ;
+    k.grid = coop ? per * N : occ * N;  // filling-retreating: enough blocks to fill every SM (L27)
+    k.kslot = (int)pl.kernels.size();
+    if (k.kslot >= kMaxKernels) return fail(p, VP_ERR_INVALID, "too many kernels");
+    pl.kernels.push_back(k);
+    return VP_OK;
+  };
+  uint32_t all[kMaskWords];
+  mask_all(all, N);
+  vp_status rc = VP_OK;
+  switch (model) {
+    case VP_RTC:
+      if (!p->fam->rtc_legal(0, S - 1))
+        return fail(p, VP_ERR_UNSUPPORTED, "RTC needs a linear pipeline without recursion, loops or global sync (L11)");
+      pl.wave_rtc = true;
+      break;
+    case VP_KBK:
+      for (int s = 0; s < S; ++s) pl.kbk_stages.push_back(s);
+      break;
+    case VP_MEGAKERNEL: {
+      int q = (b && b->blocks_per_sm[0] > 0) ? b->blocks_per_sm[0] : 0;
+      rc = add_kernel(0, S - 1, false, q, all, true);
+      break;
+    }
+    case VP_COARSE: {
+      // each stage its own persistent kernel on exclusive SMs (Fig. 4, L21)
+      for (int s = 0; s < S && rc == VP_OK; ++s) {
+        uint32_t m[kMaskWords];
+        if (b) memcpy(m, b->group_sm_mask[s], sizeof(m));
+        else mask_range(m, s * N / S, (s + 1) * N / S);
+        int q = (b && b->blocks_per_sm[s] > 0) ? b->blocks_per_sm[s] : 0;
+        rc = add_kernel(s, s, false, q, m, false);
+      }
+      break;
+    }
+    case VP_FINE: {
+      // each stage its own persistent kernel; SMs shared, blocks per (stage, SM) capped (Fig. 5)
+      int q[kMaxStages];
+      rc = fine_quotas(p, 0, S - 1, b ? b->blocks_per_sm : nullptr, q);
+      uint32_t m[kMaskWords];
+      if (b && b->num_groups == 1) memcpy(m, b->group_sm_mask[0], sizeof(m));
+      else memcpy(m, all, sizeof(m));
+      for (int s = 0; s < S && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], m, false);
+      break;
+    }
+    case VP_HYBRID: {
+      if (!b) return fail(p, VP_ERR_INVALID, "VP_HYBRID needs a vp_sm_binding");
+      int G = b->num_groups;
+      if (G < 1 || G > S) return fail(p, VP_ERR_INVALID, "num_groups must be in [1, %d]", S);
+      int lo[kMaxStages], hi[kMaxStages];
+      for (int g = 0; g < G; ++g) lo[g] = S, hi[g] = -1;
+      for (int s = 0; s < S; ++s) {
+        int g = b->group_of_stage[s];
+        if (g < 0 || g >= G) return fail(p, VP_ERR_INVALID, "group_of_stage[%d] out of range", s);
+        if (s > 0 && g != b->group_of_stage[s - 1] && g != b->group_of_stage[s - 1] + 1)
+          return fail(p, VP_ERR_INVALID, "groups must be contiguous stage ranges in order (L45)");
+        if (s == 0 && g != 0) return fail(p, VP_ERR_INVALID, "stage 0 must be in group 0");
+        lo[g] = std::min(lo[g], s);
+        hi[g] = std::max(hi[g], s);
+      }
+      uint32_t used[kMaskWords] = {};
+      for (int g = 0; g < G && rc == VP_OK; ++g) {
+        if (hi[g] < 0) return fail(p, VP_ERR_INVALID, "group %d is empty", g);
+        int gm = b->group_model[g];
+        const uint32_t* m = b->group_sm_mask[g];
+        {
+          // KBK groups reserve their SMs too: wave kernels need resources the persistent
+          // groups do not hold (otherwise the host-launched waves could never start)
+          if (mask_count(m, N) == 0) return fail(p, VP_ERR_INVALID, "group %d has no SM in its mask", g);
+          for (int w = 0; w < kMaskWords; ++w) {
+            if (used[w] & m[w]) return fail(p, VP_ERR_INVALID, "SM masks of groups overlap (coarse pipelining between groups, L27)");
+            used[w] |= m[w];
+          }
+        }
+        if (gm == VP_GROUP_RTC) {
+          if (!p->fam->rtc_legal(lo[g], hi[g]))
+            return fail(p, VP_ERR_UNSUPPORTED, "RTC group [%d,%d] has recursion, a loop or a latch", lo[g], hi[g]);
+          rc = add_kernel(lo[g], hi[g], true, b->blocks_per_sm[lo[g]], m, false);
+        } else if (gm == VP_GROUP_MEGA) {
+          rc = add_kernel(lo[g], hi[g], false, b->blocks_per_sm[lo[g]], m, false);
+        } else if (gm == VP_GROUP_FINE) {
+          int q[kMaxStages];
+          rc = fine_quotas(p, lo[g], hi[g], b->blocks_per_sm, q);
+          for (int s = lo[g]; s <= hi[g] && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], m, false);
+        } else if (gm == VP_GROUP_KBK) {
+          for (int s = lo[g]; s <= hi[g]; ++s) pl.kbk_stages.push_back(s);
+        } else {
+          return fail(p, VP_ERR_INVALID, "unknown group model %d", gm);
+        }
+      }
+      break;
+    }
+    default:
+      return fail(p, VP_ERR_INVALID, "unknown model %d", model);
+  }
+  if (rc != VP_OK) return rc;
+  // every producer batch must fit twice into its target ring, or the ring cannot drain
+  for (int s = 0; s < S; ++s)
+    for (int t = 0; t < S; ++t) {
+      int f = p->fam->fanout(s, t);
+      if (f > 0 && 2ll * pl.batch[s] * f > (1ll << p->st[t].cap_log2))
+        return fail(p, VP_ERR_INVALID, "queue_capacity of stage %d (%lld) < 2 x batch(%d) x fanout(%d) of stage %d", t,
+                    1ll << p->st[t].cap_log2, pl.batch[s], f, s);
+    }
+  pl.cfg.model = model;
+  pl.cfg.has_binding = b ? 1 : 0;
+  if (b) pl.cfg.binding = *b;
+  pl.cfg.batch = batch;
+  out = pl;
+  return VP_OK;
+}
+
+// ------------------------------------------------------------------ running
+vp_status launch_wave(vp_pipeline_s* p, const Common& c, int lo, int hi, bool rtc, int stage, long long n,
+                      cudaStream_t st, int kslot) {
+  GroupArgs g;
+  memset(&g, 0, sizeof(g));
+  g.mode = MODE_WAVE;
+  g.wave_stage = stage;
+  g.wave_n = n;
+  g.kslot = kslot;
+  for (int s = 0; s < kMaxStages; ++s) g.batch[s] = p->plan.batch[s] ? p->plan.batch[s] : 1;
+  long long grid = (n + g.batch[stage] - 1) / g.batch[stage];
+  if (grid > 0x7fffffff) grid = 0x7fffffff;
+  occupancy(p, lo, hi, rtc);  // sets the smem attribute once
+  CUDA_TRY(p, p->fam->launch(lo, hi, rtc, c, g, p->params.data(), (int)grid, false, st));
+  return VP_OK;
+}
+
+struct Avail {
+  long long ring[kMaxStages];
+  long long seeds_left[kMaxStages];
+  long long pending;
+  unsigned long long abort;
+};
+
+vp_status read_avail(vp_pipeline_s* p, cudaStream_t st, Avail& a) {
+  // the counters live on separate 128-B lines: copy the first kMaxStages*4 + 2 lines
+  size_t bytes = offsetof(Ctrl, deadline);
+  CUDA_TRY(p, cudaMemcpyAsync(p->h_ctrl, p->ctrl, bytes, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(p, cudaStreamSynchronize(st));
+  for (size_t s = 0; s < p->st.size(); ++s) {
+    a.ring[s] = (long long)p->h_ctrl->count[s].v;
+    long long sh = (long long)p->h_ctrl->seed_head[s].v;
+    long long left = (long long)p->st[s].n_seeds - sh;
+    a.seeds_left[s] = left > 0 ? left : 0;
+  }
+  a.pending = (long long)p->h_ctrl->pending.v;
+  a.abort = p->h_ctrl->abort.v;
+  return VP_OK;
+}
+
+vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uint64_t* launches) {
+  // KBK (Fig. 3b): "The pipeline logic control is implemented on the CPU side" — read the
+  // queue counts back, launch one kernel for one stage over the items present, repeat.
+  // Stage choice: most downstream non-empty stage first (bounds live items, like the
+  // task scheduler's priority).  A wave is capped so its output fits the target rings.
+  const std::vector<int>& ks = p->plan.kbk_stages;
+  const int S = (int)p->st.size();
+  auto wave_cap = [&](int s) -> long long {
+    long long cap = 1ll << 40;
+    for (int t = 0; t < S; ++t) {
+      int f = p->fam->fanout(s, t);
+      if (f > 0) cap = std::min(cap, (long long)(1ll << p->st[t].cap_log2) / (2 * f));
+    }
+    return std::max(1ll, cap);
+  };
+  for (;;) {
+    Avail a;
+    vp_status rc = read_avail(p, st, a);
+    if (rc != VP_OK) return rc;
+    if (a.abort) return VP_OK;
+    if (a.pending <= 0) return VP_OK;
+    bool launched = false;
+    if (p->plan.wave_rtc) {
+      for (int s = 0; s < S && !launched; ++s) {
+        long long n = a.ring[s] + a.seeds_left[s];
+        if (n > 0) {
+          n = std::min(n, wave_cap(s));
+          rc = launch_wave(p, c, 0, S - 1, true, s, n, st, 0);
+          if (rc != VP_OK) return rc;
+          launched = true;
+        }
+      }
+    } else {
+      for (int i = (int)ks.size() - 1; i >= 0 && !launched; --i) {
+        int s = ks[i];
+        long long n = a.ring[s] + a.seeds_left[s];
+        if (n > 0) {
+          n = std::min(n, wave_cap(s));
+          rc = launch_wave(p, c, s, s, false, s, n, st, 0);
+          if (rc != VP_OK) return rc;
+          launched = true;
+        }
+      }
+    }
+    if (launched) {
+      (*launches)++;
+    } else {
+      // hybrid: the work is in persistent groups right now; poll again shortly
+      std::this_thread::sleep_for(std::chrono::microseconds(5));
+    }
+  }
+}
+
+}  // namespace
+
+// ====================================================================== C ABI
+extern "C" {
+
+const char* vp_status_string(vp_status s) {
+  switch (s) {
+    case VP_OK: return "VP_OK";
+    case VP_ERR_INVALID: return "VP_ERR_INVALID";
+    case VP_ERR_UNSUPPORTED: return "VP_ERR_UNSUPPORTED";
+    case VP_ERR_CUDA: return "VP_ERR_CUDA";
+    case VP_ERR_OOM: return "VP_ERR_OOM";
+    case VP_ERR_QUEUE_OVERFLOW: return "VP_ERR_QUEUE_OVERFLOW";
+    case VP_ERR_TIMEOUT: return "VP_ERR_TIMEOUT";
+    case VP_ERR_BINDING: return "VP_ERR_BINDING";
+    case VP_ERR_FANOUT: return "VP_ERR_FANOUT";
+  }
+  return "VP_ERR_UNKNOWN";
+}
+
+const char* vp_last_error(void* h) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  return p ? p->err.c_str() : "";
+}
+
+vp_status vp_device_info(int device, int* num_sms, int* cc_major, int* cc_minor) {
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return VP_ERR_CUDA;
+  if (num_sms) *num_sms = prop.multiProcessorCount;
+  if (cc_major) *cc_major = prop.major;
+  if (cc_minor) *cc_minor = prop.minor;
+  return VP_OK;
+}
+
+vp_status vp_memcpy(void* dst, const void* src, size_t bytes, int kind, void* stream) {
+  cudaMemcpyKind k = kind == 0 ? cudaMemcpyHostToDevice : kind == 1 ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  cudaStream_t st = (cudaStream_t)stream;
+  if (cudaMemcpyAsync(dst, src, bytes, k, st) != cudaSuccess) return VP_ERR_CUDA;
+  if (cudaStreamSynchronize(st) != cudaSuccess) return VP_ERR_CUDA;
+  return VP_OK;
+}
+
+vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) {
+  if (!out) return VP_ERR_INVALID;
+  *out = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) return VP_ERR_CUDA;
+  DeviceGuard dg(device);
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, device) != cudaSuccess) return VP_ERR_CUDA;
+  if (prop.major < 10) return VP_ERR_UNSUPPORTED;  // sm_100a build only
+  vp_pipeline_s* p = new vp_pipeline_s();
+  p->device = device;
+  p->num_sms = std::min(prop.multiProcessorCount, kMaxSM);
+  if (d) p->desc = *d;
+  if (p->desc.max_stages <= 0 || p->desc.max_stages > VP_MAX_STAGES) p->desc.max_stages = VP_MAX_STAGES;
+  if (p->desc.watchdog_ms <= 0) p->desc.watchdog_ms = 30000;
+  p->timeout_ms = p->desc.watchdog_ms;
+  if ((p->desc.flags & VP_FLAG_TRACE) && p->desc.trace_capacity <= 0) p->desc.trace_capacity = 1 << 20;
+  auto bad = [&](cudaError_t e) {
+    if (e == cudaSuccess) return false;
+    delete p;
+    return true;
+  };
+  if (bad(cudaMalloc(&p->ctrl, sizeof(Ctrl)))) return VP_ERR_OOM;
+  if (bad(cudaMemset(p->ctrl, 0, sizeof(Ctrl)))) return VP_ERR_CUDA;
+  if (bad(cudaMalloc(&p->blk, sizeof(uint32_t) * kMaxKernels * kMaxSM))) return VP_ERR_OOM;
+  if (bad(cudaMallocHost(&p->h_ctrl, sizeof(Ctrl)))) return VP_ERR_OOM;
+  if (bad(cudaMallocHost(&p->h_blk, sizeof(uint32_t) * kMaxKernels * kMaxSM))) return VP_ERR_OOM;
+  {
+    void* ha = nullptr;
+    if (bad(cudaHostAlloc(&ha, sizeof(uint32_t) * kMaxKernels, cudaHostAllocMapped))) return VP_ERR_OOM;
+    memset(ha, 0, sizeof(uint32_t) * kMaxKernels);
+    p->h_arrive = (volatile uint32_t*)ha;
+    if (bad(cudaHostGetDevicePointer((void**)&p->d_arrive, ha, 0))) return VP_ERR_CUDA;
+  }
+  if (p->desc.flags & VP_FLAG_TRACE)
+    if (bad(cudaMalloc(&p->trace, sizeof(TraceRec) * (size_t)p->desc.trace_capacity))) return VP_ERR_OOM;
+  for (int i = 0; i < kMaxKernels; ++i) {
+    if (bad(cudaStreamCreateWithFlags(&p->streams[i], cudaStreamNonBlocking))) return VP_ERR_CUDA;
+    if (bad(cudaEventCreate(&p->ev_join[i]))) return VP_ERR_CUDA;
+    if (bad(cudaEventCreate(&p->ev_kbeg[i]))) return VP_ERR_CUDA;
+  }
+  if (bad(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming))) return VP_ERR_CUDA;
+  if (bad(cudaEventCreate(&p->ev_start)) || bad(cudaEventCreate(&p->ev_end))) return VP_ERR_CUDA;
+  *out = p;
+  return VP_OK;
+}
+
+vp_status vp_pipeline_destroy(void* h) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  DeviceGuard dg(p->device);
+  cudaDeviceSynchronize();
+  for (StageRec& r : p->st) {
+    cudaFree(r.slots);
+    cudaFree(r.seq);
+    cudaFree(r.seeds);
+  }
+  cudaFree(p->ctrl);
+  cudaFree(p->blk);
+  cudaFree(p->trace);
+  cudaFreeHost(p->h_ctrl);
+  cudaFreeHost(p->h_blk);
+  cudaFreeHost((void*)p->h_arrive);
+  for (int i = 0; i < kMaxKernels; ++i) {
+    cudaStreamDestroy(p->streams[i]);
+    cudaEventDestroy(p->ev_join[i]);
+    cudaEventDestroy(p->ev_kbeg[i]);
+  }
+  cudaEventDestroy(p->ev_fork);
+  cudaEventDestroy(p->ev_start);
+  cudaEventDestroy(p->ev_end);
+  delete p;
+  return VP_OK;
+}
+
+vp_status vp_stage_register(void* h, const vp_stage_desc* s, int* stage_id) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !s) return VP_ERR_INVALID;
+  if (p->queues_ready) return fail(p, VP_ERR_INVALID, "stages must be registered before vp_insert/vp_configure");
+  int pos = -1;
+  const FamilyOps* f = family_of_kind(s->kind, &pos);
+  if (!f) return fail(p, VP_ERR_INVALID, "unknown stage kind %d", s->kind);
+  if (p->fam && p->fam != f) return fail(p, VP_ERR_INVALID, "stage kind %d belongs to family '%s', pipeline is '%s'", s->kind, f->name, p->fam->name);
+  if (pos != (int)p->st.size())
+    return fail(p, VP_ERR_INVALID, "family '%s' stages must be registered in order: expected stage %zu, got %d", f->name, p->st.size(), pos);
+  if ((int)p->st.size() >= p->desc.max_stages) return fail(p, VP_ERR_INVALID, "max_stages exceeded");
+  if (s->item_bytes != f->stride(pos))
+    return fail(p, VP_ERR_INVALID, "item_bytes %d != %d for stage kind %d", s->item_bytes, f->stride(pos), s->kind);
+  if (s->threads_per_item != 0 && s->threads_per_item != f->threads_per_item(pos))
+    return fail(p, VP_ERR_INVALID, "threads_per_item %d unsupported for kind %d (built-in uses %d)", s->threads_per_item, s->kind, f->threads_per_item(pos));
+  if (s->params) {
+    if (s->params_bytes != f->params_bytes()) return fail(p, VP_ERR_INVALID, "params_bytes %zu != %zu", s->params_bytes, f->params_bytes());
+    std::vector<uint8_t> pr((const uint8_t*)s->params, (const uint8_t*)s->params + s->params_bytes);
+    if (!p->params.empty() && p->params != pr) return fail(p, VP_ERR_INVALID, "stages of one family must share one params struct");
+    p->params = pr;
+  }
+  p->fam = f;
+  StageRec r;
+  r.d = *s;
+  r.name = s->name ? s->name : "";
+  r.d.name = nullptr;
+  int64_t cap = s->queue_capacity > 0 ? s->queue_capacity : (p->desc.default_queue_capacity > 0 ? p->desc.default_queue_capacity : (1ll << f->default_cap_log2(pos)));
+  int lg = 0;
+  while ((1ll << lg) < cap) ++lg;
+  if (lg < 5) lg = 5;
+  r.cap_log2 = lg;
+  p->st.push_back(r);
+  if (stage_id) *stage_id = pos;
+  p->configured = false;
+  return VP_OK;
+}
+
+static vp_status finish_registration(vp_pipeline_s* p) {
+  if (!p->fam) return fail(p, VP_ERR_INVALID, "no stages registered");
+  if ((int)p->st.size() != p->fam->S) return fail(p, VP_ERR_INVALID, "family '%s' needs all %d stages registered (%zu given)", p->fam->name, p->fam->S, p->st.size());
+  if (p->params.empty()) return fail(p, VP_ERR_INVALID, "no params struct given for family '%s'", p->fam->name);
+  const char* v = p->fam->validate(p->params.data());
+  if (v) return fail(p, VP_ERR_INVALID, "%s", v);
+  return ensure_queues(p);
+}
+
+vp_status vp_insert_async(void* h, int stage_id, const void* items, size_t n, int flags, void* stream) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  DeviceGuard dg(p->device);
+  vp_status rc = finish_registration(p);
+  if (rc != VP_OK) return rc;
+  if (stage_id < 0 || stage_id >= (int)p->st.size()) return fail(p, VP_ERR_INVALID, "bad stage id %d", stage_id);
+  if (n > 0 && !items) return fail(p, VP_ERR_INVALID, "items is NULL");
+  StageRec& r = p->st[stage_id];
+  if (flags & VP_INSERT_REPLACE) r.n_seeds = 0;
+  size_t stride = (size_t)p->fam->stride(stage_id);
+  cudaStream_t st = (cudaStream_t)stream;
+  if (r.n_seeds + n > r.seed_cap) {
+    size_t ncap = std::max(r.n_seeds + n, r.seed_cap * 2);
+    uint8_t* nb = nullptr;
+    CUDA_TRY(p, cudaMalloc(&nb, ncap * stride));
+    if (r.n_seeds) CUDA_TRY(p, cudaMemcpyAsync(nb, r.seeds, r.n_seeds * stride, cudaMemcpyDeviceToDevice, st));
+    CUDA_TRY(p, cudaStreamSynchronize(st));
+    cudaFree(r.seeds);
+    r.seeds = nb;
+    r.seed_cap = ncap;
+  }
+  if (n) {
+    CUDA_TRY(p, cudaMemcpyAsync(r.seeds + r.n_seeds * stride, items, n * stride,
+                                (flags & VP_INSERT_DEVICE) ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
+  }
+  r.n_seeds += n;
+  return VP_OK;
+}
+
+vp_status vp_insert(void* h, int stage_id, const void* items, size_t n, int flags) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  vp_status rc = vp_insert_async(h, stage_id, items, n, flags, nullptr);
+  if (rc != VP_OK) return rc;
+  DeviceGuard dg(p->device);
+  CUDA_TRY(p, cudaStreamSynchronize(nullptr));
+  return VP_OK;
+}
+
+vp_status vp_configure(void* h, int model, const vp_sm_binding* b, int batch) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  DeviceGuard dg(p->device);
+  vp_status rc = finish_registration(p);
+  if (rc != VP_OK) return rc;
+  if (batch < 0) return fail(p, VP_ERR_INVALID, "batch must be >= 0");
+  Plan pl;
+  rc = build_plan(p, model, b, batch, pl);
+  if (rc != VP_OK) return rc;
+  p->plan = pl;
+  p->configured = true;
+  return VP_OK;
+}
+
+vp_status vp_configure_config(void* h, const vp_config* c) {
+  if (!c) return VP_ERR_INVALID;
+  return vp_configure(h, c->model, c->has_binding ? &c->binding : nullptr, c->batch);
+}
+
+vp_status vp_get_config(void* h, vp_config* out) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !out) return VP_ERR_INVALID;
+  if (!p->configured) return fail(p, VP_ERR_INVALID, "not configured");
+  *out = p->plan.cfg;
+  return VP_OK;
+}
+
+vp_status vp_get_output(void* h, int index, void** dev_ptr, size_t* bytes) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !dev_ptr || !bytes) return VP_ERR_INVALID;
+  if (!p->fam || p->params.empty()) return fail(p, VP_ERR_INVALID, "no family params");
+  if (!p->fam->output(p->params.data(), index, dev_ptr, bytes)) return fail(p, VP_ERR_INVALID, "no output %d", index);
+  return VP_OK;
+}
+
+vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  if (!p->configured) return fail(p, VP_ERR_INVALID, "vp_run before vp_configure/vp_autotune");
+  DeviceGuard dg(p->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const int S = (int)p->st.size();
+  if (p->dirty_queues) {
+    vp_status rc = reset_queues(p, st);
+    if (rc != VP_OK) return rc;
+  }
+  RunInit ri;
+  memset(&ri, 0, sizeof(ri));
+  for (int s = 0; s < S; ++s) {
+    ri.seeds[s] = p->st[s].n_seeds;
+    ri.pending += (long long)p->st[s].n_seeds;
+  }
+  ri.watchdog_ns = (unsigned long long)(p->timeout_ms * 1e6);
+  p->epoch++;
+  if (p->epoch == 0) p->epoch = 1;
+  Common c = make_common(p);
+  CUDA_TRY(p, cudaEventRecord(p->ev_start, st));
+  k_run_init<<<1, 256, 0, st>>>(p->ctrl, p->blk, ri);
+  CUDA_TRY(p, cudaGetLastError());
+  CUDA_TRY(p, p->fam->init_run(p->params.data(), st));
+  const Plan& pl = p->plan;
+  int nk = (int)pl.kernels.size();
+  if (nk > 0) {
+    CUDA_TRY(p, cudaEventRecord(p->ev_fork, st));
+    for (int i = 0; i < nk; ++i) {
+      const KernelPlan& k = pl.kernels[i];
+      cudaStream_t ks = p->streams[i];
+      CUDA_TRY(p, cudaStreamWaitEvent(ks, p->ev_fork, 0));
+      GroupArgs g;
+      memset(&g, 0, sizeof(g));
+      memcpy(g.sm_mask, k.mask, sizeof(g.sm_mask));
+      g.quota = k.quota;
+      g.kslot = k.kslot;
+      g.mode = MODE_PERSISTENT;
+      for (int s = 0; s < kMaxStages; ++s) g.batch[s] = pl.batch[s] ? pl.batch[s] : 1;
+      occupancy(p, k.lo, k.hi, k.rtc);
+      CUDA_TRY(p, cudaEventRecord(p->ev_kbeg[i], ks));
+      CUDA_TRY(p, p->fam->launch(k.lo, k.hi, k.rtc, c, g, p->params.data(), k.grid, k.coop, ks));
+      CUDA_TRY(p, cudaEventRecord(p->ev_join[i], ks));
+      if (i + 1 < nk) {
+        // High-level control: launch the next group's kernel only after this grid is
+        // fully dispatched, so its admitted blocks hold their SMs before the next
+        // kernel's blocks arrive (deterministic filling-retreating, L27 §5).
+        auto t0 = std::chrono::steady_clock::now();
+        while (p->h_arrive[i] != p->epoch) {
+          if (std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(2000)) break;
+        }
+      }
+    }
+  }
+  uint64_t launches = 0;
+  if (!pl.kbk_stages.empty() || pl.wave_rtc) {
+    vp_status rc = host_wave_loop(p, c, st, &launches);
+    if (rc != VP_OK) return rc;
+  }
+  for (int i = 0; i < nk; ++i) CUDA_TRY(p, cudaStreamWaitEvent(st, p->ev_join[i], 0));
+  CUDA_TRY(p, p->fam->finalize(p->params.data(), st));
+  CUDA_TRY(p, cudaEventRecord(p->ev_end, st));
+  CUDA_TRY(p, cudaMemcpyAsync(p->h_ctrl, p->ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(p, cudaMemcpyAsync(p->h_blk, p->blk, sizeof(uint32_t) * kMaxKernels * kMaxSM, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(p, cudaStreamSynchronize(st));
+  float ms = 0;
+  cudaEventElapsedTime(&ms, p->ev_start, p->ev_end);
+  const Ctrl& hc = *p->h_ctrl;
+  if (stats) {
+    memset(stats, 0, sizeof(*stats));
+    stats->device_ms = ms;
+    for (int s = 0; s < S; ++s) {
+      stats->dequeued[s] = hc.deq[s];
+      stats->enqueued[s] = hc.enq[s];
+      stats->max_depth[s] = hc.max_depth[s];
+    }
+    stats->num_kernels = nk;
+    for (int i = 0; i < nk && i < 16; ++i) {
+      stats->kernel_lo[i] = pl.kernels[i].lo;
+      stats->kernel_hi[i] = pl.kernels[i].hi;
+      stats->kernel_quota[i] = pl.kernels[i].quota;
+      float kms = 0;
+      cudaEventElapsedTime(&kms, p->ev_kbeg[i], p->ev_join[i]);
+      stats->kernel_ms[i] = kms;
+      stats->admitted[i] = hc.admitted[i].v;
+      for (int sm = 0; sm < VP_MAX_SM; ++sm) stats->blocks_on_sm[i][sm] = p->h_blk[i * kMaxSM + sm];
+    }
+    if (nk == 0) {
+      for (int sm = 0; sm < VP_MAX_SM; ++sm) stats->blocks_on_sm[0][sm] = p->h_blk[sm];
+    }
+    stats->fallback_admits = hc.fallback_admits;
+    stats->kbk_launches = launches;
+    stats->trace_records = hc.trace_n.v;
+    stats->abort_reason = (int)hc.abort.v;
+    stats->num_sms = p->num_sms;
+    for (int s = 0; s < S; ++s) {
+      stats->stage_exec_ns[s] = hc.exec_ns[s];
+      stats->stage_flush_ns[s] = hc.flush_ns[s];
+    }
+    for (int i = 0; i < kMaxKernels; ++i) stats->kernel_idle_ns[i] = hc.idle_ns[i];
+  }
+  if (hc.abort.v != ABORT_NONE) {
+    p->dirty_queues = true;
+    switch (hc.abort.v) {
+      case ABORT_TIMEOUT: return fail(p, VP_ERR_TIMEOUT, "device watchdog fired after %.3f ms", p->timeout_ms);
+      case ABORT_OVERFLOW: return fail(p, VP_ERR_QUEUE_OVERFLOW, "a ring stayed full for > 200 ms (raise queue_capacity)");
+      case ABORT_FANOUT: return fail(p, VP_ERR_FANOUT, "a stage exceeded its declared fan-out");
+      case ABORT_GUARD: return fail(p, VP_ERR_INVALID, "a stage's recursion guard fired (input outside the domain)");
+      default: return fail(p, VP_ERR_CUDA, "unknown abort reason %llu", (unsigned long long)hc.abort.v);
+    }
+  }
+  if ((long long)hc.pending.v != 0) {
+    p->dirty_queues = true;
+    return fail(p, VP_ERR_CUDA, "pipeline ended with pending = %lld", (long long)hc.pending.v);
+  }
+  if (p->desc.flags & VP_FLAG_STRICT_BINDING) {
+    for (int i = 0; i < nk; ++i) {
+      const KernelPlan& k = pl.kernels[i];
+      if (k.quota <= 0) continue;
+      for (int sm = 0; sm < p->num_sms; ++sm)
+        if ((k.mask[sm >> 5] >> (sm & 31)) & 1u)
+          if ((int)p->h_blk[i * kMaxSM + sm] < k.quota)
+            return fail(p, VP_ERR_BINDING, "kernel %d reached %u of %d blocks on SM %d", i, p->h_blk[i * kMaxSM + sm], k.quota, sm);
+    }
+  }
+  return VP_OK;
+}
+
+vp_status vp_get_trace(void* h, void** dev_ptr, size_t* n) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !dev_ptr || !n) return VP_ERR_INVALID;
+  if (!(p->desc.flags & VP_FLAG_TRACE)) return fail(p, VP_ERR_INVALID, "pipeline created without VP_FLAG_TRACE");
+  *dev_ptr = p->trace;
+  unsigned long long m = p->h_ctrl ? p->h_ctrl->trace_n.v : 0;
+  *n = (size_t)std::min<unsigned long long>(m, (unsigned long long)p->desc.trace_capacity);
+  return VP_OK;
+}
+
+vp_status vp_set_timeout(void* h, double ms) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !(ms > 0)) return VP_ERR_INVALID;
+  p->timeout_ms = ms;
+  return VP_OK;
+}
+
+vp_status vp_profile(void* h, int* max_blocks, int* regs, int* smem) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  DeviceGuard dg(p->device);
+  vp_status rc = finish_registration(p);
+  if (rc != VP_OK) return rc;
+  for (int s = 0; s < (int)p->st.size(); ++s) {
+    const void* fn = p->fam->kernel(s, s, false);
+    cudaFuncAttributes at;
+    CUDA_TRY(p, cudaFuncGetAttributes(&at, fn));
+    if (max_blocks) max_blocks[s] = occupancy(p, s, s, false);
+    if (regs) regs[s] = at.numRegs;
+    if (smem) smem[s] = (int)(at.sharedSizeBytes + p->fam->smem(s, s, false));
+  }
+  return VP_OK;
+}
+
+}  // extern "C"

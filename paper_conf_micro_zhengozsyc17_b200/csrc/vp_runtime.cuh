@@ -1,0 +1,749 @@
+// vp_runtime.cuh — device side of the VersaPipe runtime for sm_100a.
+//
+// One template kernel realises every execution model of PAPER.md §4 (L11–L27):
+//   * persistent threads (L13, L17): blocks loop "fetch item batch -> execute -> push"
+//     until the pipeline drains (pending == 0);
+//   * Megakernel (L13 Fig. 3c): one kernel over all stages, blocks "query queues in turn
+//     of priority" (Fig. 8a, L31/L37);
+//   * coarse / fine pipeline (L21 Figs. 4–5): one persistent kernel per stage, bound to
+//     SMs by check_sm() and to per-(stage,SM) block quotas by check_sm_blk();
+//   * RTC (L11): all stages of a linear group in one kernel, intermediate items passed
+//     block-locally in shared memory instead of through work queues;
+//   * KBK (L13 Fig. 3b): the same kernel in non-persistent "wave" mode, one launch per
+//     stage over the items present, driven by the host.
+//
+// B200-first mechanics: per-stage bounded MPMC rings with 64-bit
+// tickets and per-slot sequence words (Vyukov), block-aggregated claims and publishes
+// (2 L2 atomics per block batch per queue), one pending-counter atomic per batch,
+// 16-B (or 4/8-B for small items) coalesced payload movement through shared memory,
+// L1-bypassing (.cg) payload loads, release/acquire publication, %smid binding,
+// %globaltimer watchdog.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <type_traits>
+#include <utility>
+
+namespace vp {
+
+constexpr int kThreads = 256;       // the paper's block size for persistent models (L53)
+constexpr int kMaxStages = 8;
+constexpr int kMaxKernels = 16;     // kernel slots per run (binding counters)
+constexpr int kMaxSM = 256;         // table width; B200 has 148 SMs (queried at runtime)
+constexpr int kMaskWords = kMaxSM / 32;
+
+enum Abort : unsigned long long {
+  ABORT_NONE = 0,
+  ABORT_TIMEOUT = 1,   // watchdog deadline passed (VP_ERR_TIMEOUT)
+  ABORT_OVERFLOW = 2,  // a producer could not get a free ring slot (VP_ERR_QUEUE_OVERFLOW)
+  ABORT_FANOUT = 3,    // a stage emitted more items than its declared fan-out
+  ABORT_GUARD = 4,     // a stage's own recursion guard fired (invalid input)
+};
+
+// Each hot counter on its own 128-B line (no false sharing between L2 atomics).
+struct alignas(128) Line {
+  unsigned long long v;
+  unsigned long long pad[15];
+};
+
+struct Ctrl {
+  Line tail[kMaxStages];       // producer reservation ticket
+  Line head[kMaxStages];       // consumer claim ticket
+  Line count[kMaxStages];      // published-and-unclaimed items (signed)
+  Line seed_head[kMaxStages];  // claim index into the seed segment
+  Line pending;                // items alive: seeded + emitted - completed (signed)
+  Line abort;                  // Abort reason, first writer wins
+  Line deadline;               // %globaltimer deadline in ns
+  Line trace_n;
+  Line arrivals[kMaxKernels];  // blocks of each kernel that ran the binding prologue
+  Line admitted[kMaxKernels];  // blocks of each kernel that stayed
+  unsigned long long deq[kMaxStages];
+  unsigned long long enq[kMaxStages];      // includes seeds
+  unsigned long long max_depth[kMaxStages];
+  unsigned long long fallback_admits;
+  unsigned long long exec_ns[kMaxStages];   // FLAG_TIMERS: stage-in + execute per stage
+  unsigned long long flush_ns[kMaxStages];  // FLAG_TIMERS: publish (queue overhead) per stage
+  unsigned long long idle_ns[kMaxKernels];  // FLAG_TIMERS: blocks finding no work, per kernel
+};
+
+struct QueueDesc {
+  uint8_t* slots;            // [cap][stride]
+  unsigned long long* seq;   // [cap]
+  const uint8_t* seeds;      // [n_seeds][stride] (read-only during a run)
+  long long n_seeds;
+  uint32_t cap_log2;
+  uint32_t stride;
+};
+
+struct TraceRec {
+  unsigned long long id;
+  uint32_t stage, smid;
+};
+
+enum : uint32_t { FLAG_TRACE = 1u, FLAG_DEPTH = 2u, FLAG_TIMERS = 4u };
+
+struct Common {
+  QueueDesc q[kMaxStages];
+  Ctrl* ctrl;
+  uint32_t* blk;             // [kMaxKernels][kMaxSM] per-(kernel, SM) block counters (D4)
+  TraceRec* trace;
+  unsigned long long trace_cap;
+  uint32_t flags;
+  int n_stages;
+  volatile uint32_t* host_arrive;  // mapped pinned host words: grid of kernel k fully dispatched
+  uint32_t epoch;                  // run counter written into host_arrive
+};
+
+enum : int { MODE_PERSISTENT = 0, MODE_WAVE = 1 };
+
+struct GroupArgs {
+  uint32_t sm_mask[kMaskWords];  // s_flag(group, sm) (Fig. 5, L21)
+  int quota;                     // blocks per SM (check_sm_blk threshold), <= 0: no cap
+  int kslot;                     // kernel slot for the binding counters
+  int mode;                      // MODE_PERSISTENT or MODE_WAVE
+  int wave_stage;                // WAVE: the stage whose items this launch processes
+  long long wave_n;              // WAVE: number of items in this launch
+  int batch[kMaxStages];         // items per claim, per stage
+};
+
+template <class F>
+struct KArgs {
+  Common c;
+  GroupArgs g;
+  typename F::Params p;
+};
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ unsigned long long globaltimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ unsigned long long ld_acquire(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long atom_add(unsigned long long* p, long long d) {
+  return atomicAdd(p, (unsigned long long)d);
+}
+
+// Vector chunk used to move items of a given stride (16 B when possible).
+template <int STRIDE>
+struct Chunk {
+  static constexpr int bytes = (STRIDE % 16 == 0) ? 16 : (STRIDE % 8 == 0) ? 8 : 4;
+  using T = typename std::conditional<bytes == 16, uint4, typename std::conditional<bytes == 8, uint2, uint32_t>::type>::type;
+  static constexpr int per_item = STRIDE / bytes;
+};
+template <class T>
+__device__ __forceinline__ T ld_cg(const T* p) { return __ldcg(p); }
+template <class T>
+__device__ __forceinline__ void st_cg(T* p, T v) { __stcg(p, v); }
+
+// ------------------------------------------------------------------ constexpr graph helpers
+template <class F>
+struct Graph {
+  static constexpr int S = F::S;
+  static constexpr int fan(int s, int t) { return F::fanout(s, t); }
+  // true iff an edge s->t with LO <= t <= s <= HI exists (recursion / loop inside [LO,HI])
+  static constexpr bool has_back_edge(int lo, int hi) {
+    for (int s = lo; s <= hi; ++s)
+      for (int t = lo; t <= s; ++t)
+        if (fan(s, t) > 0) return true;
+    return false;
+  }
+  static constexpr bool rtc_legal(int lo, int hi) { return !has_back_edge(lo, hi) && !F::uses_latches(lo, hi); }
+  // items that can arrive block-locally at stage t of an RTC group [lo,hi]
+  static constexpr int rtc_in_cap(int lo, int t) {
+    if (t == lo) return F::max_batch(lo);
+    int n = F::max_batch(t);
+    int inc = 0;
+    for (int s = lo; s < t; ++s) inc += rtc_in_cap(lo, s) * fan(s, t);
+    return n > inc ? n : inc;
+  }
+  // out-buffer capacity (items) for target t in a kernel [lo,hi]
+  static constexpr int out_cap(int lo, int hi, bool rtc, int t) {
+    int c = 0;
+    for (int s = lo; s <= hi; ++s) {
+      if (fan(s, t) == 0) continue;
+      int n = rtc ? rtc_in_cap(lo, s) : F::max_batch(s);
+      int v = n * fan(s, t);
+      if (rtc) c += v;
+      else c = c > v ? c : v;
+    }
+    return c;
+  }
+  static constexpr int in_bytes(int lo, int hi) {
+    int b = 0;
+    for (int s = lo; s <= hi; ++s) {
+      int v = F::max_batch(s) * F::stride(s);
+      b = b > v ? b : v;
+    }
+    return b;
+  }
+  static constexpr int align128(int b) { return (b + 127) / 128 * 128; }
+  static constexpr int out_offset(int lo, int hi, bool rtc, int t) {
+    int off = align128(in_bytes(lo, hi));
+    for (int u = 0; u < t; ++u) off += align128(out_cap(lo, hi, rtc, u) * F::stride(u));
+    return off;
+  }
+  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return out_offset(lo, hi, rtc, S) + F::scratch_bytes(lo, hi); }
+  static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_offset(lo, hi, rtc, S); }
+};
+
+
+// ------------------------------------------------------------------ per-block context
+struct BlockShared {
+  int out_cnt[kMaxStages];
+  unsigned long long out_base[kMaxStages];
+  int cl_stage, cl_n, cl_seed, done, skip;
+  unsigned long long cl_base;
+  long long acc_neg;  // completions not yet subtracted from `pending` (deferred, <= 0)
+  unsigned long long deq[kMaxStages];
+  unsigned long long enq[kMaxStages];
+  unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle;
+};
+
+template <class F, int LO, int HI, bool RTC>
+struct Ctx {
+  using G = Graph<F>;
+  const KArgs<F>& a;
+  uint8_t* smem;
+  BlockShared& sh;
+  int tid;
+
+  __device__ Ctx(const KArgs<F>& a_, uint8_t* smem_, BlockShared& sh_) : a(a_), smem(smem_), sh(sh_), tid(threadIdx.x) {}
+
+  __device__ __forceinline__ const typename F::Params& params() const { return a.p; }
+  __device__ __forceinline__ uint8_t* scratch() { return smem + G::scratch_offset(LO, HI, RTC); }
+
+  template <int T>
+  __device__ __forceinline__ uint8_t* out_ptr(int slot) {
+    return smem + G::out_offset(LO, HI, RTC, T) + slot * F::stride(T);
+  }
+  template <int T>
+  static constexpr int cap() { return G::out_cap(LO, HI, RTC, T); }
+
+  // Reserve k consecutive out slots for target T (called by one thread).  The declared
+  // fan-out bounds guarantee capacity; exceeding it aborts the run (ABORT_FANOUT).
+  template <int T>
+  __device__ __forceinline__ int reserve(int k = 1) {
+    int slot = atomicAdd(&sh.out_cnt[T], k);
+    if (slot + k > cap<T>()) {
+      atomicCAS((unsigned long long*)&a.c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_FANOUT);
+      return -1;
+    }
+    return slot;
+  }
+  // Thread-level emit of a whole item (enqueue<Stage>(itemVal), Fig. 9 L37).
+  template <int T>
+  __device__ __forceinline__ void emit(const void* item) {
+    int slot = reserve<T>();
+    if (slot < 0) return;
+    constexpr int W = F::stride(T) / 4;
+    const uint32_t* src = (const uint32_t*)item;
+    uint32_t* dst = (uint32_t*)out_ptr<T>(slot);
+#pragma unroll
+    for (int i = 0; i < W; ++i) dst[i] = src[i];
+  }
+  __device__ __forceinline__ void abort(unsigned long long why) {
+    atomicCAS((unsigned long long*)&a.c.ctrl->abort.v, 0ull, why);
+  }
+};
+
+// ------------------------------------------------------------------ queue operations
+__device__ __forceinline__ bool aborted(const Ctrl* c) {
+  return *(volatile const unsigned long long*)&c->abort.v != 0ull;
+}
+
+// Thread 0: claim up to k items of stage s from its ring (published items only).
+// 2 L2 atomics per block batch: `count` (availability) then `head` (ticket range).
+__device__ __forceinline__ int claim_ring(Ctrl* c, int s, int k, unsigned long long& base) {
+  long long avail = (long long)ld_relaxed(&c->count[s].v);
+  if (avail <= 0) return 0;  // cheap L2 read first: idle blocks do not hammer atomics
+  int want = (int)(avail < k ? avail : k);
+  long long old = (long long)atom_add(&c->count[s].v, -want);
+  int got = old <= 0 ? 0 : (old < want ? (int)old : want);
+  if (got < want) atom_add(&c->count[s].v, want - got);
+  if (got == 0) return 0;
+  base = atom_add(&c->head[s].v, got);
+  return got;
+}
+// Thread 0: claim up to k seed items of stage s.
+__device__ __forceinline__ int claim_seed(Ctrl* c, const QueueDesc& q, int s, int k, unsigned long long& base) {
+  if (q.n_seeds == 0) return 0;
+  if ((long long)ld_relaxed(&c->seed_head[s].v) >= q.n_seeds) return 0;
+  long long old = (long long)atom_add(&c->seed_head[s].v, k);
+  if (old >= q.n_seeds) return 0;
+  long long got = q.n_seeds - old;
+  base = (unsigned long long)old;
+  return (int)(got < k ? got : k);
+}
+
+// Block-wide: wait until ring slots [base, base+n) hold the wanted sequence value.
+// mode 0: wait for publish (seq == t+1); mode 1: wait for free (seq == t).
+__device__ __forceinline__ void wait_slots(const Common& c, const QueueDesc& q, unsigned long long base, int n,
+                                           int mode) {
+  const unsigned long long mask = (1ull << q.cap_log2) - 1;
+  for (int k = threadIdx.x; k < n; k += blockDim.x) {
+    unsigned long long t = base + k;
+    unsigned long long want = t + (mode == 0 ? 1ull : 0ull);
+    const unsigned long long* p = q.seq + (t & mask);
+    if (ld_acquire(p) == want) continue;
+    unsigned long long t0 = globaltimer();
+    unsigned ns = 32;
+    while (ld_acquire(p) != want) {
+      __nanosleep(ns);
+      if (ns < 1024) ns <<= 1;
+      if (aborted(c.ctrl)) return;
+      unsigned long long now = globaltimer();
+      // a producer stuck > 200 ms on a full ring is a capacity failure, not progress
+      if (mode == 1 && now - t0 > 200000000ull) {
+        atomicCAS((unsigned long long*)&c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_OVERFLOW);
+        return;
+      }
+      if (now > c.ctrl->deadline.v) {
+        atomicCAS((unsigned long long*)&c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
+        return;
+      }
+    }
+  }
+}
+
+// Block-wide copies between the smem batch and a ring (wrap-aware) or the seed array,
+// in 16-B (or 8/4-B for small items) coalesced chunks; ring loads bypass L1 (.cg).
+template <int STRIDE>
+__device__ __forceinline__ void copy_in(uint8_t* dst, const uint8_t* ring, unsigned long long base, int n,
+                                        uint32_t cap_log2) {
+  using C = Chunk<STRIDE>;
+  using T = typename C::T;
+  const unsigned long long mask = (1ull << cap_log2) - 1;
+  const int total = n * C::per_item;
+  for (int i = threadIdx.x; i < total; i += blockDim.x) {
+    int k = i / C::per_item, w = i - k * C::per_item;
+    const T* src = (const T*)(ring + ((base + k) & mask) * STRIDE) + w;
+    ((T*)dst)[i] = ld_cg(src);
+  }
+}
+template <int STRIDE>
+__device__ __forceinline__ void copy_seed_in(uint8_t* dst, const uint8_t* seeds, unsigned long long base, int n) {
+  using C = Chunk<STRIDE>;
+  using T = typename C::T;
+  const T* src = (const T*)(seeds + base * STRIDE);
+  const int total = n * C::per_item;
+  for (int i = threadIdx.x; i < total; i += blockDim.x) ((T*)dst)[i] = __ldg(src + i);
+}
+template <int STRIDE>
+__device__ __forceinline__ void copy_out(uint8_t* ring, const uint8_t* src, unsigned long long base, int n,
+                                         uint32_t cap_log2) {
+  using C = Chunk<STRIDE>;
+  using T = typename C::T;
+  const unsigned long long mask = (1ull << cap_log2) - 1;
+  const int total = n * C::per_item;
+  for (int i = threadIdx.x; i < total; i += blockDim.x) {
+    int k = i / C::per_item, w = i - k * C::per_item;
+    T* d = (T*)(ring + ((base + k) & mask) * STRIDE) + w;
+    st_cg(d, ((const T*)src)[i]);
+  }
+}
+
+// ------------------------------------------------------------------ compile-time loops
+template <int I, int N, class Fn>
+__device__ __forceinline__ void static_for(Fn&& fn) {
+  if constexpr (I < N) {
+    fn(std::integral_constant<int, I>{});
+    static_for<I + 1, N>(fn);
+  }
+}
+
+// ------------------------------------------------------------------ the persistent kernel
+template <class F, int LO, int HI, bool RTC>
+struct Runner {
+  using G = Graph<F>;
+  using CtxT = Ctx<F, LO, HI, RTC>;
+  static constexpr int S = F::S;
+
+  static __device__ __forceinline__ bool is_local(int t, int local_from, int local_to) {
+    return t >= local_from && t <= local_to;
+  }
+
+  // Publish the block-staged outputs of every target outside the local chain to its
+  // ring: one `tail` atomic + one `count` atomic per (block batch, target), coalesced
+  // payload stores, per-slot release.  `completed` parents are retired here.
+  static __device__ void flush(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, int local_from, int local_to,
+                               long long completed) {
+    Ctrl* c = a.c.ctrl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      long long children = 0;
+      for (int t = 0; t < S; ++t) {
+        int n = sh.out_cnt[t];
+        if (n > G::out_cap(LO, HI, RTC, t)) n = G::out_cap(LO, HI, RTC, t);
+        sh.out_cnt[t] = n;
+        if (n == 0 || is_local(t, local_from, local_to)) continue;
+        children += n;
+      }
+      // Termination accounting: children must be counted before they become visible;
+      // completions may be deferred (pending only stays conservatively high).
+      if (children > 0) {
+        long long d = children - completed + sh.acc_neg;
+        if (d != 0) atom_add(&c->pending.v, d);
+        sh.acc_neg = 0;
+      } else {
+        sh.acc_neg -= completed;
+      }
+      for (int t = 0; t < S; ++t) {
+        int n = sh.out_cnt[t];
+        if (n == 0 || is_local(t, local_from, local_to)) continue;
+        sh.out_base[t] = atom_add(&c->tail[t].v, n);
+        sh.enq[t] += n;
+        if (a.c.flags & FLAG_DEPTH) {
+          unsigned long long h = ld_relaxed(&c->head[t].v);
+          unsigned long long d = sh.out_base[t] + n - h;
+          if (d > c->max_depth[t]) atomicMax(&c->max_depth[t], d);
+        }
+      }
+    }
+    __syncthreads();
+    bool any = false;
+    static_for<0, S>([&](auto T_) {
+      constexpr int T = decltype(T_)::value;
+      if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
+        int n = sh.out_cnt[T];
+        if (n > 0 && !is_local(T, local_from, local_to)) {
+          wait_slots(a.c, a.c.q[T], sh.out_base[T], n, 1);
+          any = true;
+        }
+      }
+    });
+    if (any) {
+      __syncthreads();
+      static_for<0, S>([&](auto T_) {
+        constexpr int T = decltype(T_)::value;
+        if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
+          int n = sh.out_cnt[T];
+          if (n > 0 && !is_local(T, local_from, local_to))
+            copy_out<F::stride(T)>(a.c.q[T].slots, ctx.template out_ptr<T>(0), sh.out_base[T], n, a.c.q[T].cap_log2);
+        }
+      });
+      __syncthreads();
+      // publish: seq = ticket + 1 (release; cumulative over the block's payload stores)
+      static_for<0, S>([&](auto T_) {
+        constexpr int T = decltype(T_)::value;
+        if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
+          int n = sh.out_cnt[T];
+          if (n > 0 && !is_local(T, local_from, local_to)) {
+            const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
+            for (int k = threadIdx.x; k < n; k += blockDim.x) {
+              unsigned long long t = sh.out_base[T] + k;
+              st_release(a.c.q[T].seq + (t & mask), t + 1);
+            }
+          }
+        }
+      });
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) {
+      for (int t = 0; t < S; ++t) {
+        if (is_local(t, local_from, local_to)) continue;
+        int n = sh.out_cnt[t];
+        if (n > 0) atom_add(&c->count[t].v, n);
+        sh.out_cnt[t] = 0;
+      }
+    }
+    __syncthreads();
+  }
+
+  static __device__ __forceinline__ void record_trace(const KArgs<F>& a, int s, const uint8_t* items, int n) {
+    if (!(a.c.flags & FLAG_TRACE)) return;
+    uint32_t sm = smid();
+    static_for<LO, HI + 1>([&](auto S_) {
+      constexpr int SS = decltype(S_)::value;
+      if (s == SS) {
+        for (int k = threadIdx.x; k < n; k += blockDim.x) {
+          unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
+          if (idx < a.c.trace_cap) {
+            a.c.trace[idx].id = F::template item_id<SS>(items + k * F::stride(SS));
+            a.c.trace[idx].stage = SS;
+            a.c.trace[idx].smid = sm;
+          }
+        }
+      }
+    });
+  }
+
+  // Execute stage s on n block-resident items, (RTC) forward block-locally through the
+  // rest of the linear group, then publish.
+  static __device__ void execute(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, int s, const uint8_t* items, int n,
+                                 unsigned long long t_start) {
+    const bool timers = a.c.flags & FLAG_TIMERS;
+    static_for<LO, HI + 1>([&](auto S_) {
+      constexpr int SS = decltype(S_)::value;
+      if (s == SS) {
+        record_trace(a, SS, items, n);
+        if (threadIdx.x == 0) sh.deq[SS] += n;
+        F::template exec<SS>(ctx, items, n);
+        int local_from = S, local_to = -1;
+        if constexpr (RTC && SS < HI) {
+          // RTC: run the remaining stages of the group on block-local items (L11 §4.1).
+          __syncthreads();
+          static_for<SS + 1, HI + 1>([&](auto T_) {
+            constexpr int TT = decltype(T_)::value;
+            int m = sh.out_cnt[TT];
+            if (m > G::out_cap(LO, HI, RTC, TT)) m = G::out_cap(LO, HI, RTC, TT);
+            if (m > 0) {
+              const uint8_t* loc = ctx.template out_ptr<TT>(0);
+              record_trace(a, TT, loc, m);
+              if (threadIdx.x == 0) sh.deq[TT] += m;
+              // block-local items were never counted in `pending` (the claimed parents
+              // keep it positive), so they are neither added nor subtracted
+              F::template exec<TT>(ctx, loc, m);
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) sh.out_cnt[TT] = 0;  // consumed locally
+            __syncthreads();
+          });
+          local_from = SS + 1;
+          local_to = HI;
+        }
+        unsigned long long t_mid = 0;
+        if (timers && threadIdx.x == 0) t_mid = globaltimer();
+        flush(a, ctx, sh, local_from, local_to, n);
+        if (timers && threadIdx.x == 0) {
+          unsigned long long t_end = globaltimer();
+          sh.t_exec[SS] += t_mid - t_start;
+          sh.t_flush[SS] += t_end - t_mid;
+        }
+      }
+    });
+  }
+
+  static __device__ bool admit(const KArgs<F>& a, BlockShared& sh) {
+    // check_sm() + check_sm_blk() (Fig. 5, L21; §5), increment-then-compare
+    // (Fig. 5's check-then-increment is racy).
+    __shared__ int ok;
+    if (threadIdx.x == 0) {
+      const GroupArgs& g = a.g;
+      Ctrl* c = a.c.ctrl;
+      int good = 1;
+      uint32_t sm = smid();
+      if (g.mode == MODE_PERSISTENT) {
+        if (sm >= (uint32_t)kMaxSM || !((g.sm_mask[sm >> 5] >> (sm & 31)) & 1u)) good = 0;
+        if (good && g.quota > 0) {
+          uint32_t slot = atomicAdd(&a.c.blk[g.kslot * kMaxSM + sm], 1u);
+          if (slot >= (uint32_t)g.quota) good = 0;
+        } else if (good && sm < (uint32_t)kMaxSM) {
+          atomicAdd(&a.c.blk[g.kslot * kMaxSM + sm], 1u);
+        }
+        if (good) atomicAdd(&c->admitted[g.kslot].v, 1ull);
+        __threadfence();
+        unsigned long long t = atomicAdd(&c->arrivals[g.kslot].v, 1ull);
+        if (t == (unsigned long long)gridDim.x - 1 && a.c.host_arrive) {
+          // every block of this grid has been dispatched and decided: tell the host it
+          // may launch the next group's kernel (deterministic SM/block binding)
+          a.c.host_arrive[g.kslot] = a.c.epoch;
+          __threadfence_system();
+        }
+        // progress guarantee: the last block of a grid to arrive stays if nobody did
+        // (binding is a performance hint; correctness never depends on it)
+        if (!good && t == (unsigned long long)gridDim.x - 1 && ld_relaxed(&c->admitted[g.kslot].v) == 0) {
+          good = 1;
+          atomicAdd(&c->admitted[g.kslot].v, 1ull);
+          atomicAdd(&c->fallback_admits, 1ull);
+        }
+      } else if (sm < (uint32_t)kMaxSM) {
+        atomicAdd(&a.c.blk[g.kslot * kMaxSM + sm], 1u);
+      }
+      ok = good;
+      for (int s = 0; s < kMaxStages; ++s) {
+        sh.out_cnt[s] = 0;
+        sh.deq[s] = sh.enq[s] = 0;
+        sh.t_exec[s] = sh.t_flush[s] = 0;
+      }
+      sh.t_idle = 0;
+      sh.acc_neg = 0;
+      sh.skip = 0;
+    }
+    __syncthreads();
+    return ok != 0;
+  }
+
+  static __device__ void flush_stats(const KArgs<F>& a, BlockShared& sh) {
+    if (threadIdx.x == 0) {
+      Ctrl* c = a.c.ctrl;
+      if (sh.acc_neg != 0) atom_add(&c->pending.v, sh.acc_neg);
+      sh.acc_neg = 0;
+      for (int s = 0; s < S; ++s) {
+        if (sh.deq[s]) atomicAdd(&c->deq[s], sh.deq[s]);
+        if (sh.enq[s]) atomicAdd(&c->enq[s], sh.enq[s]);
+        if (sh.t_exec[s]) atomicAdd(&c->exec_ns[s], sh.t_exec[s]);
+        if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
+      }
+      if (sh.t_idle) atomicAdd(&c->idle_ns[a.g.kslot], sh.t_idle);
+    }
+  }
+
+  // Claim from stage s (ring first, then seeds); thread 0 only.
+  static __device__ __forceinline__ int claim(const KArgs<F>& a, int s, int k, unsigned long long& base, int& from_seed) {
+    Ctrl* c = a.c.ctrl;
+    int got = claim_ring(c, s, k, base);
+    if (got) { from_seed = 0; return got; }
+    got = claim_seed(c, a.c.q[s], s, k, base);
+    from_seed = 1;
+    return got;
+  }
+
+  // Stage-in a claimed batch into the in-buffer (block-wide), releasing its ring slots.
+  // Returns false (block-uniformly) if the run aborted while waiting.
+  static __device__ bool stage_in(const KArgs<F>& a, BlockShared& sh, uint8_t* inbuf, int s, int n,
+                                  unsigned long long base, int from_seed) {
+    bool ok = true;
+    static_for<LO, HI + 1>([&](auto S_) {
+      constexpr int SS = decltype(S_)::value;
+      if (s == SS) {
+        const QueueDesc& q = a.c.q[SS];
+        if (from_seed) {
+          copy_seed_in<F::stride(SS)>(inbuf, q.seeds, base, n);
+        } else {
+          wait_slots(a.c, q, base, n, 0);
+          if (threadIdx.x == 0) sh.skip = aborted(a.c.ctrl) ? 1 : 0;
+          __syncthreads();
+          if (sh.skip) {
+            ok = false;
+          } else {
+            copy_in<F::stride(SS)>(inbuf, q.slots, base, n, q.cap_log2);
+            __syncthreads();
+            const unsigned long long mask = (1ull << q.cap_log2) - 1;
+            for (int k = threadIdx.x; k < n; k += blockDim.x) {
+              unsigned long long t = base + k;
+              st_release(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
+            }
+          }
+        }
+      }
+    });
+    __syncthreads();
+    return ok;
+  }
+
+  static __device__ void run(const KArgs<F>& a) {
+    extern __shared__ __align__(128) uint8_t smem[];
+    __shared__ BlockShared sh;
+    if (!admit(a, sh)) return;
+    CtxT ctx(a, smem, sh);
+    Ctrl* c = a.c.ctrl;
+    uint8_t* inbuf = smem;
+    const bool timers = a.c.flags & FLAG_TIMERS;
+
+    if (a.g.mode == MODE_WAVE) {
+      // KBK / standalone-RTC wave: this block processes items [b*batch, ...) of wave_stage.
+      const int s = a.g.wave_stage;
+      long long lo = (long long)blockIdx.x * a.g.batch[s];
+      long long rem = a.g.wave_n - lo;
+      int k = (int)(rem < a.g.batch[s] ? rem : a.g.batch[s]);
+      while (k > 0) {
+        unsigned long long t0 = 0;
+        if (threadIdx.x == 0) {
+          if (timers) t0 = globaltimer();
+          unsigned long long base = 0;
+          int fs = 0;
+          int got = aborted(c) ? 0 : claim(a, s, k, base, fs);
+          sh.cl_n = got;
+          sh.cl_base = base;
+          sh.cl_seed = fs;
+        }
+        __syncthreads();
+        const int n = sh.cl_n;
+        const unsigned long long base = sh.cl_base;
+        const int fs = sh.cl_seed;
+        __syncthreads();
+        if (n == 0) break;  // aborted, or (never) the host over-sized the wave
+        if (!stage_in(a, sh, inbuf, s, n, base, fs)) break;
+        execute(a, ctx, sh, s, inbuf, n, t0);
+        k -= n;
+      }
+      flush_stats(a, sh);
+      return;
+    }
+
+    unsigned ns = 64;
+    for (;;) {
+      unsigned long long t0 = 0;
+      if (threadIdx.x == 0) {
+        if (timers) t0 = globaltimer();
+        int got = 0, st = -1, fs = 0;
+        unsigned long long base = 0;
+        sh.done = 0;
+        if (aborted(c)) {
+          sh.done = 1;
+        } else {
+          // Task scheduler: "Query queues in turn of priority" (Fig. 8a) — downstream
+          // stages first (drains the pipeline, bounds live items), rings before seeds.
+          for (int s = HI; s >= LO && !got; --s) {
+            got = claim_ring(c, s, a.g.batch[s], base);
+            if (got) { st = s; fs = 0; }
+          }
+          for (int s = HI; s >= LO && !got; --s) {
+            got = claim_seed(c, a.c.q[s], s, a.g.batch[s], base);
+            if (got) { st = s; fs = 1; }
+          }
+          if (!got) {
+            // idle: retire deferred completions first, then test for termination
+            if (sh.acc_neg != 0) {
+              atom_add(&c->pending.v, sh.acc_neg);
+              sh.acc_neg = 0;
+            }
+            if ((long long)ld_acquire(&c->pending.v) <= 0) sh.done = 1;
+            else if (globaltimer() > c->deadline.v) {
+              atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
+              sh.done = 1;
+            }
+          }
+        }
+        sh.cl_stage = st;
+        sh.cl_n = got;
+        sh.cl_base = base;
+        sh.cl_seed = fs;
+      }
+      __syncthreads();
+      const int done = sh.done, n = sh.cl_n, s = sh.cl_stage, fs = sh.cl_seed;
+      const unsigned long long base = sh.cl_base;
+      __syncthreads();  // everyone has read the claim; thread 0 may overwrite it next round
+      if (done) break;
+      if (n == 0) {
+        __nanosleep(ns);
+        if (ns < 2048) ns <<= 1;
+        if (timers && threadIdx.x == 0) sh.t_idle += globaltimer() - t0;
+        continue;
+      }
+      ns = 64;
+      if (!stage_in(a, sh, inbuf, s, n, base, fs)) break;
+      execute(a, ctx, sh, s, inbuf, n, t0);
+    }
+    flush_stats(a, sh);
+  }
+};
+
+template <class F, int LO, int HI, bool RTC>
+__global__ void __launch_bounds__(kThreads, F::min_blocks(LO, HI, RTC)) vp_kernel(const __grid_constant__ KArgs<F> a) {
+  Runner<F, LO, HI, RTC>::run(a);
+}
+
+}  // namespace vp

@@ -1,0 +1,110 @@
+"""Workload assembly through the C ABI (argument marshalling only).
+
+Each class allocates the family's device buffers with PyTorch (plumbing), fills the
+vp_*_params struct with raw device pointers, registers the family's stages in order,
+inserts the seeded items (insertIntoQueue) and exposes run() and the
+sink outputs.  All pipeline work happens inside libvp.so.
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+from . import inputs, vp
+
+
+def _dev(device):
+    return torch.device("cuda", device)
+
+
+class ToyPipeline:
+    """Fig. 9 (L37): S1 doubles until >= threshold (recursive), S2 adds 1, S3 sink."""
+
+    def __init__(self, seeds: np.ndarray, threshold: int = inputs.TOY_THRESHOLD, device: int = 0, **kw):
+        self.n = int(seeds.size)
+        self.out = torch.zeros(max(self.n, 1), dtype=torch.int32, device=_dev(device))
+        self.n_out = torch.zeros(1, dtype=torch.int64, device=_dev(device))
+        self.prm = vp.ToyParams(threshold=threshold, out=self.out.data_ptr(), n_out=self.n_out.data_ptr())
+        self.p = vp.Pipeline(device, **kw)
+        for kind in (vp.TOY_S1, vp.TOY_S2, vp.TOY_S3):
+            self.p.register(kind, 4, self.prm)
+        self.p.insert(0, np.ascontiguousarray(seeds, np.int32))
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        st = self.p.run(stream)
+        n = int(self.n_out.item())
+        return self.out[:n].cpu().numpy(), st
+
+
+class CollatzPipeline:
+    def __init__(self, seeds: np.ndarray, max_steps: int = 1000, device: int = 0, **kw):
+        n = int(seeds.size)
+        self.steps = torch.zeros(n, dtype=torch.int32, device=_dev(device))
+        self.seen = torch.zeros(n, dtype=torch.int32, device=_dev(device))
+        self.prm = vp.CollatzParams(steps_out=self.steps.data_ptr(), seen=self.seen.data_ptr(), n_ids=n,
+                                    max_steps=max_steps)
+        self.p = vp.Pipeline(device, **kw)
+        self.p.register(vp.COLLATZ_STEP, 16, self.prm)
+        self.p.register(vp.COLLATZ_SINK, 16, self.prm)
+        self.p.insert(0, np.ascontiguousarray(seeds))
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        st = self.p.run(stream)
+        return self.steps.cpu().numpy().view(np.uint32), self.seen.cpu().numpy().view(np.uint32), st
+
+
+REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
+REYES_STRIDES = (272, 272, 272, 1968)
+
+
+class ReyesPipeline:
+    """Reyes Bound -> Split (recursive) | Dice -> Shade (Fig. 1, L3) over a ReyesScene."""
+
+    def __init__(self, scene: inputs.ReyesScene, device: int = 0, seeds_on_device: bool = True,
+                 queue_caps=None, **kw):
+        dev = _dev(device)
+        self.scene = scene
+        self.npix = scene.n_frames * scene.W * scene.H
+        self.M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).to(dev)
+        self.albedo = torch.from_numpy(np.ascontiguousarray(scene.albedo, np.float32)).to(dev)
+        self.fb = torch.empty((self.npix, 4), dtype=torch.int32, device=dev)       # {u64 key, f32 s, pad}
+        self.colour = torch.empty((scene.n_frames, scene.H, scene.W, 4), dtype=torch.float32, device=dev)
+        L = [float(np.float32(v)) for v in scene.light]
+        self.prm = vp.ReyesParams(W=scene.W, H=scene.H, n_frames=scene.n_frames,
+                                  patches_per_frame=scene.patches_per_frame, max_depth=scene.max_depth,
+                                  t_dice=scene.t_dice, near_w=scene.near_w, M=self.M.data_ptr(),
+                                  albedo=self.albedo.data_ptr(), fb=self.fb.data_ptr(),
+                                  colour=self.colour.data_ptr())
+        for i in range(4):
+            self.prm.L[i] = L[i]
+        self.p = vp.Pipeline(device, **kw)
+        caps = queue_caps or [0, 0, 0, 0]
+        for kind, stride, cap in zip(REYES_STAGES, REYES_STRIDES, caps):
+            self.p.register(kind, stride, self.prm, queue_capacity=cap)
+        seeds = np.ascontiguousarray(scene.seeds)
+        if seeds_on_device:
+            self.seeds_dev = torch.from_numpy(seeds.view(np.uint8).reshape(-1)).to(dev)
+            self.p.insert(0, self.seeds_dev, n=seeds.size)
+        else:
+            self.p.insert(0, seeds, n=seeds.size)
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def keys(self):
+        fb = self.fb.cpu().numpy()
+        key = fb[:, :2].copy().view(np.uint64).reshape(self.scene.n_frames, self.scene.H, self.scene.W)
+        s = fb[:, 2].copy().view(np.float32).reshape(self.scene.n_frames, self.scene.H, self.scene.W)
+        return key, s
+
+    def colours(self):
+        return self.colour.cpu().numpy()

@@ -1,0 +1,75 @@
+"""CPU-side checks of the boundary: libvp.so builds, loads without a GPU, and exports
+every entry point include/vp.h declares; struct layouts of the binding match the header."""
+import ctypes
+import os
+import re
+import subprocess
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HDR = os.path.join(ROOT, "include", "vp.h")
+
+
+def declared_functions():
+    src = open(HDR).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:vp_status|const char\*)\s+(vp_\w+)\s*\(", src, flags=re.M)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_micro_zhengozsyc17_b200 import build
+    path = build.build()
+    return ctypes.CDLL(path)
+
+
+def test_every_declared_symbol_is_exported(lib):
+    fns = declared_functions()
+    assert len(fns) >= 15
+    for f in fns:
+        assert hasattr(lib, f), f"libvp.so does not export {f}"
+
+
+def test_exports_are_extern_c():
+    from paper_conf_micro_zhengozsyc17_b200 import build
+    out = subprocess.run(["nm", "-D", "--defined-only", build.build()], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (vp_\w+)", out))
+    assert set(declared_functions()) <= exported
+
+
+def test_binding_declares_all_symbols():
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    assert set(declared_functions()) == set(vp.EXPORTED)
+
+
+def test_struct_sizes_match_header():
+    """Compile a tiny C program against vp.h and compare sizeof with the ctypes mirrors."""
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    prog = r'''
+#include <stdio.h>
+#include "vp.h"
+int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pipeline_desc), sizeof(vp_stage_desc),
+ sizeof(vp_sm_binding), sizeof(vp_config), sizeof(vp_run_stats), sizeof(vp_autotune_opts), sizeof(vp_tune_report),
+ sizeof(vp_toy_params), sizeof(vp_collatz_params), sizeof(vp_reyes_params));return 0;}
+'''
+    tmp = os.path.join(ROOT, "build_abi_check")
+    os.makedirs(tmp, exist_ok=True)
+    c = os.path.join(tmp, "sz.c")
+    open(c, "w").write(prog)
+    exe = os.path.join(tmp, "sz")
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe], check=True)
+    sizes = [int(x) for x in subprocess.run([exe], capture_output=True, text=True).stdout.split()]
+    mirrors = [vp.PipelineDesc, vp.StageDesc, vp.SmBinding, vp.Config, vp.RunStats, vp.AutotuneOpts, vp.TuneReport,
+               vp.ToyParams, vp.CollatzParams, vp.ReyesParams]
+    assert sizes == [ctypes.sizeof(m) for m in mirrors]
+
+
+def test_no_gpu_calls_fail_cleanly(lib):
+    """Without a GPU the library reports an error instead of crashing."""
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    with pytest.raises(vp.VPError):
+        vp.Pipeline(0)

@@ -1,0 +1,42 @@
+"""Dev tool: single-kernel launches of the hot path for `ncu` (which serialises kernels,
+so co-running persistent groups cannot be captured together).
+
+  mega      : the whole Reyes pipeline as one megakernel (config 5 shape, --frames)
+  rtc_dice  : the [Dice,Shade] RTC kernel alone: every seed patch is inserted into the
+              Dice queue, the [Bound,Split] group is an (idle) KBK group
+  kbk       : one launch per stage per wave
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch
+
+from paper_conf_micro_zhengozsyc17_b200 import inputs, vp
+from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+
+ap = argparse.ArgumentParser()
+ap.add_argument("target")
+ap.add_argument("--frames", type=int, default=64)
+ap.add_argument("--runs", type=int, default=2)
+args = ap.parse_args()
+
+scene = inputs.reyes_config5(n_frames=args.frames)
+nsm, _ = vp.device_info(0)
+rp = ReyesPipeline(scene)
+if args.target == "mega":
+    rp.configure(vp.MEGAKERNEL)
+elif args.target == "kbk":
+    rp.configure(vp.KBK)
+elif args.target == "rtc_dice":
+    rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
+    rp.p.insert(2, rp.seeds_dev, n=scene.seeds.size)
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_KBK, 0, 8), (2, 3, vp.GROUP_RTC, 8, nsm)], nsm))
+else:
+    raise SystemExit(f"unknown target {args.target}")
+for _ in range(args.runs):
+    st = rp.run()
+torch.cuda.synchronize()
+print(args.target, st["device_ms"], st["dequeued"][:4], st["kernels"])
