@@ -30,14 +30,14 @@ struct ToyF {
   static constexpr bool uses_latches(int, int) { return false; }
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int) { return 20; }
-  static constexpr int min_blocks(int, int, bool) { return 1; }
+  static constexpr int min_blocks(int, int, bool) { return 3; }
   template <int s>
   static __device__ unsigned long long item_id(const uint8_t* it) { return *(const uint32_t*)it; }
 
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
-    for (int base = 0; base < n; base += blockDim.x) {
+    for (int base = 0; base < n; base += kThreads) {
       int k = base + threadIdx.x;
       bool valid = k < n;
       int32_t v = valid ? ((const int32_t*)items)[k] : 0;
@@ -92,7 +92,7 @@ struct CollatzF {
   static constexpr bool uses_latches(int, int) { return false; }
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int) { return 20; }
-  static constexpr int min_blocks(int, int, bool) { return 1; }
+  static constexpr int min_blocks(int, int, bool) { return 3; }
   template <int s>
   static __device__ unsigned long long item_id(const uint8_t* it) {
     const CollatzItem* c = (const CollatzItem*)it;
@@ -101,7 +101,7 @@ struct CollatzF {
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
-    for (int k = threadIdx.x; k < n; k += blockDim.x) {
+    for (int k = threadIdx.x; k < n; k += kThreads) {
       CollatzItem it = ((const CollatzItem*)items)[k];
       if constexpr (s == 0) {
         if (it.v == 1) {

@@ -176,8 +176,8 @@ struct ReyesF {
   using Params = vp_reyes_params;
   static constexpr int stride(int s) { return s == SHADE ? (int)sizeof(RGrid) : (int)sizeof(RPatch); }
   static constexpr int threads_per_item(int s) { return s == BOUND ? 16 : s == SPLIT ? 16 : s == DICE ? 32 : 64; }
-  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 32 : 8; }
-  static constexpr int default_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 8 : 4; }
+  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 8 : 4; }
+  static constexpr int default_batch(int s) { return max_batch(s); }
   static constexpr int fanout(int s, int t) {
     return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
   }
@@ -185,7 +185,7 @@ struct ReyesF {
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
-  static constexpr int min_blocks(int lo, int hi, bool) { return hi == SHADE ? VP_REYES_MINB : 1; }
+  static constexpr int min_blocks(int, int, bool) { return VP_REYES_MINB; }
 
   template <int s>
   static __device__ unsigned long long item_id(const uint8_t* it) {

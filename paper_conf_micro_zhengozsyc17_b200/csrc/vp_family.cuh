@@ -104,8 +104,8 @@ struct FamilyImpl final : FamilyOps {
     a.p = *(const typename F::Params*)params;
     void* args[] = {&a};
     size_t sm = smem(lo, hi, rtc);
-    if (coop) return cudaLaunchCooperativeKernel(k, dim3(grid), dim3(kThreads), args, sm, st);
-    return cudaLaunchKernel(k, dim3(grid), dim3(kThreads), args, sm, st);
+    if (coop) return cudaLaunchCooperativeKernel(k, dim3(grid), dim3(kBlock), args, sm, st);
+    return cudaLaunchKernel(k, dim3(grid), dim3(kBlock), args, sm, st);
   }
   cudaError_t init_run(const void* params, cudaStream_t st) const override {
     return F::init_run(*(const typename F::Params*)params, st);

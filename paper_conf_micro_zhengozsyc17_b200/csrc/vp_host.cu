@@ -118,6 +118,7 @@ struct Plan {
   std::vector<int> kbk_stages;         // stages driven by the host wave loop
   bool wave_rtc = false;               // standalone RTC: waves of the [0,S-1] RTC kernel
   int batch[kMaxStages] = {};
+  int cap_log2[kMaxStages] = {};       // effective ring size this plan runs with
   vp_config cfg{};
 };
 
@@ -133,6 +134,7 @@ struct vp_pipeline_s {
   bool queues_ready = false;
   bool configured = false;
   bool dirty_queues = false;  // after an aborted run: reset rings before the next one
+  int run_cap_log2[kMaxStages] = {};  // ring size the seq words were initialised for
   Plan plan;
   Ctrl* ctrl = nullptr;
   uint32_t* blk = nullptr;
@@ -191,9 +193,9 @@ int occupancy(vp_pipeline_s* p, int lo, int hi, bool rtc) {
   const void* fn = p->fam->kernel(lo, hi, rtc);
   if (!fn) return 0;
   size_t sm = p->fam->smem(lo, hi, rtc);
-  if (sm > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+  cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
   int occ = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kThreads, sm) != cudaSuccess) occ = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, sm) != cudaSuccess) occ = 0;
   c = occ;
   return occ;
 }
@@ -220,6 +222,7 @@ vp_status ensure_queues(vp_pipeline_s* p) {
     CUDA_TRY(p, cudaMalloc(&r.slots, cap * (size_t)p->fam->stride((int)s)));
     CUDA_TRY(p, cudaMalloc(&r.seq, cap * sizeof(unsigned long long)));
     k_init_seq<<<256, 256>>>(r.seq, cap, 0);
+    p->run_cap_log2[s] = r.cap_log2;
     CUDA_TRY(p, cudaGetLastError());
   }
   CUDA_TRY(p, cudaDeviceSynchronize());
@@ -230,8 +233,9 @@ vp_status ensure_queues(vp_pipeline_s* p) {
 vp_status reset_queues(vp_pipeline_s* p, cudaStream_t st) {
   k_reset_queues<<<1, 32, 0, st>>>(p->ctrl);
   for (size_t s = 0; s < p->st.size(); ++s) {
-    size_t cap = 1ull << p->st[s].cap_log2;
-    k_init_seq<<<256, 256, 0, st>>>(p->st[s].seq, cap, 0);
+    int lg = p->plan.cap_log2[s] ? p->plan.cap_log2[s] : p->st[s].cap_log2;
+    p->run_cap_log2[s] = lg;
+    k_init_seq<<<256, 256, 0, st>>>(p->st[s].seq, 1ull << lg, 0);
   }
   CUDA_TRY(p, cudaGetLastError());
   p->dirty_queues = false;
@@ -247,7 +251,7 @@ Common make_common(vp_pipeline_s* p) {
     c.q[s].seq = r.seq;
     c.q[s].seeds = r.seeds;
     c.q[s].n_seeds = (long long)r.n_seeds;
-    c.q[s].cap_log2 = (uint32_t)r.cap_log2;
+    c.q[s].cap_log2 = (uint32_t)(p->plan.cap_log2[s] ? p->plan.cap_log2[s] : r.cap_log2);
     c.q[s].stride = (uint32_t)p->fam->stride((int)s);
   }
   c.ctrl = p->ctrl;
@@ -268,11 +272,11 @@ struct KRes {
   int regs, smem, threads;
 };
 KRes kernel_res(vp_pipeline_s* p, int lo, int hi, bool rtc) {
-  KRes r{0, 0, kThreads};
+  KRes r{0, 0, kBlock};
   cudaFuncAttributes at;
-  if (cudaFuncGetAttributes(&at, p->fam->kernel(lo, hi, rtc)) != cudaSuccess) return KRes{1 << 30, 1 << 30, kThreads};
+  if (cudaFuncGetAttributes(&at, p->fam->kernel(lo, hi, rtc)) != cudaSuccess) return KRes{1 << 30, 1 << 30, kBlock};
   int per_warp = ((at.numRegs * 32 + 255) / 256) * 256;
-  r.regs = per_warp * (kThreads / 32);
+  r.regs = per_warp * (kBlock / 32);
   r.smem = (int)(at.sharedSizeBytes + p->fam->smem(lo, hi, rtc)) + 1024;
   return r;
 }
@@ -289,10 +293,14 @@ bool fits_sm(vp_pipeline_s* p, const KRes* res, const int* q, int n) {
   return regs <= prop.regsPerMultiprocessor && smem <= (long long)prop.sharedMemPerMultiprocessor &&
          thr <= prop.maxThreadsPerMultiProcessor && blocks <= prop.maxBlocksPerMultiProcessor;
 }
-// Block quotas for the single-stage kernels of a fine group [lo,hi] sharing each SM:
-// requested quotas are checked for co-residency; missing ones are filled greedily
-// (one block each, then round-robin while the SM still fits them all).
-vp_status fine_quotas(vp_pipeline_s* p, int lo, int hi, const int* req, int* q) {
+// Block mapping of a fine group [lo,hi] (Fig. 5; Block Mapping Controller, L27): every
+// stage kernel gets the same block quota on each of its SMs (L45 pruning rule).  If all
+// stages cannot co-reside on one SM, SM j of the group hosts the cyclic window of m
+// stages {(j + i) mod n : i < m} for the largest m whose every window fits.
+// Requested quotas are checked; missing ones are filled greedily (round-robin while
+// every window still fits).
+vp_status fine_quotas(vp_pipeline_s* p, int lo, int hi, const int* req, const uint32_t* group_mask, int* q,
+                      uint32_t (*masks)[kMaskWords]) {
   const int n = hi - lo + 1;
   KRes res[kMaxStages];
   int qq[kMaxStages];
@@ -302,18 +310,45 @@ vp_status fine_quotas(vp_pipeline_s* p, int lo, int hi, const int* req, int* q) 
     fixed[i] = req && req[lo + i] > 0;
     qq[i] = fixed[i] ? req[lo + i] : 1;
   }
-  if (!fits_sm(p, res, qq, n))
+  auto windows_fit = [&](int m) {
+    for (int j = 0; j < n; ++j) {
+      KRes wr[kMaxStages];
+      int wq[kMaxStages];
+      for (int i = 0; i < m; ++i) {
+        wr[i] = res[(j + i) % n];
+        wq[i] = qq[(j + i) % n];
+      }
+      if (!fits_sm(p, wr, wq, m)) return false;
+      if (m == n) break;
+    }
+    return true;
+  };
+  int m = n;
+  while (m > 0 && !windows_fit(m)) --m;
+  if (m == 0)
     return fail(p, VP_ERR_INVALID, "fine group [%d,%d]: block quotas do not fit one SM (registers/smem/threads)", lo, hi);
   for (bool grew = true; grew;) {
     grew = false;
     for (int i = 0; i < n; ++i) {
       if (fixed[i]) continue;
       qq[i]++;
-      if (fits_sm(p, res, qq, n)) grew = true;
+      if (windows_fit(m)) grew = true;
       else qq[i]--;
     }
   }
-  for (int i = 0; i < n; ++i) q[lo + i] = qq[i];
+  for (int i = 0; i < n; ++i) {
+    q[lo + i] = qq[i];
+    memset(masks[lo + i], 0, sizeof(uint32_t) * kMaskWords);
+  }
+  int j = 0;
+  for (int sm = 0; sm < kMaxSM; ++sm) {
+    if (!((group_mask[sm >> 5] >> (sm & 31)) & 1u)) continue;
+    for (int i = 0; i < m; ++i) {
+      int st = lo + (j + i) % n;
+      masks[st][sm >> 5] |= 1u << (sm & 31);
+    }
+    ++j;
+  }
   return VP_OK;
 }
 
@@ -379,11 +414,12 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
     case VP_FINE: {
       // each stage its own persistent kernel; SMs shared, blocks per (stage, SM) capped (Fig. 5)
       int q[kMaxStages];
-      rc = fine_quotas(p, 0, S - 1, b ? b->blocks_per_sm : nullptr, q);
+      uint32_t sm_of[kMaxStages][kMaskWords];
       uint32_t m[kMaskWords];
       if (b && b->num_groups == 1) memcpy(m, b->group_sm_mask[0], sizeof(m));
       else memcpy(m, all, sizeof(m));
-      for (int s = 0; s < S && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], m, false);
+      rc = fine_quotas(p, 0, S - 1, b ? b->blocks_per_sm : nullptr, m, q, sm_of);
+      for (int s = 0; s < S && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], sm_of[s], false);
       break;
     }
     case VP_HYBRID: {
@@ -423,8 +459,9 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
           rc = add_kernel(lo[g], hi[g], false, b->blocks_per_sm[lo[g]], m, false);
         } else if (gm == VP_GROUP_FINE) {
           int q[kMaxStages];
-          rc = fine_quotas(p, lo[g], hi[g], b->blocks_per_sm, q);
-          for (int s = lo[g]; s <= hi[g] && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], m, false);
+          uint32_t sm_of[kMaxStages][kMaskWords];
+          rc = fine_quotas(p, lo[g], hi[g], b->blocks_per_sm, m, q, sm_of);
+          for (int s = lo[g]; s <= hi[g] && rc == VP_OK; ++s) rc = add_kernel(s, s, false, q[s], sm_of[s], false);
         } else if (gm == VP_GROUP_KBK) {
           for (int s = lo[g]; s <= hi[g]; ++s) pl.kbk_stages.push_back(s);
         } else {
@@ -437,13 +474,35 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       return fail(p, VP_ERR_INVALID, "unknown model %d", model);
   }
   if (rc != VP_OK) return rc;
+  // Effective ring sizes.  Persistent plans drain continuously: a ring needs room for
+  // the batches its producers hold (two out buffers per block), so it is sized to that
+  // and stays L2-resident (no dirty-line write-back to HBM).  Host-driven waves (KBK,
+  // RTC waves) need room for a whole wave: they use the full allocation.
+  for (int t = 0; t < S; ++t) {
+    int full = p->st[t].cap_log2;
+    if (!pl.kbk_stages.empty() || pl.wave_rtc) {
+      pl.cap_log2[t] = full;
+      continue;
+    }
+    long long need = 0;
+    for (const KernelPlan& k : pl.kernels) {
+      int per = k.quota > 0 ? k.quota : occupancy(p, k.lo, k.hi, k.rtc);
+      long long blocks = (long long)per * mask_count(k.mask, N);
+      long long mx = 0;
+      for (int s = k.lo; s <= k.hi; ++s) mx = std::max(mx, (long long)pl.batch[s] * p->fam->fanout(s, t));
+      need += 2 * blocks * mx;
+    }
+    int lg = 12;
+    while (lg < full && (1ll << lg) < need) ++lg;
+    pl.cap_log2[t] = std::min(lg, full);
+  }
   // every producer batch must fit twice into its target ring, or the ring cannot drain
   for (int s = 0; s < S; ++s)
     for (int t = 0; t < S; ++t) {
       int f = p->fam->fanout(s, t);
-      if (f > 0 && 2ll * pl.batch[s] * f > (1ll << p->st[t].cap_log2))
+      if (f > 0 && 2ll * pl.batch[s] * f > (1ll << pl.cap_log2[t]))
         return fail(p, VP_ERR_INVALID, "queue_capacity of stage %d (%lld) < 2 x batch(%d) x fanout(%d) of stage %d", t,
-                    1ll << p->st[t].cap_log2, pl.batch[s], f, s);
+                    1ll << pl.cap_log2[t], pl.batch[s], f, s);
     }
   pl.cfg.model = model;
   pl.cfg.has_binding = b ? 1 : 0;
@@ -463,9 +522,13 @@ vp_status launch_wave(vp_pipeline_s* p, const Common& c, int lo, int hi, bool rt
   g.wave_n = n;
   g.kslot = kslot;
   for (int s = 0; s < kMaxStages; ++s) g.batch[s] = p->plan.batch[s] ? p->plan.batch[s] : 1;
-  long long grid = (n + g.batch[stage] - 1) / g.batch[stage];
-  if (grid > 0x7fffffff) grid = 0x7fffffff;
-  occupancy(p, lo, hi, rtc);  // sets the smem attribute once
+  // one resident wave of blocks, each taking a contiguous chunk of whole batches so the
+  // fetch / execute / publish warps of a block overlap across its batches
+  long long batches = (n + g.batch[stage] - 1) / g.batch[stage];
+  long long resident = (long long)std::max(1, occupancy(p, lo, hi, rtc)) * p->num_sms;
+  long long grid = std::min(batches, resident);
+  g.wave_chunk = ((batches + grid - 1) / grid) * g.batch[stage];
+  grid = (n + g.wave_chunk - 1) / g.wave_chunk;
   CUDA_TRY(p, p->fam->launch(lo, hi, rtc, c, g, p->params.data(), (int)grid, false, st));
   return VP_OK;
 }
@@ -504,7 +567,7 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
     long long cap = 1ll << 40;
     for (int t = 0; t < S; ++t) {
       int f = p->fam->fanout(s, t);
-      if (f > 0) cap = std::min(cap, (long long)(1ll << p->st[t].cap_log2) / (2 * f));
+      if (f > 0) cap = std::min(cap, (long long)(1ll << p->plan.cap_log2[t]) / (2 * f));
     }
     return std::max(1ll, cap);
   };
@@ -792,6 +855,8 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   DeviceGuard dg(p->device);
   cudaStream_t st = (cudaStream_t)stream;
   const int S = (int)p->st.size();
+  for (int s = 0; s < S; ++s)
+    if (p->run_cap_log2[s] != (p->plan.cap_log2[s] ? p->plan.cap_log2[s] : p->st[s].cap_log2)) p->dirty_queues = true;
   if (p->dirty_queues) {
     vp_status rc = reset_queues(p, st);
     if (rc != VP_OK) return rc;

@@ -27,7 +27,9 @@
 
 namespace vp {
 
-constexpr int kThreads = 256;       // the paper's block size for persistent models (L53)
+constexpr int kThreads = 256;       // worker threads per block: the paper's block size (L53)
+constexpr int kWarpsW = kThreads / 32;
+constexpr int kBlock = kThreads + 64;  // + a fetcher warp and a publisher warp (task scheduler)
 constexpr int kMaxStages = 8;
 constexpr int kMaxKernels = 16;     // kernel slots per run (binding counters)
 constexpr int kMaxSM = 256;         // table width; B200 has 148 SMs (queried at runtime)
@@ -104,6 +106,7 @@ struct GroupArgs {
   int mode;                      // MODE_PERSISTENT or MODE_WAVE
   int wave_stage;                // WAVE: the stage whose items this launch processes
   long long wave_n;              // WAVE: number of items in this launch
+  long long wave_chunk;          // WAVE: items per block (a multiple of the batch)
   int batch[kMaxStages];         // items per claim, per stage
 };
 
@@ -190,36 +193,42 @@ struct Graph {
     }
     return c;
   }
-  static constexpr int in_bytes(int lo, int hi) {
+  static constexpr int align128(int b) { return (b + 127) / 128 * 128; }
+  static constexpr int in_region(int lo, int hi) {
     int b = 0;
     for (int s = lo; s <= hi; ++s) {
       int v = F::max_batch(s) * F::stride(s);
       b = b > v ? b : v;
     }
-    return b;
+    return align128(b);
   }
-  static constexpr int align128(int b) { return (b + 127) / 128 * 128; }
-  static constexpr int out_offset(int lo, int hi, bool rtc, int t) {
-    int off = align128(in_bytes(lo, hi));
+  static constexpr int out_off(int lo, int hi, bool rtc, int t) {
+    int off = 0;
     for (int u = 0; u < t; ++u) off += align128(out_cap(lo, hi, rtc, u) * F::stride(u));
     return off;
   }
-  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return out_offset(lo, hi, rtc, S) + F::scratch_bytes(lo, hi); }
-  static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_offset(lo, hi, rtc, S); }
+  static constexpr int out_region(int lo, int hi, bool rtc) { return out_off(lo, hi, rtc, S); }
+  // double-buffered: in[2] | out[2] | scratch
+  static constexpr int in_base(int lo, int hi, int b) { return b * in_region(lo, hi); }
+  static constexpr int out_base(int lo, int hi, bool rtc, int b) { return 2 * in_region(lo, hi) + b * out_region(lo, hi, rtc); }
+  static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_base(lo, hi, rtc, 2); }
+  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + F::scratch_bytes(lo, hi); }
 };
-
 
 // ------------------------------------------------------------------ per-block context
 struct BlockShared {
-  int out_cnt[kMaxStages];
+  int out_cnt[2][kMaxStages];          // per out buffer, per target
   unsigned long long out_base[kMaxStages];
-  int cl_stage, cl_n, cl_seed, done, skip;
-  unsigned long long cl_base;
-  long long acc_neg;  // completions not yet subtracted from `pending` (deferred, <= 0)
+  int nx_stage, nx_n, nx_seed, done;   // the batch the fetcher staged for the next round
+  unsigned long long nx_base;
+  long long acc_neg;                   // completions not yet subtracted from `pending` (<= 0)
+  long long wave_rem;                  // WAVE: items of this block's chunk not yet claimed
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle;
 };
+
+__device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
 
 template <class F, int LO, int HI, bool RTC>
 struct Ctx {
@@ -227,25 +236,25 @@ struct Ctx {
   const KArgs<F>& a;
   uint8_t* smem;
   BlockShared& sh;
-  int tid;
+  int ob;  // current out buffer
 
-  __device__ Ctx(const KArgs<F>& a_, uint8_t* smem_, BlockShared& sh_) : a(a_), smem(smem_), sh(sh_), tid(threadIdx.x) {}
+  __device__ Ctx(const KArgs<F>& a_, uint8_t* smem_, BlockShared& sh_) : a(a_), smem(smem_), sh(sh_), ob(0) {}
 
   __device__ __forceinline__ const typename F::Params& params() const { return a.p; }
   __device__ __forceinline__ uint8_t* scratch() { return smem + G::scratch_offset(LO, HI, RTC); }
 
   template <int T>
   __device__ __forceinline__ uint8_t* out_ptr(int slot) {
-    return smem + G::out_offset(LO, HI, RTC, T) + slot * F::stride(T);
+    return smem + G::out_base(LO, HI, RTC, ob) + G::out_off(LO, HI, RTC, T) + slot * F::stride(T);
   }
   template <int T>
   static constexpr int cap() { return G::out_cap(LO, HI, RTC, T); }
 
-  // Reserve k consecutive out slots for target T (called by one thread).  The declared
-  // fan-out bounds guarantee capacity; exceeding it aborts the run (ABORT_FANOUT).
+  // Reserve k consecutive out slots for target T (one thread).  The declared fan-out
+  // bounds guarantee capacity; exceeding it aborts the run (ABORT_FANOUT).
   template <int T>
   __device__ __forceinline__ int reserve(int k = 1) {
-    int slot = atomicAdd(&sh.out_cnt[T], k);
+    int slot = atomicAdd(&sh.out_cnt[ob][T], k);
     if (slot + k > cap<T>()) {
       atomicCAS((unsigned long long*)&a.c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_FANOUT);
       return -1;
@@ -273,11 +282,11 @@ __device__ __forceinline__ bool aborted(const Ctrl* c) {
   return *(volatile const unsigned long long*)&c->abort.v != 0ull;
 }
 
-// Thread 0: claim up to k items of stage s from its ring (published items only).
+// One thread: claim up to k published items of stage s from its ring.
 // 2 L2 atomics per block batch: `count` (availability) then `head` (ticket range).
 __device__ __forceinline__ int claim_ring(Ctrl* c, int s, int k, unsigned long long& base) {
   long long avail = (long long)ld_relaxed(&c->count[s].v);
-  if (avail <= 0) return 0;  // cheap L2 read first: idle blocks do not hammer atomics
+  if (avail <= 0) return 0;  // cheap L2 read first: idle fetchers do not hammer atomics
   int want = (int)(avail < k ? avail : k);
   long long old = (long long)atom_add(&c->count[s].v, -want);
   int got = old <= 0 ? 0 : (old < want ? (int)old : want);
@@ -286,7 +295,7 @@ __device__ __forceinline__ int claim_ring(Ctrl* c, int s, int k, unsigned long l
   base = atom_add(&c->head[s].v, got);
   return got;
 }
-// Thread 0: claim up to k seed items of stage s.
+// One thread: claim up to k seed items of stage s.
 __device__ __forceinline__ int claim_seed(Ctrl* c, const QueueDesc& q, int s, int k, unsigned long long& base) {
   if (q.n_seeds == 0) return 0;
   if ((long long)ld_relaxed(&c->seed_head[s].v) >= q.n_seeds) return 0;
@@ -297,12 +306,12 @@ __device__ __forceinline__ int claim_seed(Ctrl* c, const QueueDesc& q, int s, in
   return (int)(got < k ? got : k);
 }
 
-// Block-wide: wait until ring slots [base, base+n) hold the wanted sequence value.
+// Warp-wide (lane = 0..31): wait until ring slots [base, base+n) hold the wanted sequence.
 // mode 0: wait for publish (seq == t+1); mode 1: wait for free (seq == t).
 __device__ __forceinline__ void wait_slots(const Common& c, const QueueDesc& q, unsigned long long base, int n,
-                                           int mode) {
+                                           int mode, int lane) {
   const unsigned long long mask = (1ull << q.cap_log2) - 1;
-  for (int k = threadIdx.x; k < n; k += blockDim.x) {
+  for (int k = lane; k < n; k += 32) {
     unsigned long long t = base + k;
     unsigned long long want = t + (mode == 0 ? 1ull : 0ull);
     const unsigned long long* p = q.seq + (t & mask);
@@ -327,40 +336,59 @@ __device__ __forceinline__ void wait_slots(const Common& c, const QueueDesc& q, 
   }
 }
 
-// Block-wide copies between the smem batch and a ring (wrap-aware) or the seed array,
-// in 16-B (or 8/4-B for small items) coalesced chunks; ring loads bypass L1 (.cg).
+// Warp-wide copies between a smem batch and a ring (wrap-aware) or the seed array, in
+// 16-B (or 8/4-B for small items) chunks, 4 loads in flight per lane; ring loads bypass
+// L1 (.cg) so a reused slot is never served stale.
 template <int STRIDE>
 __device__ __forceinline__ void copy_in(uint8_t* dst, const uint8_t* ring, unsigned long long base, int n,
-                                        uint32_t cap_log2) {
+                                        uint32_t cap_log2, int lane) {
   using C = Chunk<STRIDE>;
   using T = typename C::T;
   const unsigned long long mask = (1ull << cap_log2) - 1;
   const int total = n * C::per_item;
-  for (int i = threadIdx.x; i < total; i += blockDim.x) {
+  int i = lane;
+  for (; i + 96 < total; i += 128) {
+    T v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      int j = i + 32 * u, k = j / C::per_item, w = j - k * C::per_item;
+      v[u] = ld_cg((const T*)(ring + ((base + k) & mask) * STRIDE) + w);
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) ((T*)dst)[i + 32 * u] = v[u];
+  }
+  for (; i < total; i += 32) {
     int k = i / C::per_item, w = i - k * C::per_item;
-    const T* src = (const T*)(ring + ((base + k) & mask) * STRIDE) + w;
-    ((T*)dst)[i] = ld_cg(src);
+    ((T*)dst)[i] = ld_cg((const T*)(ring + ((base + k) & mask) * STRIDE) + w);
   }
 }
 template <int STRIDE>
-__device__ __forceinline__ void copy_seed_in(uint8_t* dst, const uint8_t* seeds, unsigned long long base, int n) {
+__device__ __forceinline__ void copy_seed_in(uint8_t* dst, const uint8_t* seeds, unsigned long long base, int n,
+                                             int lane) {
   using C = Chunk<STRIDE>;
   using T = typename C::T;
   const T* src = (const T*)(seeds + base * STRIDE);
   const int total = n * C::per_item;
-  for (int i = threadIdx.x; i < total; i += blockDim.x) ((T*)dst)[i] = __ldg(src + i);
+  int i = lane;
+  for (; i + 96 < total; i += 128) {
+    T v[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = __ldg(src + i + 32 * u);
+#pragma unroll
+    for (int u = 0; u < 4; ++u) ((T*)dst)[i + 32 * u] = v[u];
+  }
+  for (; i < total; i += 32) ((T*)dst)[i] = __ldg(src + i);
 }
 template <int STRIDE>
 __device__ __forceinline__ void copy_out(uint8_t* ring, const uint8_t* src, unsigned long long base, int n,
-                                         uint32_t cap_log2) {
+                                         uint32_t cap_log2, int lane) {
   using C = Chunk<STRIDE>;
   using T = typename C::T;
   const unsigned long long mask = (1ull << cap_log2) - 1;
   const int total = n * C::per_item;
-  for (int i = threadIdx.x; i < total; i += blockDim.x) {
+  for (int i = lane; i < total; i += 32) {
     int k = i / C::per_item, w = i - k * C::per_item;
-    T* d = (T*)(ring + ((base + k) & mask) * STRIDE) + w;
-    st_cg(d, ((const T*)src)[i]);
+    st_cg((T*)(ring + ((base + k) & mask) * STRIDE) + w, ((const T*)src)[i]);
   }
 }
 
@@ -373,102 +401,194 @@ __device__ __forceinline__ void static_for(Fn&& fn) {
   }
 }
 
-// ------------------------------------------------------------------ the persistent kernel
+// ------------------------------------------------------------------ the persistent block
+// Warp-specialised persistent block (B200 design): warps 0..7 execute
+// batch i of their stage, while the fetcher warp claims and stages batch i+1 and the
+// publisher warp pushes the outputs of batch i-1 — the task scheduler and work-queue
+// library of Fig. 2/Fig. 8 run concurrently with the stage functions, one block
+// barrier per batch.
 template <class F, int LO, int HI, bool RTC>
 struct Runner {
   using G = Graph<F>;
   using CtxT = Ctx<F, LO, HI, RTC>;
   static constexpr int S = F::S;
+  static constexpr int W_FETCH = kWarpsW, W_PUBLISH = kWarpsW + 1;
 
-  static __device__ __forceinline__ bool is_local(int t, int local_from, int local_to) {
-    return t >= local_from && t <= local_to;
+  __device__ static __forceinline__ uint8_t* in_buf(uint8_t* smem, int b) { return smem + G::in_base(LO, HI, b); }
+  __device__ static __forceinline__ uint8_t* out_buf(uint8_t* smem, int b, int t) {
+    return smem + G::out_base(LO, HI, RTC, b) + G::out_off(LO, HI, RTC, t);
   }
 
-  // Publish the block-staged outputs of every target outside the local chain to its
-  // ring: one `tail` atomic + one `count` atomic per (block batch, target), coalesced
-  // payload stores, per-slot release.  `completed` parents are retired here.
-  static __device__ void flush(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, int local_from, int local_to,
-                               long long completed) {
+  // ---------------- publisher warp: push out buffer `pb` (outputs of a batch of
+  // `completed` items of stage ps) to the target rings, then retire the batch.
+  static __device__ void publish(const KArgs<F>& a, BlockShared& sh, uint8_t* smem, int pb, int ps, int completed,
+                                 int lane) {
     Ctrl* c = a.c.ctrl;
-    __syncthreads();
-    if (threadIdx.x == 0) {
+    const bool timers = a.c.flags & FLAG_TIMERS;
+    unsigned long long t0 = (timers && lane == 0) ? globaltimer() : 0;
+    int any = 0;
+    if (lane == 0) {
       long long children = 0;
       for (int t = 0; t < S; ++t) {
-        int n = sh.out_cnt[t];
+        int n = sh.out_cnt[pb][t];
         if (n > G::out_cap(LO, HI, RTC, t)) n = G::out_cap(LO, HI, RTC, t);
-        sh.out_cnt[t] = n;
-        if (n == 0 || is_local(t, local_from, local_to)) continue;
+        sh.out_cnt[pb][t] = n;
         children += n;
       }
-      // Termination accounting: children must be counted before they become visible;
+      // Termination accounting: children are counted before they become visible;
       // completions may be deferred (pending only stays conservatively high).
       if (children > 0) {
         long long d = children - completed + sh.acc_neg;
         if (d != 0) atom_add(&c->pending.v, d);
         sh.acc_neg = 0;
+        for (int t = 0; t < S; ++t) {
+          int n = sh.out_cnt[pb][t];
+          if (n == 0) continue;
+          sh.out_base[t] = atom_add(&c->tail[t].v, n);
+          sh.enq[t] += n;
+          if (a.c.flags & FLAG_DEPTH) {
+            unsigned long long h = ld_relaxed(&c->head[t].v);
+            unsigned long long dd = sh.out_base[t] + n - h;
+            if (dd > c->max_depth[t]) atomicMax(&c->max_depth[t], dd);
+          }
+        }
+        any = 1;
       } else {
         sh.acc_neg -= completed;
       }
-      for (int t = 0; t < S; ++t) {
-        int n = sh.out_cnt[t];
-        if (n == 0 || is_local(t, local_from, local_to)) continue;
-        sh.out_base[t] = atom_add(&c->tail[t].v, n);
-        sh.enq[t] += n;
-        if (a.c.flags & FLAG_DEPTH) {
-          unsigned long long h = ld_relaxed(&c->head[t].v);
-          unsigned long long d = sh.out_base[t] + n - h;
-          if (d > c->max_depth[t]) atomicMax(&c->max_depth[t], d);
-        }
-      }
     }
-    __syncthreads();
-    bool any = false;
-    static_for<0, S>([&](auto T_) {
-      constexpr int T = decltype(T_)::value;
-      if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
-        int n = sh.out_cnt[T];
-        if (n > 0 && !is_local(T, local_from, local_to)) {
-          wait_slots(a.c, a.c.q[T], sh.out_base[T], n, 1);
-          any = true;
-        }
-      }
-    });
+    any = __shfl_sync(0xffffffffu, any, 0);
     if (any) {
-      __syncthreads();
+      __syncwarp();
       static_for<0, S>([&](auto T_) {
         constexpr int T = decltype(T_)::value;
         if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
-          int n = sh.out_cnt[T];
-          if (n > 0 && !is_local(T, local_from, local_to))
-            copy_out<F::stride(T)>(a.c.q[T].slots, ctx.template out_ptr<T>(0), sh.out_base[T], n, a.c.q[T].cap_log2);
+          int n = sh.out_cnt[pb][T];
+          if (n > 0) {
+            wait_slots(a.c, a.c.q[T], sh.out_base[T], n, 1, lane);
+            __syncwarp();  // every slot of the range is free before any lane writes into it
+            copy_out<F::stride(T)>(a.c.q[T].slots, out_buf(smem, pb, T), sh.out_base[T], n, a.c.q[T].cap_log2, lane);
+          }
         }
       });
-      __syncthreads();
-      // publish: seq = ticket + 1 (release; cumulative over the block's payload stores)
+      __syncwarp();
+      // publish: seq = ticket + 1 (release; cumulative over the warp's payload stores)
       static_for<0, S>([&](auto T_) {
         constexpr int T = decltype(T_)::value;
         if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
-          int n = sh.out_cnt[T];
-          if (n > 0 && !is_local(T, local_from, local_to)) {
+          int n = sh.out_cnt[pb][T];
+          if (n > 0) {
             const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
-            for (int k = threadIdx.x; k < n; k += blockDim.x) {
+            for (int k = lane; k < n; k += 32) {
               unsigned long long t = sh.out_base[T] + k;
               st_release(a.c.q[T].seq + (t & mask), t + 1);
             }
           }
         }
       });
-      __syncthreads();
+      __syncwarp();
+      if (lane == 0)
+        for (int t = 0; t < S; ++t)
+          if (sh.out_cnt[pb][t] > 0) atom_add(&c->count[t].v, sh.out_cnt[pb][t]);
     }
-    if (threadIdx.x == 0) {
-      for (int t = 0; t < S; ++t) {
-        if (is_local(t, local_from, local_to)) continue;
-        int n = sh.out_cnt[t];
-        if (n > 0) atom_add(&c->count[t].v, n);
-        sh.out_cnt[t] = 0;
+    if (lane == 0) {
+      for (int t = 0; t < S; ++t) sh.out_cnt[pb][t] = 0;
+      if (timers) sh.t_flush[ps] += globaltimer() - t0;
+    }
+  }
+
+  // ---------------- fetcher warp: claim the next batch (task scheduler) and stage it
+  // into in buffer nb.  quiescent: this block holds no batch and flushes nothing now.
+  static __device__ void fetch(const KArgs<F>& a, BlockShared& sh, uint8_t* smem, int nb, bool quiescent, int lane) {
+    Ctrl* c = a.c.ctrl;
+    const bool timers = a.c.flags & FLAG_TIMERS;
+    if (lane == 0) {
+      unsigned long long t0 = timers ? globaltimer() : 0;
+      int got = 0, st = -1, fs = 0;
+      unsigned long long base = 0;
+      sh.done = 0;
+      if (aborted(c)) {
+        sh.done = 1;
+      } else if (a.g.mode == MODE_WAVE) {
+        const int s = a.g.wave_stage;
+        int k = (int)(sh.wave_rem < a.g.batch[s] ? sh.wave_rem : a.g.batch[s]);
+        if (k > 0) {
+          got = claim_ring(c, s, k, base);
+          fs = 0;
+          if (!got) {
+            got = claim_seed(c, a.c.q[s], s, k, base);
+            fs = 1;
+          }
+          st = s;
+          sh.wave_rem -= got;
+          if (!got) sh.wave_rem = 0;  // cannot happen when the host sized the wave
+        }
+        if (!got && quiescent) sh.done = 1;
+      } else {
+        // "Query queues in turn of priority" (Fig. 8a): downstream stages first (drains
+        // the pipeline, bounds live items), rings before seeds.
+        for (int s = HI; s >= LO && !got; --s) {
+          got = claim_ring(c, s, a.g.batch[s], base);
+          if (got) { st = s; fs = 0; }
+        }
+        for (int s = HI; s >= LO && !got; --s) {
+          got = claim_seed(c, a.c.q[s], s, a.g.batch[s], base);
+          if (got) { st = s; fs = 1; }
+        }
+        if (!got && quiescent) {
+          // idle: retire deferred completions first, then test for termination
+          if (sh.acc_neg != 0) {
+            atom_add(&c->pending.v, sh.acc_neg);
+            sh.acc_neg = 0;
+          }
+          if ((long long)ld_acquire(&c->pending.v) <= 0) {
+            sh.done = 1;
+          } else if (globaltimer() > c->deadline.v) {
+            atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
+            sh.done = 1;
+          } else {
+            __nanosleep(256);
+          }
+        }
       }
+      sh.nx_stage = st;
+      sh.nx_n = got;
+      sh.nx_base = base;
+      sh.nx_seed = fs;
+      if (timers && !got) sh.t_idle += globaltimer() - t0;
     }
-    __syncthreads();
+    __syncwarp();
+    const int n = sh.nx_n;
+    if (n == 0) return;
+    const int s = sh.nx_stage;
+    const unsigned long long base = sh.nx_base;
+    uint8_t* dst = in_buf(smem, nb);
+    static_for<LO, HI + 1>([&](auto S_) {
+      constexpr int SS = decltype(S_)::value;
+      if (s == SS) {
+        const QueueDesc& q = a.c.q[SS];
+        if (sh.nx_seed) {
+          copy_seed_in<F::stride(SS)>(dst, q.seeds, base, n, lane);
+        } else {
+          wait_slots(a.c, q, base, n, 0, lane);
+          __syncwarp();
+          if (aborted(a.c.ctrl)) {  // never hand unpublished slots to the workers
+            if (lane == 0) {
+              sh.nx_n = 0;
+              sh.done = 1;
+            }
+            return;
+          }
+          copy_in<F::stride(SS)>(dst, q.slots, base, n, q.cap_log2, lane);
+          __syncwarp();
+          const unsigned long long mask = (1ull << q.cap_log2) - 1;
+          for (int k = lane; k < n; k += 32) {
+            unsigned long long t = base + k;
+            st_release(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
+          }
+        }
+      }
+    });
   }
 
   static __device__ __forceinline__ void record_trace(const KArgs<F>& a, int s, const uint8_t* items, int n) {
@@ -477,7 +597,7 @@ struct Runner {
     static_for<LO, HI + 1>([&](auto S_) {
       constexpr int SS = decltype(S_)::value;
       if (s == SS) {
-        for (int k = threadIdx.x; k < n; k += blockDim.x) {
+        for (int k = threadIdx.x; k < n; k += kThreads) {
           unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
           if (idx < a.c.trace_cap) {
             a.c.trace[idx].id = F::template item_id<SS>(items + k * F::stride(SS));
@@ -489,48 +609,37 @@ struct Runner {
     });
   }
 
-  // Execute stage s on n block-resident items, (RTC) forward block-locally through the
-  // rest of the linear group, then publish.
-  static __device__ void execute(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, int s, const uint8_t* items, int n,
-                                 unsigned long long t_start) {
+  // ---------------- worker warps: execute stage s on n staged items into out buffer
+  // ctx.ob; RTC groups then run the rest of the linear group on block-local items.
+  static __device__ void execute(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, int s, const uint8_t* items, int n) {
     const bool timers = a.c.flags & FLAG_TIMERS;
+    unsigned long long t0 = (timers && threadIdx.x == 0) ? globaltimer() : 0;
     static_for<LO, HI + 1>([&](auto S_) {
       constexpr int SS = decltype(S_)::value;
       if (s == SS) {
         record_trace(a, SS, items, n);
         if (threadIdx.x == 0) sh.deq[SS] += n;
         F::template exec<SS>(ctx, items, n);
-        int local_from = S, local_to = -1;
         if constexpr (RTC && SS < HI) {
-          // RTC: run the remaining stages of the group on block-local items (L11 §4.1).
-          __syncthreads();
+          // RTC (L11 §4.1): the remaining stages of the linear group, block-locally.
+          // Local items were never counted in `pending` (the claimed parents keep it
+          // positive), so they are neither added nor retired.
           static_for<SS + 1, HI + 1>([&](auto T_) {
             constexpr int TT = decltype(T_)::value;
-            int m = sh.out_cnt[TT];
+            worker_sync();
+            int m = sh.out_cnt[ctx.ob][TT];
             if (m > G::out_cap(LO, HI, RTC, TT)) m = G::out_cap(LO, HI, RTC, TT);
             if (m > 0) {
               const uint8_t* loc = ctx.template out_ptr<TT>(0);
               record_trace(a, TT, loc, m);
               if (threadIdx.x == 0) sh.deq[TT] += m;
-              // block-local items were never counted in `pending` (the claimed parents
-              // keep it positive), so they are neither added nor subtracted
               F::template exec<TT>(ctx, loc, m);
             }
-            __syncthreads();
-            if (threadIdx.x == 0) sh.out_cnt[TT] = 0;  // consumed locally
-            __syncthreads();
+            worker_sync();
+            if (threadIdx.x == 0) sh.out_cnt[ctx.ob][TT] = 0;  // consumed locally
           });
-          local_from = SS + 1;
-          local_to = HI;
         }
-        unsigned long long t_mid = 0;
-        if (timers && threadIdx.x == 0) t_mid = globaltimer();
-        flush(a, ctx, sh, local_from, local_to, n);
-        if (timers && threadIdx.x == 0) {
-          unsigned long long t_end = globaltimer();
-          sh.t_exec[SS] += t_mid - t_start;
-          sh.t_flush[SS] += t_end - t_mid;
-        }
+        if (timers && threadIdx.x == 0) sh.t_exec[SS] += globaltimer() - t0;
       }
     });
   }
@@ -556,8 +665,8 @@ struct Runner {
         __threadfence();
         unsigned long long t = atomicAdd(&c->arrivals[g.kslot].v, 1ull);
         if (t == (unsigned long long)gridDim.x - 1 && a.c.host_arrive) {
-          // every block of this grid has been dispatched and decided: tell the host it
-          // may launch the next group's kernel (deterministic SM/block binding)
+          // every block of this grid has been dispatched and decided: the host may launch
+          // the next group's kernel (deterministic SM/block binding)
           a.c.host_arrive[g.kslot] = a.c.epoch;
           __threadfence_system();
         }
@@ -573,13 +682,22 @@ struct Runner {
       }
       ok = good;
       for (int s = 0; s < kMaxStages; ++s) {
-        sh.out_cnt[s] = 0;
+        sh.out_cnt[0][s] = sh.out_cnt[1][s] = 0;
         sh.deq[s] = sh.enq[s] = 0;
         sh.t_exec[s] = sh.t_flush[s] = 0;
       }
       sh.t_idle = 0;
       sh.acc_neg = 0;
-      sh.skip = 0;
+      sh.done = 0;
+      sh.nx_n = 0;
+      sh.nx_stage = -1;
+      if (g.mode == MODE_WAVE) {
+        long long lo = (long long)blockIdx.x * g.wave_chunk;
+        long long rem = g.wave_n - lo;
+        sh.wave_rem = rem < 0 ? 0 : (rem < g.wave_chunk ? rem : g.wave_chunk);
+      } else {
+        sh.wave_rem = 0;
+      }
     }
     __syncthreads();
     return ok != 0;
@@ -600,149 +718,41 @@ struct Runner {
     }
   }
 
-  // Claim from stage s (ring first, then seeds); thread 0 only.
-  static __device__ __forceinline__ int claim(const KArgs<F>& a, int s, int k, unsigned long long& base, int& from_seed) {
-    Ctrl* c = a.c.ctrl;
-    int got = claim_ring(c, s, k, base);
-    if (got) { from_seed = 0; return got; }
-    got = claim_seed(c, a.c.q[s], s, k, base);
-    from_seed = 1;
-    return got;
-  }
-
-  // Stage-in a claimed batch into the in-buffer (block-wide), releasing its ring slots.
-  // Returns false (block-uniformly) if the run aborted while waiting.
-  static __device__ bool stage_in(const KArgs<F>& a, BlockShared& sh, uint8_t* inbuf, int s, int n,
-                                  unsigned long long base, int from_seed) {
-    bool ok = true;
-    static_for<LO, HI + 1>([&](auto S_) {
-      constexpr int SS = decltype(S_)::value;
-      if (s == SS) {
-        const QueueDesc& q = a.c.q[SS];
-        if (from_seed) {
-          copy_seed_in<F::stride(SS)>(inbuf, q.seeds, base, n);
-        } else {
-          wait_slots(a.c, q, base, n, 0);
-          if (threadIdx.x == 0) sh.skip = aborted(a.c.ctrl) ? 1 : 0;
-          __syncthreads();
-          if (sh.skip) {
-            ok = false;
-          } else {
-            copy_in<F::stride(SS)>(inbuf, q.slots, base, n, q.cap_log2);
-            __syncthreads();
-            const unsigned long long mask = (1ull << q.cap_log2) - 1;
-            for (int k = threadIdx.x; k < n; k += blockDim.x) {
-              unsigned long long t = base + k;
-              st_release(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
-            }
-          }
-        }
-      }
-    });
-    __syncthreads();
-    return ok;
-  }
-
   static __device__ void run(const KArgs<F>& a) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ BlockShared sh;
     if (!admit(a, sh)) return;
     CtxT ctx(a, smem, sh);
-    Ctrl* c = a.c.ctrl;
-    uint8_t* inbuf = smem;
-    const bool timers = a.c.flags & FLAG_TIMERS;
-
-    if (a.g.mode == MODE_WAVE) {
-      // KBK / standalone-RTC wave: this block processes items [b*batch, ...) of wave_stage.
-      const int s = a.g.wave_stage;
-      long long lo = (long long)blockIdx.x * a.g.batch[s];
-      long long rem = a.g.wave_n - lo;
-      int k = (int)(rem < a.g.batch[s] ? rem : a.g.batch[s]);
-      while (k > 0) {
-        unsigned long long t0 = 0;
-        if (threadIdx.x == 0) {
-          if (timers) t0 = globaltimer();
-          unsigned long long base = 0;
-          int fs = 0;
-          int got = aborted(c) ? 0 : claim(a, s, k, base, fs);
-          sh.cl_n = got;
-          sh.cl_base = base;
-          sh.cl_seed = fs;
-        }
-        __syncthreads();
-        const int n = sh.cl_n;
-        const unsigned long long base = sh.cl_base;
-        const int fs = sh.cl_seed;
-        __syncthreads();
-        if (n == 0) break;  // aborted, or (never) the host over-sized the wave
-        if (!stage_in(a, sh, inbuf, s, n, base, fs)) break;
-        execute(a, ctx, sh, s, inbuf, n, t0);
-        k -= n;
-      }
-      flush_stats(a, sh);
-      return;
-    }
-
-    unsigned ns = 64;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    // prologue: stage the first batch into in[0]
+    if (warp == W_FETCH) fetch(a, sh, smem, 0, true, lane);
+    __syncthreads();
+    int b = 0, prev_s = -1, prev_n = 0;
     for (;;) {
-      unsigned long long t0 = 0;
-      if (threadIdx.x == 0) {
-        if (timers) t0 = globaltimer();
-        int got = 0, st = -1, fs = 0;
-        unsigned long long base = 0;
-        sh.done = 0;
-        if (aborted(c)) {
-          sh.done = 1;
-        } else {
-          // Task scheduler: "Query queues in turn of priority" (Fig. 8a) — downstream
-          // stages first (drains the pipeline, bounds live items), rings before seeds.
-          for (int s = HI; s >= LO && !got; --s) {
-            got = claim_ring(c, s, a.g.batch[s], base);
-            if (got) { st = s; fs = 0; }
-          }
-          for (int s = HI; s >= LO && !got; --s) {
-            got = claim_seed(c, a.c.q[s], s, a.g.batch[s], base);
-            if (got) { st = s; fs = 1; }
-          }
-          if (!got) {
-            // idle: retire deferred completions first, then test for termination
-            if (sh.acc_neg != 0) {
-              atom_add(&c->pending.v, sh.acc_neg);
-              sh.acc_neg = 0;
-            }
-            if ((long long)ld_acquire(&c->pending.v) <= 0) sh.done = 1;
-            else if (globaltimer() > c->deadline.v) {
-              atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
-              sh.done = 1;
-            }
-          }
+      const int done = sh.done, cur_s = sh.nx_stage, cur_n = sh.nx_n;
+      __syncthreads();  // everyone has read the round's batch; the fetcher may overwrite it
+      if (done) break;
+      if (warp < kWarpsW) {
+        if (cur_n > 0) {
+          ctx.ob = b;
+          execute(a, ctx, sh, cur_s, in_buf(smem, b), cur_n);
         }
-        sh.cl_stage = st;
-        sh.cl_n = got;
-        sh.cl_base = base;
-        sh.cl_seed = fs;
+      } else if (warp == W_FETCH) {
+        fetch(a, sh, smem, b ^ 1, cur_n == 0 && prev_n == 0, lane);
+      } else {
+        if (prev_n > 0) publish(a, sh, smem, b ^ 1, prev_s, prev_n, lane);
       }
       __syncthreads();
-      const int done = sh.done, n = sh.cl_n, s = sh.cl_stage, fs = sh.cl_seed;
-      const unsigned long long base = sh.cl_base;
-      __syncthreads();  // everyone has read the claim; thread 0 may overwrite it next round
-      if (done) break;
-      if (n == 0) {
-        __nanosleep(ns);
-        if (ns < 2048) ns <<= 1;
-        if (timers && threadIdx.x == 0) sh.t_idle += globaltimer() - t0;
-        continue;
-      }
-      ns = 64;
-      if (!stage_in(a, sh, inbuf, s, n, base, fs)) break;
-      execute(a, ctx, sh, s, inbuf, n, t0);
+      prev_s = cur_s;
+      prev_n = cur_n;
+      b ^= 1;
     }
     flush_stats(a, sh);
   }
 };
 
 template <class F, int LO, int HI, bool RTC>
-__global__ void __launch_bounds__(kThreads, F::min_blocks(LO, HI, RTC)) vp_kernel(const __grid_constant__ KArgs<F> a) {
+__global__ void __launch_bounds__(kBlock, F::min_blocks(LO, HI, RTC)) vp_kernel(const __grid_constant__ KArgs<F> a) {
   Runner<F, LO, HI, RTC>::run(a);
 }
 
