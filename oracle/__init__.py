@@ -228,3 +228,49 @@ def reyes_shade_factor(n3, L4):
 
 
 REYES_CULL, REYES_SPLIT, REYES_DICE = 0, 1, 2
+
+
+# ------------------------------------------------------------------ Rasterization
+class RasterSceneC(C.Structure):
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P)]
+
+
+class RasterOutC(C.Structure):
+    _fields_ = [("key", P), ("colour", P), ("n_vertex", C.c_uint64), ("n_clip", C.c_uint64),
+                ("n_raster", C.c_uint64), ("n_fragment", C.c_uint64), ("n_frag_pixels", C.c_uint64),
+                ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t)]
+
+
+def _raster_run(fname, scene, trace_cap=0):
+    L = lib()
+    fn = getattr(L, fname)
+    fn.argtypes = [P, P]
+    M = np.ascontiguousarray(scene.M, np.float32).reshape(-1)
+    pos = np.ascontiguousarray(scene.pos, np.float32)
+    col = np.ascontiguousarray(scene.col, np.float32)
+    sc = RasterSceneC(W=scene.W, H=scene.H, n_tris=pos.shape[0], M=M.ctypes.data, pos=pos.ctypes.data,
+                      col=col.ctypes.data)
+    npix = scene.W * scene.H
+    key = np.empty(npix, np.uint64)
+    colour = np.empty((npix, 4), np.float32)
+    o = RasterOutC(key=key.ctypes.data, colour=colour.ctypes.data)
+    trace = np.zeros(max(trace_cap, 1), TRACE_DTYPE)
+    if trace_cap:
+        o.trace, o.trace_cap = trace.ctypes.data, trace_cap
+    rc = fn(C.byref(sc), C.byref(o))
+    assert rc == 0, rc
+    res = dict(key=key.reshape(scene.H, scene.W), colour=colour.reshape(scene.H, scene.W, 4),
+               n_vertex=o.n_vertex, n_clip=o.n_clip, n_raster=o.n_raster, n_fragment=o.n_fragment,
+               n_frag_pixels=o.n_frag_pixels)
+    if trace_cap:
+        assert o.trace_n <= trace_cap, "trace_cap too small"
+        res["trace"] = trace[: o.trace_n].copy()
+    return res
+
+
+def raster_definition(scene):
+    return _raster_run("orc_raster_definition", scene)
+
+
+def raster_pipeline(scene, trace_cap=0):
+    return _raster_run("orc_raster_pipeline", scene, trace_cap)

@@ -112,4 +112,24 @@ void orc_reyes_dice(const orc_reyes_scene* sc, const orc_patch* p, float grid[6]
 void orc_reyes_project(const float M[16], const float p[4], float c[4]);
 float orc_reyes_shade_factor(const float n[3], const float L[4]);
 
+/* ---------------- Rasterization (raster.c) ---------------- */
+typedef struct orc_raster_scene {
+  int32_t W, H;
+  int64_t n_tris;
+  const float* M;   /* [16] row-major                                   */
+  const float* pos; /* [n_tris][3][4] (x_px, y_px, z, 1)                 */
+  const float* col; /* [n_tris][3][4] (r, g, b, 0)                       */
+} orc_raster_scene;
+
+typedef struct orc_raster_out {
+  uint64_t* key;   /* [H*W] min (zkey(z) << 32 | tri), UINT64_MAX if empty */
+  float* colour;   /* [H*W][4]                                          */
+  uint64_t n_vertex, n_clip, n_raster, n_fragment, n_frag_pixels;
+  orc_trace_rec* trace; size_t trace_cap, trace_n;
+} orc_raster_out;
+
+int orc_raster_definition(const orc_raster_scene* sc, orc_raster_out* out);
+int orc_raster_pipeline(const orc_raster_scene* sc, orc_raster_out* out);
+void orc_raster_vertex(const orc_raster_scene* sc, uint32_t tri, float clip[3][4]);
+
 #endif

@@ -191,6 +191,78 @@ def reyes_config5(n_frames: int = 512, n_side: int = 64, frame0: int = 0, seed: 
                       extra={"frame0": frame0})
 
 
+@dataclass
+class RasterScene:
+    """BASELINE config 4 inputs: triangles in pixel space."""
+    W: int
+    H: int
+    M: np.ndarray      # [16] float32 pixel -> NDC, w = 1
+    pos: np.ndarray    # [n, 3, 4] float32 (x_px, y_px, z, 1)
+    col: np.ndarray    # [n, 3, 4] float32 (r, g, b, 0)
+
+    @property
+    def n_tris(self):
+        return self.pos.shape[0]
+
+
+def pixel_to_ndc(W: int, H: int) -> np.ndarray:
+    M = np.zeros((4, 4))
+    M[0, 0], M[0, 3] = 2.0 / W, -1.0
+    M[1, 1], M[1, 3] = 2.0 / H, -1.0
+    M[2, 2] = 1.0
+    M[3, 3] = 1.0
+    return M.astype(np.float32).reshape(16)
+
+
+def raster_scene(n: int = 1 << 20, W: int = 1920, H: int = 1080, seed: int = seed_for(4),
+                 area_range=(0.5, 512.0), aspect_range=(0.25, 4.0)) -> RasterScene:
+    """Synthetic triangles: centres U(screen), area log-uniform on
+    [0.5, 512] px^2, aspect log-uniform on [1/4, 4], random rotation, z ~ U(0.05, 0.95)
+    per vertex, colours U[0,1)^3.  Shape: base b, height h (b*h/2 = area, b/h = aspect),
+    vertices (-b/2, -h/3), (b/2, -h/3), (0, 2h/3) about the centre, then rotated."""
+    u = uniform01(seed, n * 17).reshape(n, 17)
+    cx, cy = u[:, 0] * W, u[:, 1] * H
+    la, lb = math.log(area_range[0]), math.log(area_range[1])
+    area = np.exp(la + u[:, 2] * (lb - la))
+    sa, sb = math.log(aspect_range[0]), math.log(aspect_range[1])
+    aspect = np.exp(sa + u[:, 3] * (sb - sa))
+    th = 2 * math.pi * u[:, 4]
+    b = np.sqrt(2 * area * aspect)
+    h = 2 * area / b
+    lx = np.stack([-b / 2, b / 2, np.zeros(n)], 1)
+    ly = np.stack([-h / 3, -h / 3, 2 * h / 3], 1)
+    c, s = np.cos(th)[:, None], np.sin(th)[:, None]
+    pos = np.zeros((n, 3, 4), np.float32)
+    pos[:, :, 0] = cx[:, None] + c * lx - s * ly
+    pos[:, :, 1] = cy[:, None] + s * lx + c * ly
+    pos[:, :, 2] = 0.05 + 0.9 * u[:, 5:8]
+    pos[:, :, 3] = 1.0
+    col = np.zeros((n, 3, 4), np.float32)
+    col[:, :, :3] = u[:, 8:17].reshape(n, 3, 3)
+    return RasterScene(W=W, H=H, M=pixel_to_ndc(W, H), pos=pos, col=col)
+
+
+def raster_quad_mesh(W: int, H: int, cell: int = 8, z: float = 0.5) -> RasterScene:
+    """Watertightness pin: a full-screen grid of cell x cell squares, each split into two
+    triangles along a diagonal (alternating), all at depth z."""
+    tris = []
+    for y in range(0, H, cell):
+        for x in range(0, W, cell):
+            a, b_, c_, d = (x, y), (x + cell, y), (x + cell, y + cell), (x, y + cell)
+            if ((x // cell) + (y // cell)) % 2 == 0:
+                tris += [(a, b_, c_), (a, c_, d)]
+            else:
+                tris += [(a, b_, d), (b_, c_, d)]
+    n = len(tris)
+    pos = np.zeros((n, 3, 4), np.float32)
+    for i, t in enumerate(tris):
+        for k, (px, py) in enumerate(t):
+            pos[i, k] = (px, py, z, 1.0)
+    col = np.full((n, 3, 4), 0.5, np.float32)
+    col[:, :, 3] = 0
+    return RasterScene(W=W, H=H, M=pixel_to_ndc(W, H), pos=pos, col=col)
+
+
 def reyes_planar(S_px: float, W: int = 64, H: int = 64, x0: float = 8.0, y0: float = 8.0,
                  max_depth: int = 8, albedo=(0.5, 0.25, 0.75)) -> ReyesScene:
     """Closed-form special case (SURVEY c-1 pin 4): a planar patch parallel to the image
