@@ -69,7 +69,10 @@ typedef enum vp_stage_kind {
   /* Collatz queue stress (not in the paper): step (recursive), sink */
   VP_COLLATZ_STEP = 10, VP_COLLATZ_SINK = 11,
   /* Reyes (Fig. 1, L3; L55): Bound, Split (recursive via Bound), Dice, Shade */
-  VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23
+  VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23,
+  /* Rasterization (Fig. 16, L59): Vertex + Clip (the paper's Clip), Raster (its
+   * Interpolate: triangle -> 8x8 tiles), Fragment (its Shade: coverage + z-buffer) */
+  VP_RASTER_VERTEX = 30, VP_RASTER_CLIP = 31, VP_RASTER_RASTER = 32, VP_RASTER_FRAGMENT = 33
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -144,6 +147,13 @@ typedef struct vp_run_stats {
   uint64_t stage_exec_ns[VP_MAX_STAGES];
   uint64_t stage_flush_ns[VP_MAX_STAGES];
   uint64_t kernel_idle_ns[16];
+  /* ring state at the end of the run (diagnostics after an abort): reserved tickets,
+   * claimed tickets, published-unclaimed items, seeds claimed; final pending count */
+  uint64_t ring_tail[VP_MAX_STAGES], ring_head[VP_MAX_STAGES];
+  int64_t ring_count[VP_MAX_STAGES];
+  uint64_t seed_head[VP_MAX_STAGES];
+  int64_t pending;
+  uint64_t kernel_rounds[16];               /* persistent-loop rounds summed over blocks  */
 } vp_run_stats;
 
 typedef struct vp_autotune_opts {
@@ -192,6 +202,17 @@ typedef struct vp_reyes_params {
                              /* reset by vp_run; key = UINT64_MAX when uncovered           */
   float* colour;             /* [n_frames*H*W][4] resolved colour, written by vp_run       */
 } vp_reyes_params;
+
+typedef struct vp_raster_params {
+  int32_t W, H;
+  int64_t n_tris;            /* vertex stage items are triangle ids in [0, n_tris)        */
+  const float* M;            /* [16] row-major vertex transform (pixel -> clip)            */
+  const float* pos;          /* [n_tris][3][4] vertex positions (x, y, z, w), 16-B aligned */
+  const float* col;          /* [n_tris][3][4] vertex colours (r, g, b, -)                  */
+  void* setup;               /* [n_tris] x 128 B scratch (per-triangle setup), 128-B aligned */
+  unsigned long long* fb;    /* [H*W] depth keys (zkey(z) << 32 | tri), reset by vp_run    */
+  float* colour;             /* [H*W][4] resolved colour, written by vp_run                */
+} vp_raster_params;
 
 /* ---------------- calls ---------------- */
 const char* vp_status_string(vp_status s);

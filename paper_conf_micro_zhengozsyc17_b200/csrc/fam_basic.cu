@@ -27,7 +27,7 @@ struct ToyF {
   static constexpr int max_batch(int) { return 1024; }
   static constexpr int default_batch(int) { return 256; }
   static constexpr int fanout(int s, int t) { return (s == 0 && (t == 0 || t == 1)) || (s == 1 && t == 2) ? 1 : 0; }
-  static constexpr bool uses_latches(int, int) { return false; }
+  static constexpr bool rtc_ok(int, int) { return true; }
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int) { return 20; }
   static constexpr int min_blocks(int, int, bool) { return 3; }
@@ -89,7 +89,7 @@ struct CollatzF {
   static constexpr int max_batch(int) { return 512; }
   static constexpr int default_batch(int) { return 256; }
   static constexpr int fanout(int s, int t) { return s == 0 ? 1 : 0; }
-  static constexpr bool uses_latches(int, int) { return false; }
+  static constexpr bool rtc_ok(int, int) { return true; }
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int) { return 20; }
   static constexpr int min_blocks(int, int, bool) { return 3; }

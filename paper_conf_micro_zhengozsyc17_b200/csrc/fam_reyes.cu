@@ -181,7 +181,7 @@ struct ReyesF {
   static constexpr int fanout(int s, int t) {
     return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
   }
-  static constexpr bool uses_latches(int, int) { return false; }
+  static constexpr bool rtc_ok(int, int) { return true; }
   static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM

@@ -89,7 +89,7 @@ struct FamilyImpl final : FamilyOps {
   int threads_per_item(int s) const override { return F::threads_per_item(s); }
   int fanout(int s, int t) const override { return F::fanout(s, t); }
   bool rtc_legal(int lo, int hi) const override { return fn[lo][hi][1] != nullptr; }
-  bool latched(int lo, int hi) const override { return F::uses_latches(lo, hi); }
+  bool latched(int lo, int hi) const override { return !F::rtc_ok(lo, hi); }
   int default_cap_log2(int s) const override { return F::default_cap_log2(s); }
   size_t params_bytes() const override { return sizeof(typename F::Params); }
   const void* kernel(int lo, int hi, bool rtc) const override { return fn[lo][hi][rtc ? 1 : 0]; }
@@ -123,5 +123,6 @@ struct FamilyImpl final : FamilyOps {
 const FamilyOps* family_toy();
 const FamilyOps* family_collatz();
 const FamilyOps* family_reyes();
+const FamilyOps* family_raster();
 
 }  // namespace vp

@@ -21,12 +21,13 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
     all_families[0] = family_toy();
     all_families[1] = family_collatz();
     all_families[2] = family_reyes();
+    all_families[3] = family_raster();
   }
 }
 const FamilyOps* family_of_kind(int kind, int* pos) {
@@ -67,7 +68,10 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
     c->exec_ns[t] = 0;
     c->flush_ns[t] = 0;
   }
-  if (t < kMaxKernels) c->idle_ns[t] = 0;
+  if (t < kMaxKernels) {
+    c->idle_ns[t] = 0;
+    c->rounds[t] = 0;
+  }
   if (t < kMaxKernels) {
     c->arrivals[t].v = 0;
     c->admitted[t].v = 0;
@@ -194,6 +198,10 @@ int occupancy(vp_pipeline_s* p, int lo, int hi, bool rtc) {
   if (!fn) return 0;
   size_t sm = p->fam->smem(lo, hi, rtc);
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+  // One shared-memory carveout for every kernel: an SM configured for a small carveout
+  // cannot take a block of a kernel that needs a larger one until it drains, which would
+  // stop co-resident persistent groups (coarse/fine/hybrid) from ever starting.
+  cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   int occ = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, sm) != cudaSuccess) occ = 0;
   c = occ;
@@ -950,7 +958,17 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       stats->stage_exec_ns[s] = hc.exec_ns[s];
       stats->stage_flush_ns[s] = hc.flush_ns[s];
     }
-    for (int i = 0; i < kMaxKernels; ++i) stats->kernel_idle_ns[i] = hc.idle_ns[i];
+    for (int i = 0; i < kMaxKernels; ++i) {
+      stats->kernel_idle_ns[i] = hc.idle_ns[i];
+      stats->kernel_rounds[i] = hc.rounds[i];
+    }
+    for (int s = 0; s < S; ++s) {
+      stats->ring_tail[s] = hc.tail[s].v;
+      stats->ring_head[s] = hc.head[s].v;
+      stats->ring_count[s] = (int64_t)hc.count[s].v;
+      stats->seed_head[s] = hc.seed_head[s].v;
+    }
+    stats->pending = (int64_t)hc.pending.v;
   }
   if (hc.abort.v != ABORT_NONE) {
     p->dirty_queues = true;

@@ -67,6 +67,7 @@ struct Ctrl {
   unsigned long long exec_ns[kMaxStages];   // FLAG_TIMERS: stage-in + execute per stage
   unsigned long long flush_ns[kMaxStages];  // FLAG_TIMERS: publish (queue overhead) per stage
   unsigned long long idle_ns[kMaxKernels];  // FLAG_TIMERS: blocks finding no work, per kernel
+  unsigned long long rounds[kMaxKernels];   // persistent-loop rounds, summed over blocks, per kernel
 };
 
 struct QueueDesc {
@@ -172,7 +173,7 @@ struct Graph {
         if (fan(s, t) > 0) return true;
     return false;
   }
-  static constexpr bool rtc_legal(int lo, int hi) { return !has_back_edge(lo, hi) && !F::uses_latches(lo, hi); }
+  static constexpr bool rtc_legal(int lo, int hi) { return !has_back_edge(lo, hi) && F::rtc_ok(lo, hi); }
   // items that can arrive block-locally at stage t of an RTC group [lo,hi]
   static constexpr int rtc_in_cap(int lo, int t) {
     if (t == lo) return F::max_batch(lo);
@@ -225,7 +226,7 @@ struct BlockShared {
   long long wave_rem;                  // WAVE: items of this block's chunk not yet claimed
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
-  unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle;
+  unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
 };
 
 __device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
@@ -687,6 +688,7 @@ struct Runner {
         sh.t_exec[s] = sh.t_flush[s] = 0;
       }
       sh.t_idle = 0;
+      sh.rounds = 0;
       sh.acc_neg = 0;
       sh.done = 0;
       sh.nx_n = 0;
@@ -715,6 +717,7 @@ struct Runner {
         if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
       }
       if (sh.t_idle) atomicAdd(&c->idle_ns[a.g.kslot], sh.t_idle);
+      atomicAdd(&c->rounds[a.g.kslot], sh.rounds);
     }
   }
 
@@ -743,6 +746,7 @@ struct Runner {
         if (prev_n > 0) publish(a, sh, smem, b ^ 1, prev_s, prev_n, lane);
       }
       __syncthreads();
+      if (threadIdx.x == 0) sh.rounds++;
       prev_s = cur_s;
       prev_n = cur_n;
       b ^= 1;

@@ -32,6 +32,7 @@ GROUP_RTC, GROUP_KBK, GROUP_MEGA, GROUP_FINE = range(4)
 TOY_S1, TOY_S2, TOY_S3 = 1, 2, 3
 COLLATZ_STEP, COLLATZ_SINK = 10, 11
 REYES_BOUND, REYES_SPLIT, REYES_DICE, REYES_SHADE = 20, 21, 22, 23
+RASTER_VERTEX, RASTER_CLIP, RASTER_RASTER, RASTER_FRAGMENT = 30, 31, 32, 33
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS = 1, 2, 4, 8
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
@@ -67,7 +68,9 @@ class RunStats(C.Structure):
                 ("admitted", C.c_uint64 * 16), ("fallback_admits", C.c_uint64), ("kbk_launches", C.c_uint64),
                 ("trace_records", C.c_uint64), ("abort_reason", C.c_int), ("num_sms", C.c_int),
                 ("stage_exec_ns", C.c_uint64 * MAX_STAGES), ("stage_flush_ns", C.c_uint64 * MAX_STAGES),
-                ("kernel_idle_ns", C.c_uint64 * 16)]
+                ("kernel_idle_ns", C.c_uint64 * 16), ("ring_tail", C.c_uint64 * MAX_STAGES),
+                ("ring_head", C.c_uint64 * MAX_STAGES), ("ring_count", C.c_int64 * MAX_STAGES),
+                ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16)]
 
 
 class AutotuneOpts(C.Structure):
@@ -94,6 +97,11 @@ class ReyesParams(C.Structure):
     _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_frames", C.c_int32), ("patches_per_frame", C.c_int32),
                 ("max_depth", C.c_int32), ("pad0", C.c_int32), ("t_dice", C.c_float), ("near_w", C.c_float),
                 ("M", P), ("albedo", P), ("L", C.c_float * 4), ("fb", P), ("colour", P)]
+
+
+class RasterParams(C.Structure):
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P),
+                ("setup", P), ("fb", P), ("colour", P)]
 
 
 def _decl(name, args, res=C.c_int):
@@ -292,7 +300,9 @@ def stats_dict(st: RunStats):
                 admitted=list(st.admitted[:nk]), fallback_admits=st.fallback_admits,
                 kbk_launches=st.kbk_launches, trace_records=st.trace_records, abort_reason=st.abort_reason,
                 num_sms=st.num_sms, stage_exec_ns=list(st.stage_exec_ns), stage_flush_ns=list(st.stage_flush_ns),
-                kernel_idle_ns=list(st.kernel_idle_ns[:max(nk, 1)]))
+                kernel_idle_ns=list(st.kernel_idle_ns[:max(nk, 1)]), ring_tail=list(st.ring_tail),
+                ring_head=list(st.ring_head), ring_count=list(st.ring_count), seed_head=list(st.seed_head),
+                pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]))
 
 
 def config_to_string(cfg: Config) -> str:

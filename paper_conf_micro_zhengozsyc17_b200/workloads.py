@@ -59,6 +59,41 @@ class CollatzPipeline:
         return self.steps.cpu().numpy().view(np.uint32), self.seen.cpu().numpy().view(np.uint32), st
 
 
+class RasterPipeline:
+    """Vertex -> Clip -> Raster -> Fragment (+ colour resolve) over a RasterScene (Fig. 16, L59)."""
+
+    def __init__(self, scene: inputs.RasterScene, device: int = 0, **kw):
+        dev = _dev(device)
+        self.scene = scene
+        n = scene.n_tris
+        self.M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).to(dev)
+        self.pos = torch.from_numpy(np.ascontiguousarray(scene.pos, np.float32)).to(dev)
+        self.col = torch.from_numpy(np.ascontiguousarray(scene.col, np.float32)).to(dev)
+        self.setup = torch.empty((n, 32), dtype=torch.float32, device=dev)          # 128 B per triangle
+        self.fb = torch.empty((scene.H, scene.W), dtype=torch.int64, device=dev)
+        self.colour = torch.empty((scene.H, scene.W, 4), dtype=torch.float32, device=dev)
+        self.prm = vp.RasterParams(W=scene.W, H=scene.H, n_tris=n, M=self.M.data_ptr(), pos=self.pos.data_ptr(),
+                                   col=self.col.data_ptr(), setup=self.setup.data_ptr(), fb=self.fb.data_ptr(),
+                                   colour=self.colour.data_ptr())
+        self.p = vp.Pipeline(device, **kw)
+        for kind, stride in zip((vp.RASTER_VERTEX, vp.RASTER_CLIP, vp.RASTER_RASTER, vp.RASTER_FRAGMENT), (4, 4, 4, 8)):
+            self.p.register(kind, stride, self.prm)
+        self.ids = torch.arange(n, dtype=torch.int32, device=dev)
+        self.p.insert(0, self.ids, n=n)
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def keys(self):
+        return self.fb.cpu().numpy().view(np.uint64)
+
+    def colours(self):
+        return self.colour.cpu().numpy()
+
+
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
 REYES_STRIDES = (272, 272, 272, 1968)
 

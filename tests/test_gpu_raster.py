@@ -1,0 +1,96 @@
+"""GPU parity for rasterization (Fig. 16, L59; BASELINE config 4) through the C ABI:
+bit-exact depth keys, colours (<= 1e-4, bit-exact expected), per-stage counts and the
+trace multiset against the CPU oracle, under every legal execution model."""
+import numpy as np
+import pytest
+
+from paper_conf_micro_zhengozsyc17_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module")
+def vpm():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    return vp
+
+
+def configure(vp, rp, model):
+    nsm, _ = vp.device_info(0)
+    if model in ("kbk", "megakernel", "coarse", "fine"):
+        rp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+    elif model == "hybrid_rtc_mega":      # [Vertex,Clip] RTC (the paper's Clip) | [Raster,Fragment] megakernel
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_RTC, 0, 40), (2, 3, vp.GROUP_MEGA, 40, nsm)], nsm))
+    elif model == "hybrid_rtc_rtc":       # [Vertex,Clip] RTC | [Raster,Fragment] RTC
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_RTC, 0, 40), (2, 3, vp.GROUP_RTC, 40, nsm)], nsm))
+    elif model == "hybrid_fine":          # [Vertex..Raster] megakernel | [Fragment] fine
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 2, vp.GROUP_MEGA, 0, 30), (3, 3, vp.GROUP_FINE, 30, nsm)], nsm))
+    else:
+        raise ValueError(model)
+
+
+def check(orc, scene, rp, st):
+    ref = orc.raster_pipeline(scene)
+    key = rp.keys()
+    assert np.array_equal(key, ref["key"]), f"{(key != ref['key']).sum()} keys differ"
+    col = rp.colours()
+    assert np.max(np.abs(col - ref["colour"])) <= TOL
+    assert np.array_equal(col, ref["colour"])
+    assert st["dequeued"][:4] == [ref["n_vertex"], ref["n_clip"], ref["n_raster"], ref["n_fragment"]]
+    return ref
+
+
+MODELS = ["kbk", "megakernel", "coarse", "fine", "hybrid_rtc_mega", "hybrid_rtc_rtc", "hybrid_fine"]
+
+
+@pytest.mark.parametrize("model", MODELS)
+def test_raster_reduced(vpm, orc, model):
+    """10^4 triangles at 320x180 (SURVEY §8(d) reduced size)."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_scene(10_000, W=320, H=180)
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, model)
+    for _ in range(2):
+        check(orc, scene, rp, rp.run())
+
+
+def test_raster_rtc_whole_pipeline_rejected(vpm):
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    vp = vpm
+    rp = RasterPipeline(inputs.raster_scene(100, W=64, H=64))
+    with pytest.raises(vp.VPError) as e:
+        rp.configure(vp.RTC)   # Raster's fan-out cannot be expanded block-locally
+    assert e.value.status == vp.VP_ERR_UNSUPPORTED
+
+
+def test_raster_tiny_brute_force_scene(vpm, orc):
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    vp = vpm
+    scene = inputs.raster_scene(200, W=64, H=64, seed=inputs.seed_for(4, 1), area_range=(0.5, 200.0))
+    rp = RasterPipeline(scene)
+    rp.configure(vp.MEGAKERNEL)
+    check(orc, scene, rp, rp.run())
+
+
+def test_raster_watertight(vpm, orc):
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    vp = vpm
+    scene = inputs.raster_quad_mesh(320, 176, cell=16)
+    rp = RasterPipeline(scene)
+    rp.configure(vp.MEGAKERNEL)
+    check(orc, scene, rp, rp.run())
+    assert np.all(rp.keys() != np.uint64(0xFFFFFFFFFFFFFFFF))
+
+
+def test_raster_full_config4_sampled(vpm, orc):
+    """Full config 4 (1M triangles, 1920x1080) in the hybrid launch configuration; the
+    oracle runs the whole frame (~5 s) and everything is compared."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_scene()
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, "hybrid_rtc_mega")
+    check(orc, scene, rp, rp.run())
