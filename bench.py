@@ -53,7 +53,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="vp", choices=["vp", "reference"])
     ap.add_argument("--frames", type=int, default=TOTAL_FRAMES)
-    ap.add_argument("--model", default="hybrid", help="hybrid|megakernel|kbk|coarse|fine")
+    ap.add_argument("--model", default="tuned", help="tuned (auto-tuner) | hybrid | megakernel | kbk | coarse | fine")
+    ap.add_argument("--tune-seconds", type=float, default=30.0)
     ap.add_argument("--split", type=int, default=44, help="SMs for the [Bound,Split] group (hybrid)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baselines", action="store_true")
@@ -205,7 +206,19 @@ def main():
     f1 = (rank + 1) * args.frames // world
     scene = inputs.reyes_config5(n_frames=f1 - f0, n_side=PATCH_SIDE, frame0=f0)
     rp = ReyesPipeline(scene, device=local)
-    configure(vp, rp, args.model, nsm, args.split)
+    tune = None
+    if args.model == "tuned":
+        # the paper's offline auto-tuner (L41-L45, Fig. 10) picks {grouping, models, SM
+        # split, batch} on this shard before anything is timed
+        t_tune = time.perf_counter()
+        best_cfg, rep = rp.p.autotune(time_budget_s=args.tune_seconds, sm_granularity=4, batch_choices=(1, 2))
+        tune = {"seconds": round(time.perf_counter() - t_tune, 2), "candidates_run": rep.candidates_run,
+                "candidates_total": rep.candidates_total, "timed_out": rep.candidates_timed_out,
+                "best_ms": rep.best_ms, "kbk_ms": rep.baseline_kbk_ms, "megakernel_ms": rep.baseline_mega_ms,
+                "config": vp.config_to_string(best_cfg)}
+    else:
+        configure(vp, rp, args.model, nsm, args.split)
+    main_cfg = rp.p.get_config()
     stream = torch.cuda.current_stream()
     for _ in range(max(args.warmup, 3) if args.warmup >= 3 else args.warmup):
         rp.run(stream)
@@ -250,9 +263,11 @@ def main():
     # for bit-exactness), at clocks.max.sm
     alu_peak = nsm * 128 * sm_max * 1e6 / 1e12
     achieved = dom_flop / (kmean[dom] / 1e3) / 1e12
+    b = main_cfg.binding
+    is_rtc = bool(main_cfg.has_binding and b.group_model[b.group_of_stage[lo]] == vp.GROUP_RTC)
     roofline = {"bound": "alu", "achieved": achieved, "peak": alu_peak, "unit": "TFLOP/s",
                 "frac": achieved / alu_peak, "traffic": None,
-                "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if args.model == 'hybrid' and lo == 2 else 'MEGA'}>",
+                "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if is_rtc else 'MEGA'}>",
                 "peak_source": "derived: SMs x 128 fp32 lanes x clocks.max.sm (MEASURED_PEAKS sm_max_mhz), non-FMA",
                 "kernel_ms": float(kmean[dom]), "kernel_share_of_step": float(kmean[dom] / ms_per_step)}
     hbm = pk.get("hbm_gbs", 6548.5)
@@ -274,7 +289,7 @@ def main():
                 dist.all_reduce(bt_t, op=dist.ReduceOp.MAX)
             extra[name] = {"ms_per_step": float(bt_t.item()) / max(1, min(args.steps, 3)),
                            "launches_per_step": int(bst["kbk_launches"])}
-        configure(vp, rp, args.model, nsm, args.split)
+        rp.p.configure_config(main_cfg)
 
     # ---- e2e through the public API with HOST buffers: H2D seeds + run + D2H colours
     e2e = None
@@ -346,7 +361,8 @@ def main():
                 "note": "ALU/latency-bound workload (SURVEY §8(d) d5); % HBM reported, not the bound"},
         "speedup_vs_kbk": (extra["kbk"]["ms_per_step"] / ms_per_step) if "kbk" in extra else None,
         "baselines": extra, "e2e": e2e, "gather_ms": gather_ms, "clocks": clocks, "gpu_launches": launches * args.steps,
-        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs",
+        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune,
+        "config_string": vp.config_to_string(main_cfg),
     }
     if rank == 0:
         print(json.dumps(line), flush=True)

@@ -85,6 +85,8 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
   }
 }
 
+__global__ void k_set_abort(Ctrl* c, unsigned long long why) { atomicCAS(&c->abort.v, 0ull, why); }
+
 __global__ void k_reset_queues(Ctrl* c) {
   int t = threadIdx.x;
   if (t < kMaxStages) {
@@ -579,12 +581,19 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
     }
     return std::max(1ll, cap);
   };
+  const auto t_start = std::chrono::steady_clock::now();
   for (;;) {
     Avail a;
     vp_status rc = read_avail(p, st, a);
     if (rc != VP_OK) return rc;
     if (a.abort) return VP_OK;
     if (a.pending <= 0) return VP_OK;
+    if (std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count() > p->timeout_ms) {
+      // host-side watchdog for wave-driven models (timeoutexec): abort the device run
+      k_set_abort<<<1, 1, 0, st>>>(p->ctrl, ABORT_TIMEOUT);
+      CUDA_TRY(p, cudaStreamSynchronize(st));
+      return VP_OK;
+    }
     bool launched = false;
     if (p->plan.wave_rtc) {
       for (int s = 0; s < S && !launched; ++s) {
@@ -1006,6 +1015,23 @@ vp_status vp_get_trace(void* h, void** dev_ptr, size_t* n) {
   *n = (size_t)std::min<unsigned long long>(m, (unsigned long long)p->desc.trace_capacity);
   return VP_OK;
 }
+
+// ---- internal accessors for the auto-tuner (vp_tune.cu); not part of vp.h
+int vpi_num_stages(void* h) { return h ? (int)((vp_pipeline_s*)h)->st.size() : 0; }
+int vpi_num_sms(void* h) { return h ? ((vp_pipeline_s*)h)->num_sms : 0; }
+int vpi_rtc_legal(void* h, int lo, int hi) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  return p && p->fam && p->fam->rtc_legal(lo, hi) ? 1 : 0;
+}
+int vpi_default_batch(void* h, int s) { return ((vp_pipeline_s*)h)->fam->default_batch(s); }
+uint32_t vpi_swap_flags(void* h, uint32_t flags) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  uint32_t old = p->desc.flags;
+  p->desc.flags = flags;
+  return old;
+}
+double vpi_timeout(void* h) { return ((vp_pipeline_s*)h)->timeout_ms; }
+void vpi_set_error(void* h, const char* msg) { ((vp_pipeline_s*)h)->err = msg; }
 
 vp_status vp_set_timeout(void* h, double ms) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;

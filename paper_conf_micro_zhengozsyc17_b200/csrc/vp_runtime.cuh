@@ -510,6 +510,10 @@ struct Runner {
       sh.done = 0;
       if (aborted(c)) {
         sh.done = 1;
+      } else if (globaltimer() > c->deadline.v) {
+        // watchdog, checked every round even by busy blocks (the tuner's timeoutexec)
+        atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
+        sh.done = 1;
       } else if (a.g.mode == MODE_WAVE) {
         const int s = a.g.wave_stage;
         int k = (int)(sh.wave_rem < a.g.batch[s] ? sh.wave_rem : a.g.batch[s]);
@@ -573,7 +577,9 @@ struct Runner {
         } else {
           wait_slots(a.c, q, base, n, 0, lane);
           __syncwarp();
-          if (aborted(a.c.ctrl)) {  // never hand unpublished slots to the workers
+          // warp-uniform decision (lanes may observe the abort flag at different times)
+          const bool abort_now = __shfl_sync(0xffffffffu, aborted(a.c.ctrl) ? 1 : 0, 0) != 0;
+          if (abort_now) {  // never hand unpublished slots to the workers
             if (lane == 0) {
               sh.nx_n = 0;
               sh.done = 1;

@@ -73,3 +73,17 @@ def test_no_gpu_calls_fail_cleanly(lib):
     from paper_conf_micro_zhengozsyc17_b200 import vp
     with pytest.raises(vp.VPError):
         vp.Pipeline(0)
+
+
+def test_config_string_roundtrip():
+    """vp_config_to_string / vp_config_from_string are host-only (no GPU needed)."""
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    b = vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 44), (2, 3, vp.GROUP_RTC, 44, 148)], 148,
+                        blocks_per_sm=[2, 0, 3, 0], batch=[32, 16, 8, 4])
+    c = vp.Config(model=vp.HYBRID, has_binding=1, binding=b, batch=0)
+    s = vp.config_to_string(c)
+    c2 = vp.config_from_string(s)
+    assert ctypes.string_at(ctypes.addressof(c), ctypes.sizeof(c)) == ctypes.string_at(ctypes.addressof(c2), ctypes.sizeof(c2))
+    assert vp.config_to_string(c2) == s
+    with pytest.raises(vp.VPError):
+        vp.config_from_string("garbage")
