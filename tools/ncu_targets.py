@@ -23,10 +23,19 @@ ap.add_argument("--frames", type=int, default=64)
 ap.add_argument("--runs", type=int, default=2)
 args = ap.parse_args()
 
-scene = inputs.reyes_config5(n_frames=args.frames)
 nsm, _ = vp.device_info(0)
-rp = ReyesPipeline(scene)
-if args.target == "mega":
+if args.target.startswith("raster"):
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_scene()
+    rp = RasterPipeline(scene)
+else:
+    scene = inputs.reyes_config5(n_frames=args.frames)
+    rp = ReyesPipeline(scene)
+if args.target == "raster_mega":
+    rp.configure(vp.MEGAKERNEL)
+elif args.target == "raster_kbk":
+    rp.configure(vp.KBK)
+elif args.target == "mega":
     rp.configure(vp.MEGAKERNEL)
 elif args.target == "kbk":
     rp.configure(vp.KBK)
