@@ -202,8 +202,8 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     nsm, cc = vp.device_info(local)
     # ---- shard: rank r renders frames [r*F/P, (r+1)*F/P) of the orbit
-    f0 = rank * args.frames // world
-    f1 = (rank + 1) * args.frames // world
+    from paper_conf_micro_zhengozsyc17_b200 import shard
+    f0, f1 = shard.shard_range(rank, world, args.frames)
     scene = inputs.reyes_config5(n_frames=f1 - f0, n_side=PATCH_SIDE, frame0=f0)
     rp = ReyesPipeline(scene, device=local)
     tune = None
@@ -234,14 +234,8 @@ def main():
     t_ms, st, kms = time_steps(torch, rp, args.steps, stream)
     barrier()
     clocks = clk.stop()
-    t = torch.tensor([t_ms], dtype=torch.float64, device="cuda")
-    items_local = sum(st["dequeued"][:4])
-    cnt = torch.tensor([items_local, f1 - f0], dtype=torch.float64, device="cuda")
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(cnt, op=dist.ReduceOp.SUM)
-    t_ms = float(t.item())
-    items_all, frames_all = float(cnt[0].item()), float(cnt[1].item())
+    t_ms = shard.max_over_ranks(t_ms, "cuda")
+    items_all, frames_all = shard.sum_over_ranks([sum(st["dequeued"][:4]), f1 - f0], "cuda")
     ms_per_step = t_ms / args.steps
     fps = frames_all * args.steps / (t_ms / 1e3)
     ips = items_all * args.steps / (t_ms / 1e3)
@@ -321,17 +315,15 @@ def main():
 
     # ---- NCCL output gather (config 5), timed separately
     gather_ms = None
-    if world > 1 and (f1 - f0) * world == args.frames:
-        out = torch.empty((args.frames,) + tuple(rp.colour.shape[1:]), dtype=torch.float32, device="cuda")
+    if world > 1:
         barrier()
         g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         g0.record(stream)
-        dist.all_gather_into_tensor(out, rp.colour)
+        out = shard.gather_frames(rp.colour, args.frames)  # NCCL over NVLink
         g1.record(stream)
         torch.cuda.synchronize()
-        gt = torch.tensor([g0.elapsed_time(g1)], dtype=torch.float64, device="cuda")
-        dist.all_reduce(gt, op=dist.ReduceOp.MAX)
-        gather_ms = float(gt.item())
+        assert out.shape[0] == args.frames
+        gather_ms = shard.max_over_ranks(g0.elapsed_time(g1), "cuda")
 
     cpu = None
     if rank == 0 and world == 1:

@@ -268,6 +268,68 @@ def _raster_run(fname, scene, trace_cap=0):
     return res
 
 
+class PyrSceneC(C.Structure):
+    _fields_ = [("S", C.c_int32), ("n_img", C.c_int32), ("rgb", P)]
+
+
+class PyrOutC(C.Structure):
+    _fields_ = [("gray", P), ("hist", P), ("lut", P), ("pyr", P), ("n_gray", C.c_uint64), ("n_cdf", C.c_uint64),
+                ("n_map", C.c_uint64), ("n_resize", C.c_uint64), ("trace", P), ("trace_cap", C.c_size_t),
+                ("trace_n", C.c_size_t)]
+
+
+def pyr_levels(S):
+    return lib().orc_pyr_levels(S)
+
+
+def pyr_level_offset(S, l):
+    f = lib().orc_pyr_level_offset
+    f.restype = C.c_size_t
+    return int(f(S, l))
+
+
+def histeq_lut(hist, N):
+    h = np.ascontiguousarray(hist, np.uint32)
+    lut = np.zeros(256, np.uint8)
+    f = lib().orc_histeq_lut
+    f.argtypes = [P, C.c_uint64, P]
+    f(_ptr(h), N, _ptr(lut))
+    return lut
+
+
+def _pyr_run(fname, rgb, trace_cap=0):
+    rgb = np.ascontiguousarray(rgb, np.uint8)
+    n, S = rgb.shape[0], rgb.shape[1]
+    L = pyr_levels(S)
+    total = pyr_level_offset(S, L)
+    gray = np.zeros((n, S * S), np.uint8)
+    hist = np.zeros((n, 256), np.uint32)
+    lut = np.zeros((n, 256), np.uint8)
+    pyr = np.zeros((n, total), np.uint8)
+    sc = PyrSceneC(S=S, n_img=n, rgb=rgb.ctypes.data)
+    o = PyrOutC(gray=gray.ctypes.data, hist=hist.ctypes.data, lut=lut.ctypes.data, pyr=pyr.ctypes.data)
+    trace = np.zeros(max(trace_cap, 1), TRACE_DTYPE)
+    if trace_cap:
+        o.trace, o.trace_cap = trace.ctypes.data, trace_cap
+    fn = getattr(lib(), fname)
+    fn.argtypes = [P, P]
+    rc = fn(C.byref(sc), C.byref(o))
+    assert rc == 0, rc
+    res = dict(gray=gray, hist=hist, lut=lut, pyr=pyr, n_gray=o.n_gray, n_cdf=o.n_cdf, n_map=o.n_map,
+               n_resize=o.n_resize, levels=L)
+    if trace_cap:
+        res["trace"] = trace[: o.trace_n].copy()
+    return res
+
+
+def pyr_definition(rgb):
+    return _pyr_run("orc_pyr_definition", rgb)
+
+
+def pyr_pipeline(rgb, trace_cap=0):
+    return _pyr_run("orc_pyr_pipeline", rgb, trace_cap)
+
+
 def raster_definition(scene):
     return _raster_run("orc_raster_definition", scene)
 

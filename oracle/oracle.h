@@ -128,6 +128,28 @@ typedef struct orc_raster_out {
   orc_trace_rec* trace; size_t trace_cap, trace_n;
 } orc_raster_out;
 
+/* ---------------- Image pyramid (pyramid.c) ---------------- */
+typedef struct orc_pyr_scene {
+  int32_t S;          /* image side, a power of two >= 64 */
+  int32_t n_img;
+  const uint8_t* rgb; /* [n_img][S][S][3] */
+} orc_pyr_scene;
+
+typedef struct orc_pyr_out {
+  uint8_t* gray;  /* [n_img][S*S] level-0 grayscale (before equalisation) */
+  uint32_t* hist; /* [n_img][256] */
+  uint8_t* lut;   /* [n_img][256] */
+  uint8_t* pyr;   /* [n_img][sum_l (S>>l)^2] levels concatenated, level 0 equalised */
+  uint64_t n_gray, n_cdf, n_map, n_resize;
+  orc_trace_rec* trace; size_t trace_cap, trace_n;
+} orc_pyr_out;
+
+int orc_pyr_levels(int S);
+size_t orc_pyr_level_offset(int S, int l);
+void orc_histeq_lut(const uint32_t hist[256], uint64_t N, uint8_t lut[256]);
+int orc_pyr_definition(const orc_pyr_scene* sc, orc_pyr_out* out);
+int orc_pyr_pipeline(const orc_pyr_scene* sc, orc_pyr_out* out);
+
 int orc_raster_definition(const orc_raster_scene* sc, orc_raster_out* out);
 int orc_raster_pipeline(const orc_raster_scene* sc, orc_raster_out* out);
 void orc_raster_vertex(const orc_raster_scene* sc, uint32_t tri, float clip[3][4]);

@@ -263,6 +263,17 @@ def raster_quad_mesh(W: int, H: int, cell: int = 8, z: float = 0.5) -> RasterSce
     return RasterScene(W=W, H=H, M=pixel_to_ndc(W, H), pos=pos, col=col)
 
 
+def pyramid_images(n_img: int = 32, S: int = 4096, seed: int = seed_for(3)) -> np.ndarray:
+    """BASELINE config 3 (pyramid half) inputs: n_img RGB8 images S x S (SURVEY §8(d)
+    d3a): 8x8 constant blocks U(0,255) per channel, scaled by 3/4, plus a horizontal
+    gradient 0..63.  uint8 [n_img, S, S, 3]."""
+    nb = S // 8
+    vals = (splitmix64(seed, n_img * nb * nb * 3) % np.uint64(256)).astype(np.int32).reshape(n_img, nb, nb, 3)
+    blocks = np.repeat(np.repeat(vals, 8, axis=1), 8, axis=2)
+    grad = (np.arange(S, dtype=np.int32) * 64 // S)[None, None, :, None]
+    return np.minimum(255, blocks * 3 // 4 + grad).astype(np.uint8)
+
+
 def reyes_planar(S_px: float, W: int = 64, H: int = 64, x0: float = 8.0, y0: float = 8.0,
                  max_depth: int = 8, albedo=(0.5, 0.25, 0.75)) -> ReyesScene:
     """Closed-form special case (SURVEY c-1 pin 4): a planar patch parallel to the image

@@ -1,0 +1,70 @@
+"""Multi-process (gloo, world_size 2 and 3, CPU) test of the frame sharder used by
+bench.py for config 5: partition, per-rank rendering (the CPU oracle stands in for the
+GPU compute here), counter reduction and frame gather reproduce a single-process run."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.multiprocessing as mp
+
+from paper_conf_micro_zhengozsyc17_b200 import shard
+
+
+def test_shard_range_partition():
+    for world in (1, 2, 3, 4, 7, 8):
+        for total in (0, 1, 5, 64, 512):
+            ranges = [shard.shard_range(r, world, total) for r in range(world)]
+            assert ranges[0][0] == 0 and ranges[-1][1] == total
+            assert all(a[1] == b[0] for a, b in zip(ranges, ranges[1:]))
+            sizes = [b - a for a, b in ranges]
+            assert max(sizes) - min(sizes) <= 1
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, total, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_micro_zhengozsyc17_b200 import inputs
+        f0, f1 = shard.shard_range(rank, world, total)
+        sc = inputs.reyes_config5(n_frames=f1 - f0, n_side=8, frame0=f0, W=48, H=48)
+        r = oracle.reyes_pipeline(sc)
+        local = torch.from_numpy(r["colour"].copy())
+        full = shard.gather_frames(local, total)
+        counts = shard.sum_over_ranks([r["n_bound"], r["n_split"], r["n_dice"], r["n_shade"]], "cpu")
+        t = shard.max_over_ranks(float(rank + 1), "cpu")
+        if rank == 0:
+            q.put((full.numpy(), counts, t))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_render_equals_single_process(orc, world):
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    total = 5
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, total, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    full, counts, t = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    ref = orc.reyes_pipeline(inputs.reyes_config5(n_frames=total, n_side=8, W=48, H=48))
+    assert np.array_equal(full, ref["colour"])
+    assert counts == [ref["n_bound"], ref["n_split"], ref["n_dice"], ref["n_shade"]]
+    assert t == float(world)
