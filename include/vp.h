@@ -72,7 +72,10 @@ typedef enum vp_stage_kind {
   VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23,
   /* Rasterization (Fig. 16, L59): Vertex + Clip (the paper's Clip), Raster (its
    * Interpolate: triangle -> 8x8 tiles), Fragment (its Shade: coverage + z-buffer) */
-  VP_RASTER_VERTEX = 30, VP_RASTER_CLIP = 31, VP_RASTER_RASTER = 32, VP_RASTER_FRAGMENT = 33
+  VP_RASTER_VERTEX = 30, VP_RASTER_CLIP = 31, VP_RASTER_RASTER = 32, VP_RASTER_FRAGMENT = 33,
+  /* Image pyramid (Fig. 12, L53): Grayscale, HistEq as CDF + Map, Resize (recursive);
+   * dependency latches between them */
+  VP_PYR_GRAY = 40, VP_PYR_CDF = 41, VP_PYR_MAP = 42, VP_PYR_RESIZE = 43
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -213,6 +216,18 @@ typedef struct vp_raster_params {
   unsigned long long* fb;    /* [H*W] depth keys (zkey(z) << 32 | tri), reset by vp_run    */
   float* colour;             /* [H*W][4] resolved colour, written by vp_run                */
 } vp_raster_params;
+
+typedef struct vp_pyramid_params {
+  int32_t S;                 /* image side: power of two in [64, 4096]                     */
+  int32_t n_img;             /* Gray items are {img, 0, ty, tx} for the 64x64 tiles        */
+  const uint8_t* rgb;        /* [n_img][S][S][3] input, 16-B aligned                       */
+  uint8_t* gray;             /* [n_img][S*S] scratch: level-0 grayscale                    */
+  uint8_t* pyr;              /* [n_img][stride] output pyramid, levels concatenated;       */
+                             /* stride = sum_l (S>>l)^2 rounded up to a multiple of 128    */
+  uint32_t* hist;            /* [n_img][256] histograms (reset by vp_run)                  */
+  uint8_t* lut;              /* [n_img][256] equalisation LUTs (output)                    */
+  int32_t* latch;            /* [n_img][1 + sum_{l>=1} tiles_l^2] dependency latches       */
+} vp_pyramid_params;
 
 /* ---------------- calls ---------------- */
 const char* vp_status_string(vp_status s);

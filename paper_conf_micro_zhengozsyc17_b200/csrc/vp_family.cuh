@@ -124,5 +124,6 @@ const FamilyOps* family_toy();
 const FamilyOps* family_collatz();
 const FamilyOps* family_reyes();
 const FamilyOps* family_raster();
+const FamilyOps* family_pyramid();
 
 }  // namespace vp

@@ -21,13 +21,14 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
     all_families[0] = family_toy();
     all_families[1] = family_collatz();
     all_families[2] = family_reyes();
     all_families[3] = family_raster();
+    all_families[4] = family_pyramid();
   }
 }
 const FamilyOps* family_of_kind(int kind, int* pos) {

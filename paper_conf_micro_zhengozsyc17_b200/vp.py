@@ -33,6 +33,7 @@ TOY_S1, TOY_S2, TOY_S3 = 1, 2, 3
 COLLATZ_STEP, COLLATZ_SINK = 10, 11
 REYES_BOUND, REYES_SPLIT, REYES_DICE, REYES_SHADE = 20, 21, 22, 23
 RASTER_VERTEX, RASTER_CLIP, RASTER_RASTER, RASTER_FRAGMENT = 30, 31, 32, 33
+PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS = 1, 2, 4, 8
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
@@ -102,6 +103,11 @@ class ReyesParams(C.Structure):
 class RasterParams(C.Structure):
     _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P),
                 ("setup", P), ("fb", P), ("colour", P)]
+
+
+class PyramidParams(C.Structure):
+    _fields_ = [("S", C.c_int32), ("n_img", C.c_int32), ("rgb", P), ("gray", P), ("pyr", P), ("hist", P),
+                ("lut", P), ("latch", P)]
 
 
 def _decl(name, args, res=C.c_int):

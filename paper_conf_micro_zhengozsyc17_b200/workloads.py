@@ -94,6 +94,58 @@ class RasterPipeline:
         return self.colour.cpu().numpy()
 
 
+def pyramid_levels(S):
+    L = 0
+    while (S >> L) >= 1:
+        L += 1
+    return L
+
+
+def pyramid_latches_per_img(S):
+    n = 1
+    for l in range(1, pyramid_levels(S)):
+        t = max(1, (S >> l) // 64)
+        n += t * t
+    return n
+
+
+class PyramidPipeline:
+    """Grayscale -> HistEq (CDF, Map) -> Resize (recursive) over n_img RGB8 images (Fig. 12, L53)."""
+
+    def __init__(self, rgb: np.ndarray, device: int = 0, rgb_on_device=None, **kw):
+        dev = _dev(device)
+        n, S = rgb.shape[0], rgb.shape[1]
+        self.n_img, self.S = n, S
+        self.total = sum((S >> l) ** 2 for l in range(pyramid_levels(S)))
+        self.stride = (self.total + 127) // 128 * 128
+        self.rgb = rgb_on_device if rgb_on_device is not None else torch.from_numpy(np.ascontiguousarray(rgb)).to(dev)
+        self.gray = torch.empty((n, S * S), dtype=torch.uint8, device=dev)
+        self.pyr = torch.empty((n, self.stride), dtype=torch.uint8, device=dev)
+        self.hist = torch.empty((n, 256), dtype=torch.int32, device=dev)
+        self.lut = torch.empty((n, 256), dtype=torch.uint8, device=dev)
+        self.latch = torch.empty((n, pyramid_latches_per_img(S)), dtype=torch.int32, device=dev)
+        self.prm = vp.PyramidParams(S=S, n_img=n, rgb=self.rgb.data_ptr(), gray=self.gray.data_ptr(),
+                                    pyr=self.pyr.data_ptr(), hist=self.hist.data_ptr(), lut=self.lut.data_ptr(),
+                                    latch=self.latch.data_ptr())
+        self.p = vp.Pipeline(device, **kw)
+        for kind in (vp.PYR_GRAY, vp.PYR_CDF, vp.PYR_MAP, vp.PYR_RESIZE):
+            self.p.register(kind, 16, self.prm)
+        nt = S // 64
+        ii, yy, xx = np.meshgrid(np.arange(n), np.arange(nt), np.arange(nt), indexing="ij")
+        seeds = np.zeros((n * nt * nt, 4), np.uint32)
+        seeds[:, 0], seeds[:, 2], seeds[:, 3] = ii.ravel(), yy.ravel(), xx.ravel()
+        self.p.insert(0, seeds, n=seeds.shape[0])
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def pyramid(self):
+        return self.pyr.cpu().numpy()[:, : self.total]
+
+
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
 REYES_STRIDES = (272, 272, 272, 1968)
 

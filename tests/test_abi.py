@@ -49,9 +49,10 @@ def test_struct_sizes_match_header():
     prog = r'''
 #include <stdio.h>
 #include "vp.h"
-int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pipeline_desc), sizeof(vp_stage_desc),
+int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pipeline_desc), sizeof(vp_stage_desc),
  sizeof(vp_sm_binding), sizeof(vp_config), sizeof(vp_run_stats), sizeof(vp_autotune_opts), sizeof(vp_tune_report),
- sizeof(vp_toy_params), sizeof(vp_collatz_params), sizeof(vp_reyes_params));return 0;}
+ sizeof(vp_toy_params), sizeof(vp_collatz_params), sizeof(vp_reyes_params), sizeof(vp_raster_params),
+ sizeof(vp_pyramid_params));return 0;}
 '''
     tmp = os.path.join(ROOT, "build_abi_check")
     os.makedirs(tmp, exist_ok=True)
@@ -61,7 +62,7 @@ int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pip
     subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe], check=True)
     sizes = [int(x) for x in subprocess.run([exe], capture_output=True, text=True).stdout.split()]
     mirrors = [vp.PipelineDesc, vp.StageDesc, vp.SmBinding, vp.Config, vp.RunStats, vp.AutotuneOpts, vp.TuneReport,
-               vp.ToyParams, vp.CollatzParams, vp.ReyesParams]
+               vp.ToyParams, vp.CollatzParams, vp.ReyesParams, vp.RasterParams, vp.PyramidParams]
     assert sizes == [ctypes.sizeof(m) for m in mirrors]
 
 
