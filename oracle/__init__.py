@@ -330,6 +330,47 @@ def pyr_pipeline(rgb, trace_cap=0):
     return _pyr_run("orc_pyr_pipeline", rgb, trace_cap)
 
 
+class CfdSceneC(C.Structure):
+    _fields_ = [("G", C.c_int32), ("T", C.c_int32), ("n_outer", C.c_int32), ("pad", C.c_int32), ("vars0", P),
+                ("area", P), ("nb", P), ("normals", P), ("ff", C.c_float * 5)]
+
+
+class CfdOutC(C.Structure):
+    _fields_ = [("vars", P), ("n_copy", C.c_uint64), ("n_step", C.c_uint64), ("n_flux", C.c_uint64),
+                ("n_time", C.c_uint64), ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t)]
+
+
+def _cfd_run(fname, scene, n_outer=None, trace_cap=0):
+    arrs = [np.ascontiguousarray(scene.vars0, np.float32), np.ascontiguousarray(scene.area, np.float32),
+            np.ascontiguousarray(scene.nb, np.int32), np.ascontiguousarray(scene.normals, np.float32)]
+    sc = CfdSceneC(G=scene.G, T=scene.T, n_outer=scene.n_outer if n_outer is None else n_outer,
+                   vars0=arrs[0].ctypes.data, area=arrs[1].ctypes.data, nb=arrs[2].ctypes.data,
+                   normals=arrs[3].ctypes.data)
+    for i in range(5):
+        sc.ff[i] = float(scene.ff[i])
+    out = np.zeros((5, scene.G * scene.G), np.float32)
+    o = CfdOutC(vars=out.ctypes.data)
+    trace = np.zeros(max(trace_cap, 1), TRACE_DTYPE)
+    if trace_cap:
+        o.trace, o.trace_cap = trace.ctypes.data, trace_cap
+    fn = getattr(lib(), fname)
+    fn.argtypes = [P, P]
+    rc = fn(C.byref(sc), C.byref(o))
+    assert rc == 0, rc
+    res = dict(vars=out, n_copy=o.n_copy, n_step=o.n_step, n_flux=o.n_flux, n_time=o.n_time)
+    if trace_cap:
+        res["trace"] = trace[: o.trace_n].copy()
+    return res
+
+
+def cfd_definition(scene, n_outer=None):
+    return _cfd_run("orc_cfd_definition", scene, n_outer)
+
+
+def cfd_pipeline(scene, n_outer=None, trace_cap=0):
+    return _cfd_run("orc_cfd_pipeline", scene, n_outer, trace_cap)
+
+
 def raster_definition(scene):
     return _raster_run("orc_raster_definition", scene)
 

@@ -150,6 +150,28 @@ void orc_histeq_lut(const uint32_t hist[256], uint64_t N, uint8_t lut[256]);
 int orc_pyr_definition(const orc_pyr_scene* sc, orc_pyr_out* out);
 int orc_pyr_pipeline(const orc_pyr_scene* sc, orc_pyr_out* out);
 
+/* ---------------- CFD (cfd.c) ---------------- */
+typedef struct orc_cfd_scene {
+  int32_t G;              /* grid side (cells)                                     */
+  int32_t T;              /* cells per tile item (divides G)                        */
+  int32_t n_outer;        /* outer iterations (each: Copy, StepFactor, 3 x RK)      */
+  int32_t pad;
+  const float* vars0;     /* [5][G*G] initial conserved variables (SoA)              */
+  const float* area;      /* [G*G]                                                  */
+  const int32_t* nb;      /* [4][G*G] neighbour cell or -1 (wall) / -2 (far field)  */
+  const float* normals;   /* [4][3][G*G]                                            */
+  float ff[5];            /* far-field conserved state                               */
+} orc_cfd_scene;
+
+typedef struct orc_cfd_out {
+  float* vars;            /* [5][G*G] final state                                    */
+  uint64_t n_copy, n_step, n_flux, n_time;
+  orc_trace_rec* trace; size_t trace_cap, trace_n;
+} orc_cfd_out;
+
+int orc_cfd_definition(const orc_cfd_scene* sc, orc_cfd_out* out);
+int orc_cfd_pipeline(const orc_cfd_scene* sc, orc_cfd_out* out);
+
 int orc_raster_definition(const orc_raster_scene* sc, orc_raster_out* out);
 int orc_raster_pipeline(const orc_raster_scene* sc, orc_raster_out* out);
 void orc_raster_vertex(const orc_raster_scene* sc, uint32_t tri, float clip[3][4]);

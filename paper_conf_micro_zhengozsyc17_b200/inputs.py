@@ -263,6 +263,66 @@ def raster_quad_mesh(W: int, H: int, cell: int = 8, z: float = 0.5) -> RasterSce
     return RasterScene(W=W, H=H, M=pixel_to_ndc(W, H), pos=pos, col=col)
 
 
+@dataclass
+class CfdScene:
+    """BASELINE config 3 (CFD half) inputs: a structured G x G grid with
+    Rodinia euler3d semantics.  All arrays SoA float32 / int32."""
+    G: int
+    T: int
+    n_outer: int
+    vars0: np.ndarray     # [5, G*G] density, momentum x, y, z, density energy
+    area: np.ndarray      # [G*G]
+    nb: np.ndarray        # [4, G*G] int32 neighbour or -2 (far field)
+    normals: np.ndarray   # [4, 3, G*G]
+    ff: np.ndarray        # [5] far-field conserved state
+
+    @property
+    def n_cells(self):
+        return self.G * self.G
+
+
+def cfd_far_field() -> np.ndarray:
+    """Rodinia euler3d far field: rho 1.4, p 1, Mach 1.2, angle of attack 0 (float64 ->
+    float32): (rho, rho*u, 0, 0, rho*|u|^2/2 + p/(gamma-1))."""
+    gamma, rho, p, mach = 1.4, 1.4, 1.0, 1.2
+    c = math.sqrt(gamma * p / rho)
+    u = mach * c
+    return np.array([rho, rho * u, 0.0, 0.0, rho * 0.5 * u * u + p / (gamma - 1)], np.float32)
+
+
+def cfd_scene(G: int = 4096, n_outer: int = 10, seed: int = seed_for(3, 1), T: int = 0, bump_amp: float = 0.05,
+              uniform: bool = False) -> CfdScene:
+    """Grid cell (r, c) has index r*G + c; faces j = 0..3 are -x, +x, -y, +y with unit
+    normals (-1,0,0), (1,0,0), (0,-1,0), (0,1,0), area 1; off-grid neighbours are far
+    field.  Initial state = far field x (1 + amp * bump), bump = sum of 8 seeded
+    Gaussians (float64 on the host).  Tiles are T = min(1024, G) cells of a row."""
+    n = G * G
+    T = T or min(1024, G)
+    ff = cfd_far_field()
+    r = np.repeat(np.arange(G), G)
+    c = np.tile(np.arange(G), G)
+    if uniform:
+        scale = np.ones(n)
+    else:
+        u = uniform01(seed, 8 * 3).reshape(8, 3)
+        bump = np.zeros(n)
+        for g in range(8):
+            r0, c0, s = u[g, 0] * G, u[g, 1] * G, G / 16.0 * (0.5 + u[g, 2])
+            bump += np.exp(-((r - r0) ** 2 + (c - c0) ** 2) / (2 * s * s))
+        scale = 1.0 + bump_amp * bump
+    vars0 = (ff.astype(np.float64)[:, None] * scale[None, :]).astype(np.float32)
+    nb = np.full((4, n), -2, np.int32)
+    idx = np.arange(n, dtype=np.int64)
+    nb[0] = np.where(c > 0, idx - 1, -2)
+    nb[1] = np.where(c < G - 1, idx + 1, -2)
+    nb[2] = np.where(r > 0, idx - G, -2)
+    nb[3] = np.where(r < G - 1, idx + G, -2)
+    normals = np.zeros((4, 3, n), np.float32)
+    normals[0, 0], normals[1, 0], normals[2, 1], normals[3, 1] = -1.0, 1.0, -1.0, 1.0
+    return CfdScene(G=G, T=T, n_outer=n_outer, vars0=vars0, area=np.ones(n, np.float32), nb=nb,
+                    normals=normals, ff=ff)
+
+
 def pyramid_images(n_img: int = 32, S: int = 4096, seed: int = seed_for(3)) -> np.ndarray:
     """BASELINE config 3 (pyramid half) inputs: n_img RGB8 images S x S (SURVEY §8(d)
     d3a): 8x8 constant blocks U(0,255) per channel, scaled by 3/4, plus a horizontal
