@@ -75,7 +75,10 @@ typedef enum vp_stage_kind {
   VP_RASTER_VERTEX = 30, VP_RASTER_CLIP = 31, VP_RASTER_RASTER = 32, VP_RASTER_FRAGMENT = 33,
   /* Image pyramid (Fig. 12, L53): Grayscale, HistEq as CDF + Map, Resize (recursive);
    * dependency latches between them */
-  VP_PYR_GRAY = 40, VP_PYR_CDF = 41, VP_PYR_MAP = 42, VP_PYR_RESIZE = 43
+  VP_PYR_GRAY = 40, VP_PYR_CDF = 41, VP_PYR_MAP = 42, VP_PYR_RESIZE = 43,
+  /* CFD (Fig. 15, L55; Rodinia euler3d): Copy, Step Factor, Flux, Time Step; loop of 3 RK
+   * steps per outer iteration; tiles of T cells (composite items, L37) */
+  VP_CFD_COPY = 50, VP_CFD_STEP_FACTOR = 51, VP_CFD_FLUX = 52, VP_CFD_TIME_STEP = 53
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -228,6 +231,24 @@ typedef struct vp_pyramid_params {
   uint8_t* lut;              /* [n_img][256] equalisation LUTs (output)                    */
   int32_t* latch;            /* [n_img][1 + sum_{l>=1} tiles_l^2] dependency latches       */
 } vp_pyramid_params;
+
+typedef struct vp_cfd_params {
+  int32_t G;                 /* grid side; N = G*G cells                                   */
+  int32_t T;                 /* cells per tile item (divides G, multiple of 4)             */
+  int32_t n_outer;           /* outer iterations; the final state is vars[(3*n_outer) & 1] */
+  int32_t pad0;
+  const float* vars0;        /* [5][N] initial state (density, momentum x/y/z, energy)     */
+  float* vars;               /* [2][5][N] ping-pong state, 16-B aligned (output)           */
+  float* old;                /* [5][N] scratch                                             */
+  float* sf;                 /* [N] step factors (scratch)                                 */
+  float* flux;               /* [5][N] scratch                                             */
+  const float* area;         /* [N]                                                        */
+  const int32_t* nb;         /* [4][N] neighbour cell, -1 wall, -2 far field               */
+  const float* normals;      /* [4][3][N] face normals                                     */
+  float ff[5];               /* far-field conserved state                                  */
+  int32_t pad1;
+  int32_t* latch;            /* [2][N/T] dependency latches (scratch)                      */
+} vp_cfd_params;
 
 /* ---------------- calls ---------------- */
 const char* vp_status_string(vp_status s);

@@ -125,5 +125,6 @@ const FamilyOps* family_collatz();
 const FamilyOps* family_reyes();
 const FamilyOps* family_raster();
 const FamilyOps* family_pyramid();
+const FamilyOps* family_cfd();
 
 }  // namespace vp

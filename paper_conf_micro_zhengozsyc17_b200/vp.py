@@ -34,6 +34,7 @@ COLLATZ_STEP, COLLATZ_SINK = 10, 11
 REYES_BOUND, REYES_SPLIT, REYES_DICE, REYES_SHADE = 20, 21, 22, 23
 RASTER_VERTEX, RASTER_CLIP, RASTER_RASTER, RASTER_FRAGMENT = 30, 31, 32, 33
 PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
+CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS = 1, 2, 4, 8
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
@@ -108,6 +109,12 @@ class RasterParams(C.Structure):
 class PyramidParams(C.Structure):
     _fields_ = [("S", C.c_int32), ("n_img", C.c_int32), ("rgb", P), ("gray", P), ("pyr", P), ("hist", P),
                 ("lut", P), ("latch", P)]
+
+
+class CfdParams(C.Structure):
+    _fields_ = [("G", C.c_int32), ("T", C.c_int32), ("n_outer", C.c_int32), ("pad0", C.c_int32), ("vars0", P),
+                ("vars", P), ("old", P), ("sf", P), ("flux", P), ("area", P), ("nb", P), ("normals", P),
+                ("ff", C.c_float * 5), ("pad1", C.c_int32), ("latch", P)]
 
 
 def _decl(name, args, res=C.c_int):

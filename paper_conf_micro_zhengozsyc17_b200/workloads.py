@@ -146,6 +146,45 @@ class PyramidPipeline:
         return self.pyr.cpu().numpy()[:, : self.total]
 
 
+class CfdPipeline:
+    """Copy -> StepFactor -> 3 x (Flux -> TimeStep), looped (Fig. 15, L55; Rodinia euler3d)."""
+
+    def __init__(self, scene: inputs.CfdScene, device: int = 0, **kw):
+        dev = _dev(device)
+        self.scene = scene
+        N = scene.n_cells
+        t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+        self.vars0, self.area, self.nb, self.normals = t(scene.vars0), t(scene.area), t(scene.nb), t(scene.normals)
+        self.vars = torch.empty((2, 5, N), dtype=torch.float32, device=dev)
+        self.old = torch.empty((5, N), dtype=torch.float32, device=dev)
+        self.sf = torch.empty((N,), dtype=torch.float32, device=dev)
+        self.flux = torch.empty((5, N), dtype=torch.float32, device=dev)
+        self.ntiles = N // scene.T
+        self.latch = torch.empty((2, self.ntiles), dtype=torch.int32, device=dev)
+        self.prm = vp.CfdParams(G=scene.G, T=scene.T, n_outer=scene.n_outer, vars0=self.vars0.data_ptr(),
+                                vars=self.vars.data_ptr(), old=self.old.data_ptr(), sf=self.sf.data_ptr(),
+                                flux=self.flux.data_ptr(), area=self.area.data_ptr(), nb=self.nb.data_ptr(),
+                                normals=self.normals.data_ptr(), latch=self.latch.data_ptr())
+        for i in range(5):
+            self.prm.ff[i] = float(scene.ff[i])
+        self.p = vp.Pipeline(device, **kw)
+        for kind in (vp.CFD_COPY, vp.CFD_STEP_FACTOR, vp.CFD_FLUX, vp.CFD_TIME_STEP):
+            self.p.register(kind, 16, self.prm)
+        seeds = np.zeros((self.ntiles, 4), np.uint32)
+        seeds[:, 0] = np.arange(self.ntiles)
+        if scene.n_outer > 0:
+            self.p.insert(0, seeds, n=self.ntiles)
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def state(self):
+        return self.vars[(3 * self.scene.n_outer) & 1].cpu().numpy()
+
+
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
 REYES_STRIDES = (272, 272, 272, 1968)
 
