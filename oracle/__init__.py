@@ -371,6 +371,62 @@ def cfd_pipeline(scene, n_outer=None, trace_cap=0):
     return _cfd_run("orc_cfd_pipeline", scene, n_outer, trace_cap)
 
 
+class FdSceneC(C.Structure):
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_frames", C.c_int32), ("n_stages", C.c_int32), ("rgb", P),
+                ("n_weak", C.c_int32 * 16), ("thr", C.c_int32 * 16), ("weak", P)]
+
+
+class FdOutC(C.Structure):
+    _fields_ = [("levels", P), ("lbp", P), ("hist", P), ("lut", P), ("det", P), ("det_cap", C.c_size_t),
+                ("n_det", C.c_size_t), ("survivors", C.c_uint64 * 16), ("windows", C.c_uint64),
+                ("deq", C.c_uint64 * 8), ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t)]
+
+
+def fd_levels(W, H):
+    Ws, Hs = (C.c_int * 8)(), (C.c_int * 8)()
+    L = lib().orc_fd_levels(W, H, Ws, Hs)
+    return [(Ws[i], Hs[i]) for i in range(L)]
+
+
+def _fd_run(fname, scene, det_cap=1 << 16, trace_cap=0):
+    rgb = np.ascontiguousarray(scene.rgb, np.uint8)
+    weak = np.ascontiguousarray(scene.weak, np.int32)
+    sc = FdSceneC(W=scene.W, H=scene.H, n_frames=rgb.shape[0], n_stages=len(scene.n_weak), rgb=rgb.ctypes.data,
+                  weak=weak.ctypes.data)
+    for k, (n, t) in enumerate(zip(scene.n_weak, scene.thr)):
+        sc.n_weak[k], sc.thr[k] = int(n), int(t)
+    per = sum(w * h for w, h in fd_levels(scene.W, scene.H))
+    F = rgb.shape[0]
+    levels = np.zeros((F, per), np.uint8)
+    lbp = np.zeros((F, per), np.uint8)
+    hist = np.zeros((F, 256), np.uint32)
+    lut = np.zeros((F, 256), np.uint8)
+    det = np.zeros((det_cap, 4), np.uint32)
+    o = FdOutC(levels=levels.ctypes.data, lbp=lbp.ctypes.data, hist=hist.ctypes.data, lut=lut.ctypes.data,
+               det=det.ctypes.data, det_cap=det_cap)
+    trace = np.zeros(max(trace_cap, 1), TRACE_DTYPE)
+    if trace_cap:
+        o.trace, o.trace_cap = trace.ctypes.data, trace_cap
+    fn = getattr(lib(), fname)
+    fn.argtypes = [P, P]
+    rc = fn(C.byref(sc), C.byref(o))
+    assert rc == 0, rc
+    assert o.n_det <= det_cap
+    res = dict(levels=levels, lbp=lbp, hist=hist, lut=lut, det=det[: o.n_det].copy(), n_det=o.n_det,
+               survivors=list(o.survivors[: len(scene.n_weak)]), windows=o.windows, deq=list(o.deq[:6]))
+    if trace_cap:
+        res["trace"] = trace[: o.trace_n].copy()
+    return res
+
+
+def fd_definition(scene, det_cap=1 << 16):
+    return _fd_run("orc_fd_definition", scene, det_cap)
+
+
+def fd_pipeline(scene, det_cap=1 << 16, trace_cap=0):
+    return _fd_run("orc_fd_pipeline", scene, det_cap, trace_cap)
+
+
 def raster_definition(scene):
     return _raster_run("orc_raster_definition", scene)
 

@@ -172,6 +172,32 @@ typedef struct orc_cfd_out {
 int orc_cfd_definition(const orc_cfd_scene* sc, orc_cfd_out* out);
 int orc_cfd_pipeline(const orc_cfd_scene* sc, orc_cfd_out* out);
 
+/* ---------------- LBP face detection (facedet.c) ---------------- */
+typedef struct orc_fd_scene {
+  int32_t W, H, n_frames, n_stages;
+  const uint8_t* rgb;      /* [n_frames][H][W][3]                                   */
+  int32_t n_weak[16];      /* weak classifiers per cascade stage                     */
+  int32_t thr[16];         /* stage thresholds                                       */
+  const int32_t* weak;     /* [sum n_weak][12]: cx, cy, mask[8], in, out             */
+} orc_fd_scene;
+
+typedef struct orc_fd_out {
+  uint8_t* levels;         /* [n_frames][sum_l W_l*H_l] equalised pyramid             */
+  uint8_t* lbp;            /* [n_frames][sum_l W_l*H_l] LBP codes                    */
+  uint32_t* hist;          /* [n_frames][256]                                        */
+  uint8_t* lut;            /* [n_frames][256]                                        */
+  uint32_t* det;           /* [det_cap][4] frame, level, x, y                         */
+  size_t det_cap, n_det;
+  uint64_t survivors[16];  /* windows passing cascade stage k                         */
+  uint64_t windows;        /* windows evaluated                                       */
+  uint64_t deq[8];
+  orc_trace_rec* trace; size_t trace_cap, trace_n;
+} orc_fd_out;
+
+int orc_fd_levels(int W, int H, int* Ws, int* Hs);
+int orc_fd_definition(const orc_fd_scene* sc, orc_fd_out* out);
+int orc_fd_pipeline(const orc_fd_scene* sc, orc_fd_out* out);
+
 int orc_raster_definition(const orc_raster_scene* sc, orc_raster_out* out);
 int orc_raster_pipeline(const orc_raster_scene* sc, orc_raster_out* out);
 void orc_raster_vertex(const orc_raster_scene* sc, uint32_t tri, float clip[3][4]);

@@ -323,6 +323,61 @@ def cfd_scene(G: int = 4096, n_outer: int = 10, seed: int = seed_for(3, 1), T: i
                     normals=normals, ff=ff)
 
 
+@dataclass
+class FaceScene:
+    """BASELINE config 2 inputs: RGB frames and a synthetic LBP cascade."""
+    W: int
+    H: int
+    rgb: np.ndarray          # [n_frames, H, W, 3] uint8
+    n_weak: np.ndarray       # [K] int32
+    thr: np.ndarray          # [K] int32
+    weak: np.ndarray         # [sum n_weak, 12] int32: cx, cy, mask[8], in, out
+    planted: np.ndarray      # [n_frames, n_planted, 2] level-0 (x, y) of the constant templates
+
+    @property
+    def n_frames(self):
+        return self.rgb.shape[0]
+
+
+def face_scene(W: int = 1920, H: int = 1080, n_frames: int = 1, seed: int = seed_for(2), n_planted: int = 24,
+               K: int = 12) -> FaceScene:
+    """Frames: 8x8 constant blocks U(0,255) + per-pixel noise in [-8, 8] (clamped), plus
+    n_planted noise-free constant 24x24 templates (their interior LBP code is 255).
+    Cascade: K stages, stage k has 2+k weak classifiers with cells
+    U([1,22]^2), 256-bit masks with bit probability 1/2 and the template code (255) forced
+    on, leaves +/-1000, threshold 1000 * (2*ceil(0.6 n_k) - n_k)."""
+    nb_w, nb_h = (W + 7) // 8, (H + 7) // 8
+    rgb = np.zeros((n_frames, H, W, 3), np.uint8)
+    planted = np.zeros((n_frames, n_planted, 2), np.int32)
+    for f in range(n_frames):
+        s = seed + 1000 * f
+        blocks = (splitmix64(s, nb_h * nb_w * 3) % np.uint64(256)).astype(np.int32).reshape(nb_h, nb_w, 3)
+        img = np.repeat(np.repeat(blocks, 8, 0), 8, 1)[:H, :W]
+        noise = (splitmix64(s + 1, H * W * 3) % np.uint64(17)).astype(np.int32).reshape(H, W, 3) - 8
+        img = np.clip(img + noise, 0, 255)
+        pos = splitmix64(s + 2, n_planted * 2).reshape(n_planted, 2)
+        for t in range(n_planted):
+            x = int(pos[t, 0] % np.uint64(W - 24))
+            y = int(pos[t, 1] % np.uint64(H - 24))
+            img[y:y + 24, x:x + 24] = 200
+            planted[f, t] = (x, y)
+        rgb[f] = img.astype(np.uint8)
+    n_weak = np.array([2 + k for k in range(K)], np.int32)
+    nw = int(n_weak.sum())
+    r = splitmix64(seed + 77, nw * 11).reshape(nw, 11)
+    weak = np.zeros((nw, 12), np.int64)
+    weak[:, 0] = 1 + (r[:, 0] % np.uint64(22)).astype(np.int64)
+    weak[:, 1] = 1 + (r[:, 1] % np.uint64(22)).astype(np.int64)
+    masks = r[:, 2:6]                                 # 4 x 64 random bits = 256
+    for w in range(8):
+        weak[:, 2 + w] = ((masks[:, w // 2] >> np.uint64(32 * (w % 2))) & np.uint64(0xFFFFFFFF)).astype(np.int64)
+    weak[:, 2 + 7] |= 1 << 31                         # code 255 -> word 7, bit 31
+    weak[:, 10], weak[:, 11] = 1000, -1000
+    weak = weak.astype(np.uint32).view(np.int32).reshape(nw, 12)
+    thr = np.array([1000 * (2 * math.ceil(0.6 * n) - n) for n in n_weak], np.int32)
+    return FaceScene(W=W, H=H, rgb=rgb, n_weak=n_weak, thr=thr, weak=np.ascontiguousarray(weak), planted=planted)
+
+
 def pyramid_images(n_img: int = 32, S: int = 4096, seed: int = seed_for(3)) -> np.ndarray:
     """BASELINE config 3 (pyramid half) inputs: n_img RGB8 images S x S (SURVEY §8(d)
     d3a): 8x8 constant blocks U(0,255) per channel, scaled by 3/4, plus a horizontal
