@@ -78,7 +78,10 @@ typedef enum vp_stage_kind {
   VP_PYR_GRAY = 40, VP_PYR_CDF = 41, VP_PYR_MAP = 42, VP_PYR_RESIZE = 43,
   /* CFD (Fig. 15, L55; Rodinia euler3d): Copy, Step Factor, Flux, Time Step; loop of 3 RK
    * steps per outer iteration; tiles of T cells (composite items, L37) */
-  VP_CFD_COPY = 50, VP_CFD_STEP_FACTOR = 51, VP_CFD_FLUX = 52, VP_CFD_TIME_STEP = 53
+  VP_CFD_COPY = 50, VP_CFD_STEP_FACTOR = 51, VP_CFD_FLUX = 52, VP_CFD_TIME_STEP = 53,
+  /* LBP face detection (Fig. 14, L55): Grayscale, HistEq as CDF + Map, Resize
+   * (recursive), Feature Extraction (LBP), Scanning (rows of 24x24 windows) */
+  VP_FD_GRAY = 60, VP_FD_CDF = 61, VP_FD_MAP = 62, VP_FD_RESIZE = 63, VP_FD_LBP = 64, VP_FD_SCAN = 65
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -249,6 +252,28 @@ typedef struct vp_cfd_params {
   int32_t pad1;
   int32_t* latch;            /* [2][N/T] dependency latches (scratch)                      */
 } vp_cfd_params;
+
+typedef struct vp_facedet_params {
+  int32_t W, H;              /* level-0 frame size (H <= 2048)                             */
+  int32_t n_frames;          /* Gray items are {frame, 0, band, 0}, bands of 32 rows        */
+  int32_t n_stages;          /* cascade stages K <= 16                                     */
+  int32_t n_weak[16];        /* weak classifiers per stage                                 */
+  int32_t thr[16];           /* stage thresholds                                           */
+  int32_t n_weak_total;      /* sum(n_weak) <= 128                                         */
+  int32_t pad0;
+  const uint8_t* rgb;        /* [n_frames][H][W][3]                                         */
+  uint8_t* levels;           /* [n_frames][sum_l W_l*H_l] equalised pyramid (scratch/out)  */
+  uint8_t* lbp;              /* [n_frames][sum_l W_l*H_l] LBP codes (scratch/out)          */
+  uint32_t* hist;            /* [n_frames][256]                                            */
+  uint8_t* lut;              /* [n_frames][256]                                            */
+  const int32_t* weak;       /* [n_weak_total][12]: cx, cy, mask[8], in, out               */
+  uint32_t* det;             /* [det_cap][4] detections {frame, level, x, y}, 16-B aligned */
+  unsigned long long* det_count;   /* device counter (reset by vp_run)                     */
+  unsigned long long det_cap;
+  unsigned long long* survivors;   /* [16] windows passing stage k (reset by vp_run)       */
+  unsigned long long* windows;     /* windows evaluated (reset by vp_run)                  */
+  int32_t* latch;            /* [n_frames][1 + 3 * sum_l bands_l] dependency latches       */
+} vp_facedet_params;
 
 /* ---------------- calls ---------------- */
 const char* vp_status_string(vp_status s);

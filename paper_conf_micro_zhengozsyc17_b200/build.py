@@ -6,7 +6,7 @@ import sys
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libvp.so")
-SOURCES = ["vp_host.cu", "vp_tune.cu", "fam_basic.cu", "fam_reyes.cu", "fam_raster.cu", "fam_pyramid.cu", "fam_cfd.cu"]
+SOURCES = ["vp_host.cu", "vp_tune.cu", "fam_basic.cu", "fam_reyes.cu", "fam_raster.cu", "fam_pyramid.cu", "fam_cfd.cu", "fam_facedet.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          # no FMA contraction, IEEE div/sqrt, no fast math -> bit-exact vs oracle

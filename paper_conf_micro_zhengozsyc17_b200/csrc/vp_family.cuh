@@ -126,5 +126,6 @@ const FamilyOps* family_reyes();
 const FamilyOps* family_raster();
 const FamilyOps* family_pyramid();
 const FamilyOps* family_cfd();
+const FamilyOps* family_facedet();
 
 }  // namespace vp

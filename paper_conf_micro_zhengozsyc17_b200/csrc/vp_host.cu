@@ -21,10 +21,11 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
     all_families[5] = family_cfd();
+    all_families[6] = family_facedet();
     all_families[0] = family_toy();
     all_families[1] = family_collatz();
     all_families[2] = family_reyes();

@@ -35,6 +35,7 @@ REYES_BOUND, REYES_SPLIT, REYES_DICE, REYES_SHADE = 20, 21, 22, 23
 RASTER_VERTEX, RASTER_CLIP, RASTER_RASTER, RASTER_FRAGMENT = 30, 31, 32, 33
 PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
+FD_GRAY, FD_CDF, FD_MAP, FD_RESIZE, FD_LBP, FD_SCAN = 60, 61, 62, 63, 64, 65
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS = 1, 2, 4, 8
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
@@ -115,6 +116,14 @@ class CfdParams(C.Structure):
     _fields_ = [("G", C.c_int32), ("T", C.c_int32), ("n_outer", C.c_int32), ("pad0", C.c_int32), ("vars0", P),
                 ("vars", P), ("old", P), ("sf", P), ("flux", P), ("area", P), ("nb", P), ("normals", P),
                 ("ff", C.c_float * 5), ("pad1", C.c_int32), ("latch", P)]
+
+
+class FaceDetParams(C.Structure):
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_frames", C.c_int32), ("n_stages", C.c_int32),
+                ("n_weak", C.c_int32 * 16), ("thr", C.c_int32 * 16), ("n_weak_total", C.c_int32),
+                ("pad0", C.c_int32), ("rgb", P), ("levels", P), ("lbp", P), ("hist", P), ("lut", P), ("weak", P),
+                ("det", P), ("det_count", P), ("det_cap", C.c_uint64), ("survivors", P), ("windows", P),
+                ("latch", P)]
 
 
 def _decl(name, args, res=C.c_int):

@@ -185,6 +185,63 @@ class CfdPipeline:
         return self.vars[(3 * self.scene.n_outer) & 1].cpu().numpy()
 
 
+def face_levels(W, H):
+    out, w, h = [], W, H
+    while len(out) < 8 and w >= 24 and h >= 24:
+        out.append((w, h))
+        w, h = 4 * w // 5, 4 * h // 5
+    return out
+
+
+class FaceDetPipeline:
+    """Gray -> HistEq (CDF, Map) -> Resize (recursive) -> LBP -> Scan over RGB frames (Fig. 14, L55)."""
+
+    def __init__(self, scene: inputs.FaceScene, device: int = 0, det_cap: int = 1 << 20, **kw):
+        dev = _dev(device)
+        self.scene = scene
+        F, W, H = scene.n_frames, scene.W, scene.H
+        lv = face_levels(W, H)
+        per = sum(w * h for w, h in lv)
+        bands = [-(-h // 32) for _, h in lv]
+        self.rgb = torch.from_numpy(np.ascontiguousarray(scene.rgb)).to(dev)
+        self.levels = torch.empty((F, per), dtype=torch.uint8, device=dev)
+        self.lbp = torch.empty((F, per), dtype=torch.uint8, device=dev)
+        self.hist = torch.empty((F, 256), dtype=torch.int32, device=dev)
+        self.lut = torch.empty((F, 256), dtype=torch.uint8, device=dev)
+        self.weak = torch.from_numpy(np.ascontiguousarray(scene.weak)).to(dev)
+        self.det = torch.empty((det_cap, 4), dtype=torch.int32, device=dev)
+        self.counters = torch.zeros(32, dtype=torch.int64, device=dev)   # [0] det_count, [1] windows, [16:32] survivors
+        self.latch = torch.empty((F, 1 + 3 * sum(bands)), dtype=torch.int32, device=dev)
+        base = self.counters.data_ptr()
+        self.prm = vp.FaceDetParams(W=W, H=H, n_frames=F, n_stages=len(scene.n_weak),
+                                    n_weak_total=int(scene.n_weak.sum()), rgb=self.rgb.data_ptr(),
+                                    levels=self.levels.data_ptr(), lbp=self.lbp.data_ptr(),
+                                    hist=self.hist.data_ptr(), lut=self.lut.data_ptr(), weak=self.weak.data_ptr(),
+                                    det=self.det.data_ptr(), det_count=base, det_cap=det_cap,
+                                    survivors=base + 16 * 8, windows=base + 8, latch=self.latch.data_ptr())
+        for k, (n, t) in enumerate(zip(scene.n_weak, scene.thr)):
+            self.prm.n_weak[k], self.prm.thr[k] = int(n), int(t)
+        self.p = vp.Pipeline(device, **kw)
+        for kind in (vp.FD_GRAY, vp.FD_CDF, vp.FD_MAP, vp.FD_RESIZE, vp.FD_LBP, vp.FD_SCAN):
+            self.p.register(kind, 16, self.prm)
+        seeds = np.zeros((F * bands[0], 4), np.uint32)
+        seeds[:, 0] = np.repeat(np.arange(F), bands[0])
+        seeds[:, 2] = np.tile(np.arange(bands[0]), F)
+        self.p.insert(0, seeds, n=seeds.shape[0])
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def results(self):
+        c = self.counters.cpu().numpy()
+        n = int(c[0])
+        det = self.det[: min(n, self.det.shape[0])].cpu().numpy().astype(np.int64)
+        return dict(det=det, n_det=n, windows=int(c[1]), survivors=[int(x) for x in c[16:16 + len(self.scene.n_weak)]])
+
+
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
 REYES_STRIDES = (272, 272, 272, 1968)
 
