@@ -58,6 +58,8 @@ def parse():
     ap.add_argument("--split", type=int, default=44, help="SMs for the [Bound,Split] group (hybrid)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-baselines", action="store_true")
+    ap.add_argument("--no-suite", action="store_true", help="skip the configs 1-4 secondary measurements")
+    ap.add_argument("--suite-tune-seconds", type=float, default=8.0)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     return ap.parse_args()
 
@@ -182,6 +184,64 @@ def run_reference(args, rank, world):
             "cpu_baseline": {"value": v, "unit": "frames/s", "cores": info[0], "kind": "oracle", "sample": info[1]},
             "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
+    """Secondary measurements: every BASELINE workload (configs 1-4) through the same
+    runtime, auto-tuned, vs KBK; items/s, frames/s and % of measured HBM where the
+    workload is HBM-bound."""
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    from paper_conf_micro_zhengozsyc17_b200.workloads import (CfdPipeline, FaceDetPipeline, PyramidPipeline,
+                                                              RasterPipeline, ReyesPipeline)
+
+    def measure(pipe, frames, alg_bytes=None, reps=3):
+        best, rep = pipe.p.autotune(time_budget_s=tune_s, sm_granularity=4, batch_choices=(1, 2))
+        tuned_cfg = vp.config_to_string(best)
+
+        def t_run():
+            pipe.run(stream)
+            ts = []
+            st = None
+            for _ in range(reps):
+                st = pipe.run(stream)
+                ts.append(st["device_ms"])
+            return min(ts), st
+
+        ms, st = t_run()
+        pipe.configure(vp.KBK)
+        kbk_ms, _ = t_run()
+        pipe.configure(vp.MEGAKERNEL)
+        mega_ms, _ = t_run()
+        pipe.p.configure_config(best)
+        items = sum(st["dequeued"][:8])
+        r = {"ms": ms, "frames_per_s": frames / (ms / 1e3), "items_per_s": items / (ms / 1e3),
+             "items": items, "kbk_ms": kbk_ms, "megakernel_ms": mega_ms, "speedup_vs_kbk": kbk_ms / ms,
+             "speedup_vs_megakernel": mega_ms / ms, "tuned": tuned_cfg.split(" mask")[0]}
+        if alg_bytes:
+            gbs = alg_bytes / (ms / 1e3) / 1e9
+            r.update({"alg_bytes": alg_bytes, "achieved_gbs": gbs, "pct_hbm_measured": 100 * gbs / hbm_gbs})
+        return r
+
+    out = {}
+    sc1 = inputs.reyes_config1()
+    out["reyes_config1"] = measure(ReyesPipeline(sc1), 1)
+    fs = inputs.face_scene()
+    fp = FaceDetPipeline(fs)
+    out["facedet_config2"] = measure(fp, fs.n_frames)
+    out["facedet_config2"]["windows_per_s"] = fp.results()["windows"] / (out["facedet_config2"]["ms"] / 1e3)
+    n_img, S = 32, 4096
+    rgb = inputs.pyramid_images(n_img, S)
+    # Gray: RGB read; Map: RGB read + level-0 write; Resize: read + write per level; hist negligible
+    per_img = 3 * S * S + (3 * S * S + S * S) + sum(((S >> l) ** 2) * 5 for l in range(1, 13))
+    out["pyramid_config3"] = measure(PyramidPipeline(rgb), n_img, alg_bytes=n_img * per_img)
+    del rgb
+    cs = inputs.cfd_scene(G=4096, n_outer=10)
+    out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
+    out["cfd_config3"]["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (out["cfd_config3"]["ms"] / 1e3)
+    rs = inputs.raster_scene()
+    out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
+    out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)
+    return out
 
 
 def main():
@@ -325,6 +385,13 @@ def main():
         assert out.shape[0] == args.frames
         gather_ms = shard.max_over_ranks(g0.elapsed_time(g1), "cuda")
 
+    suite = None
+    if world == 1 and not args.no_suite:
+        try:
+            suite = workload_suite(torch, vp, stream, args.suite_tune_seconds, pk.get("hbm_gbs", 6548.5))
+        except Exception as ex:  # secondary numbers must never lose the headline line
+            suite = {"error": repr(ex)}
+
     cpu = None
     if rank == 0 and world == 1:
         try:
@@ -353,7 +420,7 @@ def main():
                 "note": "ALU/latency-bound workload (SURVEY §8(d) d5); % HBM reported, not the bound"},
         "speedup_vs_kbk": (extra["kbk"]["ms_per_step"] / ms_per_step) if "kbk" in extra else None,
         "baselines": extra, "e2e": e2e, "gather_ms": gather_ms, "clocks": clocks, "gpu_launches": launches * args.steps,
-        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune,
+        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune, "workloads": suite,
         "config_string": vp.config_to_string(main_cfg),
     }
     if rank == 0:
