@@ -5,7 +5,10 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libvp.so")
+# VP_LIB_NAME: dev variants (e.g. libvp_m4.so built with other VP_NVCC_EXTRA), still in-tree
+LIB_NAME = os.environ.get("VP_LIB_NAME", "libvp.so")
+LIB = os.path.join(HERE, LIB_NAME)
+OBJDIR = os.path.join(HERE, "build" if LIB_NAME == "libvp.so" else "build_" + LIB_NAME.split(".")[0])
 SOURCES = ["vp_host.cu", "vp_tune.cu", "fam_basic.cu", "fam_reyes.cu", "fam_raster.cu", "fam_pyramid.cu", "fam_cfd.cu", "fam_facedet.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
@@ -28,9 +31,9 @@ def build(force=False, verbose=False, jobs=None):
         return LIB
     objs = []
     procs = []
-    os.makedirs(os.path.join(HERE, "build"), exist_ok=True)
+    os.makedirs(OBJDIR, exist_ok=True)
     for src in SOURCES:
-        obj = os.path.join(HERE, "build", src.replace(".cu", ".o"))
+        obj = os.path.join(OBJDIR, src.replace(".cu", ".o"))
         cmd = [NVCC, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True)))
         objs.append(obj)
@@ -41,7 +44,7 @@ def build(force=False, verbose=False, jobs=None):
         if p.returncode != 0:
             sys.stderr.write(out)
             raise RuntimeError(f"nvcc failed for {src}")
-    with open(os.path.join(HERE, "build", "ptxas.log"), "w") as f:
+    with open(os.path.join(OBJDIR, "ptxas.log"), "w") as f:
         f.write("\n".join(logs))
     cmd = [NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", LIB, *objs, "-lcudart"]
     subprocess.run(cmd, check=True)

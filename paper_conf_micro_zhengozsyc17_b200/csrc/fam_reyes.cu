@@ -142,6 +142,31 @@ __device__ __forceinline__ void cover(const vp_reyes_params& p, FbRec* fb, I ax,
   }
 }
 
+// One triangle of a micropolygon in the int32 quad path: three edge functions biased so
+// that "inside or owned boundary" (reading R-R9) is w >= 0, evaluated incrementally
+// along a pixel row (exact integer arithmetic, so identical to a direct evaluation).
+struct TriEdges {
+  int w[3], dx[3], dy[3];  // w at the row-start sample; per-pixel-step and per-row-step increments
+  bool live;
+};
+__device__ __forceinline__ void tri_setup(TriEdges& T, int ax, int ay, int bx, int by, int cx, int cy, int X0, int Y0) {
+  const int area = edge(ax, ay, bx, by, cx, cy);
+  T.live = area != 0;
+  if (area < 0) {  // positive orientation: (a, c, b)
+    int tx = bx, ty = by;
+    bx = cx; by = cy; cx = tx; cy = ty;
+  }
+  const int ex[3] = {ax, bx, cx}, ey[3] = {ay, by, cy};
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    const int px = ex[k], py = ey[k], qx = ex[(k + 1) % 3], qy = ey[(k + 1) % 3];
+    const int bias = owns(px, py, qx, qy) ? 0 : -1;
+    T.w[k] = edge(px, py, qx, qy, X0, Y0) + bias;
+    T.dx[k] = -(qy - py) * 256;
+    T.dy[k] = (qx - px) * 256;
+  }
+}
+
 __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, long long ay, long long bx, long long by,
                            long long cx, long long cy, unsigned long long key, float s) {
   long long xmin = min(ax, min(bx, cx)), xmax = max(ax, max(bx, cx));
@@ -335,6 +360,48 @@ struct ReyesF {
   }
 
   // -------------------------------------------------------------- Dice (warp/patch)
+  // One warp evaluates the 9x9 grid of patch P into `out` (reading R-R7/R-R9).
+  static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane) {
+    uint32_t frame = P->id >> 12;
+    if (frame >= (uint32_t)p.n_frames) frame = 0;
+    const float* M = p.M + 16 * (size_t)frame;
+    for (int g = lane; g < kNP; g += 32) {
+      const int i = g / kNG, j = g - i * kNG;
+      float Bu[4], Bv[4];
+      bernstein((float)i * 0.125f, Bu);
+      bernstein((float)j * 0.125f, Bv);
+      float x = 0.0f, y = 0.0f, z = 0.0f;
+#pragma unroll
+      for (int a = 0; a < 4; ++a)
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+          const float w = Bu[a] * Bv[b];
+          const float4 cp = P->cp[4 * a + b];
+          x = x + w * cp.x;
+          y = y + w * cp.y;
+          z = z + w * cp.z;
+        }
+      float4 c = project(M, x, y, z, 1.0f);
+      float sx, sy, zs;
+      screen(p, c, sx, sy, zs);
+      out->g[0][g] = x;
+      out->g[1][g] = y;
+      out->g[2][g] = z;
+      // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
+      const float X = sx * 256.0f, Y = sy * 256.0f;
+      const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
+      out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
+      out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
+      out->g[5][g] = zs;
+    }
+    if (lane == 0) {
+      out->id = P->id;
+      out->path = P->path;
+      out->depth = P->depth;
+      out->dirs = P->dirs;
+    }
+  }
+
   template <class Ctx>
   static __device__ void dice(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
@@ -342,104 +409,133 @@ struct ReyesF {
     for (int r0 = 0; r0 < n; r0 += kThreads / 32) {
       const int k = r0 + (threadIdx.x >> 5);
       if (k >= n) break;  // warp-uniform
-      const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
-      uint32_t frame = P->id >> 12;
-      if (frame >= (uint32_t)p.n_frames) frame = 0;
-      const float* M = p.M + 16 * (size_t)frame;
       int slot = 0;
       if (lane == 0) slot = ctx.template reserve<SHADE>();
       slot = __shfl_sync(0xffffffffu, slot, 0);
       if (slot < 0) continue;
-      RGrid* out = (RGrid*)ctx.template out_ptr<SHADE>(slot);
-      for (int g = lane; g < kNP; g += 32) {
-        const int i = g / kNG, j = g - i * kNG;
-        float Bu[4], Bv[4];
-        bernstein((float)i * 0.125f, Bu);
-        bernstein((float)j * 0.125f, Bv);
-        float x = 0.0f, y = 0.0f, z = 0.0f;
-#pragma unroll
-        for (int a = 0; a < 4; ++a)
-#pragma unroll
-          for (int b = 0; b < 4; ++b) {
-            const float w = Bu[a] * Bv[b];
-            const float4 cp = P->cp[4 * a + b];
-            x = x + w * cp.x;
-            y = y + w * cp.y;
-            z = z + w * cp.z;
-          }
-        float4 c = project(M, x, y, z, 1.0f);
-        float sx, sy, zs;
-        screen(p, c, sx, sy, zs);
-        out->g[0][g] = x;
-        out->g[1][g] = y;
-        out->g[2][g] = z;
-        // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
-        const float X = sx * 256.0f, Y = sy * 256.0f;
-        const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
-        out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
-        out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
-        out->g[5][g] = zs;
-      }
-      if (lane == 0) {
-        out->id = P->id;
-        out->path = P->path;
-        out->depth = P->depth;
-        out->dirs = P->dirs;
-      }
+      dice_patch(p, (const RPatch*)(items + (size_t)k * sizeof(RPatch)), (RGrid*)ctx.template out_ptr<SHADE>(slot), lane);
     }
   }
 
-  // -------------------------------------------------------------- Shade (64 thr/grid)
+  // -------------------------------------------------------------- Shade (per micropolygon)
+  // Micropolygon q = 8i + j of grid Gd: the quad (i,j)..(i+1,j+1), split into the
+  // triangles (v0,v1,v2), (v0,v2,v3) (reading R-R8..R-R10).
+  static __device__ __forceinline__ void shade_mp(const Params& p, const RGrid* Gd, int q) {
+    const uint32_t frame = Gd->id >> 12, patch = Gd->id & 0xFFFu;
+    if (frame >= (uint32_t)p.n_frames) return;
+    const int i = q >> 3, j = q & 7;
+    const int g00 = i * kNG + j, g10 = (i + 1) * kNG + j, g01 = i * kNG + j + 1, g11 = (i + 1) * kNG + j + 1;
+    // Coverage first: the two triangles cover exactly the pixel centres inside either
+    // one, all within the quad's box; a micropolygon whose box holds no pixel centre
+    // (most of them at config 5: ~0.25 px^2 each) writes nothing, so its shading is
+    // never computed.
+    const int gi[4] = {g00, g10, g11, g01};
+    int vx[4], vy[4];
+    bool ok = true;
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      vx[v] = __float_as_int(Gd->g[3][gi[v]]);
+      vy[v] = __float_as_int(Gd->g[4][gi[v]]);
+      if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
+    }
+    if (!ok) return;
+    const int xmin = min(min(vx[0], vx[1]), min(vx[2], vx[3])), xmax = max(max(vx[0], vx[1]), max(vx[2], vx[3]));
+    const int ymin = min(min(vy[0], vy[1]), min(vy[2], vy[3])), ymax = max(max(vy[0], vy[1]), max(vy[2], vy[3]));
+    // |coords| < 2^30: these int expressions cannot overflow
+    int px0 = -((128 - xmin) >> 8), px1 = (xmax - 128) >> 8;  // ceil / floor of (v - 128) / 256
+    int py0 = -((128 - ymin) >> 8), py1 = (ymax - 128) >> 8;
+    px0 = max(px0, 0);
+    py0 = max(py0, 0);
+    px1 = min(px1, p.W - 1);
+    py1 = min(py1, p.H - 1);
+    if (px0 > px1 || py0 > py1) return;
+    float e1[3], e2[3];
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+      e1[c] = Gd->g[c][g10] - Gd->g[c][g00];
+      e2[c] = Gd->g[c][g01] - Gd->g[c][g00];
+    }
+    float nx = e1[1] * e2[2] - e1[2] * e2[1];
+    float ny = e1[2] * e2[0] - e1[0] * e2[2];
+    float nz = e1[0] * e2[1] - e1[1] * e2[0];
+    float nn = nx * nx + ny * ny;
+    nn = nn + nz * nz;
+    float s;
+    if (nn == 0.0f) {
+      s = 0.1f;
+    } else {
+      float d = nx * p.L[0] + ny * p.L[1];
+      d = d + nz * p.L[2];
+      float t = d / sqrtf(nn);
+      if (!(t > 0.0f)) t = 0.0f;
+      s = 0.1f + 0.9f * t;
+    }
+    const float zq = ((Gd->g[5][g00] + Gd->g[5][g10]) + (Gd->g[5][g11] + Gd->g[5][g01])) * 0.25f;
+    const uint32_t mp = (patch << 18) | ((Gd->path & 0xFFu) << 10) | ((Gd->depth & 0xFu) << 6) | (uint32_t)q;
+    const unsigned long long key = ((unsigned long long)zkey(zq) << 32) | mp;
+    FbRec* fb = (FbRec*)p.fb + (size_t)frame * p.W * p.H;
+    if ((unsigned)xmax - (unsigned)xmin < (1u << 14) && (unsigned)ymax - (unsigned)ymin < (1u << 14)) {
+      // int32 quad path: coordinates relative to the box corner, |products| < 2^29
+      int ax[4], ay[4];
+#pragma unroll
+      for (int v = 0; v < 4; ++v) {
+        ax[v] = vx[v] - xmin;
+        ay[v] = vy[v] - ymin;
+      }
+      const int X0 = px0 * 256 + 128 - xmin, Y0 = py0 * 256 + 128 - ymin;
+      TriEdges A, B;
+      tri_setup(A, ax[0], ay[0], ax[1], ay[1], ax[2], ay[2], X0, Y0);
+      tri_setup(B, ax[0], ay[0], ax[2], ay[2], ax[3], ay[3], X0, Y0);
+      for (int py = py0; py <= py1; ++py) {
+        int a0 = A.w[0], a1 = A.w[1], a2 = A.w[2], b0 = B.w[0], b1 = B.w[1], b2 = B.w[2];
+        FbRec* row = fb + (size_t)py * p.W;
+        for (int px = px0; px <= px1; ++px) {
+          const bool in = (A.live && (a0 | a1 | a2) >= 0) || (B.live && (b0 | b1 | b2) >= 0);
+          if (in) fb_min(row + px, key, s);  // idempotent: a pixel in both writes once
+          a0 += A.dx[0]; a1 += A.dx[1]; a2 += A.dx[2];
+          b0 += B.dx[0]; b1 += B.dx[1]; b2 += B.dx[2];
+        }
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+          A.w[k] += A.dy[k];
+          B.w[k] += B.dy[k];
+        }
+      }
+    } else {
+      raster_tri(p, fb, vx[0], vy[0], vx[1], vy[1], vx[2], vy[2], key, s);
+      raster_tri(p, fb, vx[0], vy[0], vx[2], vy[2], vx[3], vy[3], key, s);
+    }
+  }
+
   template <class Ctx>
   static __device__ void shade(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
     const int q = threadIdx.x & 63;
-    const int i = q >> 3, j = q & 7;
     for (int r0 = 0; r0 < n; r0 += kThreads / 64) {
       const int k = r0 + (threadIdx.x >> 6);
       if (k >= n) break;  // uniform per pair of warps
-      const RGrid* Gd = (const RGrid*)(items + (size_t)k * sizeof(RGrid));
-      const uint32_t frame = Gd->id >> 12, patch = Gd->id & 0xFFFu;
-      if (frame >= (uint32_t)p.n_frames) continue;
-      const int g00 = i * kNG + j, g10 = (i + 1) * kNG + j, g01 = i * kNG + j + 1, g11 = (i + 1) * kNG + j + 1;
-      float e1[3], e2[3];
-#pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        e1[c] = Gd->g[c][g10] - Gd->g[c][g00];
-        e2[c] = Gd->g[c][g01] - Gd->g[c][g00];
-      }
-      float nx = e1[1] * e2[2] - e1[2] * e2[1];
-      float ny = e1[2] * e2[0] - e1[0] * e2[2];
-      float nz = e1[0] * e2[1] - e1[1] * e2[0];
-      float nn = nx * nx + ny * ny;
-      nn = nn + nz * nz;
-      float s;
-      if (nn == 0.0f) {
-        s = 0.1f;
-      } else {
-        float d = nx * p.L[0] + ny * p.L[1];
-        d = d + nz * p.L[2];
-        float t = d / sqrtf(nn);
-        if (!(t > 0.0f)) t = 0.0f;
-        s = 0.1f + 0.9f * t;
-      }
-      const float zq = ((Gd->g[5][g00] + Gd->g[5][g10]) + (Gd->g[5][g11] + Gd->g[5][g01])) * 0.25f;
-      const uint32_t mp = (patch << 18) | ((Gd->path & 0xFFu) << 10) | ((Gd->depth & 0xFu) << 6) | (uint32_t)q;
-      const unsigned long long key = ((unsigned long long)zkey(zq) << 32) | mp;
-      const int gi[4] = {g00, g10, g11, g01};
-      long long vx[4], vy[4];
-      bool ok = true;
-#pragma unroll
-      for (int v = 0; v < 4; ++v) {
-        const int X = __float_as_int(Gd->g[3][gi[v]]), Y = __float_as_int(Gd->g[4][gi[v]]);
-        if (X == INT_MIN || Y == INT_MIN) ok = false;
-        vx[v] = X;
-        vy[v] = Y;
-      }
-      if (!ok) continue;
-      FbRec* fb = (FbRec*)p.fb + (size_t)frame * p.W * p.H;
-      raster_tri(p, fb, vx[0], vy[0], vx[1], vy[1], vx[2], vy[2], key, s);
-      raster_tri(p, fb, vx[0], vy[0], vx[2], vy[2], vx[3], vy[3], key, s);
+      shade_mp(p, (const RGrid*)(items + (size_t)k * sizeof(RGrid)), q);
+    }
+  }
+
+  // -------------------------------------------------------------- RTC [Dice, Shade]
+  // Warp-granular run-to-completion: each warp dices one patch into a
+  // block-local grid slot and shades it itself (2 micropolygons per lane), so the chain
+  // needs no block barrier between the two stages.
+  static constexpr bool fused_rtc(int s, int hi) { return s == DICE && hi == SHADE; }
+  template <int S0, int HI, class Ctx>
+  static __device__ void exec_rtc_chain(Ctx& ctx, const uint8_t* items, int n) {
+    static_assert(S0 == DICE && HI == SHADE, "only the [Dice, Shade] chain is fused");
+    static_assert(Ctx::template cap<SHADE>() >= max_batch(DICE), "one grid slot per diced patch");
+    const Params& p = ctx.params();
+    const int lane = threadIdx.x & 31;
+    for (int k = threadIdx.x >> 5; k < n; k += kThreads / 32) {
+      RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(k);
+      dice_patch(p, (const RPatch*)(items + (size_t)k * sizeof(RPatch)), g, lane);
+      __syncwarp();
+      if (lane == 0) ctx.template note_local<SHADE>((const uint8_t*)g);
+      shade_mp(p, g, lane);
+      shade_mp(p, g, lane + 32);
     }
   }
 

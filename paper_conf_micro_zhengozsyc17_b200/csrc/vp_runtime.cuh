@@ -148,6 +148,52 @@ __device__ __forceinline__ void st_relaxed(unsigned long long* p, unsigned long 
 __device__ __forceinline__ unsigned long long atom_add(unsigned long long* p, long long d) {
   return atomicAdd(p, (unsigned long long)d);
 }
+__device__ __forceinline__ void red_add(unsigned long long* p, long long d) {
+  asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"((unsigned long long)d) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+
+// Bulk (TMA, non-tensor) copies between global memory and shared memory (sm_90+).
+// Ring ranges are contiguous up to the wrap point, so one claimed batch moves with one
+// or two instructions issued by one thread instead of ~n*stride/16 per-lane accesses.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned long long* m, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(m)), "r"(count) : "memory");
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long* m, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned long long* m, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(m)), "r"(parity)
+        : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* m) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   smem_u32(dst)),
+               "l"(src), "r"(bytes), "r"(smem_u32(m))
+               : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_commit_wait_all() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+// generic-proxy shared-memory writes -> later async-proxy (bulk) reads of them
+__device__ __forceinline__ void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+// async-proxy global writes/reads <-> generic-proxy release/acquire on the slot sequence words
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
 
 // Vector chunk used to move items of a given stride (16 B when possible).
 template <int STRIDE>
@@ -216,6 +262,30 @@ struct Graph {
   static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + F::scratch_bytes(lo, hi); }
 };
 
+// A family may run an RTC chain [s, hi] itself (F::fused_rtc(s, hi) and
+// F::exec_rtc_chain<s, hi>), e.g. with warp-granular hand-off instead of block barriers.
+template <class F, class = void>
+struct HasFusedRtc : std::false_type {};
+template <class F>
+struct HasFusedRtc<F, std::void_t<decltype(F::fused_rtc(0, 0))>> : std::true_type {};
+template <class F, bool kHas = HasFusedRtc<F>::value>
+struct FusedChain {
+  template <int S0, int HI, class C>
+  static __device__ __forceinline__ void run(C&, const uint8_t*, int) {}
+};
+template <class F>
+struct FusedChain<F, true> {
+  template <int S0, int HI, class C>
+  static __device__ __forceinline__ void run(C& ctx, const uint8_t* items, int n) {
+    F::template exec_rtc_chain<S0, HI>(ctx, items, n);
+  }
+};
+template <class F>
+constexpr bool fused_chain(int s, int hi) {
+  if constexpr (HasFusedRtc<F>::value) return F::fused_rtc(s, hi);
+  else return false;
+}
+
 // ------------------------------------------------------------------ per-block context
 struct BlockShared {
   int out_cnt[2][kMaxStages];          // per out buffer, per target
@@ -227,6 +297,8 @@ struct BlockShared {
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
+  unsigned long long mbar[2];          // bulk-copy completion, one per in buffer
+  uint32_t mbar_phase[2];
 };
 
 __device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
@@ -242,14 +314,25 @@ struct Ctx {
   __device__ Ctx(const KArgs<F>& a_, uint8_t* smem_, BlockShared& sh_) : a(a_), smem(smem_), sh(sh_), ob(0) {}
 
   __device__ __forceinline__ const typename F::Params& params() const { return a.p; }
-  __device__ __forceinline__ uint8_t* scratch() { return smem + G::scratch_offset(LO, HI, RTC); }
+  // layout constants are forced to compile time (nvcc does not always fold the
+  // recursive constexpr helpers when they appear in runtime expressions)
+  static constexpr int kScratch = G::scratch_offset(LO, HI, RTC);
+  static constexpr int kOutBase0 = G::out_base(LO, HI, RTC, 0);
+  static constexpr int kOutRegion = G::out_region(LO, HI, RTC);
+  template <int T>
+  struct OutT {
+    static constexpr int off = G::out_off(LO, HI, RTC, T);
+    static constexpr int cap = G::out_cap(LO, HI, RTC, T);
+  };
+
+  __device__ __forceinline__ uint8_t* scratch() { return smem + kScratch; }
 
   template <int T>
   __device__ __forceinline__ uint8_t* out_ptr(int slot) {
-    return smem + G::out_base(LO, HI, RTC, ob) + G::out_off(LO, HI, RTC, T) + slot * F::stride(T);
+    return smem + kOutBase0 + ob * kOutRegion + OutT<T>::off + slot * F::stride(T);
   }
   template <int T>
-  static constexpr int cap() { return G::out_cap(LO, HI, RTC, T); }
+  static constexpr int cap() { return OutT<T>::cap; }
 
   // Reserve k consecutive out slots for target T (one thread).  The declared fan-out
   // bounds guarantee capacity; exceeding it aborts the run (ABORT_FANOUT).
@@ -261,6 +344,20 @@ struct Ctx {
       return -1;
     }
     return slot;
+  }
+  // A fused RTC chain executed one block-local item of stage T (one thread per item):
+  // the per-stage task count and, with FLAG_TRACE, the trace record.
+  template <int T>
+  __device__ __forceinline__ void note_local(const uint8_t* item) {
+    atomicAdd(&sh.deq[T], 1ull);
+    if (a.c.flags & FLAG_TRACE) {
+      unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
+      if (idx < a.c.trace_cap) {
+        a.c.trace[idx].id = F::template item_id<T>(item);
+        a.c.trace[idx].stage = T;
+        a.c.trace[idx].smid = smid();
+      }
+    }
   }
   // Thread-level emit of a whole item (enqueue<Stage>(itemVal), Fig. 9 L37).
   template <int T>
@@ -288,6 +385,16 @@ __device__ __forceinline__ bool aborted(const Ctrl* c) {
 __device__ __forceinline__ int claim_ring(Ctrl* c, int s, int k, unsigned long long& base) {
   long long avail = (long long)ld_relaxed(&c->count[s].v);
   if (avail <= 0) return 0;  // cheap L2 read first: idle fetchers do not hammer atomics
+  int want = (int)(avail < k ? avail : k);
+  long long old = (long long)atom_add(&c->count[s].v, -want);
+  int got = old <= 0 ? 0 : (old < want ? (int)old : want);
+  if (got < want) atom_add(&c->count[s].v, want - got);
+  if (got == 0) return 0;
+  base = atom_add(&c->head[s].v, got);
+  return got;
+}
+// As claim_ring, with `avail` already polled (the fetcher polls all stages at once).
+__device__ __forceinline__ int claim_ring_avail(Ctrl* c, int s, int k, long long avail, unsigned long long& base) {
   int want = (int)(avail < k ? avail : k);
   long long old = (long long)atom_add(&c->count[s].v, -want);
   int got = old <= 0 ? 0 : (old < want ? (int)old : want);
@@ -393,6 +500,25 @@ __device__ __forceinline__ void copy_out(uint8_t* ring, const uint8_t* src, unsi
   }
 }
 
+// One thread: bulk copies of ring tickets [base, base+n) <-> a contiguous smem batch.
+template <int STRIDE>
+__device__ __forceinline__ void bulk_in(uint8_t* dst, const uint8_t* ring, unsigned long long base, int n,
+                                        uint32_t cap_log2, unsigned long long* m) {
+  const unsigned long long cap = 1ull << cap_log2, i0 = base & (cap - 1);
+  const int n1 = (cap - i0) < (unsigned long long)n ? (int)(cap - i0) : n;
+  mbar_arrive_expect_tx(m, (uint32_t)(n * STRIDE));
+  bulk_g2s(dst, ring + i0 * STRIDE, (uint32_t)(n1 * STRIDE), m);
+  if (n1 < n) bulk_g2s(dst + n1 * STRIDE, ring, (uint32_t)((n - n1) * STRIDE), m);
+}
+template <int STRIDE>
+__device__ __forceinline__ void bulk_out(uint8_t* ring, const uint8_t* src, unsigned long long base, int n,
+                                         uint32_t cap_log2) {
+  const unsigned long long cap = 1ull << cap_log2, i0 = base & (cap - 1);
+  const int n1 = (cap - i0) < (unsigned long long)n ? (int)(cap - i0) : n;
+  bulk_s2g(ring + i0 * STRIDE, src, (uint32_t)(n1 * STRIDE));
+  if (n1 < n) bulk_s2g(ring, src + n1 * STRIDE, (uint32_t)((n - n1) * STRIDE));
+}
+
 // ------------------------------------------------------------------ compile-time loops
 template <int I, int N, class Fn>
 __device__ __forceinline__ void static_for(Fn&& fn) {
@@ -415,87 +541,121 @@ struct Runner {
   static constexpr int S = F::S;
   static constexpr int W_FETCH = kWarpsW, W_PUBLISH = kWarpsW + 1;
 
-  __device__ static __forceinline__ uint8_t* in_buf(uint8_t* smem, int b) { return smem + G::in_base(LO, HI, b); }
-  __device__ static __forceinline__ uint8_t* out_buf(uint8_t* smem, int b, int t) {
-    return smem + G::out_base(LO, HI, RTC, b) + G::out_off(LO, HI, RTC, t);
+  static constexpr int kInRegion = G::in_region(LO, HI);
+  __device__ static __forceinline__ uint8_t* in_buf(uint8_t* smem, int b) { return smem + b * kInRegion; }
+  template <int T>
+  __device__ static __forceinline__ uint8_t* out_buf(uint8_t* smem, int b) {
+    return smem + CtxT::kOutBase0 + b * CtxT::kOutRegion + CtxT::template OutT<T>::off;
   }
 
   // ---------------- publisher warp: push out buffer `pb` (outputs of a batch of
   // `completed` items of stage ps) to the target rings, then retire the batch.
+  // Lane T handles target T's reservation, so every L2 round trip of a publish is taken
+  // once for all targets: tail reservations (1), free-slot check (1), bulk payload
+  // store + completion (1), sequence release.
   static __device__ void publish(const KArgs<F>& a, BlockShared& sh, uint8_t* smem, int pb, int ps, int completed,
                                  int lane) {
     Ctrl* c = a.c.ctrl;
     const bool timers = a.c.flags & FLAG_TIMERS;
     unsigned long long t0 = (timers && lane == 0) ? globaltimer() : 0;
-    int any = 0;
-    if (lane == 0) {
-      long long children = 0;
-      for (int t = 0; t < S; ++t) {
-        int n = sh.out_cnt[pb][t];
-        if (n > G::out_cap(LO, HI, RTC, t)) n = G::out_cap(LO, HI, RTC, t);
-        sh.out_cnt[pb][t] = n;
-        children += n;
+    int myn = 0;  // lane T: items for target T (clamped to the declared capacity)
+    static_for<0, S>([&](auto T_) {
+      constexpr int T = decltype(T_)::value;
+      constexpr int capT = CtxT::template cap<T>();
+      if (lane == T) {
+        const int n = sh.out_cnt[pb][T];
+        myn = n > capT ? capT : n;
       }
-      // Termination accounting: children are counted before they become visible;
-      // completions may be deferred (pending only stays conservatively high).
-      if (children > 0) {
-        long long d = children - completed + sh.acc_neg;
-        if (d != 0) atom_add(&c->pending.v, d);
-        sh.acc_neg = 0;
-        for (int t = 0; t < S; ++t) {
-          int n = sh.out_cnt[pb][t];
-          if (n == 0) continue;
-          sh.out_base[t] = atom_add(&c->tail[t].v, n);
-          sh.enq[t] += n;
-          if (a.c.flags & FLAG_DEPTH) {
-            unsigned long long h = ld_relaxed(&c->head[t].v);
-            unsigned long long dd = sh.out_base[t] + n - h;
-            if (dd > c->max_depth[t]) atomicMax(&c->max_depth[t], dd);
-          }
-        }
-        any = 1;
-      } else {
+    });
+    int children = myn;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) children += __shfl_xor_sync(0xffffffffu, children, o);
+    if (children == 0) {
+      if (lane == 0) {
         sh.acc_neg -= completed;
+        if (timers) sh.t_flush[ps] += globaltimer() - t0;
+      }
+      return;
+    }
+    // Termination accounting: children are counted in `pending` before they become
+    // visible (the release stores below order this reduction before them); completions
+    // may be deferred (pending only stays conservatively high).
+    if (lane == 0) {
+      const long long d = children - completed + sh.acc_neg;
+      if (d != 0) red_add(&c->pending.v, d);
+      sh.acc_neg = 0;
+    }
+    unsigned long long mybase = 0;
+    if (myn > 0) {
+      mybase = atom_add(&c->tail[lane].v, myn);
+      sh.enq[lane] += myn;
+      if (a.c.flags & FLAG_DEPTH) {
+        const unsigned long long h = ld_relaxed(&c->head[lane].v);
+        const unsigned long long dd = mybase + myn - h;
+        if (dd > c->max_depth[lane]) atomicMax(&c->max_depth[lane], dd);
       }
     }
-    any = __shfl_sync(0xffffffffu, any, 0);
-    if (any) {
-      __syncwarp();
+    // free-slot check: relaxed loads of every target's slots, then one acquire fence
+    bool free_ok = true;
+    static_for<0, S>([&](auto T_) {
+      constexpr int T = decltype(T_)::value;
+      if constexpr (CtxT::template cap<T>() > 0) {
+        const int n = __shfl_sync(0xffffffffu, myn, T);
+        const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
+        const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
+        for (int k = lane; k < n; k += 32) free_ok &= ld_relaxed(a.c.q[T].seq + ((base + k) & mask)) == base + k;
+      }
+    });
+    if (!__all_sync(0xffffffffu, free_ok)) {
+      // a consumer is still reading the previous lap of some slot (full ring): spin
       static_for<0, S>([&](auto T_) {
         constexpr int T = decltype(T_)::value;
-        if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
-          int n = sh.out_cnt[pb][T];
-          if (n > 0) {
-            wait_slots(a.c, a.c.q[T], sh.out_base[T], n, 1, lane);
-            __syncwarp();  // every slot of the range is free before any lane writes into it
-            copy_out<F::stride(T)>(a.c.q[T].slots, out_buf(smem, pb, T), sh.out_base[T], n, a.c.q[T].cap_log2, lane);
-          }
+        if constexpr (CtxT::template cap<T>() > 0) {
+          const int n = __shfl_sync(0xffffffffu, myn, T);
+          const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
+          if (n > 0) wait_slots(a.c, a.c.q[T], base, n, 1, lane);
         }
       });
-      __syncwarp();
-      // publish: seq = ticket + 1 (release; cumulative over the warp's payload stores)
-      static_for<0, S>([&](auto T_) {
-        constexpr int T = decltype(T_)::value;
-        if constexpr (G::out_cap(LO, HI, RTC, T) > 0) {
-          int n = sh.out_cnt[pb][T];
-          if (n > 0) {
-            const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
-            for (int k = lane; k < n; k += 32) {
-              unsigned long long t = sh.out_base[T] + k;
-              st_release(a.c.q[T].seq + (t & mask), t + 1);
+    }
+    fence_acq_rel_gpu();
+    __syncwarp();  // every slot of every range is free before any payload is written
+    bool bulk_used = false;
+    static_for<0, S>([&](auto T_) {
+      constexpr int T = decltype(T_)::value;
+      if constexpr (CtxT::template cap<T>() > 0) {
+        const int n = __shfl_sync(0xffffffffu, myn, T);
+        const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
+        if (n > 0) {
+          if constexpr (F::stride(T) % 16 == 0) {
+            if (lane == 0) {
+              fence_proxy_async_global();
+              bulk_out<F::stride(T)>(a.c.q[T].slots, out_buf<T>(smem, pb), base, n, a.c.q[T].cap_log2);
             }
+            bulk_used = true;
+          } else {
+            copy_out<F::stride(T)>(a.c.q[T].slots, out_buf<T>(smem, pb), base, n, a.c.q[T].cap_log2, lane);
           }
         }
-      });
-      __syncwarp();
-      if (lane == 0)
-        for (int t = 0; t < S; ++t)
-          if (sh.out_cnt[pb][t] > 0) atom_add(&c->count[t].v, sh.out_cnt[pb][t]);
+      }
+    });
+    if (bulk_used && lane == 0) {
+      bulk_commit_wait_all();       // payload written (and the smem batch read) ...
+      fence_proxy_async_global();   // ... and ordered before the generic release below
     }
-    if (lane == 0) {
-      for (int t = 0; t < S; ++t) sh.out_cnt[pb][t] = 0;
-      if (timers) sh.t_flush[ps] += globaltimer() - t0;
-    }
+    __syncwarp();
+    // publish: seq = ticket + 1 (release; cumulative over the warp's payload stores)
+    static_for<0, S>([&](auto T_) {
+      constexpr int T = decltype(T_)::value;
+      if constexpr (CtxT::template cap<T>() > 0) {
+        const int n = __shfl_sync(0xffffffffu, myn, T);
+        const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
+        const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
+        for (int k = lane; k < n; k += 32) st_release(a.c.q[T].seq + ((base + k) & mask), base + k + 1);
+      }
+    });
+    if (myn > 0) red_add(&c->count[lane].v, myn);
+    if (lane < S) sh.out_cnt[pb][lane] = 0;
+    if (timers && lane == 0) sh.t_flush[ps] += globaltimer() - t0;
   }
 
   // ---------------- fetcher warp: claim the next batch (task scheduler) and stage it
@@ -503,6 +663,20 @@ struct Runner {
   static __device__ void fetch(const KArgs<F>& a, BlockShared& sh, uint8_t* smem, int nb, bool quiescent, int lane) {
     Ctrl* c = a.c.ctrl;
     const bool timers = a.c.flags & FLAG_TIMERS;
+    constexpr int NS = HI - LO + 1;
+    // One warp-wide poll of every ring's `count` and seed cursor (one L2 round trip
+    // instead of one per stage); lane l looks at stage HI - l (downstream first).
+    long long avail = 0;
+    bool seeds_left = false;
+    if (a.g.mode != MODE_WAVE && lane < NS) {
+      const int s = HI - lane;
+      avail = (long long)ld_relaxed(&c->count[s].v);
+      const long long ns = a.c.q[s].n_seeds;
+      seeds_left = ns > 0 && (long long)ld_relaxed(&c->seed_head[s].v) < ns;
+    }
+    long long av[NS];
+    static_for<0, NS>([&](auto L_) { av[decltype(L_)::value] = __shfl_sync(0xffffffffu, avail, decltype(L_)::value); });
+    const unsigned seed_mask = __ballot_sync(0xffffffffu, seeds_left);
     if (lane == 0) {
       unsigned long long t0 = timers ? globaltimer() : 0;
       int got = 0, st = -1, fs = 0;
@@ -532,14 +706,20 @@ struct Runner {
       } else {
         // "Query queues in turn of priority" (Fig. 8a): downstream stages first (drains
         // the pipeline, bounds live items), rings before seeds.
-        for (int s = HI; s >= LO && !got; --s) {
-          got = claim_ring(c, s, a.g.batch[s], base);
-          if (got) { st = s; fs = 0; }
-        }
-        for (int s = HI; s >= LO && !got; --s) {
-          got = claim_seed(c, a.c.q[s], s, a.g.batch[s], base);
-          if (got) { st = s; fs = 1; }
-        }
+        static_for<0, NS>([&](auto L_) {
+          constexpr int l = decltype(L_)::value, s = HI - l;
+          if (!got && av[l] > 0) {
+            got = claim_ring_avail(c, s, a.g.batch[s], av[l], base);
+            if (got) { st = s; fs = 0; }
+          }
+        });
+        static_for<0, NS>([&](auto L_) {
+          constexpr int l = decltype(L_)::value, s = HI - l;
+          if (!got && ((seed_mask >> l) & 1u)) {
+            got = claim_seed(c, a.c.q[s], s, a.g.batch[s], base);
+            if (got) { st = s; fs = 1; }
+          }
+        });
         if (!got && quiescent) {
           // idle: retire deferred completions first, then test for termination
           if (sh.acc_neg != 0) {
@@ -568,14 +748,31 @@ struct Runner {
     const int s = sh.nx_stage;
     const unsigned long long base = sh.nx_base;
     uint8_t* dst = in_buf(smem, nb);
+    unsigned long long* mb = &sh.mbar[nb];
     static_for<LO, HI + 1>([&](auto S_) {
       constexpr int SS = decltype(S_)::value;
+      constexpr bool kBulk = F::stride(SS) % 16 == 0;
       if (s == SS) {
         const QueueDesc& q = a.c.q[SS];
+        if (kBulk) fence_proxy_async_smem();  // earlier generic writes of this buffer -> bulk writes
         if (sh.nx_seed) {
-          copy_seed_in<F::stride(SS)>(dst, q.seeds, base, n, lane);
+          if constexpr (kBulk) {
+            if (lane == 0) {
+              mbar_arrive_expect_tx(mb, (uint32_t)(n * F::stride(SS)));
+              bulk_g2s(dst, q.seeds + base * F::stride(SS), (uint32_t)(n * F::stride(SS)), mb);
+              mbar_wait(mb, sh.mbar_phase[nb]);
+              sh.mbar_phase[nb] ^= 1u;
+            }
+          } else {
+            copy_seed_in<F::stride(SS)>(dst, q.seeds, base, n, lane);
+          }
         } else {
-          wait_slots(a.c, q, base, n, 0, lane);
+          // published? relaxed loads first, one acquire fence; spin only if a producer lags
+          const unsigned long long mask = (1ull << q.cap_log2) - 1;
+          bool ok = true;
+          for (int k = lane; k < n; k += 32) ok &= ld_relaxed(q.seq + ((base + k) & mask)) == base + k + 1;
+          if (!__all_sync(0xffffffffu, ok)) wait_slots(a.c, q, base, n, 0, lane);
+          fence_acq_rel_gpu();
           __syncwarp();
           // warp-uniform decision (lanes may observe the abort flag at different times)
           const bool abort_now = __shfl_sync(0xffffffffu, aborted(a.c.ctrl) ? 1 : 0, 0) != 0;
@@ -586,9 +783,17 @@ struct Runner {
             }
             return;
           }
-          copy_in<F::stride(SS)>(dst, q.slots, base, n, q.cap_log2, lane);
+          if constexpr (kBulk) {
+            if (lane == 0) {
+              fence_proxy_async_global();  // acquired payload -> async-proxy reads
+              bulk_in<F::stride(SS)>(dst, q.slots, base, n, q.cap_log2, mb);
+              mbar_wait(mb, sh.mbar_phase[nb]);  // bytes landed: the slots' reads are done
+              sh.mbar_phase[nb] ^= 1u;
+            }
+          } else {
+            copy_in<F::stride(SS)>(dst, q.slots, base, n, q.cap_log2, lane);
+          }
           __syncwarp();
-          const unsigned long long mask = (1ull << q.cap_log2) - 1;
           for (int k = lane; k < n; k += 32) {
             unsigned long long t = base + k;
             st_release(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
@@ -626,6 +831,9 @@ struct Runner {
       if (s == SS) {
         record_trace(a, SS, items, n);
         if (threadIdx.x == 0) sh.deq[SS] += n;
+        if constexpr (RTC && SS < HI && fused_chain<F>(SS, HI)) {
+          FusedChain<F>::template run<SS, HI>(ctx, items, n);
+        } else {
         F::template exec<SS>(ctx, items, n);
         if constexpr (RTC && SS < HI) {
           // RTC (L11 §4.1): the remaining stages of the linear group, block-locally.
@@ -635,7 +843,8 @@ struct Runner {
             constexpr int TT = decltype(T_)::value;
             worker_sync();
             int m = sh.out_cnt[ctx.ob][TT];
-            if (m > G::out_cap(LO, HI, RTC, TT)) m = G::out_cap(LO, HI, RTC, TT);
+            constexpr int capT = CtxT::template cap<TT>();
+            if (m > capT) m = capT;
             if (m > 0) {
               const uint8_t* loc = ctx.template out_ptr<TT>(0);
               record_trace(a, TT, loc, m);
@@ -646,6 +855,8 @@ struct Runner {
             if (threadIdx.x == 0) sh.out_cnt[ctx.ob][TT] = 0;  // consumed locally
           });
         }
+        }
+        fence_proxy_async_smem();  // out-buffer writes -> the publisher's bulk reads
         if (timers && threadIdx.x == 0) sh.t_exec[SS] += globaltimer() - t0;
       }
     });
@@ -695,6 +906,10 @@ struct Runner {
       }
       sh.t_idle = 0;
       sh.rounds = 0;
+      for (int b = 0; b < 2; ++b) {
+        mbar_init(&sh.mbar[b], 1);
+        sh.mbar_phase[b] = 0;
+      }
       sh.acc_neg = 0;
       sh.done = 0;
       sh.nx_n = 0;

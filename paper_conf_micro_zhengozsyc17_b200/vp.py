@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libvp.so")
+LIB_PATH = os.path.join(_HERE, os.environ.get("VP_LIB_NAME", "libvp.so"))
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libvp.so not built at {LIB_PATH}: run `python -c 'import __graft_entry__ as g; g.build()'` "
