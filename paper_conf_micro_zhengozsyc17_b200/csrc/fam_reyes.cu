@@ -201,7 +201,13 @@ struct ReyesF {
   using Params = vp_reyes_params;
   static constexpr int stride(int s) { return s == SHADE ? (int)sizeof(RGrid) : (int)sizeof(RPatch); }
   static constexpr int threads_per_item(int s) { return s == BOUND ? 16 : s == SPLIT ? 16 : s == DICE ? 32 : 64; }
-  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 8 : 4; }
+  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 32 : 4; }
+  // Dice batches above 8 only in the fused RTC [Dice, Shade] kernel, whose grids stay in
+  // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
+  static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
+    return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
+  }
+  static constexpr int fused_local_cap(int, int, int) { return kThreads / 32; }
   static constexpr int default_batch(int s) { return max_batch(s); }
   static constexpr int fanout(int s, int t) {
     return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
@@ -526,16 +532,17 @@ struct ReyesF {
   template <int S0, int HI, class Ctx>
   static __device__ void exec_rtc_chain(Ctx& ctx, const uint8_t* items, int n) {
     static_assert(S0 == DICE && HI == SHADE, "only the [Dice, Shade] chain is fused");
-    static_assert(Ctx::template cap<SHADE>() >= max_batch(DICE), "one grid slot per diced patch");
+    static_assert(Ctx::template cap<SHADE>() >= kThreads / 32, "one grid slot per worker warp");
     const Params& p = ctx.params();
     const int lane = threadIdx.x & 31;
+    RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(threadIdx.x >> 5);
     for (int k = threadIdx.x >> 5; k < n; k += kThreads / 32) {
-      RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(k);
       dice_patch(p, (const RPatch*)(items + (size_t)k * sizeof(RPatch)), g, lane);
       __syncwarp();
       if (lane == 0) ctx.template note_local<SHADE>((const uint8_t*)g);
       shade_mp(p, g, lane);
       shade_mp(p, g, lane + 32);
+      __syncwarp();  // the slot is re-diced next
     }
   }
 

@@ -29,6 +29,7 @@ struct FamilyOps {
   virtual ~FamilyOps() {}
   virtual int stride(int s) const = 0;
   virtual int max_batch(int s) const = 0;
+  virtual int max_batch_k(int lo, int hi, bool rtc, int s) const = 0;  // per-kernel cap
   virtual int default_batch(int s) const = 0;
   virtual int threads_per_item(int s) const = 0;
   virtual int fanout(int s, int t) const = 0;
@@ -85,6 +86,7 @@ struct FamilyImpl final : FamilyOps {
   }
   int stride(int s) const override { return F::stride(s); }
   int max_batch(int s) const override { return F::max_batch(s); }
+  int max_batch_k(int lo, int hi, bool rtc, int s) const override { return kernel_max_batch<F>(lo, hi, rtc, s); }
   int default_batch(int s) const override { return F::default_batch(s); }
   int threads_per_item(int s) const override { return F::threads_per_item(s); }
   int fanout(int s, int t) const override { return F::fanout(s, t); }

@@ -487,6 +487,13 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       return fail(p, VP_ERR_INVALID, "unknown model %d", model);
   }
   if (rc != VP_OK) return rc;
+  // per-kernel batch caps (a stage is fetched by exactly one kernel or wave kind)
+  auto clamp_batch = [&](int lo, int hi, bool rtc) {
+    for (int s = lo; s <= hi; ++s) pl.batch[s] = std::min(pl.batch[s], p->fam->max_batch_k(lo, hi, rtc, s));
+  };
+  for (const KernelPlan& k : pl.kernels) clamp_batch(k.lo, k.hi, k.rtc);
+  for (int s : pl.kbk_stages) clamp_batch(s, s, false);
+  if (pl.wave_rtc) clamp_batch(0, S - 1, true);
   // Effective ring sizes.  Persistent plans drain continuously: a ring needs room for
   // the batches its producers hold (two out buffers per block), so it is sized to that
   // and stays L2-resident (no dirty-line write-back to HBM).  Host-driven waves (KBK,

@@ -207,61 +207,6 @@ __device__ __forceinline__ T ld_cg(const T* p) { return __ldcg(p); }
 template <class T>
 __device__ __forceinline__ void st_cg(T* p, T v) { __stcg(p, v); }
 
-// ------------------------------------------------------------------ constexpr graph helpers
-template <class F>
-struct Graph {
-  static constexpr int S = F::S;
-  static constexpr int fan(int s, int t) { return F::fanout(s, t); }
-  // true iff an edge s->t with LO <= t <= s <= HI exists (recursion / loop inside [LO,HI])
-  static constexpr bool has_back_edge(int lo, int hi) {
-    for (int s = lo; s <= hi; ++s)
-      for (int t = lo; t <= s; ++t)
-        if (fan(s, t) > 0) return true;
-    return false;
-  }
-  static constexpr bool rtc_legal(int lo, int hi) { return !has_back_edge(lo, hi) && F::rtc_ok(lo, hi); }
-  // items that can arrive block-locally at stage t of an RTC group [lo,hi]
-  static constexpr int rtc_in_cap(int lo, int t) {
-    if (t == lo) return F::max_batch(lo);
-    int n = F::max_batch(t);
-    int inc = 0;
-    for (int s = lo; s < t; ++s) inc += rtc_in_cap(lo, s) * fan(s, t);
-    return n > inc ? n : inc;
-  }
-  // out-buffer capacity (items) for target t in a kernel [lo,hi]
-  static constexpr int out_cap(int lo, int hi, bool rtc, int t) {
-    int c = 0;
-    for (int s = lo; s <= hi; ++s) {
-      if (fan(s, t) == 0) continue;
-      int n = rtc ? rtc_in_cap(lo, s) : F::max_batch(s);
-      int v = n * fan(s, t);
-      if (rtc) c += v;
-      else c = c > v ? c : v;
-    }
-    return c;
-  }
-  static constexpr int align128(int b) { return (b + 127) / 128 * 128; }
-  static constexpr int in_region(int lo, int hi) {
-    int b = 0;
-    for (int s = lo; s <= hi; ++s) {
-      int v = F::max_batch(s) * F::stride(s);
-      b = b > v ? b : v;
-    }
-    return align128(b);
-  }
-  static constexpr int out_off(int lo, int hi, bool rtc, int t) {
-    int off = 0;
-    for (int u = 0; u < t; ++u) off += align128(out_cap(lo, hi, rtc, u) * F::stride(u));
-    return off;
-  }
-  static constexpr int out_region(int lo, int hi, bool rtc) { return out_off(lo, hi, rtc, S); }
-  // double-buffered: in[2] | out[2] | scratch
-  static constexpr int in_base(int lo, int hi, int b) { return b * in_region(lo, hi); }
-  static constexpr int out_base(int lo, int hi, bool rtc, int b) { return 2 * in_region(lo, hi) + b * out_region(lo, hi, rtc); }
-  static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_base(lo, hi, rtc, 2); }
-  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + F::scratch_bytes(lo, hi); }
-};
-
 // A family may run an RTC chain [s, hi] itself (F::fused_rtc(s, hi) and
 // F::exec_rtc_chain<s, hi>), e.g. with warp-granular hand-off instead of block barriers.
 template <class F, class = void>
@@ -285,6 +230,80 @@ constexpr bool fused_chain(int s, int hi) {
   if constexpr (HasFusedRtc<F>::value) return F::fused_rtc(s, hi);
   else return false;
 }
+
+// A family may cap a stage's batch per kernel (F::kernel_max_batch(lo, hi, rtc, s)),
+// e.g. a larger batch only where its outputs stay block-local; default F::max_batch(s).
+template <class F, class = void>
+struct HasKernelMaxBatch : std::false_type {};
+template <class F>
+struct HasKernelMaxBatch<F, std::void_t<decltype(F::kernel_max_batch(0, 0, false, 0))>> : std::true_type {};
+template <class F>
+constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
+  if constexpr (HasKernelMaxBatch<F>::value) return F::kernel_max_batch(lo, hi, rtc, s);
+  else return F::max_batch(s);
+}
+template <class F>
+constexpr int fused_local_cap(int lo, int hi, int t) {
+  if constexpr (HasFusedRtc<F>::value) return F::fused_local_cap(lo, hi, t);
+  else return 0;
+}
+
+// ------------------------------------------------------------------ constexpr graph helpers
+template <class F>
+struct Graph {
+  static constexpr int S = F::S;
+  static constexpr int fan(int s, int t) { return F::fanout(s, t); }
+  // true iff an edge s->t with LO <= t <= s <= HI exists (recursion / loop inside [LO,HI])
+  static constexpr bool has_back_edge(int lo, int hi) {
+    for (int s = lo; s <= hi; ++s)
+      for (int t = lo; t <= s; ++t)
+        if (fan(s, t) > 0) return true;
+    return false;
+  }
+  static constexpr bool rtc_legal(int lo, int hi) { return !has_back_edge(lo, hi) && F::rtc_ok(lo, hi); }
+  static constexpr int mb(int lo, int hi, bool rtc, int s) { return kernel_max_batch<F>(lo, hi, rtc, s); }
+  // items that can arrive block-locally at stage t of an RTC group [lo,hi]
+  static constexpr int rtc_in_cap(int lo, int hi, int t) {
+    if (t == lo) return mb(lo, hi, true, lo);
+    int n = mb(lo, hi, true, t);
+    int inc = 0;
+    for (int s = lo; s < t; ++s) inc += rtc_in_cap(lo, hi, s) * fan(s, t);
+    return n > inc ? n : inc;
+  }
+  // out-buffer capacity (items) for target t in a kernel [lo,hi]
+  static constexpr int out_cap(int lo, int hi, bool rtc, int t) {
+    if (rtc && lo < t && t <= hi && fused_chain<F>(lo, hi)) return fused_local_cap<F>(lo, hi, t);
+    int c = 0;
+    for (int s = lo; s <= hi; ++s) {
+      if (fan(s, t) == 0) continue;
+      int n = rtc ? rtc_in_cap(lo, hi, s) : mb(lo, hi, false, s);
+      int v = n * fan(s, t);
+      if (rtc) c += v;
+      else c = c > v ? c : v;
+    }
+    return c;
+  }
+  static constexpr int align128(int b) { return (b + 127) / 128 * 128; }
+  static constexpr int in_region(int lo, int hi, bool rtc) {
+    int b = 0;
+    for (int s = lo; s <= hi; ++s) {
+      int v = mb(lo, hi, rtc, s) * F::stride(s);
+      b = b > v ? b : v;
+    }
+    return align128(b);
+  }
+  static constexpr int out_off(int lo, int hi, bool rtc, int t) {
+    int off = 0;
+    for (int u = 0; u < t; ++u) off += align128(out_cap(lo, hi, rtc, u) * F::stride(u));
+    return off;
+  }
+  static constexpr int out_region(int lo, int hi, bool rtc) { return out_off(lo, hi, rtc, S); }
+  // double-buffered: in[2] | out[2] | scratch
+  static constexpr int in_base(int lo, int hi, bool rtc, int b) { return b * in_region(lo, hi, rtc); }
+  static constexpr int out_base(int lo, int hi, bool rtc, int b) { return 2 * in_region(lo, hi, rtc) + b * out_region(lo, hi, rtc); }
+  static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_base(lo, hi, rtc, 2); }
+  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + F::scratch_bytes(lo, hi); }
+};
 
 // ------------------------------------------------------------------ per-block context
 struct BlockShared {
@@ -541,7 +560,7 @@ struct Runner {
   static constexpr int S = F::S;
   static constexpr int W_FETCH = kWarpsW, W_PUBLISH = kWarpsW + 1;
 
-  static constexpr int kInRegion = G::in_region(LO, HI);
+  static constexpr int kInRegion = G::in_region(LO, HI, RTC);
   __device__ static __forceinline__ uint8_t* in_buf(uint8_t* smem, int b) { return smem + b * kInRegion; }
   template <int T>
   __device__ static __forceinline__ uint8_t* out_buf(uint8_t* smem, int b) {
