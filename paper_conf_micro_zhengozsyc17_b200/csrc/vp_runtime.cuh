@@ -614,7 +614,8 @@ struct Runner {
         if (dd > c->max_depth[lane]) atomicMax(&c->max_depth[lane], dd);
       }
     }
-    // free-slot check: relaxed loads of every target's slots, then one acquire fence
+    // free-slot check: acquire loads of every target's slots (LDG + L1 invalidate, no
+    // membar), all issued before any is tested
     bool free_ok = true;
     static_for<0, S>([&](auto T_) {
       constexpr int T = decltype(T_)::value;
@@ -622,7 +623,7 @@ struct Runner {
         const int n = __shfl_sync(0xffffffffu, myn, T);
         const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
         const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
-        for (int k = lane; k < n; k += 32) free_ok &= ld_relaxed(a.c.q[T].seq + ((base + k) & mask)) == base + k;
+        for (int k = lane; k < n; k += 32) free_ok &= ld_acquire(a.c.q[T].seq + ((base + k) & mask)) == base + k;
       }
     });
     if (!__all_sync(0xffffffffu, free_ok)) {
@@ -636,7 +637,6 @@ struct Runner {
         }
       });
     }
-    fence_acq_rel_gpu();
     __syncwarp();  // every slot of every range is free before any payload is written
     bool bulk_used = false;
     static_for<0, S>([&](auto T_) {
@@ -662,14 +662,16 @@ struct Runner {
       fence_proxy_async_global();   // ... and ordered before the generic release below
     }
     __syncwarp();
-    // publish: seq = ticket + 1 (release; cumulative over the warp's payload stores)
+    // publish: seq = ticket + 1.  One release fence for every target's sequence stores
+    // (fence + relaxed stores = the release pattern; one membar per publish).
+    fence_acq_rel_gpu();
     static_for<0, S>([&](auto T_) {
       constexpr int T = decltype(T_)::value;
       if constexpr (CtxT::template cap<T>() > 0) {
         const int n = __shfl_sync(0xffffffffu, myn, T);
         const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
         const unsigned long long mask = (1ull << a.c.q[T].cap_log2) - 1;
-        for (int k = lane; k < n; k += 32) st_release(a.c.q[T].seq + ((base + k) & mask), base + k + 1);
+        for (int k = lane; k < n; k += 32) st_relaxed(a.c.q[T].seq + ((base + k) & mask), base + k + 1);
       }
     });
     if (myn > 0) red_add(&c->count[lane].v, myn);
@@ -786,12 +788,11 @@ struct Runner {
             copy_seed_in<F::stride(SS)>(dst, q.seeds, base, n, lane);
           }
         } else {
-          // published? relaxed loads first, one acquire fence; spin only if a producer lags
+          // published? acquire loads (no membar); spin only if a producer lags
           const unsigned long long mask = (1ull << q.cap_log2) - 1;
           bool ok = true;
-          for (int k = lane; k < n; k += 32) ok &= ld_relaxed(q.seq + ((base + k) & mask)) == base + k + 1;
+          for (int k = lane; k < n; k += 32) ok &= ld_acquire(q.seq + ((base + k) & mask)) == base + k + 1;
           if (!__all_sync(0xffffffffu, ok)) wait_slots(a.c, q, base, n, 0, lane);
-          fence_acq_rel_gpu();
           __syncwarp();
           // warp-uniform decision (lanes may observe the abort flag at different times)
           const bool abort_now = __shfl_sync(0xffffffffu, aborted(a.c.ctrl) ? 1 : 0, 0) != 0;
@@ -813,9 +814,10 @@ struct Runner {
             copy_in<F::stride(SS)>(dst, q.slots, base, n, q.cap_log2, lane);
           }
           __syncwarp();
+          fence_acq_rel_gpu();  // the batch's reads before the slots' release (one membar)
           for (int k = lane; k < n; k += 32) {
             unsigned long long t = base + k;
-            st_release(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
+            st_relaxed(q.seq + (t & mask), t + (1ull << q.cap_log2));  // free for ticket t + cap
           }
         }
       }

@@ -225,10 +225,12 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
     }
   }
   R.candidates_total = (int)shapes.size() + 2;
+  // Phase 1 runs with a lenient limit (2x the best so far): a shape whose seed split is
+  // off still gets a time, so it can be ranked and refined in phase 2.
   std::vector<std::pair<double, Shape>> scored;
   for (const Shape& sh : shapes) {
     if (elapsed() > budget_s || R.candidates_run >= max_cand) break;
-    double t = consider(to_config(p, S, sh), mintime);
+    double t = consider(to_config(p, S, sh), 2.0 * mintime);
     if (t > 0) scored.push_back({t, sh});
   }
   if (((allowed >> VP_GROUP_RTC) & 1) && vpi_rtc_legal(p, 0, S - 1) && elapsed() < budget_s) {
@@ -241,7 +243,7 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
 
   // ---- phase 2: SM-split and batch refinement around the best phase-1 shapes
   std::sort(scored.begin(), scored.end(), [](const auto& a, const auto& b) { return a.first < b.first; });
-  const int top = std::min<int>(3, (int)scored.size());
+  const int top = std::min<int>(4, (int)scored.size());
   for (int k = 0; k < top; ++k) {
     Shape base = scored[k].second;
     std::vector<Shape> nb;
