@@ -194,6 +194,14 @@ __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, lo
   }
 }
 
+// Scratch of the fused [Dice, Shade] chain.
+struct ChainScratch {
+  float4 W[4][kNP];            // W[a][g] = {Bu[a]Bv[0], .., Bu[a]Bv[3]} at grid point g = 9i + j
+  float4 M[kWarpsW][4];        // per-warp copy of the patch's frame matrix (rows)
+  uint8_t list[kWarpsW][64];   // per-warp compacted list of pixel-covering micropolygons
+  int ready;                   // W built (scratch is zeroed at block start)
+};
+
 struct ReyesF {
   static constexpr int S = 4;
   static constexpr int BOUND = 0, SPLIT = 1, DICE = 2, SHADE = 3;
@@ -213,7 +221,7 @@ struct ReyesF {
     return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
   }
   static constexpr bool rtc_ok(int, int) { return true; }
-  static constexpr int scratch_bytes(int, int) { return 0; }
+  static constexpr int scratch_bytes(int lo, int hi) { return (lo == DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0; }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
   static constexpr int min_blocks(int, int, bool) { return VP_REYES_MINB; }
@@ -526,23 +534,117 @@ struct ReyesF {
 
   // -------------------------------------------------------------- RTC [Dice, Shade]
   // Warp-granular run-to-completion: each warp dices one patch into a
-  // block-local grid slot and shades it itself (2 micropolygons per lane), so the chain
-  // needs no block barrier between the two stages.
+  // block-local grid slot and shades it itself, so the chain needs no block barrier
+  // between the two stages.  The same arithmetic as dice_patch / shade_mp, restaged:
+  // the Bernstein products Bu[a]*Bv[b] come from a per-block table (identical float
+  // products), the frame matrix from shared memory, and only the micropolygons whose box
+  // holds a pixel centre (~1 in 4 at config 5) are shaded, compacted onto the warp's lanes.
   static constexpr bool fused_rtc(int s, int hi) { return s == DICE && hi == SHADE; }
+
+  static __device__ __forceinline__ void dice_patch_tab(const Params& p, const RPatch* P, RGrid* out, int lane,
+                                                        const ChainScratch& cs, const float4* Mr) {
+    for (int g = lane; g < kNP; g += 32) {
+      float x = 0.0f, y = 0.0f, z = 0.0f;
+#pragma unroll
+      for (int a = 0; a < 4; ++a) {
+        const float4 w4 = cs.W[a][g];
+        const float w[4] = {w4.x, w4.y, w4.z, w4.w};
+#pragma unroll
+        for (int b = 0; b < 4; ++b) {
+          const float4 cp = P->cp[4 * a + b];
+          x = x + w[b] * cp.x;
+          y = y + w[b] * cp.y;
+          z = z + w[b] * cp.z;
+        }
+      }
+      float c[4];
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {
+        const float4 m = Mr[r];
+        float acc = m.x * x;
+        acc = acc + m.y * y;
+        acc = acc + m.z * z;
+        acc = acc + m.w * 1.0f;
+        c[r] = acc;
+      }
+      float sx, sy, zs;
+      screen(p, make_float4(c[0], c[1], c[2], c[3]), sx, sy, zs);
+      out->g[0][g] = x;
+      out->g[1][g] = y;
+      out->g[2][g] = z;
+      const float X = sx * 256.0f, Y = sy * 256.0f;
+      const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
+      out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
+      out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
+      out->g[5][g] = zs;
+    }
+    if (lane == 0) {
+      out->id = P->id;
+      out->path = P->path;
+      out->depth = P->depth;
+      out->dirs = P->dirs;
+    }
+  }
+
+  // shade_mp's early exit alone: does micropolygon q's box hold a pixel centre?
+  static __device__ __forceinline__ bool mp_box(const Params& p, const RGrid* Gd, int q) {
+    if ((Gd->id >> 12) >= (uint32_t)p.n_frames) return false;
+    const int i = q >> 3, j = q & 7;
+    const int gi[4] = {i * kNG + j, (i + 1) * kNG + j, (i + 1) * kNG + j + 1, i * kNG + j + 1};
+    int vx[4], vy[4];
+    bool ok = true;
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      vx[v] = __float_as_int(Gd->g[3][gi[v]]);
+      vy[v] = __float_as_int(Gd->g[4][gi[v]]);
+      if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
+    }
+    const int xmin = min(min(vx[0], vx[1]), min(vx[2], vx[3])), xmax = max(max(vx[0], vx[1]), max(vx[2], vx[3]));
+    const int ymin = min(min(vy[0], vy[1]), min(vy[2], vy[3])), ymax = max(max(vy[0], vy[1]), max(vy[2], vy[3]));
+    const int px0 = max(-((128 - xmin) >> 8), 0), px1 = min((xmax - 128) >> 8, p.W - 1);
+    const int py0 = max(-((128 - ymin) >> 8), 0), py1 = min((ymax - 128) >> 8, p.H - 1);
+    return ok && px0 <= px1 && py0 <= py1;
+  }
+
   template <int S0, int HI, class Ctx>
   static __device__ void exec_rtc_chain(Ctx& ctx, const uint8_t* items, int n) {
     static_assert(S0 == DICE && HI == SHADE, "only the [Dice, Shade] chain is fused");
-    static_assert(Ctx::template cap<SHADE>() >= kThreads / 32, "one grid slot per worker warp");
+    static_assert(Ctx::template cap<SHADE>() >= kWarpsW, "one grid slot per worker warp");
     const Params& p = ctx.params();
-    const int lane = threadIdx.x & 31;
-    RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(threadIdx.x >> 5);
-    for (int k = threadIdx.x >> 5; k < n; k += kThreads / 32) {
-      dice_patch(p, (const RPatch*)(items + (size_t)k * sizeof(RPatch)), g, lane);
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    ChainScratch& cs = *(ChainScratch*)ctx.scratch();
+    if (!cs.ready) {  // first batch of this block (uniform: read before anyone sets it)
+      for (int e = threadIdx.x; e < 4 * kNP; e += kThreads) {
+        const int a = e / kNP, g = e - a * kNP, i = g / kNG, j = g - i * kNG;
+        float Bu[4], Bv[4];
+        bernstein((float)i * 0.125f, Bu);
+        bernstein((float)j * 0.125f, Bv);
+        cs.W[a][g] = make_float4(Bu[a] * Bv[0], Bu[a] * Bv[1], Bu[a] * Bv[2], Bu[a] * Bv[3]);
+      }
+      worker_sync();
+      if (threadIdx.x == 0) cs.ready = 1;
+    }
+    RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(warp);
+    float* Mw = (float*)cs.M[warp];
+    uint8_t* list = cs.list[warp];
+    for (int k = warp; k < n; k += kWarpsW) {
+      const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
+      uint32_t frame = P->id >> 12;
+      if (frame >= (uint32_t)p.n_frames) frame = 0;
+      if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+      __syncwarp();
+      dice_patch_tab(p, P, g, lane, cs, cs.M[warp]);
       __syncwarp();
       if (lane == 0) ctx.template note_local<SHADE>((const uint8_t*)g);
-      shade_mp(p, g, lane);
-      shade_mp(p, g, lane + 32);
-      __syncwarp();  // the slot is re-diced next
+      const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
+      const unsigned m0 = __ballot_sync(0xffffffffu, a0), m1 = __ballot_sync(0xffffffffu, a1);
+      const unsigned lt = (1u << lane) - 1u;
+      const int c0 = __popc(m0), tot = c0 + __popc(m1);
+      if (a0) list[__popc(m0 & lt)] = (uint8_t)lane;
+      if (a1) list[c0 + __popc(m1 & lt)] = (uint8_t)(lane + 32);
+      __syncwarp();
+      for (int t = lane; t < tot; t += 32) shade_mp(p, g, list[t]);
+      __syncwarp();  // the slot, the matrix and the list are rewritten next
     }
   }
 

@@ -968,6 +968,9 @@ struct Runner {
     __shared__ BlockShared sh;
     if (!admit(a, sh)) return;
     CtxT ctx(a, smem, sh);
+    if constexpr (F::scratch_bytes(LO, HI) > 0) {  // family scratch starts zeroed
+      for (int i = threadIdx.x; i < F::scratch_bytes(LO, HI) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+    }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // prologue: stage the first batch into in[0]
     if (warp == W_FETCH) fetch(a, sh, smem, 0, true, lane);

@@ -5,6 +5,8 @@ so co-running persistent groups cannot be captured together).
   rtc_dice  : the [Dice,Shade] RTC kernel alone: every seed patch is inserted into the
               Dice queue, the [Bound,Split] group is an (idle) KBK group
   kbk       : one launch per stage per wave
+  rtc_leaf  : the [Dice,Shade] RTC kernel alone on representative leaf patches
+              (tools/reyes_leaves.py: numpy approximation of the Bound/Split recursion)
 """
 import argparse
 import os
@@ -42,6 +44,15 @@ elif args.target == "kbk":
 elif args.target == "rtc_dice":
     rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
     rp.p.insert(2, rp.seeds_dev, n=scene.seeds.size)
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_KBK, 0, 8), (2, 3, vp.GROUP_RTC, 8, nsm)], nsm))
+elif args.target == "rtc_leaf":
+    import numpy as np
+    sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
+    import reyes_leaves
+    lv = np.ascontiguousarray(reyes_leaves.leaves(scene, args.frames))
+    leaves_dev = torch.from_numpy(lv.view(np.uint8).reshape(-1)).cuda()
+    rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
+    rp.p.insert(2, leaves_dev, n=lv.size)
     rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_KBK, 0, 8), (2, 3, vp.GROUP_RTC, 8, nsm)], nsm))
 else:
     raise SystemExit(f"unknown target {args.target}")
