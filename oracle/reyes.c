@@ -13,7 +13,8 @@
  *  Split dir: L_u = max_b(|sx[3][b]-sx[0][b]| + |sy[3][b]-sy[0][b]|), L_v likewise
  *             along b; split u iff L_u >= L_v (tie -> u).
  *  Split:     de Casteljau at t = 1/2 on the 4 curves along that direction.
- *  Dice:      (G+1)^2 = 81 points, Bernstein basis, sum a outer / b inner, project.
+ *  Dice:      (G+1)^2 = 81 points, separable Bernstein evaluation (v-sums over b into
+ *             the u-curve points C_a(v_j), then u-sums over a), project.
  *  Shade:     per micropolygon q = (i,j): n = cross(p10-p00, p01-p00),
  *             s = 0.1 + 0.9*max(0, n.L/|n|) (0.1 if |n| = 0); coverage of the two
  *             triangles (v00,v10,v11), (v00,v11,v01) at pixel centres, Q8 fixed point,
@@ -152,23 +153,35 @@ static void bernstein(float t, float B[4]) {
   B[3] = (t * t) * t;
 }
 
-/* Dice: grid[0..5][g], g = i*9 + j, rows x,y,z (object) and sx,sy,zs (screen). */
+/* Dice: grid[0..5][g], g = i*9 + j, rows x,y,z (object) and sx,sy,zs (screen).
+ * Reading R-R7: the tensor-product Bezier surface S(u,v) = sum_a B_a(u) sum_b B_b(v) P_ab
+ * evaluated in its separable (two-stage) form at u_i = i/8, v_j = j/8: first the four
+ * u-curve control points at v_j, C_a(v_j) = sum_b B_b(v_j) P_ab (b = 0..3 in order), then
+ * S(u_i, v_j) = sum_a B_a(u_i) C_a(v_j) (a = 0..3 in order); every sum starts at 0. */
 void orc_reyes_dice(const orc_reyes_scene* sc, const orc_patch* p, float grid[6][81]) {
   const float* M = frame_M(sc, p->id);
+  float C[4][NG][3];
+  for (int a = 0; a < 4; ++a)
+    for (int j = 0; j < NG; ++j) {
+      float Bv[4];
+      bernstein((float)j * 0.125f, Bv);
+      for (int k = 0; k < 3; ++k) {
+        float acc = 0.0f;
+        for (int b = 0; b < 4; ++b) acc = acc + Bv[b] * p->cp[4 * a + b][k];
+        C[a][j][k] = acc;
+      }
+    }
   for (int i = 0; i < NG; ++i) {
     float Bu[4];
     bernstein((float)i * 0.125f, Bu);
     for (int j = 0; j < NG; ++j) {
-      float Bv[4];
-      bernstein((float)j * 0.125f, Bv);
-      float x = 0.0f, y = 0.0f, z = 0.0f;
-      for (int a = 0; a < 4; ++a)
-        for (int b = 0; b < 4; ++b) {
-          float w = Bu[a] * Bv[b];
-          x = x + w * p->cp[4 * a + b][0];
-          y = y + w * p->cp[4 * a + b][1];
-          z = z + w * p->cp[4 * a + b][2];
-        }
+      float xyz[3];
+      for (int k = 0; k < 3; ++k) {
+        float acc = 0.0f;
+        for (int a = 0; a < 4; ++a) acc = acc + Bu[a] * C[a][j][k];
+        xyz[k] = acc;
+      }
+      const float x = xyz[0], y = xyz[1], z = xyz[2];
       float q[4] = {x, y, z, 1.0f}, c[4];
       orc_reyes_project(M, q, c);
       int g = i * NG + j;

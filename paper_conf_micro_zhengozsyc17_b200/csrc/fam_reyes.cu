@@ -196,10 +196,8 @@ __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, lo
 
 // Scratch of the fused [Dice, Shade] chain.
 struct ChainScratch {
-  float4 W[4][kNP];            // W[a][g] = {Bu[a]Bv[0], .., Bu[a]Bv[3]} at grid point g = 9i + j
   float4 M[kWarpsW][4];        // per-warp copy of the patch's frame matrix (rows)
   uint8_t list[kWarpsW][64];   // per-warp compacted list of pixel-covering micropolygons
-  int ready;                   // W built (scratch is zeroed at block start)
 };
 
 struct ReyesF {
@@ -374,39 +372,87 @@ struct ReyesF {
   }
 
   // -------------------------------------------------------------- Dice (warp/patch)
-  // One warp evaluates the 9x9 grid of patch P into `out` (reading R-R7/R-R9).
-  static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane) {
+  // One warp evaluates the 9x9 grid of patch P into `out` (readings R-R7, R-R9): the
+  // separable Bernstein form, the 36 u-curve points C_a(v_j) staged in the (not yet
+  // written) screen rows of `out`, then the 81 surface points, projection and Q8 snap.
+  // Ms: the frame matrix rows in shared memory (fused chain), else read from p.M.
+  template <bool kSmemM = false>
+  static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
+                                                    const float4* Ms = nullptr) {
     uint32_t frame = P->id >> 12;
     if (frame >= (uint32_t)p.n_frames) frame = 0;
     const float* M = p.M + 16 * (size_t)frame;
-    for (int g = lane; g < kNP; g += 32) {
-      const int i = g / kNG, j = g - i * kNG;
-      float Bu[4], Bv[4];
-      bernstein((float)i * 0.125f, Bu);
+    for (int e = lane; e < 4 * kNG; e += 32) {  // C_a(v_j), e = 9a + j
+      const int a = e / kNG, j = e - a * kNG;
+      float Bv[4];
       bernstein((float)j * 0.125f, Bv);
-      float x = 0.0f, y = 0.0f, z = 0.0f;
+      float cx = 0.0f, cy = 0.0f, cz = 0.0f;
 #pragma unroll
-      for (int a = 0; a < 4; ++a)
+      for (int b = 0; b < 4; ++b) {
+        const float4 cp = P->cp[4 * a + b];
+        cx = cx + Bv[b] * cp.x;
+        cy = cy + Bv[b] * cp.y;
+        cz = cz + Bv[b] * cp.z;
+      }
+      out->g[3][e] = cx;
+      out->g[4][e] = cy;
+      out->g[5][e] = cz;
+    }
+    __syncwarp();
+    float xs[3], ys[3], zs_[3];
 #pragma unroll
-        for (int b = 0; b < 4; ++b) {
-          const float w = Bu[a] * Bv[b];
-          const float4 cp = P->cp[4 * a + b];
-          x = x + w * cp.x;
-          y = y + w * cp.y;
-          z = z + w * cp.z;
+    for (int r = 0; r < 3; ++r) {
+      const int g = lane + 32 * r;
+      if (g < kNP) {
+        const int i = g / kNG, j = g - i * kNG;
+        float Bu[4];
+        bernstein((float)i * 0.125f, Bu);
+        float x = 0.0f, y = 0.0f, z = 0.0f;
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+          x = x + Bu[a] * out->g[3][a * kNG + j];
+          y = y + Bu[a] * out->g[4][a * kNG + j];
+          z = z + Bu[a] * out->g[5][a * kNG + j];
         }
-      float4 c = project(M, x, y, z, 1.0f);
-      float sx, sy, zs;
-      screen(p, c, sx, sy, zs);
-      out->g[0][g] = x;
-      out->g[1][g] = y;
-      out->g[2][g] = z;
-      // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
-      const float X = sx * 256.0f, Y = sy * 256.0f;
-      const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
-      out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
-      out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
-      out->g[5][g] = zs;
+        xs[r] = x;
+        ys[r] = y;
+        zs_[r] = z;
+      }
+    }
+    __syncwarp();  // every C read before the screen rows are written
+#pragma unroll
+    for (int r = 0; r < 3; ++r) {
+      const int g = lane + 32 * r;
+      if (g < kNP) {
+        const float x = xs[r], y = ys[r], z = zs_[r];
+        float4 c;
+        if constexpr (kSmemM) {
+          float cc[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const float4 m = Ms[q];
+            float acc = m.x * x;
+            acc = acc + m.y * y;
+            acc = acc + m.z * z;
+            acc = acc + m.w * 1.0f;
+            cc[q] = acc;
+          }
+          c = make_float4(cc[0], cc[1], cc[2], cc[3]);
+        } else {
+          c = project(M, x, y, z, 1.0f);
+        }
+        float sx, sy, zs;
+        screen(p, c, sx, sy, zs);
+        out->g[0][g] = x;
+        out->g[1][g] = y;
+        out->g[2][g] = z;
+        // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
+        const float X = sx * 256.0f, Y = sy * 256.0f;
+        const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
+        out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
+        out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
+        out->g[5][g] = zs;
+      }
     }
     if (lane == 0) {
       out->id = P->id;
@@ -536,55 +582,9 @@ struct ReyesF {
   // Warp-granular run-to-completion: each warp dices one patch into a
   // block-local grid slot and shades it itself, so the chain needs no block barrier
   // between the two stages.  The same arithmetic as dice_patch / shade_mp, restaged:
-  // the Bernstein products Bu[a]*Bv[b] come from a per-block table (identical float
-  // products), the frame matrix from shared memory, and only the micropolygons whose box
+  // the frame matrix comes from shared memory, and only the micropolygons whose box
   // holds a pixel centre (~1 in 4 at config 5) are shaded, compacted onto the warp's lanes.
   static constexpr bool fused_rtc(int s, int hi) { return s == DICE && hi == SHADE; }
-
-  static __device__ __forceinline__ void dice_patch_tab(const Params& p, const RPatch* P, RGrid* out, int lane,
-                                                        const ChainScratch& cs, const float4* Mr) {
-    for (int g = lane; g < kNP; g += 32) {
-      float x = 0.0f, y = 0.0f, z = 0.0f;
-#pragma unroll
-      for (int a = 0; a < 4; ++a) {
-        const float4 w4 = cs.W[a][g];
-        const float w[4] = {w4.x, w4.y, w4.z, w4.w};
-#pragma unroll
-        for (int b = 0; b < 4; ++b) {
-          const float4 cp = P->cp[4 * a + b];
-          x = x + w[b] * cp.x;
-          y = y + w[b] * cp.y;
-          z = z + w[b] * cp.z;
-        }
-      }
-      float c[4];
-#pragma unroll
-      for (int r = 0; r < 4; ++r) {
-        const float4 m = Mr[r];
-        float acc = m.x * x;
-        acc = acc + m.y * y;
-        acc = acc + m.z * z;
-        acc = acc + m.w * 1.0f;
-        c[r] = acc;
-      }
-      float sx, sy, zs;
-      screen(p, make_float4(c[0], c[1], c[2], c[3]), sx, sy, zs);
-      out->g[0][g] = x;
-      out->g[1][g] = y;
-      out->g[2][g] = z;
-      const float X = sx * 256.0f, Y = sy * 256.0f;
-      const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
-      out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
-      out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
-      out->g[5][g] = zs;
-    }
-    if (lane == 0) {
-      out->id = P->id;
-      out->path = P->path;
-      out->depth = P->depth;
-      out->dirs = P->dirs;
-    }
-  }
 
   // shade_mp's early exit alone: does micropolygon q's box hold a pixel centre?
   static __device__ __forceinline__ bool mp_box(const Params& p, const RGrid* Gd, int q) {
@@ -613,17 +613,6 @@ struct ReyesF {
     const Params& p = ctx.params();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     ChainScratch& cs = *(ChainScratch*)ctx.scratch();
-    if (!cs.ready) {  // first batch of this block (uniform: read before anyone sets it)
-      for (int e = threadIdx.x; e < 4 * kNP; e += kThreads) {
-        const int a = e / kNP, g = e - a * kNP, i = g / kNG, j = g - i * kNG;
-        float Bu[4], Bv[4];
-        bernstein((float)i * 0.125f, Bu);
-        bernstein((float)j * 0.125f, Bv);
-        cs.W[a][g] = make_float4(Bu[a] * Bv[0], Bu[a] * Bv[1], Bu[a] * Bv[2], Bu[a] * Bv[3]);
-      }
-      worker_sync();
-      if (threadIdx.x == 0) cs.ready = 1;
-    }
     RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(warp);
     float* Mw = (float*)cs.M[warp];
     uint8_t* list = cs.list[warp];
@@ -633,7 +622,7 @@ struct ReyesF {
       if (frame >= (uint32_t)p.n_frames) frame = 0;
       if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
       __syncwarp();
-      dice_patch_tab(p, P, g, lane, cs, cs.M[warp]);
+      dice_patch<true>(p, P, g, lane, cs.M[warp]);
       __syncwarp();
       if (lane == 0) ctx.template note_local<SHADE>((const uint8_t*)g);
       const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
