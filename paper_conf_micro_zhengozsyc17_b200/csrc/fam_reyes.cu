@@ -219,7 +219,9 @@ struct ReyesF {
     return (s == BOUND && (t == SPLIT || t == DICE)) ? 1 : (s == SPLIT && t == BOUND) ? 2 : (s == DICE && t == SHADE) ? 1 : 0;
   }
   static constexpr bool rtc_ok(int, int) { return true; }
-  static constexpr int scratch_bytes(int lo, int hi) { return (lo == DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0; }
+  // every kernel whose range ends in [Dice, Shade] may run the fused chain (an RTC
+  // kernel [Split..Shade] fuses its Dice batches too), so each reserves the chain scratch
+  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0; }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
   static constexpr int min_blocks(int, int, bool) { return VP_REYES_MINB; }

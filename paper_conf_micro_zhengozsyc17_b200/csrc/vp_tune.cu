@@ -63,7 +63,9 @@ vp_config to_config(void* p, int S, const Shape& sh) {
 
 // timeoutexec(mintime, config): configure, one warm run with a generous limit, then
 // `reps` runs with the watchdog at `limit_ms`; best device ms, or < 0 (invalid / timeout).
-double timeoutexec(void* p, const vp_config& c, double limit_ms, int reps, bool* timed_out) {
+// A CUDA error (e.g. an illegal address) is sticky for the context: *fatal is set and
+// the search stops instead of ranking the remaining candidates on a dead context.
+double timeoutexec(void* p, const vp_config& c, double limit_ms, int reps, bool* timed_out, vp_status* fatal) {
   *timed_out = false;
   if (vp_configure_config(p, &c) != VP_OK) return -1.0;
   vp_run_stats st;
@@ -71,6 +73,7 @@ double timeoutexec(void* p, const vp_config& c, double limit_ms, int reps, bool*
   vp_status rc = vp_run(p, nullptr, &st);
   if (rc != VP_OK) {
     *timed_out = rc == VP_ERR_TIMEOUT;
+    if (rc == VP_ERR_CUDA) *fatal = rc;
     return -1.0;
   }
   double best = 1e30;
@@ -79,6 +82,7 @@ double timeoutexec(void* p, const vp_config& c, double limit_ms, int reps, bool*
     rc = vp_run(p, nullptr, &st);
     if (rc != VP_OK) {
       *timed_out = rc == VP_ERR_TIMEOUT;
+      if (rc == VP_ERR_CUDA) *fatal = rc;
       return -1.0;
     }
     best = std::min(best, st.device_ms);
@@ -120,17 +124,20 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
   memset(&best, 0, sizeof(best));
   bool have_best = false;
   const bool debug = getenv("VP_TUNE_DEBUG") != nullptr;
+  vp_status fatal = VP_OK;
   auto consider = [&](const vp_config& c, double limit) -> double {
     bool to = false;
+    if (fatal != VP_OK) return -1.0;
     if (debug) {
       char buf[4096];
       vp_config_to_string(&c, buf, sizeof(buf));
       fprintf(stderr, "[vp_tune %.2fs] try limit=%.3fms %.160s\n", elapsed(), limit, buf);
       fflush(stderr);
     }
-    double t = timeoutexec(p, c, limit, reps, &to);
+    double t = timeoutexec(p, c, limit, reps, &to, &fatal);
     if (debug) {
-      fprintf(stderr, "[vp_tune %.2fs]   -> %.3f ms%s\n", elapsed(), t, to ? " (timeout)" : "");
+      fprintf(stderr, "[vp_tune %.2fs]   -> %.3f ms%s%s\n", elapsed(), t, to ? " (timeout)" : "",
+              fatal != VP_OK ? " (CUDA error: search stopped)" : "");
       fflush(stderr);
     }
     R.candidates_run++;
@@ -284,6 +291,7 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
   }
 
   vp_set_timeout(p, saved_timeout);
+  if (fatal != VP_OK) return fatal;  // vp_last_error holds the CUDA message
   if (!have_best) {
     vpi_set_error(p, "autotune: no candidate ran successfully");
     return VP_ERR_CUDA;

@@ -41,6 +41,9 @@ def configure(vp, rp, model):
     elif model == "hybrid_4":             # each stage its own group: coarse pipeline of groups
         rp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, 30), (1, 1, vp.GROUP_MEGA, 30, 50),
                                                  (2, 2, vp.GROUP_MEGA, 50, 100), (3, 3, vp.GROUP_MEGA, 100, nsm)], nsm))
+    elif model == "hybrid_mega_rtc3":     # [Bound] megakernel | [Split,Dice,Shade] RTC (fused Dice batches)
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, 24), (1, 3, vp.GROUP_RTC, 24, nsm)], nsm,
+                                                batch=[32, 16, 32, 4]))
     else:
         raise ValueError(model)
 
@@ -63,7 +66,8 @@ def check_against_oracle(orc, scene, rp, st, trace=None):
     return ref
 
 
-MODELS = ["kbk", "megakernel", "coarse", "fine", "hybrid_mega_rtc", "hybrid_fine_rtc", "hybrid_kbk", "hybrid_4"]
+MODELS = ["kbk", "megakernel", "coarse", "fine", "hybrid_mega_rtc", "hybrid_fine_rtc", "hybrid_kbk", "hybrid_4",
+          "hybrid_mega_rtc3"]
 
 
 @pytest.mark.parametrize("model", MODELS)
