@@ -33,7 +33,9 @@ MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
 
 # Algorithmic fp32 operations per task (counted from the stage
 # definitions, excluding per-point constant Bernstein tables and integer coverage work):
-FLOP_DICE = 81 * (16 * 7 + 28 + 9)   # 16-term tensor sum (w, 3 mul+add), M.p, screen = 12069
+# Dice (reading R-R7, separable form): 36 u-curve points x 3 coords x (4 mul + 3 add), then
+# per grid point 3 coords x 7 + M.p 28 + screen 9 (3 div, 6 mul/add) + Q8 snap 2 = 5616
+FLOP_DICE = 36 * 3 * 7 + 81 * (3 * 7 + 28 + 9 + 2)
 FLOP_SHADE = 64 * 41                 # edges, cross, |n|, n.L, sqrt/div, shade, zq, Q8 snap = 2624
 FLOP_BOUND = 16 * (28 + 9) + 40      # 16 projections + split metric = 632
 FLOP_SPLIT = 3 * 4 * 12              # de Casteljau, 3 coords x 4 curves = 144

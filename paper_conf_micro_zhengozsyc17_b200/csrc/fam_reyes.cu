@@ -207,7 +207,7 @@ struct ReyesF {
   using Params = vp_reyes_params;
   static constexpr int stride(int s) { return s == SHADE ? (int)sizeof(RGrid) : (int)sizeof(RPatch); }
   static constexpr int threads_per_item(int s) { return s == BOUND ? 16 : s == SPLIT ? 16 : s == DICE ? 32 : 64; }
-  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 32 : 4; }
+  static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 64 : 4; }
   // Dice batches above 8 only in the fused RTC [Dice, Shade] kernel, whose grids stay in
   // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
   static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
@@ -618,7 +618,15 @@ struct ReyesF {
     RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(warp);
     float* Mw = (float*)cs.M[warp];
     uint8_t* list = cs.list[warp];
-    for (int k = warp; k < n; k += kWarpsW) {
+    // Patches are handed out dynamically: shade work per patch varies with its size on
+    // screen, so a static warp -> patch map leaves warps idle at the round barrier.
+    int* next = ctx.work_counter();
+    if (threadIdx.x == 0) ctx.template note_local_count<SHADE>(n);  // Dice emits one grid per patch
+    for (;;) {
+      int k = 0;
+      if (lane == 0) k = atomicAdd(next, 1);
+      k = __shfl_sync(0xffffffffu, k, 0);
+      if (k >= n) break;
       const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
       uint32_t frame = P->id >> 12;
       if (frame >= (uint32_t)p.n_frames) frame = 0;
@@ -626,7 +634,7 @@ struct ReyesF {
       __syncwarp();
       dice_patch<true>(p, P, g, lane, cs.M[warp]);
       __syncwarp();
-      if (lane == 0) ctx.template note_local<SHADE>((const uint8_t*)g);
+      if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
       const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
       const unsigned m0 = __ballot_sync(0xffffffffu, a0), m1 = __ballot_sync(0xffffffffu, a1);
       const unsigned lt = (1u << lane) - 1u;

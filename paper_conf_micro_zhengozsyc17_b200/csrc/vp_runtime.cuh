@@ -318,6 +318,7 @@ struct BlockShared {
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
   unsigned long long mbar[2];          // bulk-copy completion, one per in buffer
   uint32_t mbar_phase[2];
+  int work_next;                       // per-round work counter (dynamic hand-out within a batch)
 };
 
 __device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
@@ -345,6 +346,9 @@ struct Ctx {
   };
 
   __device__ __forceinline__ uint8_t* scratch() { return smem + kScratch; }
+  // Zero at the start of every round: worker warps may hand out the batch's items among
+  // themselves with atomicAdd on it (dynamic load balance inside a batch).
+  __device__ __forceinline__ int* work_counter() { return &sh.work_next; }
 
   template <int T>
   __device__ __forceinline__ uint8_t* out_ptr(int slot) {
@@ -364,11 +368,15 @@ struct Ctx {
     }
     return slot;
   }
-  // A fused RTC chain executed one block-local item of stage T (one thread per item):
-  // the per-stage task count and, with FLAG_TRACE, the trace record.
+  // A fused RTC chain executed n block-local items of stage T: the per-stage task count
+  // (one thread per chain call).
   template <int T>
-  __device__ __forceinline__ void note_local(const uint8_t* item) {
-    atomicAdd(&sh.deq[T], 1ull);
+  __device__ __forceinline__ void note_local_count(int n) {
+    sh.deq[T] += (unsigned long long)n;
+  }
+  // ... and, with FLAG_TRACE, the trace record of one of them (one thread per item).
+  template <int T>
+  __device__ __forceinline__ void trace_local(const uint8_t* item) {
     if (a.c.flags & FLAG_TRACE) {
       unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
       if (idx < a.c.trace_cap) {
@@ -933,6 +941,7 @@ struct Runner {
       }
       sh.acc_neg = 0;
       sh.done = 0;
+      sh.work_next = 0;
       sh.nx_n = 0;
       sh.nx_stage = -1;
       if (g.mode == MODE_WAVE) {
@@ -978,6 +987,9 @@ struct Runner {
     int b = 0, prev_s = -1, prev_n = 0;
     for (;;) {
       const int done = sh.done, cur_s = sh.nx_stage, cur_n = sh.nx_n;
+      // the previous round's users of work_next finished at its end barrier; this round's
+      // start after the next one
+      if (threadIdx.x == 0) sh.work_next = 0;
       __syncthreads();  // everyone has read the round's batch; the fetcher may overwrite it
       if (done) break;
       if (warp < kWarpsW) {
