@@ -35,10 +35,20 @@ struct CPrim {
   float fmx[3], fmy[3], fmz[3], fe[3];
 };
 
+// a / b, exactly (IEEE round-to-nearest).  A zero dividend over a finite nonzero divisor
+// is the signed zero, returned without the division: the IEEE division sequence takes its
+// slow path for a zero dividend, and momentum components are exactly zero here (rho*w is
+// 0 everywhere on this mesh; rho*v is 0 in the free stream).
+__device__ __forceinline__ float div_rn_zero(float a, float b) {
+  if (a == 0.0f && b != 0.0f && fabsf(b) <= 3.402823466e38f)
+    return __uint_as_float((__float_as_uint(a) ^ __float_as_uint(b)) & 0x80000000u);
+  return a / b;
+}
+
 __device__ __forceinline__ void cfd_prim(const CCell& c, CPrim& q) {
-  q.vx = c.mx / c.d;
-  q.vy = c.my / c.d;
-  q.vz = c.mz / c.d;
+  q.vx = div_rn_zero(c.mx, c.d);
+  q.vy = div_rn_zero(c.my, c.d);
+  q.vz = div_rn_zero(c.mz, c.d);
   float sq = q.vx * q.vx + q.vy * q.vy;
   q.sq = sq + q.vz * q.vz;
   q.p = (kGamma - 1.0f) * (c.e - 0.5f * c.d * q.sq);
@@ -92,7 +102,6 @@ struct CfdF {
                                                                                                                  : 0;
   }
   static constexpr bool rtc_ok(int, int) { return true; }  // back edges already exclude the loop
-  static constexpr int scratch_bytes(int, int) { return 0; }
   static constexpr int default_cap_log2(int) { return 16; }
   static constexpr int min_blocks(int, int, bool) { return VP_CFD_MINB; }
 
@@ -123,6 +132,167 @@ struct CfdF {
     }
   }
 
+  // Flux shares one primitive-variable record per cell through shared memory, so a cell's
+  // primitives are computed once per chunk instead of once per face that sees it
+  // (Rodinia recomputes them per face; the values are identical, every op is the same).
+  static constexpr int kShare = 20;        // d mx my mz e | speed c p | fmx[3] fmy[3] fmz[3] fe[3]
+  static constexpr int kHalo = 8;          // left/right halo cell per chunk, <= 4 chunks per item
+  static constexpr int kLd = kThreads + kHalo;
+  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= FLUX && FLUX <= hi) ? kShare * kLd * 4 : 0; }
+
+  static __device__ __forceinline__ void share_put(float* sh, int col, const CCell& c, const CPrim& q, float speed) {
+    const float v[kShare] = {c.d, c.mx, c.my, c.mz, c.e, speed, q.c, q.p, q.fmx[0], q.fmx[1], q.fmx[2],
+                             q.fmy[0], q.fmy[1], q.fmy[2], q.fmz[0], q.fmz[1], q.fmz[2], q.fe[0], q.fe[1], q.fe[2]};
+#pragma unroll
+    for (int f = 0; f < kShare; ++f) sh[f * kLd + col] = v[f];
+  }
+  struct NbRec {
+    float d, mx, my, mz, e, speed, c, fmx[3], fmy[3], fmz[3], fe[3];
+  };
+  static __device__ __forceinline__ void share_get(const float* sh, int col, NbRec& r) {
+    r.d = sh[0 * kLd + col]; r.mx = sh[1 * kLd + col]; r.my = sh[2 * kLd + col]; r.mz = sh[3 * kLd + col];
+    r.e = sh[4 * kLd + col]; r.speed = sh[5 * kLd + col]; r.c = sh[6 * kLd + col];
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      r.fmx[a] = sh[(8 + a) * kLd + col];
+      r.fmy[a] = sh[(11 + a) * kLd + col];
+      r.fmz[a] = sh[(14 + a) * kLd + col];
+      r.fe[a] = sh[(17 + a) * kLd + col];
+    }
+  }
+  // offsets are 32-bit: validate() bounds 16 * N < 2^31
+  static __device__ __forceinline__ void gather(const float* cur, uint32_t N, uint32_t nb, NbRec& r) {
+    const CCell cn{cur[nb], cur[N + nb], cur[2 * N + nb], cur[3 * N + nb], cur[4 * N + nb]};
+    CPrim qn;
+    cfd_prim(cn, qn);
+    r.d = cn.d; r.mx = cn.mx; r.my = cn.my; r.mz = cn.mz; r.e = cn.e;
+    r.speed = sqrtf(qn.sq);
+    r.c = qn.c;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+      r.fmx[a] = qn.fmx[a]; r.fmy[a] = qn.fmy[a]; r.fmz[a] = qn.fmz[a]; r.fe[a] = qn.fe[a];
+    }
+  }
+
+  // Rodinia compute_flux over one tile item (orc_cfd_flux_cell, the same operation order).
+  // Plain (L1-cacheable) loads of `cur` are coherent here: the item was acquired from its
+  // ring after the producers' release (and the acquire invalidates L1), and the workers are
+  // ordered after the fetcher by the round barrier.
+  template <class Ctx>
+  static __device__ void flux_item(Ctx& ctx, const Params& p, const CfdItem& ci) {
+    const size_t N = (size_t)p.G * p.G;
+    const float* cur = p.vars + (size_t)(ci.k & 1u) * 5 * N;
+    const size_t i0 = (size_t)ci.tile * p.T;
+    float* sh = (float*)ctx.scratch();
+    const int t = threadIdx.x, nchunks = (p.T + kThreads - 1) / kThreads;
+    const CCell ffc{p.ff[0], p.ff[1], p.ff[2], p.ff[3], p.ff[4]};
+    // halo records: chunk h/2's left (h even) or right (h odd) neighbour cell, one per warp
+    if ((t & 31) == 0 && (t >> 5) < 2 * nchunks) {
+      const int h = t >> 5, ch = h >> 1;
+      const long long lo = (long long)i0 + (long long)ch * kThreads;
+      const long long hi = lo + min(kThreads, p.T - ch * kThreads);
+      const long long cell = (h & 1) ? hi : lo - 1;
+      if (cell >= 0 && cell < (long long)N) {
+        NbRec r;
+        gather(cur, (uint32_t)N, (uint32_t)cell, r);
+        const CCell cc{r.d, r.mx, r.my, r.mz, r.e};
+        CPrim q;
+        q.c = r.c; q.p = 0.0f;
+#pragma unroll
+        for (int a = 0; a < 3; ++a) { q.fmx[a] = r.fmx[a]; q.fmy[a] = r.fmy[a]; q.fmz[a] = r.fmz[a]; q.fe[a] = r.fe[a]; }
+        share_put(sh, kThreads + h, cc, q, r.speed);
+      }
+    }
+    const uint32_t N32 = (uint32_t)N;
+    for (int c0 = 0; c0 < p.T; c0 += kThreads) {
+      const int nch = min(kThreads, p.T - c0), chunk = c0 / kThreads;
+      const long long lo = (long long)i0 + c0, hi = lo + nch;
+      const bool act = t < nch;
+      const uint32_t c = (uint32_t)lo + (act ? t : 0);
+      // this cell's faces: neighbour ids and normals are loaded before the barrier, so
+      // their latency overlaps the primitive-variable computation
+      int nbv[4];
+      float nrm[4][3];
+      if (act) {
+        const CCell ic{cur[c], cur[N32 + c], cur[2 * N32 + c], cur[3 * N32 + c], cur[4 * N32 + c]};
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          nbv[j] = __ldg(p.nb + (j * N32 + c));
+#pragma unroll
+          for (int a = 0; a < 3; ++a) nrm[j][a] = __ldg(p.normals + ((j * 3 + a) * N32 + c));
+        }
+        CPrim qi;
+        cfd_prim(ic, qi);
+        share_put(sh, t, ic, qi, sqrtf(qi.sq));
+      }
+      worker_sync();
+      if (act) {
+        // this cell's record is read back from shared memory where it is used (registers
+        // are the limit here: 3 resident blocks of 320 threads)
+        const float* me = sh + t;
+#define ME(f) me[(f) * kLd]
+        float fd = 0.0f, fe = 0.0f, fx = 0.0f, fy = 0.0f, fz = 0.0f;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int nb = nbv[j];
+          const float nx = nrm[j][0], ny = nrm[j][1], nz = nrm[j][2];
+          float nlen = nx * nx + ny * ny;
+          nlen = sqrtf(nlen + nz * nz);
+          const float nn[3] = {nx, ny, nz};
+          if (nb >= 0) {
+            int col = -1;
+            if ((long long)nb >= lo && (long long)nb < hi) col = (int)((long long)nb - lo);
+            else if ((long long)nb == lo - 1) col = kThreads + 2 * chunk;
+            else if ((long long)nb == hi) col = kThreads + 2 * chunk + 1;
+            NbRec r;
+            if (col >= 0) share_get(sh, col, r);
+            else gather(cur, N32, (uint32_t)nb, r);
+            float factor = -nlen * kSmooth * 0.5f * (ME(5) + r.speed + ME(6) + r.c);
+            fd += factor * (ME(0) - r.d);
+            fe += factor * (ME(4) - r.e);
+            fx += factor * (ME(1) - r.mx);
+            fy += factor * (ME(2) - r.my);
+            fz += factor * (ME(3) - r.mz);
+            const float mn[3] = {r.mx, r.my, r.mz};
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+              factor = 0.5f * nn[a];
+              fd += factor * (mn[a] + ME(1 + a));
+              fe += factor * (r.fe[a] + ME(17 + a));
+              fx += factor * (r.fmx[a] + ME(8 + a));
+              fy += factor * (r.fmy[a] + ME(11 + a));
+              fz += factor * (r.fmz[a] + ME(14 + a));
+            }
+          } else if (nb == -1) {
+            fx += nx * ME(7);
+            fy += ny * ME(7);
+            fz += nz * ME(7);
+          } else if (nb == -2) {
+            CPrim qf;
+            cfd_prim(ffc, qf);
+            const float mf[3] = {ffc.mx, ffc.my, ffc.mz};
+#pragma unroll
+            for (int a = 0; a < 3; ++a) {
+              const float factor = 0.5f * nn[a];
+              fd += factor * (mf[a] + ME(1 + a));
+              fe += factor * (qf.fe[a] + ME(17 + a));
+              fx += factor * (qf.fmx[a] + ME(8 + a));
+              fy += factor * (qf.fmy[a] + ME(11 + a));
+              fz += factor * (qf.fmz[a] + ME(14 + a));
+            }
+          }
+        }
+#undef ME
+        __stcg(p.flux + c, fd);
+        __stcg(p.flux + (N32 + c), fx);
+        __stcg(p.flux + (2 * N32 + c), fy);
+        __stcg(p.flux + (3 * N32 + c), fz);
+        __stcg(p.flux + (4 * N32 + c), fe);
+      }
+      worker_sync();  // the chunk's records are rewritten next
+    }
+  }
+
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
@@ -133,85 +303,40 @@ struct CfdF {
       const uint32_t k = ci.k;
       const float* cur = p.vars + (size_t)(k & 1u) * 5 * N;
       if constexpr (s == COPY) {
-        for (int v = 0; v < 5; ++v)
-          for (int i = threadIdx.x * 4; i < p.T; i += kThreads * 4)
-            __stcg((float4*)(p.old + (size_t)v * N + i0 + i), __ldcg((const float4*)(cur + (size_t)v * N + i0 + i)));
+        // all five loads in flight before the stores (the arrays do not alias)
+        for (int i = threadIdx.x * 4; i < p.T; i += kThreads * 4) {
+          float4 v[5];
+#pragma unroll
+          for (int q = 0; q < 5; ++q) v[q] = *(const float4*)(cur + (size_t)q * N + i0 + i);
+#pragma unroll
+          for (int q = 0; q < 5; ++q) __stcg((float4*)(p.old + (size_t)q * N + i0 + i), v[q]);
+        }
         worker_sync();
         if (threadIdx.x == 0) ctx.template emit<STEP>(&ci);
       } else if constexpr (s == STEP) {
-        for (int i = threadIdx.x; i < p.T; i += kThreads) {
+        for (int i = threadIdx.x * 4; i < p.T; i += kThreads * 4) {
           const size_t c = i0 + i;
-          CCell cc = cfd_load(cur, N, c);
-          CPrim q;
-          cfd_prim(cc, q);
-          p.sf[c] = 0.5f / (sqrtf(__ldg(p.area + c)) * (sqrtf(q.sq) + q.c));
+          float4 v[5];
+#pragma unroll
+          for (int q = 0; q < 5; ++q) v[q] = *(const float4*)(cur + (size_t)q * N + c);
+          const float4 ar = __ldg((const float4*)(p.area + c));
+          const float* vf = (const float*)v;
+          const float* af = (const float*)&ar;
+          float4 r;
+          float* rf = (float*)&r;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const CCell cc{vf[u], vf[4 + u], vf[8 + u], vf[12 + u], vf[16 + u]};
+            CPrim q;
+            cfd_prim(cc, q);
+            rf[u] = 0.5f / (sqrtf(af[u]) * (sqrtf(q.sq) + q.c));
+          }
+          __stcg((float4*)(p.sf + c), r);
         }
         worker_sync();
         if (threadIdx.x == 0) arrive(ctx, p, ci.tile, k);
       } else if constexpr (s == FLUX) {
-        CCell ffc{p.ff[0], p.ff[1], p.ff[2], p.ff[3], p.ff[4]};
-        CPrim qf;
-        cfd_prim(ffc, qf);
-        for (int i = threadIdx.x; i < p.T; i += kThreads) {
-          const size_t c = i0 + i;
-          const CCell ic = cfd_load(cur, N, c);
-          CPrim qi;
-          cfd_prim(ic, qi);
-          const float speed_i = sqrtf(qi.sq);
-          float fd = 0.0f, fe = 0.0f, fx = 0.0f, fy = 0.0f, fz = 0.0f;
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            const int nb = __ldg(p.nb + (size_t)j * N + c);
-            const float nx = __ldg(p.normals + ((size_t)j * 3 + 0) * N + c);
-            const float ny = __ldg(p.normals + ((size_t)j * 3 + 1) * N + c);
-            const float nz = __ldg(p.normals + ((size_t)j * 3 + 2) * N + c);
-            float nlen = nx * nx + ny * ny;
-            nlen = sqrtf(nlen + nz * nz);
-            const float nn[3] = {nx, ny, nz};
-            if (nb >= 0) {
-              const CCell cn = cfd_load(cur, N, (size_t)nb);
-              CPrim qn;
-              cfd_prim(cn, qn);
-              float factor = -nlen * kSmooth * 0.5f * (speed_i + sqrtf(qn.sq) + qi.c + qn.c);
-              fd += factor * (ic.d - cn.d);
-              fe += factor * (ic.e - cn.e);
-              fx += factor * (ic.mx - cn.mx);
-              fy += factor * (ic.my - cn.my);
-              fz += factor * (ic.mz - cn.mz);
-              const float mn[3] = {cn.mx, cn.my, cn.mz}, mi[3] = {ic.mx, ic.my, ic.mz};
-#pragma unroll
-              for (int a = 0; a < 3; ++a) {
-                factor = 0.5f * nn[a];
-                fd += factor * (mn[a] + mi[a]);
-                fe += factor * (qn.fe[a] + qi.fe[a]);
-                fx += factor * (qn.fmx[a] + qi.fmx[a]);
-                fy += factor * (qn.fmy[a] + qi.fmy[a]);
-                fz += factor * (qn.fmz[a] + qi.fmz[a]);
-              }
-            } else if (nb == -1) {
-              fx += nx * qi.p;
-              fy += ny * qi.p;
-              fz += nz * qi.p;
-            } else if (nb == -2) {
-              const float mf[3] = {ffc.mx, ffc.my, ffc.mz}, mi[3] = {ic.mx, ic.my, ic.mz};
-#pragma unroll
-              for (int a = 0; a < 3; ++a) {
-                const float factor = 0.5f * nn[a];
-                fd += factor * (mf[a] + mi[a]);
-                fe += factor * (qf.fe[a] + qi.fe[a]);
-                fx += factor * (qf.fmx[a] + qi.fmx[a]);
-                fy += factor * (qf.fmy[a] + qi.fmy[a]);
-                fz += factor * (qf.fmz[a] + qi.fmz[a]);
-              }
-            }
-          }
-          __stcg(p.flux + c, fd);
-          __stcg(p.flux + N + c, fx);
-          __stcg(p.flux + 2 * N + c, fy);
-          __stcg(p.flux + 3 * N + c, fz);
-          __stcg(p.flux + 4 * N + c, fe);
-        }
-        worker_sync();
+        flux_item(ctx, p, ci);
         if (threadIdx.x == 0) ctx.template emit<TIME>(&ci);
       } else {  // TimeStep
         const int rk = (int)(k % kRK);
@@ -220,33 +345,46 @@ struct CfdF {
         const float denom = (float)(kRK + 1 - rk);
         for (int i = threadIdx.x * 4; i < p.T; i += kThreads * 4) {
           const size_t c = i0 + i;
-          const float4 sf = __ldcg((const float4*)(p.sf + c));
+          // every load in flight before any store (old / flux / sf never alias nxt)
+          const float4 sf = *(const float4*)(p.sf + c);
+          float4 o[5], fl[5];
+#pragma unroll
+          for (int v = 0; v < 5; ++v) {
+            o[v] = *(const float4*)(p.old + (size_t)v * N + c);
+            fl[v] = *(const float4*)(p.flux + (size_t)v * N + c);
+          }
           float4 f4;
           f4.x = sf.x / denom;
           f4.y = sf.y / denom;
           f4.z = sf.z / denom;
           f4.w = sf.w / denom;
+#pragma unroll
           for (int v = 0; v < 5; ++v) {
-            const float4 o = __ldcg((const float4*)(p.old + (size_t)v * N + c));
-            const float4 fl = __ldcg((const float4*)(p.flux + (size_t)v * N + c));
             float4 r;
-            r.x = o.x + f4.x * fl.x;
-            r.y = o.y + f4.y * fl.y;
-            r.z = o.z + f4.z * fl.z;
-            r.w = o.w + f4.w * fl.w;
+            r.x = o[v].x + f4.x * fl[v].x;
+            r.y = o[v].y + f4.y * fl[v].y;
+            r.z = o[v].z + f4.z * fl[v].z;
+            r.w = o[v].w + f4.w * fl[v].w;
             __stcg((float4*)(nxt + (size_t)v * N + c), r);
           }
         }
         worker_sync();
-        if (threadIdx.x == 0 && outer + (rk == kRK - 1 ? 1u : 0u) < (uint32_t)p.n_outer) {
+        // latch arrivals: thread j < m arrives on neighbour j, thread m on the tile itself
+        // (or emits the next outer iteration's Copy) -- the fences and atomics of one item
+        // overlap instead of running back to back on one thread
+        if (threadIdx.x < 5 && outer + (rk == kRK - 1 ? 1u : 0u) < (uint32_t)p.n_outer) {
           uint32_t nbt[4];
           const int m = tile_neighbours(p, ci.tile, nbt);
-          for (int j = 0; j < m; ++j) arrive(ctx, p, nbt[j], k + 1);
-          if (rk < kRK - 1) {
-            arrive(ctx, p, ci.tile, k + 1);
-          } else {
-            CfdItem cp{ci.tile, k + 1, 0, 0};
-            ctx.template emit<COPY>(&cp);
+          const int j = threadIdx.x;
+          if (j < m) {
+            arrive(ctx, p, nbt[j], k + 1);
+          } else if (j == m) {
+            if (rk < kRK - 1) {
+              arrive(ctx, p, ci.tile, k + 1);
+            } else {
+              CfdItem cp{ci.tile, k + 1, 0, 0};
+              ctx.template emit<COPY>(&cp);
+            }
           }
         }
       }
@@ -267,6 +405,8 @@ struct CfdF {
   }
   static const char* validate(const Params& p) {
     if (p.G < 4 || p.T < 4 || p.T > p.G || p.G % p.T || p.T % 4) return "vp_cfd_params: T must divide G, T % 4 == 0";
+    if ((long long)p.G * p.G * 16 >= (1ll << 31)) return "vp_cfd_params: G <= 8191 (32-bit cell offsets)";
+    if (p.T > kThreads * (kHalo / 2)) return "vp_cfd_params: T <= 1024 (four 256-cell Flux chunks per item)";
     if (p.n_outer < 0) return "vp_cfd_params: n_outer >= 0";
     if (!p.vars0 || !p.vars || !p.old || !p.sf || !p.flux || !p.area || !p.nb || !p.normals || !p.latch)
       return "vp_cfd_params: all buffers are required";

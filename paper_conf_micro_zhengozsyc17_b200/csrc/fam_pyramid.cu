@@ -85,7 +85,7 @@ struct PyramidF {
   }
   // CDF's fan-out must not be expanded block-locally from a batch of latch-fired items
   static constexpr bool rtc_ok(int lo, int hi) { return !(lo < CDF && hi >= CDF); }
-  static constexpr int scratch_bytes(int, int) { return 256 * 4 + 256; }  // histogram / LUT staging
+  static constexpr int scratch_bytes(int, int) { return kWarpsW * 256 * 4; }  // sub-histograms / CDF / LUT staging
   static constexpr int default_cap_log2(int s) { return s == MAP ? 16 : 15; }
   static constexpr int min_blocks(int, int, bool) { return VP_PYR_MINB; }
 
@@ -97,47 +97,81 @@ struct PyramidF {
 
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
-    for (int k = 0; k < n; ++k) {
-      const PyrItem it = ((const PyrItem*)items)[k];
-      if constexpr (s == GRAY) gray(ctx, it);
-      else if constexpr (s == CDF) cdf(ctx, it);
-      else if constexpr (s == MAP) map(ctx, it);
-      else resize(ctx, it);
-      worker_sync();  // the block-wide stage functions reuse the scratch between items
+    if constexpr (s == GRAY) {
+      gray_batch(ctx, (const PyrItem*)items, n);
+    } else if constexpr (s == RESIZE) {
+      resize_batch(ctx, (const PyrItem*)items, n);
+    } else {
+      for (int k = 0; k < n; ++k) {
+        const PyrItem it = ((const PyrItem*)items)[k];
+        if constexpr (s == CDF) cdf(ctx, it);
+        else map(ctx, it);
+        worker_sync();  // the block-wide stage functions reuse the scratch between items
+      }
     }
   }
 
   // ------------------------------------------------------------ Gray (block per tile)
+  // A batch of tiles accumulates into per-warp sub-histograms in shared memory (each
+  // thread adds runs of equal values once), flushed to the image's global histogram when
+  // the image changes and at the end of the batch; the CDF latch of every image is then
+  // arrived on once with the batch's tile count for it.
   template <class Ctx>
-  static __device__ void gray(Ctx& ctx, const PyrItem& it) {
+  static __device__ void gray_batch(Ctx& ctx, const PyrItem* items, int n) {
     const Params& p = ctx.params();
-    if (it.img >= (uint32_t)p.n_img) return;
-    uint32_t* hs = (uint32_t*)ctx.scratch();
-    const int t = threadIdx.x;
-    hs[t] = 0;
+    uint32_t* hs = (uint32_t*)ctx.scratch();  // [kWarpsW][256]
+    const int t = threadIdx.x, w = t >> 5;
+    for (int i = t; i < kWarpsW * 256; i += kThreads) hs[i] = 0;
     worker_sync();
     const size_t npx = (size_t)p.S * p.S;
-    // 4096 pixels: thread t handles 16 consecutive pixels of row t/4
-    const int y = t >> 2, x0 = (t & 3) * 16;
-    const size_t row = (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + x0;
-    const uint4* src = (const uint4*)(p.rgb + ((size_t)it.img * npx + row) * 3);
-    uint4 v[3];
+    const int y = t >> 2, x0 = (t & 3) * 16;  // thread t: 16 consecutive pixels of tile row t/4
+    int k0 = 0;
+    for (int k = 0; k < n; ++k) {
+      const PyrItem it = items[k];
+      if (it.img < (uint32_t)p.n_img) {
+        const size_t row = (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + x0;
+        const uint4* src = (const uint4*)(p.rgb + ((size_t)it.img * npx + row) * 3);
+        uint4 v[3];
 #pragma unroll
-    for (int q = 0; q < 3; ++q) v[q] = __ldg(src + q);
-    const uint8_t* b = (const uint8_t*)v;
-    __align__(16) uint8_t g[16];
+        for (int q = 0; q < 3; ++q) v[q] = __ldg(src + q);
+        const uint8_t* b = (const uint8_t*)v;
+        __align__(16) uint8_t g[16];
 #pragma unroll
-    for (int i = 0; i < 16; ++i) {
-      g[i] = (uint8_t)((77u * b[3 * i] + 150u * b[3 * i + 1] + 29u * b[3 * i + 2] + 128u) >> 8);
-      atomicAdd(&hs[g[i]], 1u);
-    }
-    *(uint4*)(p.gray + (size_t)it.img * npx + row) = *(const uint4*)g;
-    worker_sync();
-    if (hs[t]) atomicAdd(&p.hist[(size_t)it.img * 256 + t], hs[t]);
-    worker_sync();
-    if (t == 0 && latch_arrive(p.latch + (size_t)it.img * pyr_latches_per_img(p.S), 1)) {
-      PyrItem c{it.img, 0, 0, 0};
-      ctx.template emit<CDF>(&c);
+        for (int i = 0; i < 16; ++i) g[i] = (uint8_t)((77u * b[3 * i] + 150u * b[3 * i + 1] + 29u * b[3 * i + 2] + 128u) >> 8);
+        *(uint4*)(p.gray + (size_t)it.img * npx + row) = *(const uint4*)g;
+        uint32_t cur = g[0], cnt = 1;
+#pragma unroll
+        for (int i = 1; i < 16; ++i) {
+          if (g[i] == cur) {
+            ++cnt;
+          } else {
+            atomicAdd(&hs[w * 256 + cur], cnt);
+            cur = g[i];
+            cnt = 1;
+          }
+        }
+        atomicAdd(&hs[w * 256 + cur], cnt);
+      }
+      const bool last = k + 1 == n || items[k + 1].img != it.img;
+      if (last) {  // flush the image's counts (block-uniform branch)
+        worker_sync();
+        if (it.img < (uint32_t)p.n_img) {
+          uint32_t sum = 0;
+#pragma unroll
+          for (int q = 0; q < kWarpsW; ++q) {
+            sum += hs[q * 256 + t];
+            hs[q * 256 + t] = 0;
+          }
+          if (sum) atomicAdd(&p.hist[(size_t)it.img * 256 + t], sum);
+        }
+        worker_sync();
+        if (t == 0 && it.img < (uint32_t)p.n_img &&
+            latch_arrive(p.latch + (size_t)it.img * pyr_latches_per_img(p.S), k + 1 - k0)) {
+          PyrItem c{it.img, 0, 0, 0};
+          ctx.template emit<CDF>(&c);
+        }
+        k0 = k + 1;
+      }
     }
   }
 
@@ -199,14 +233,27 @@ struct PyramidF {
     const uint8_t* g = p.gray + (size_t)it.img * npx;
     uint8_t* dst = p.pyr + (size_t)it.img * total;
     const int vec_per_row = wpx / 16, nvec = kPT * vec_per_row;
-    for (int i = t; i < nvec; i += kThreads) {
-      const int y = i / vec_per_row, xv = i - y * vec_per_row;
-      const size_t off = (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16;
-      uint4 v = __ldcg((const uint4*)(g + off));
-      uint8_t* b = (uint8_t*)&v;
+    // up to 8 vectors per thread, all loads in flight before the lookups and stores
+    constexpr int kV = kMapSeg * kPT * kPT / 16 / kThreads;
+    uint4 v[kV];
 #pragma unroll
-      for (int q = 0; q < 16; ++q) b[q] = lut[b[q]];
-      *(uint4*)(dst + off) = v;
+    for (int u = 0; u < kV; ++u) {
+      const int i = t + u * kThreads;
+      if (i < nvec) {
+        const int y = i / vec_per_row, xv = i - y * vec_per_row;
+        v[u] = *(const uint4*)(g + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < kV; ++u) {
+      const int i = t + u * kThreads;
+      if (i < nvec) {
+        const int y = i / vec_per_row, xv = i - y * vec_per_row;
+        uint8_t* b = (uint8_t*)&v[u];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) b[q] = lut[b[q]];
+        *(uint4*)(dst + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16) = v[u];
+      }
     }
     worker_sync();
     // latch arrivals on level 1: each level-1 tile gets one count per source tile
@@ -227,8 +274,31 @@ struct PyramidF {
   }
 
   // ------------------------------------------------------------ Resize (2x2 box)
+  // The batch's tiles are independent (disjoint outputs): all are computed, then one
+  // barrier, then thread k arrives on item k's next-level latch (the fences overlap).
   template <class Ctx>
-  static __device__ void resize(Ctx& ctx, const PyrItem& it) {
+  static __device__ void resize_batch(Ctx& ctx, const PyrItem* items, int n) {
+    for (int k = 0; k < n; ++k) resize_tile(ctx, items[k]);
+    worker_sync();
+    const Params& p = ctx.params();
+    const int t = threadIdx.x;
+    if (t < n) {
+      const PyrItem it = items[t];
+      const int l = (int)it.level, L = pyr_levels(p.S);
+      if (it.img < (uint32_t)p.n_img && l >= 1 && l + 1 < L) {
+        const int nt1 = pyr_tiles(p.S, l + 1);
+        const int by = (int)it.ty / 2, bx = (int)it.tx / 2;
+        int* lat = p.latch + (size_t)it.img * pyr_latches_per_img(p.S) + pyr_latch_off(p.S, l + 1) + (size_t)by * nt1 + bx;
+        if (latch_arrive(lat, 1)) {
+          PyrItem r{it.img, (uint32_t)(l + 1), (uint32_t)by, (uint32_t)bx};
+          ctx.template emit<RESIZE>(&r);
+        }
+      }
+    }
+  }
+
+  template <class Ctx>
+  static __device__ void resize_tile(Ctx& ctx, const PyrItem& it) {
     const Params& p = ctx.params();
     if (it.img >= (uint32_t)p.n_img) return;
     const int l = (int)it.level, L = pyr_levels(p.S);
@@ -245,7 +315,7 @@ struct PyramidF {
       const int gy = (int)it.ty * kPT + y, gx = (int)it.tx * kPT + x0;
       const uint4* r0 = (const uint4*)(src + (size_t)(2 * gy) * sp + 2 * gx);
       const uint4* r1 = (const uint4*)(src + (size_t)(2 * gy + 1) * sp + 2 * gx);
-      const uint4 a0 = __ldcg(r0), a1 = __ldcg(r0 + 1), b0 = __ldcg(r1), b1 = __ldcg(r1 + 1);
+      const uint4 a0 = r0[0], a1 = r0[1], b0 = r1[0], b1 = r1[1];
       __align__(16) uint8_t ra[32];
       __align__(16) uint8_t rb[32];
       __align__(16) uint8_t o[16];
@@ -260,19 +330,9 @@ struct PyramidF {
     } else {
       for (int i = t; i < w * w; i += kThreads) {
         const int y = i / w, x = i - y * w;
-        unsigned a = __ldcg(src + (size_t)(2 * y) * sp + 2 * x), b = __ldcg(src + (size_t)(2 * y) * sp + 2 * x + 1);
-        unsigned c = __ldcg(src + (size_t)(2 * y + 1) * sp + 2 * x), d = __ldcg(src + (size_t)(2 * y + 1) * sp + 2 * x + 1);
+        unsigned a = src[(size_t)(2 * y) * sp + 2 * x], b = src[(size_t)(2 * y) * sp + 2 * x + 1];
+        unsigned c = src[(size_t)(2 * y + 1) * sp + 2 * x], d = src[(size_t)(2 * y + 1) * sp + 2 * x + 1];
         dst[(size_t)y * s + x] = (uint8_t)((a + b + c + d + 2u) >> 2);
-      }
-    }
-    worker_sync();
-    if (t == 0 && l + 1 < L) {
-      const int nt1 = pyr_tiles(p.S, l + 1);
-      const int by = (int)it.ty / 2, bx = (int)it.tx / 2;
-      int* lat = p.latch + (size_t)it.img * pyr_latches_per_img(p.S) + pyr_latch_off(p.S, l + 1) + (size_t)by * nt1 + bx;
-      if (latch_arrive(lat, 1)) {
-        PyrItem r{it.img, (uint32_t)(l + 1), (uint32_t)by, (uint32_t)bx};
-        ctx.template emit<RESIZE>(&r);
       }
     }
   }
