@@ -55,7 +55,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="vp", choices=["vp", "reference"])
     ap.add_argument("--frames", type=int, default=TOTAL_FRAMES)
-    ap.add_argument("--model", default="tuned", help="tuned (auto-tuner) | hybrid | megakernel | kbk | coarse | fine")
+    ap.add_argument("--model", default="tuned",
+                    help="tuned (auto-tuner) | hybrid | megakernel | kbk | kbk_graph | coarse | fine")
     ap.add_argument("--tune-seconds", type=float, default=30.0)
     ap.add_argument("--split", type=int, default=44, help="SMs for the [Bound,Split] group (hybrid)")
     ap.add_argument("--no-e2e", action="store_true")
@@ -117,7 +118,8 @@ def configure(vp, rp, model, nsm, split):
     if model == "hybrid":
         rp.configure(vp.HYBRID, hybrid_binding(vp, nsm, split))
     else:
-        rp.configure({"megakernel": vp.MEGAKERNEL, "kbk": vp.KBK, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+        rp.configure({"megakernel": vp.MEGAKERNEL, "kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "coarse": vp.COARSE,
+                      "fine": vp.FINE}[model])
 
 
 def time_steps(torch, rp, steps, stream):
@@ -188,6 +190,35 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def queue_microbench(torch, vp, stream):
+    """the ring queues alone.  Chains (fan-out 1) and binary trees
+    (fan-out 2) of 4 / 16 / 272-B items under the megakernel and both KBK flavours; tasks/s
+    and ring payload GB/s (each task reads its item and writes its children)."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import QBenchPipeline
+    out = {}
+    for ib in (4, 16, 272):
+        for fan, depth in ((1, 99), (2, 16)):
+            # chains: 2^20 (2^18) live items; trees: the last level (n * 2^16) must fit the ring
+            n = (1 << 20 if ib < 272 else 1 << 18) if fan == 1 else (1 << 7 if ib < 272 else 1 << 4)
+            qb = QBenchPipeline(n, ib, fan, depth)
+            r = {}
+            for name, model in (("megakernel", vp.MEGAKERNEL), ("kbk", vp.KBK), ("kbk_graph", vp.KBK_GRAPH)):
+                qb.configure(model)
+                qb.run(stream)
+                ts = []
+                for _ in range(3):
+                    res, st = qb.run(stream)
+                    assert res["bad"] == 0 and st["dequeued"][qb.stage] == qb.tasks()
+                    ts.append(st["device_ms"])
+                ms = min(ts)
+                r[name] = {"ms": ms, "mtasks_per_s": qb.tasks() / ms / 1e3,
+                           # every task reads its item once; every non-seed item was written once
+                           "ring_gbs": (2 * qb.tasks() - n) * ib / ms / 1e6}
+            out[f"item{ib}_fan{fan}"] = {"tasks": qb.tasks(), **r}
+            del qb
+    return out
+
+
 def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
     """Secondary measurements: every BASELINE workload (configs 1-4) through the same
     runtime, auto-tuned, vs KBK; items/s, frames/s and % of measured HBM where the
@@ -212,12 +243,15 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         ms, st = t_run()
         pipe.configure(vp.KBK)
         kbk_ms, _ = t_run()
+        pipe.configure(vp.KBK_GRAPH)
+        kbkg_ms, _ = t_run()
         pipe.configure(vp.MEGAKERNEL)
         mega_ms, _ = t_run()
         pipe.p.configure_config(best)
         items = sum(st["dequeued"][:8])
         r = {"ms": ms, "frames_per_s": frames / (ms / 1e3), "items_per_s": items / (ms / 1e3),
-             "items": items, "kbk_ms": kbk_ms, "megakernel_ms": mega_ms, "speedup_vs_kbk": kbk_ms / ms,
+             "items": items, "kbk_ms": kbk_ms, "kbk_graph_ms": kbkg_ms, "megakernel_ms": mega_ms,
+             "speedup_vs_kbk": kbk_ms / ms, "speedup_vs_kbk_graph": kbkg_ms / ms,
              "speedup_vs_megakernel": mega_ms / ms, "tuned": tuned_cfg.split(" mask")[0]}
         if alg_bytes:
             gbs = alg_bytes / (ms / 1e3) / 1e9
@@ -334,7 +368,7 @@ def main():
     # ---- baselines on the same shard: KBK (one launch per stage per wave) + megakernel
     extra = {}
     if not args.no_baselines:
-        for name in ("kbk", "megakernel"):
+        for name in ("kbk", "kbk_graph", "megakernel"):
             if name == args.model:
                 continue
             configure(vp, rp, name, nsm, args.split)
@@ -345,6 +379,8 @@ def main():
                 dist.all_reduce(bt_t, op=dist.ReduceOp.MAX)
             extra[name] = {"ms_per_step": float(bt_t.item()) / max(1, min(args.steps, 3)),
                            "launches_per_step": int(bst["kbk_launches"])}
+            if name == "kbk_graph":  # + one planner per wave and one loop-condition kernel per iteration
+                extra[name]["launches_per_step"] = int(bst["kbk_launches"]) * 2 + int(bst["kbk_launches"]) // 4
         rp.p.configure_config(main_cfg)
 
     # ---- e2e through the public API with HOST buffers: H2D seeds + run + D2H colours
@@ -388,11 +424,16 @@ def main():
         gather_ms = shard.max_over_ranks(g0.elapsed_time(g1), "cuda")
 
     suite = None
+    qbench = None
     if world == 1 and not args.no_suite:
         try:
             suite = workload_suite(torch, vp, stream, args.suite_tune_seconds, pk.get("hbm_gbs", 6548.5))
         except Exception as ex:  # secondary numbers must never lose the headline line
             suite = {"error": repr(ex)}
+        try:
+            qbench = queue_microbench(torch, vp, stream)
+        except Exception as ex:
+            qbench = {"error": repr(ex)}
 
     cpu = None
     if rank == 0 and world == 1:
@@ -421,8 +462,10 @@ def main():
                 "pct_of_measured": 100.0 * bytes_step * world / (ms_per_step / 1e3) / 1e9 / hbm,
                 "note": "ALU/latency-bound workload (SURVEY §8(d) d5); % HBM reported, not the bound"},
         "speedup_vs_kbk": (extra["kbk"]["ms_per_step"] / ms_per_step) if "kbk" in extra else None,
+        "speedup_vs_kbk_graph": (extra["kbk_graph"]["ms_per_step"] / ms_per_step) if "kbk_graph" in extra else None,
         "baselines": extra, "e2e": e2e, "gather_ms": gather_ms, "clocks": clocks, "gpu_launches": launches * args.steps,
         "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune, "workloads": suite,
+        "queue_microbench": qbench,
         "config_string": vp.config_to_string(main_cfg),
     }
     if rank == 0:

@@ -47,7 +47,13 @@ typedef enum vp_model {
   VP_MEGAKERNEL = 2,
   VP_COARSE = 3,
   VP_FINE = 4,
-  VP_HYBRID = 5
+  VP_HYBRID = 5,
+  /* KBK with its control loop on the device: the same per-stage wave kernels, sized by a
+   * planner kernel from the live queue counts and repeated by a CUDA-graph while node until
+   * the pipeline drains (no host round trip per wave).  A stronger per-stage-kernel
+   * baseline than the paper's host-driven KBK (Fig. 3b, L13: "pipeline logic control is
+   * implemented on the CPU side"); SURVEY §8 a11. */
+  VP_KBK_GRAPH = 6
 } vp_model;
 
 /* Per-group models inside VP_HYBRID (the auto-tuner explores "RTC, KBK, Megakernel,
@@ -81,7 +87,11 @@ typedef enum vp_stage_kind {
   VP_CFD_COPY = 50, VP_CFD_STEP_FACTOR = 51, VP_CFD_FLUX = 52, VP_CFD_TIME_STEP = 53,
   /* LBP face detection (Fig. 14, L55): Grayscale, HistEq as CDF + Map, Resize
    * (recursive), Feature Extraction (LBP), Scanning (rows of 24x24 windows) */
-  VP_FD_GRAY = 60, VP_FD_CDF = 61, VP_FD_MAP = 62, VP_FD_RESIZE = 63, VP_FD_LBP = 64, VP_FD_SCAN = 65
+  VP_FD_GRAY = 60, VP_FD_CDF = 61, VP_FD_MAP = 62, VP_FD_RESIZE = 63, VP_FD_LBP = 64, VP_FD_SCAN = 65,
+  /* Queue microbenchmark (not a paper workload): three independent
+   * self-recursive stages with 4-, 16- and 272-B items (Fig. 9's int; Table 2's window /
+   * tile items; the Reyes patch, L61 §8.5).  See vp_qbench_params. */
+  VP_QB_ITEM4 = 70, VP_QB_ITEM16 = 71, VP_QB_ITEM272 = 72
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -92,6 +102,10 @@ typedef enum vp_stage_kind {
 #define VP_FLAG_QUEUE_DEPTH 0x2u    /* track max ring depth per stage (one extra read/flush) */
 #define VP_FLAG_STRICT_BINDING 0x4u /* vp_run fails with VP_ERR_BINDING on quota shortfall   */
 #define VP_FLAG_TIMERS 0x8u         /* in-kernel %globaltimer accumulators per stage/kernel  */
+#define VP_FLAG_FULL_RINGS 0x10u    /* persistent plans keep every ring at its registered     */
+                                    /* capacity instead of shrinking it to what the producer  */
+                                    /* blocks can hold (needed when a recursive stage's live   */
+                                    /* frontier is larger, e.g. breadth-first fan-out-2 trees) */
 
 typedef struct vp_pipeline_desc {
   int max_stages;                 /* <= VP_MAX_STAGES                                      */
@@ -193,6 +207,19 @@ typedef struct vp_toy_params {
   int32_t* out;              /* sink output values, capacity >= #seeds                     */
   unsigned long long* n_out; /* device counter, reset by every vp_run                      */
 } vp_toy_params;
+
+/* Queue microbenchmark.  Item word 0 = id (24 bits) | remaining depth << 24; words 1..
+ * = payload id * 2654435761 + k * 40503 (mod 2^32).  A task with fanout > 0 and depth > 0
+ * emits `fanout` copies of its item with depth - 1 (whole payload copied); a leaf checks
+ * its payload and adds to the per-stage counters.  Tasks per seed: 1 (fan-out 0),
+ * depth + 1 (fan-out 1), 2^(depth+1) - 1 (fan-out 2). */
+typedef struct vp_qbench_params {
+  uint32_t fanout;             /* 0, 1 or 2                                                */
+  uint32_t depth;              /* informational (seeds carry their own depth); <= 255      */
+  unsigned long long* leaves;  /* [3] leaves per stage (reset by vp_run)                   */
+  unsigned long long* idsum;   /* [3] sum of leaf ids per stage                            */
+  unsigned long long* bad;     /* [3] leaves whose payload was corrupted                   */
+} vp_qbench_params;
 
 typedef struct vp_collatz_params {
   uint32_t* steps_out;       /* [n ids] stopping time per id                               */

@@ -74,6 +74,7 @@ class ReyesOutC(C.Structure):
 def _declare(L):
     L.orc_toy_definition.argtypes = [P, C.c_size_t, C.c_int32, P, P]
     L.orc_toy_pipeline.argtypes = [P, C.c_size_t, C.c_int32, P, P, P]
+    L.orc_qbench_pipeline.argtypes = [P, C.c_size_t, C.c_size_t, C.c_uint32, P, P, P, P]
     L.orc_collatz_definition.argtypes = [P, C.c_size_t, P]
     L.orc_collatz_pipeline.argtypes = [P, C.c_size_t, C.c_uint32, P, P, P]
     L.orc_reyes_definition.argtypes = [P, P, C.c_size_t, P]
@@ -109,6 +110,19 @@ def toy_pipeline(seeds: np.ndarray, threshold: int):
     rc = lib().orc_toy_pipeline(_ptr(seeds), seeds.size, threshold, _ptr(out), C.byref(n_out), C.byref(st))
     assert rc == 0
     return out[: n_out.value], list(st.deq[:3]), list(st.enq[:3])
+
+
+def qbench_pipeline(seeds: np.ndarray, item_bytes: int, fanout: int):
+    """Queue microbenchmark (qbench.c): returns (leaves, id sum, bad payloads, tasks dequeued)."""
+    seeds = np.ascontiguousarray(seeds, np.uint32)
+    assert seeds.size * 4 % item_bytes == 0
+    n = seeds.size * 4 // item_bytes
+    lv, ids, bad = C.c_uint64(0), C.c_uint64(0), C.c_uint64(0)
+    st = Stats()
+    rc = lib().orc_qbench_pipeline(_ptr(seeds), n, item_bytes, fanout, C.byref(lv), C.byref(ids), C.byref(bad),
+                                   C.byref(st))
+    assert rc == 0
+    return lv.value, ids.value, bad.value, int(st.deq[0])
 
 
 def collatz_definition(seeds: np.ndarray):

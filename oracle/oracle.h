@@ -62,6 +62,9 @@ typedef struct orc_stats { uint64_t deq[ORC_MAX_STAGES], enq[ORC_MAX_STAGES]; } 
 int orc_toy_definition(const int32_t* in, size_t n, int32_t threshold, int32_t* out, uint64_t* s1_passes);
 int orc_toy_pipeline(const int32_t* in, size_t n, int32_t threshold, int32_t* out, size_t* n_out,
                      orc_stats* st);
+/* qbench.c: queue microbenchmark */
+int orc_qbench_pipeline(const void* seeds, size_t n, size_t item_bytes, uint32_t fanout, uint64_t* leaves,
+                        uint64_t* idsum, uint64_t* bad, orc_stats* st);
 
 /* ---------------- Collatz queue stress (collatz.c) ---------------- */
 typedef struct orc_collatz_item { uint32_t id, steps; uint64_t v; } orc_collatz_item;

@@ -1,0 +1,110 @@
+// fam_qbench.cu — queue microbenchmark family (not a paper workload).
+//
+// Three independent self-recursive stages that differ only in their item size: 4 B (the
+// toy's int, Fig. 9 L37), 16 B (the window / tile items of Table 2) and 272 B (the
+// Reyes patch, "the largest data item structure in the queue", L61 §8.5).  A run seeds
+// ONE of them.  Every item carries {id, remaining depth}; a non-leaf item emits `fanout`
+// copies of itself one level down (fan-out 0: every seed is a leaf; 1: a chain of depth+1
+// tasks; 2: a binary tree of 2^(depth+1)-1 tasks).  Children copy the whole payload, so
+// every task moves stride bytes in and stride*fanout bytes out through the rings.  Leaves
+// check the payload and add to per-stage counters (warp-aggregated).  The task count per
+// seed is closed-form, which is what the tests pin.
+#include "../../include/vp.h"
+#include "vp_family.cuh"
+
+namespace vp {
+
+struct QBenchF {
+  static constexpr int S = 3;
+  static constexpr int kinds[S] = {VP_QB_ITEM4, VP_QB_ITEM16, VP_QB_ITEM272};
+  using Params = vp_qbench_params;
+  static constexpr int stride(int s) { return s == 0 ? 4 : s == 1 ? 16 : 272; }
+  static constexpr int threads_per_item(int) { return 1; }
+  static constexpr int max_batch(int s) { return s == 2 ? 64 : 1024; }
+  static constexpr int default_batch(int s) { return s == 2 ? 32 : 256; }
+  static constexpr int fanout(int s, int t) { return s == t ? 2 : 0; }
+  static constexpr bool rtc_ok(int, int) { return true; }
+  static constexpr int scratch_bytes(int, int) { return 0; }
+  static constexpr int default_cap_log2(int) { return 16; }  // callers size the seeded ring
+  static constexpr int min_blocks(int, int, bool) { return 2; }
+
+  // word 0: id (low 24 bits) | remaining depth << 24; words 1..: payload(id, k)
+  static __device__ __forceinline__ uint32_t payload(uint32_t id, int k) { return id * 2654435761u + (uint32_t)k * 40503u; }
+  template <int s>
+  static __device__ unsigned long long item_id(const uint8_t* it) {
+    uint32_t w = *(const uint32_t*)it;
+    return ((unsigned long long)(w >> 24) << 32) | (w & 0xffffffu);
+  }
+
+  template <int s, class Ctx>
+  static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    constexpr int W = stride(s) / 4;
+    const int lane = threadIdx.x & 31;
+    for (int base = 0; base < n; base += kThreads) {
+      const int k = base + threadIdx.x;
+      const bool valid = k < n;
+      bool leaf = false, bad = false;
+      uint32_t id = 0;
+      if (valid) {
+        const uint32_t* src = (const uint32_t*)(items + (size_t)k * stride(s));
+        const uint32_t w0 = src[0];
+        id = w0 & 0xffffffu;
+        const uint32_t d = w0 >> 24;
+        if (p.fanout == 0 || d == 0) {
+          leaf = true;
+#pragma unroll 4
+          for (int i = 1; i < W; ++i) bad |= src[i] != payload(id, i);
+        } else {
+          const int slot = ctx.template reserve<s>((int)p.fanout);
+          if (slot >= 0) {
+            for (uint32_t c = 0; c < p.fanout; ++c) {
+              uint32_t* dst = (uint32_t*)ctx.template out_ptr<s>(slot + (int)c);
+              dst[0] = id | ((d - 1) << 24);
+#pragma unroll 4
+              for (int i = 1; i < W; ++i) dst[i] = src[i];
+            }
+          }
+        }
+      }
+      // warp-aggregated sink counters: one atomic per warp per counter
+      const unsigned lm = __ballot_sync(0xffffffffu, leaf);
+      const unsigned bm = __ballot_sync(0xffffffffu, bad);
+      unsigned long long ids = leaf ? (unsigned long long)id : 0ull;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) ids += __shfl_xor_sync(0xffffffffu, ids, o);
+      if (lane == 0 && lm) {
+        atomicAdd(&p.leaves[s], (unsigned long long)__popc(lm));
+        atomicAdd(&p.idsum[s], ids);
+        if (bm) atomicAdd(&p.bad[s], (unsigned long long)__popc(bm));
+      }
+    }
+  }
+  static cudaError_t init_run(const Params& p, cudaStream_t st) {
+    cudaError_t e = cudaMemsetAsync(p.leaves, 0, 3 * sizeof(unsigned long long), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(p.idsum, 0, 3 * sizeof(unsigned long long), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(p.bad, 0, 3 * sizeof(unsigned long long), st);
+    return e;
+  }
+  static cudaError_t finalize(const Params&, cudaStream_t) { return cudaSuccess; }
+  static bool output(const Params& p, int idx, void** ptr, size_t* bytes) {
+    if (idx == 0) { *ptr = p.leaves; *bytes = 24; return true; }
+    if (idx == 1) { *ptr = p.idsum; *bytes = 24; return true; }
+    if (idx == 2) { *ptr = p.bad; *bytes = 24; return true; }
+    return false;
+  }
+  static const char* validate(const Params& p) {
+    if (!p.leaves || !p.idsum || !p.bad) return "vp_qbench_params: leaves/idsum/bad must be device pointers";
+    if (p.fanout > 2) return "vp_qbench_params: fanout must be 0, 1 or 2";
+    if (p.depth > 255) return "vp_qbench_params: depth must be <= 255";
+    if (p.fanout == 2 && p.depth > 30) return "vp_qbench_params: depth must be <= 30 with fan-out 2";
+    return nullptr;
+  }
+};
+
+const FamilyOps* family_qbench() {
+  static FamilyImpl<QBenchF> f("qbench");
+  return &f;
+}
+
+}  // namespace vp

@@ -129,5 +129,6 @@ const FamilyOps* family_raster();
 const FamilyOps* family_pyramid();
 const FamilyOps* family_cfd();
 const FamilyOps* family_facedet();
+const FamilyOps* family_qbench();
 
 }  // namespace vp

@@ -21,9 +21,10 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
+    all_families[7] = family_qbench();
     all_families[5] = family_cfd();
     all_families[6] = family_facedet();
     all_families[0] = family_toy();
@@ -79,7 +80,9 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
     c->arrivals[t].v = 0;
     c->admitted[t].v = 0;
   }
+  if (t < kMaxStages) c->wave_n[t] = 0;
   if (t == 0) {
+    c->graph_iters = 0;
     c->pending.v = (unsigned long long)ri.pending;
     c->abort.v = 0;
     c->trace_n.v = 0;
@@ -89,6 +92,69 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
 }
 
 __global__ void k_set_abort(Ctrl* c, unsigned long long why) { atomicCAS(&c->abort.v, 0ull, why); }
+
+// Wave sizing shared by the host-driven and the device-driven KBK loops: the largest wave
+// of stage s whose children are guaranteed ring space while no other stage runs.
+//  * target t != s: n * f <= cap_t - count_t.
+//  * t == s (recursion): every claim takes a ring item while ring items remain, and a
+//    block releases a claimed slot before it publishes that item's children, so the
+//    ring holds at most count_s + f*n - (ring items claimed) slots: with n_r = min(n,
+//    count_s) ring items claimed, count_s + f*n - n_r <= cap_s.
+// Zero means "not now" (a downstream wave has to drain a target first).
+__host__ __device__ inline long long wave_size(int s, long long ring_s, long long seeds_left, const long long* count,
+                                               const long long* cap, const int* fan, int S) {
+  long long n = ring_s + seeds_left;
+  for (int t = 0; t < S; ++t) {
+    const long long f = fan[t];
+    if (f <= 0) continue;
+    const long long freec = cap[t] - count[t];
+    if (freec <= 0) return 0;
+    if (t != s) {
+      n = n < freec / f ? n : freec / f;
+    } else if (f == 1) {
+      // children replace claimed ring items one for one; only seed claims need space
+      const long long m = ring_s + freec;
+      n = n < m ? n : m;
+    } else {
+      // n <= ring_s: (f-1)*n <= free;  beyond ring_s every extra (seed) item needs f slots
+      long long a = freec / (f - 1);
+      if (a < ring_s) {
+        n = n < a ? n : a;
+      } else {
+        const long long extra = (freec - (f - 1) * ring_s) / f;
+        n = n < ring_s + extra ? n : ring_s + extra;
+      }
+    }
+  }
+  return n > 0 ? n : 0;
+}
+
+// Device-driven KBK (VP_KBK_GRAPH): the host loop's control logic (read the counts,
+// size the next wave) moved into a one-thread planner kernel, and the loop itself into a
+// CUDA-graph while node.  Same wave kernels, same wave sizing rule, no host round trip.
+struct WavePlan {
+  long long n_seeds;            // seeds of this stage
+  long long cap[kMaxStages];    // ring slots per stage
+  int fan[kMaxStages];          // fan-out of this stage to each stage
+  int S;
+};
+__global__ void k_wave_plan(Ctrl* c, int s, WavePlan wp) {
+  long long count[kMaxStages];
+  for (int t = 0; t < kMaxStages; ++t) count[t] = t < wp.S ? (long long)c->count[t].v : 0;
+  long long left = wp.n_seeds - (long long)c->seed_head[s].v;
+  long long n = wave_size(s, count[s], left > 0 ? left : 0, count, wp.cap, wp.fan, wp.S);
+  if (c->abort.v != 0) n = 0;
+  c->wave_n[s] = n;
+}
+__global__ void k_wave_cond(Ctrl* c, cudaGraphConditionalHandle h) {
+  bool more = (long long)c->pending.v > 0 && c->abort.v == 0;
+  if (more && globaltimer() > c->deadline.v) {  // the wave kernels' watchdog, also for empty waves
+    atomicCAS(&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
+    more = false;
+  }
+  c->graph_iters++;
+  cudaGraphSetConditional(h, more ? 1u : 0u);
+}
 
 __global__ void k_reset_queues(Ctrl* c) {
   int t = threadIdx.x;
@@ -126,6 +192,7 @@ struct Plan {
   std::vector<KernelPlan> kernels;     // persistent kernels
   std::vector<int> kbk_stages;         // stages driven by the host wave loop
   bool wave_rtc = false;               // standalone RTC: waves of the [0,S-1] RTC kernel
+  bool kbk_graph = false;              // KBK waves driven on the device by a CUDA-graph while loop
   int batch[kMaxStages] = {};
   int cap_log2[kMaxStages] = {};       // effective ring size this plan runs with
   vp_config cfg{};
@@ -159,6 +226,10 @@ struct vp_pipeline_s {
   std::string err;
   int kernel_occ_cache[kMaxStages][kMaxStages][2] = {};
   double timeout_ms = 30000;
+  // device-driven KBK: instantiated graph and the launch arguments it was captured with
+  cudaGraph_t kg_graph = nullptr;
+  cudaGraphExec_t kg_exec = nullptr;
+  std::vector<uint8_t> kg_key;
 };
 
 namespace {
@@ -406,7 +477,9 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       pl.wave_rtc = true;
       break;
     case VP_KBK:
+    case VP_KBK_GRAPH:
       for (int s = 0; s < S; ++s) pl.kbk_stages.push_back(s);
+      pl.kbk_graph = model == VP_KBK_GRAPH;
       break;
     case VP_MEGAKERNEL: {
       int q = (b && b->blocks_per_sm[0] > 0) ? b->blocks_per_sm[0] : 0;
@@ -500,7 +573,7 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
   // RTC waves) need room for a whole wave: they use the full allocation.
   for (int t = 0; t < S; ++t) {
     int full = p->st[t].cap_log2;
-    if (!pl.kbk_stages.empty() || pl.wave_rtc) {
+    if (!pl.kbk_stages.empty() || pl.wave_rtc || (p->desc.flags & VP_FLAG_FULL_RINGS)) {
       pl.cap_log2[t] = full;
       continue;
     }
@@ -583,13 +656,13 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
   // task scheduler's priority).  A wave is capped so its output fits the target rings.
   const std::vector<int>& ks = p->plan.kbk_stages;
   const int S = (int)p->st.size();
-  auto wave_cap = [&](int s) -> long long {
-    long long cap = 1ll << 40;
-    for (int t = 0; t < S; ++t) {
-      int f = p->fam->fanout(s, t);
-      if (f > 0) cap = std::min(cap, (long long)(1ll << p->plan.cap_log2[t]) / (2 * f));
-    }
-    return std::max(1ll, cap);
+  long long caps[kMaxStages] = {};
+  int fans[kMaxStages][kMaxStages] = {};
+  for (int t = 0; t < S; ++t) caps[t] = 1ll << p->plan.cap_log2[t];
+  for (int s = 0; s < S; ++s)
+    for (int t = 0; t < S; ++t) fans[s][t] = p->fam->fanout(s, t);
+  auto wave_n = [&](int s, const Avail& a) -> long long {
+    return wave_size(s, a.ring[s], a.seeds_left[s], a.ring, caps, fans[s], S);
   };
   const auto t_start = std::chrono::steady_clock::now();
   for (;;) {
@@ -607,9 +680,8 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
     bool launched = false;
     if (p->plan.wave_rtc) {
       for (int s = 0; s < S && !launched; ++s) {
-        long long n = a.ring[s] + a.seeds_left[s];
+        long long n = wave_n(s, a);
         if (n > 0) {
-          n = std::min(n, wave_cap(s));
           rc = launch_wave(p, c, 0, S - 1, true, s, n, st, 0);
           if (rc != VP_OK) return rc;
           launched = true;
@@ -618,9 +690,8 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
     } else {
       for (int i = (int)ks.size() - 1; i >= 0 && !launched; --i) {
         int s = ks[i];
-        long long n = a.ring[s] + a.seeds_left[s];
+        long long n = wave_n(s, a);
         if (n > 0) {
-          n = std::min(n, wave_cap(s));
           rc = launch_wave(p, c, s, s, false, s, n, st, 0);
           if (rc != VP_OK) return rc;
           launched = true;
@@ -634,6 +705,84 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
       std::this_thread::sleep_for(std::chrono::microseconds(5));
     }
   }
+}
+
+// Device-driven KBK: one CUDA graph whose while node repeats
+//   for s = S-1 .. 0 (downstream first, the host loop's priority):
+//     k_wave_plan(s)  -> wave size from the live counts, capped like host_wave_loop
+//     wave kernel(s)  -> fixed grid of resident blocks; blocks past the wave exit at once
+//   k_wave_cond      -> continue while pending > 0 (and no abort / watchdog)
+// The graph is captured once per (plan, queue layout, params) and relaunched.
+vp_status graph_wave_run(vp_pipeline_s* p, const Common& c0, cudaStream_t st, uint64_t* launches) {
+  const int S = (int)p->st.size();
+  Common c = c0;
+  c.epoch = 0;  // only persistent blocks use it
+  std::vector<uint8_t> key(sizeof(Common) + p->params.size() + sizeof(p->plan.batch) + sizeof(p->plan.cap_log2));
+  memcpy(key.data(), &c, sizeof(Common));
+  memcpy(key.data() + sizeof(Common), p->params.data(), p->params.size());
+  memcpy(key.data() + sizeof(Common) + p->params.size(), p->plan.batch, sizeof(p->plan.batch));
+  memcpy(key.data() + sizeof(Common) + p->params.size() + sizeof(p->plan.batch), p->plan.cap_log2, sizeof(p->plan.cap_log2));
+  if (!p->kg_exec || key != p->kg_key) {
+    if (p->kg_exec) cudaGraphExecDestroy(p->kg_exec);
+    if (p->kg_graph) cudaGraphDestroy(p->kg_graph);
+    p->kg_exec = nullptr;
+    p->kg_graph = nullptr;
+    cudaGraph_t g;
+    CUDA_TRY(p, cudaGraphCreate(&g, 0));
+    p->kg_graph = g;
+    cudaGraphConditionalHandle h;
+    CUDA_TRY(p, cudaGraphConditionalHandleCreate(&h, g, 1u, cudaGraphCondAssignDefault));
+    cudaGraphNodeParams np = {};
+    np.type = cudaGraphNodeTypeConditional;
+    np.conditional.handle = h;
+    np.conditional.type = cudaGraphCondTypeWhile;
+    np.conditional.size = 1;
+    cudaGraphNode_t node;
+    CUDA_TRY(p, cudaGraphAddNode(&node, g, nullptr, 0, &np));
+    cudaGraph_t body = np.conditional.phGraph_out[0];
+    cudaStream_t cs;
+    CUDA_TRY(p, cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    cudaError_t ce = cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeRelaxed);
+    if (ce != cudaSuccess) {
+      cudaStreamDestroy(cs);
+      CUDA_TRY(p, ce);
+    }
+    const std::vector<int>& ks = p->plan.kbk_stages;
+    for (int i = (int)ks.size() - 1; i >= 0 && ce == cudaSuccess; --i) {
+      const int s = ks[i];
+      WavePlan wp;
+      memset(&wp, 0, sizeof(wp));
+      wp.n_seeds = (long long)p->st[s].n_seeds;
+      wp.S = S;
+      for (int t = 0; t < S; ++t) {
+        wp.fan[t] = p->fam->fanout(s, t);
+        wp.cap[t] = 1ll << p->plan.cap_log2[t];
+      }
+      k_wave_plan<<<1, 1, 0, cs>>>(p->ctrl, s, wp);
+      GroupArgs ga;
+      memset(&ga, 0, sizeof(ga));
+      ga.mode = MODE_WAVE;
+      ga.wave_stage = s;
+      ga.wave_n_dev = &p->ctrl->wave_n[s];
+      for (int t = 0; t < kMaxStages; ++t) ga.batch[t] = p->plan.batch[t] ? p->plan.batch[t] : 1;
+      int grid = std::max(1, occupancy(p, s, s, false)) * p->num_sms;
+      ce = p->fam->launch(s, s, false, c, ga, p->params.data(), grid, false, cs);
+    }
+    if (ce == cudaSuccess) {
+      k_wave_cond<<<1, 1, 0, cs>>>(p->ctrl, h);
+      ce = cudaGetLastError();
+    }
+    cudaGraph_t outg = nullptr;
+    cudaError_t ee = cudaStreamEndCapture(cs, &outg);
+    cudaStreamDestroy(cs);
+    CUDA_TRY(p, ce);
+    CUDA_TRY(p, ee);
+    CUDA_TRY(p, cudaGraphInstantiate(&p->kg_exec, g, 0));
+    p->kg_key = key;
+  }
+  CUDA_TRY(p, cudaGraphLaunch(p->kg_exec, st));
+  (void)launches;  // counted from Ctrl::graph_iters after the run
+  return VP_OK;
 }
 
 }  // namespace
@@ -746,6 +895,8 @@ vp_status vp_pipeline_destroy(void* h) {
     cudaEventDestroy(p->ev_join[i]);
     cudaEventDestroy(p->ev_kbeg[i]);
   }
+  if (p->kg_exec) cudaGraphExecDestroy(p->kg_exec);
+  if (p->kg_graph) cudaGraphDestroy(p->kg_graph);
   cudaEventDestroy(p->ev_fork);
   cudaEventDestroy(p->ev_start);
   cudaEventDestroy(p->ev_end);
@@ -933,7 +1084,10 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
     }
   }
   uint64_t launches = 0;
-  if (!pl.kbk_stages.empty() || pl.wave_rtc) {
+  if (pl.kbk_graph) {
+    vp_status rc = graph_wave_run(p, c, st, &launches);
+    if (rc != VP_OK) return rc;
+  } else if (!pl.kbk_stages.empty() || pl.wave_rtc) {
     vp_status rc = host_wave_loop(p, c, st, &launches);
     if (rc != VP_OK) return rc;
   }
@@ -969,7 +1123,7 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       for (int sm = 0; sm < VP_MAX_SM; ++sm) stats->blocks_on_sm[0][sm] = p->h_blk[sm];
     }
     stats->fallback_admits = hc.fallback_admits;
-    stats->kbk_launches = launches;
+    stats->kbk_launches = pl.kbk_graph ? hc.graph_iters * pl.kbk_stages.size() : launches;
     stats->trace_records = hc.trace_n.v;
     stats->abort_reason = (int)hc.abort.v;
     stats->num_sms = p->num_sms;

@@ -68,6 +68,8 @@ struct Ctrl {
   unsigned long long flush_ns[kMaxStages];  // FLAG_TIMERS: publish (queue overhead) per stage
   unsigned long long idle_ns[kMaxKernels];  // FLAG_TIMERS: blocks finding no work, per kernel
   unsigned long long rounds[kMaxKernels];   // persistent-loop rounds, summed over blocks, per kernel
+  unsigned long long graph_iters;           // device-driven KBK: iterations of the graph's while loop
+  long long wave_n[kMaxStages];             // device-driven KBK: size of each stage's current wave
 };
 
 struct QueueDesc {
@@ -108,6 +110,8 @@ struct GroupArgs {
   int wave_stage;                // WAVE: the stage whose items this launch processes
   long long wave_n;              // WAVE: number of items in this launch
   long long wave_chunk;          // WAVE: items per block (a multiple of the batch)
+  const long long* wave_n_dev;   // WAVE, device-driven KBK: wave size written by the planner
+                                 // kernel just before this launch (overrides wave_n/chunk)
   int batch[kMaxStages];         // items per claim, per stage
 };
 
@@ -945,9 +949,19 @@ struct Runner {
       sh.nx_n = 0;
       sh.nx_stage = -1;
       if (g.mode == MODE_WAVE) {
-        long long lo = (long long)blockIdx.x * g.wave_chunk;
-        long long rem = g.wave_n - lo;
-        sh.wave_rem = rem < 0 ? 0 : (rem < g.wave_chunk ? rem : g.wave_chunk);
+        long long wn = g.wave_n, wc = g.wave_chunk;
+        if (g.wave_n_dev) {
+          // device-driven KBK (CUDA graph): the planner kernel sized this wave; split it
+          // into whole batches over the fixed grid exactly like launch_wave does on the host
+          wn = *g.wave_n_dev;
+          const long long bt = g.batch[g.wave_stage];
+          const long long batches = (wn + bt - 1) / bt;
+          wc = ((batches + gridDim.x - 1) / gridDim.x) * bt;
+          if (wc < bt) wc = bt;
+        }
+        long long lo = (long long)blockIdx.x * wc;
+        long long rem = wn - lo;
+        sh.wave_rem = rem < 0 ? 0 : (rem < wc ? rem : wc);
       } else {
         sh.wave_rem = 0;
       }

@@ -379,7 +379,7 @@ vp_status vp_config_from_string(const char* str, vp_config* out) {
       return VP_ERR_INVALID;
     }
   }
-  if (c.model < VP_RTC || c.model > VP_HYBRID) return VP_ERR_INVALID;
+  if (c.model < VP_RTC || c.model > VP_KBK_GRAPH) return VP_ERR_INVALID;
   *out = c;
   return VP_OK;
 }

@@ -52,6 +52,19 @@ def toy_seeds(n: int, seed: int = seed_for(0), threshold: int = TOY_THRESHOLD) -
     return (np.uint64(1) + x % np.uint64(threshold - 1)).astype(np.int32)
 
 
+def qbench_seeds(n: int, item_bytes: int, depth: int, id0: int = 0) -> np.ndarray:
+    """Queue-microbenchmark seeds, as a flat uint32 array of n items:
+    word 0 = id | depth << 24 (ids id0.. mod 2^24), words 1.. = id * 2654435761 + k * 40503
+    (mod 2^32), a payload every task copies and every leaf checks."""
+    W = item_bytes // 4
+    ids = (np.arange(n, dtype=np.uint64) + np.uint64(id0)) & np.uint64(0xFFFFFF)
+    a = np.empty((n, W), np.uint32)
+    a[:, 0] = (ids | np.uint64(depth << 24)).astype(np.uint32)
+    k = np.arange(1, W, dtype=np.uint64)
+    a[:, 1:] = ((ids[:, None] * np.uint64(2654435761) + k[None, :] * np.uint64(40503)) & np.uint64(0xFFFFFFFF)).astype(np.uint32)
+    return a.reshape(-1)
+
+
 COLLATZ_DTYPE = np.dtype([("id", "<u4"), ("steps", "<u4"), ("v", "<u8")])  # 16 B
 
 

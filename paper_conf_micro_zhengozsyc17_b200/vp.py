@@ -26,8 +26,9 @@ MAX_SM = 256
 # ---- enums (vp.h)
 VP_OK, VP_ERR_INVALID, VP_ERR_UNSUPPORTED, VP_ERR_CUDA, VP_ERR_OOM, VP_ERR_QUEUE_OVERFLOW, VP_ERR_TIMEOUT, \
     VP_ERR_BINDING, VP_ERR_FANOUT = range(9)
-RTC, KBK, MEGAKERNEL, COARSE, FINE, HYBRID = range(6)
-MODEL_NAMES = {RTC: "rtc", KBK: "kbk", MEGAKERNEL: "megakernel", COARSE: "coarse", FINE: "fine", HYBRID: "hybrid"}
+RTC, KBK, MEGAKERNEL, COARSE, FINE, HYBRID, KBK_GRAPH = range(7)
+MODEL_NAMES = {RTC: "rtc", KBK: "kbk", MEGAKERNEL: "megakernel", COARSE: "coarse", FINE: "fine", HYBRID: "hybrid",
+               KBK_GRAPH: "kbk_graph"}
 GROUP_RTC, GROUP_KBK, GROUP_MEGA, GROUP_FINE = range(4)
 TOY_S1, TOY_S2, TOY_S3 = 1, 2, 3
 COLLATZ_STEP, COLLATZ_SINK = 10, 11
@@ -36,7 +37,8 @@ RASTER_VERTEX, RASTER_CLIP, RASTER_RASTER, RASTER_FRAGMENT = 30, 31, 32, 33
 PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
 FD_GRAY, FD_CDF, FD_MAP, FD_RESIZE, FD_LBP, FD_SCAN = 60, 61, 62, 63, 64, 65
-FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS = 1, 2, 4, 8
+QB_ITEM4, QB_ITEM16, QB_ITEM272 = 70, 71, 72
+FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS = 1, 2, 4, 8, 16
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
 P = C.c_void_p
@@ -90,6 +92,10 @@ class TuneReport(C.Structure):
 
 class ToyParams(C.Structure):
     _fields_ = [("threshold", C.c_int32), ("pad", C.c_int32), ("out", P), ("n_out", P)]
+
+
+class QBenchParams(C.Structure):
+    _fields_ = [("fanout", C.c_uint32), ("depth", C.c_uint32), ("leaves", P), ("idsum", P), ("bad", P)]
 
 
 class CollatzParams(C.Structure):

@@ -39,6 +39,41 @@ class ToyPipeline:
         return self.out[:n].cpu().numpy(), st
 
 
+class QBenchPipeline:
+    """Queue microbenchmark: n seeds of item_bytes (4 / 16 / 272) into
+    the matching self-recursive stage; each task re-enqueues `fanout` copies until depth 0."""
+
+    SIZES = (4, 16, 272)
+
+    def __init__(self, n: int, item_bytes: int, fanout: int, depth: int, device: int = 0, **kw):
+        self.stage = self.SIZES.index(item_bytes)
+        self.n, self.item_bytes, self.fanout, self.depth = n, item_bytes, fanout, depth
+        self.cnt = torch.zeros(9, dtype=torch.int64, device=_dev(device))
+        ptr = self.cnt.data_ptr()
+        self.prm = vp.QBenchParams(fanout=fanout, depth=depth, leaves=ptr, idsum=ptr + 24, bad=ptr + 48)
+        # full rings: a breadth-first fan-out-2 tree's frontier is a whole tree level
+        kw["flags"] = kw.get("flags", 0) | vp.FLAG_FULL_RINGS
+        self.p = vp.Pipeline(device, **kw)
+        # only the seeded stage gets a large ring (a whole tree level must fit for KBK waves)
+        big = 1 << (21 if item_bytes == 272 else 24)
+        for kind, sz in zip((vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272), self.SIZES):
+            self.p.register(kind, sz, self.prm, queue_capacity=big if sz == item_bytes else 1 << 12)
+        self.seeds = inputs.qbench_seeds(n, item_bytes, depth)
+        self.p.insert(self.stage, self.seeds, n=n)
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def tasks(self) -> int:
+        per = 1 if self.fanout == 0 else (self.depth + 1 if self.fanout == 1 else (1 << (self.depth + 1)) - 1)
+        return self.n * per
+
+    def run(self, stream=None):
+        st = self.p.run(stream)
+        c = self.cnt.cpu().numpy().astype(np.uint64)
+        return {"leaves": int(c[self.stage]), "idsum": int(c[3 + self.stage]), "bad": int(c[6 + self.stage])}, st
+
+
 class CollatzPipeline:
     def __init__(self, seeds: np.ndarray, max_steps: int = 1000, device: int = 0, **kw):
         n = int(seeds.size)

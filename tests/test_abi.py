@@ -49,10 +49,10 @@ def test_struct_sizes_match_header():
     prog = r'''
 #include <stdio.h>
 #include "vp.h"
-int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pipeline_desc), sizeof(vp_stage_desc),
+int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(vp_pipeline_desc), sizeof(vp_stage_desc),
  sizeof(vp_sm_binding), sizeof(vp_config), sizeof(vp_run_stats), sizeof(vp_autotune_opts), sizeof(vp_tune_report),
  sizeof(vp_toy_params), sizeof(vp_collatz_params), sizeof(vp_reyes_params), sizeof(vp_raster_params),
- sizeof(vp_pyramid_params));return 0;}
+ sizeof(vp_pyramid_params), sizeof(vp_cfd_params), sizeof(vp_facedet_params), sizeof(vp_qbench_params));return 0;}
 '''
     tmp = os.path.join(ROOT, "build_abi_check")
     os.makedirs(tmp, exist_ok=True)
@@ -62,7 +62,8 @@ int main(void){printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeo
     subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), c, "-o", exe], check=True)
     sizes = [int(x) for x in subprocess.run([exe], capture_output=True, text=True).stdout.split()]
     mirrors = [vp.PipelineDesc, vp.StageDesc, vp.SmBinding, vp.Config, vp.RunStats, vp.AutotuneOpts, vp.TuneReport,
-               vp.ToyParams, vp.CollatzParams, vp.ReyesParams, vp.RasterParams, vp.PyramidParams]
+               vp.ToyParams, vp.CollatzParams, vp.ReyesParams, vp.RasterParams, vp.PyramidParams, vp.CfdParams,
+               vp.FaceDetParams, vp.QBenchParams]
     assert sizes == [ctypes.sizeof(m) for m in mirrors]
 
 
@@ -82,6 +83,8 @@ def test_config_string_roundtrip():
     b = vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 44), (2, 3, vp.GROUP_RTC, 44, 148)], 148,
                         blocks_per_sm=[2, 0, 3, 0], batch=[32, 16, 8, 4])
     c = vp.Config(model=vp.HYBRID, has_binding=1, binding=b, batch=0)
+    g = vp.Config(model=vp.KBK_GRAPH, has_binding=0, batch=0)
+    assert vp.config_from_string(vp.config_to_string(g)).model == vp.KBK_GRAPH
     s = vp.config_to_string(c)
     c2 = vp.config_from_string(s)
     assert ctypes.string_at(ctypes.addressof(c), ctypes.sizeof(c)) == ctypes.string_at(ctypes.addressof(c2), ctypes.sizeof(c2))

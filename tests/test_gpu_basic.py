@@ -22,7 +22,7 @@ def hybrid_toy(vp, nsm):
     return vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, nsm // 2), (1, 2, vp.GROUP_RTC, nsm // 2, nsm)], nsm)
 
 
-@pytest.mark.parametrize("model", ["kbk", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
 def test_toy_all_models(vpm, orc, model):
     from paper_conf_micro_zhengozsyc17_b200.workloads import ToyPipeline
     vp = vpm
@@ -36,7 +36,7 @@ def test_toy_all_models(vpm, orc, model):
     elif model == "hybrid_kbk":
         tp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, nsm // 2), (1, 2, vp.GROUP_KBK, nsm // 2, nsm)], nsm))
     else:
-        tp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+        tp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
     for _ in range(2):  # repeated runs reuse the rings (monotonic tickets)
         out, st = tp.run()
         assert np.array_equal(np.sort(out), np.sort(ref_out))
@@ -64,7 +64,7 @@ def test_toy_fig9_ten_items(vpm, orc):
     assert sorted(out.tolist()) == sorted(ref.tolist()) and st["dequeued"][:3] == deq
 
 
-@pytest.mark.parametrize("model", ["kbk", "megakernel", "coarse", "fine"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine"])
 @pytest.mark.parametrize("batch", [0, 1, 32])
 def test_collatz_conservation(vpm, orc, model, batch):
     from paper_conf_micro_zhengozsyc17_b200.workloads import CollatzPipeline
@@ -73,7 +73,7 @@ def test_collatz_conservation(vpm, orc, model, batch):
     rc, ref, seen_ref, deq_ref, _ = orc.collatz_pipeline(seeds)
     assert rc == 0
     cp = CollatzPipeline(seeds)
-    cp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model], None, batch)
+    cp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model], None, batch)
     steps, seen, st = cp.run()
     assert np.array_equal(steps, ref)
     assert np.all(seen == 1)                                    # each id reaches the sink exactly once

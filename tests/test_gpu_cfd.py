@@ -21,8 +21,8 @@ def vpm():
 
 def configure(vp, cp, model):
     nsm, _ = vp.device_info(0)
-    if model in ("kbk", "megakernel", "coarse", "fine"):
-        cp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+    if model in ("kbk", "kbk_graph", "megakernel", "coarse", "fine"):
+        cp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
     elif model == "hybrid":           # [Copy, StepFactor] RTC | [Flux, TimeStep] megakernel
         cp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_RTC, 0, 24), (2, 3, vp.GROUP_MEGA, 24, nsm)], nsm))
     elif model == "hybrid_fine":      # [Copy, StepFactor] mega | [Flux, TimeStep] fine
@@ -39,7 +39,7 @@ def check(orc, sc, cp, st):
     assert st["dequeued"][:4] == [ref["n_copy"], ref["n_step"], ref["n_flux"], ref["n_time"]]
 
 
-@pytest.mark.parametrize("model", ["kbk", "megakernel", "coarse", "fine", "hybrid", "hybrid_fine"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_fine"])
 def test_cfd_64_two_iterations(vpm, orc, model):
     from paper_conf_micro_zhengozsyc17_b200.workloads import CfdPipeline
     sc = inputs.cfd_scene(G=64, n_outer=2)

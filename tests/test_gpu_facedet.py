@@ -21,8 +21,8 @@ def vpm():
 
 def configure(vp, fp, model):
     nsm, _ = vp.device_info(0)
-    if model in ("kbk", "megakernel", "coarse", "fine"):
-        fp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+    if model in ("kbk", "kbk_graph", "megakernel", "coarse", "fine"):
+        fp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
     elif model == "hybrid":      # [Gray..LBP] megakernel | [Scan] fine on most SMs
         fp.configure(vp.HYBRID, vp.make_binding([(0, 4, vp.GROUP_MEGA, 0, 40), (5, 5, vp.GROUP_MEGA, 40, nsm)], nsm))
     elif model == "hybrid_kbk":  # [Gray] mega | [CDF] KBK | [Map..Scan] mega
@@ -45,7 +45,7 @@ def check(orc, sc, fp, st):
     assert st["dequeued"][:6] == ref["deq"]
 
 
-@pytest.mark.parametrize("model", ["kbk", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
 def test_facedet_reduced(vpm, orc, model):
     """480x270 frame (SURVEY §8(d) reduced size), 2 frames."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import FaceDetPipeline

@@ -20,8 +20,8 @@ def vpm():
 
 def configure(vp, pp, model):
     nsm, _ = vp.device_info(0)
-    if model in ("kbk", "megakernel", "coarse", "fine"):
-        pp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+    if model in ("kbk", "kbk_graph", "megakernel", "coarse", "fine"):
+        pp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
     elif model == "hybrid":        # [Gray] mega | [CDF, Map, Resize] mega
         pp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, 100), (1, 3, vp.GROUP_MEGA, 100, nsm)], nsm))
     elif model == "hybrid_kbk":    # [Gray] mega | [CDF] KBK | [Map, Resize] fine
@@ -39,7 +39,7 @@ def check(orc, rgb, pp, st):
     assert st["dequeued"][:4] == [ref["n_gray"], ref["n_cdf"], ref["n_map"], ref["n_resize"]]
 
 
-@pytest.mark.parametrize("model", ["kbk", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
 def test_pyramid_reduced(vpm, orc, model):
     """512^2 x 2 images (SURVEY §8(d) reduced size)."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import PyramidPipeline

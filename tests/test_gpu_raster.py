@@ -21,8 +21,8 @@ def vpm():
 
 def configure(vp, rp, model):
     nsm, _ = vp.device_info(0)
-    if model in ("kbk", "megakernel", "coarse", "fine"):
-        rp.configure({"kbk": vp.KBK, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
+    if model in ("kbk", "kbk_graph", "megakernel", "coarse", "fine"):
+        rp.configure({"kbk": vp.KBK, "kbk_graph": vp.KBK_GRAPH, "megakernel": vp.MEGAKERNEL, "coarse": vp.COARSE, "fine": vp.FINE}[model])
     elif model == "hybrid_rtc_mega":      # [Vertex,Clip] RTC (the paper's Clip) | [Raster,Fragment] megakernel
         rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_RTC, 0, 40), (2, 3, vp.GROUP_MEGA, 40, nsm)], nsm))
     elif model == "hybrid_rtc_rtc":       # [Vertex,Clip] RTC | [Raster,Fragment] RTC
@@ -44,7 +44,7 @@ def check(orc, scene, rp, st):
     return ref
 
 
-MODELS = ["kbk", "megakernel", "coarse", "fine", "hybrid_rtc_mega", "hybrid_rtc_rtc", "hybrid_fine"]
+MODELS = ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid_rtc_mega", "hybrid_rtc_rtc", "hybrid_fine"]
 
 
 @pytest.mark.parametrize("model", MODELS)

@@ -25,6 +25,8 @@ def configure(vp, rp, model):
     h = nsm // 2
     if model == "kbk":
         rp.configure(vp.KBK)
+    elif model == "kbk_graph":            # KBK with the wave loop in a CUDA-graph while node
+        rp.configure(vp.KBK_GRAPH)
     elif model == "megakernel":
         rp.configure(vp.MEGAKERNEL)
     elif model == "coarse":
@@ -66,7 +68,7 @@ def check_against_oracle(orc, scene, rp, st, trace=None):
     return ref
 
 
-MODELS = ["kbk", "megakernel", "coarse", "fine", "hybrid_mega_rtc", "hybrid_fine_rtc", "hybrid_kbk", "hybrid_4",
+MODELS = ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid_mega_rtc", "hybrid_fine_rtc", "hybrid_kbk", "hybrid_4",
           "hybrid_mega_rtc3"]
 
 
@@ -94,7 +96,7 @@ def test_reyes_rtc_rejected(vpm):
     assert e.value.status == vp.VP_ERR_UNSUPPORTED
 
 
-@pytest.mark.parametrize("model", ["megakernel", "hybrid_mega_rtc", "kbk"])
+@pytest.mark.parametrize("model", ["megakernel", "hybrid_mega_rtc", "kbk", "kbk_graph"])
 def test_reyes_trace_multiset(vpm, orc, model):
     """Each (stage, node) is dequeued exactly once and the multiset equals the oracle's."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
@@ -130,7 +132,7 @@ def test_reyes_batch_sizes(vpm, orc, batch):
     check_against_oracle(orc, scene, rp, rp.run())
 
 
-@pytest.mark.parametrize("model", ["megakernel", "hybrid_mega_rtc", "kbk"])
+@pytest.mark.parametrize("model", ["megakernel", "hybrid_mega_rtc", "kbk", "kbk_graph"])
 def test_reyes_config5_reduced(vpm, orc, model):
     """Config 5 at CI size: 8 frames x 256 patches (SURVEY §8(d) reduced sizes)."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
