@@ -24,7 +24,8 @@ struct QBenchF {
   static constexpr int default_batch(int s) { return s == 2 ? 32 : 256; }
   static constexpr int fanout(int s, int t) { return s == t ? 2 : 0; }
   static constexpr bool rtc_ok(int, int) { return true; }
-  static constexpr int scratch_bytes(int, int) { return 0; }
+  static constexpr int kMaxBatch = 1024;
+  static constexpr int scratch_bytes(int, int) { return 2 * kMaxBatch * 4; }
   static constexpr int default_cap_log2(int) { return 16; }  // callers size the seeded ring
   static constexpr int min_blocks(int, int, bool) { return 2; }
 
@@ -36,48 +37,72 @@ struct QBenchF {
     return ((unsigned long long)(w >> 24) << 32) | (w & 0xffffffu);
   }
 
+  // Block-cooperative task: (1) one thread per item decides leaf / inner and reserves its
+  // children's out slots (one shared-memory atomic per warp); (2) one thread per (item,
+  // 16-B chunk) copies the payload into the children or checks a leaf's payload; (3) the
+  // per-item payload verdicts are counted (one global atomic per warp per counter).
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
-    constexpr int W = stride(s) / 4;
+    using V = typename Chunk<stride(s)>::T;
+    constexpr int CW = Chunk<stride(s)>::per_item;   // chunks per item
+    constexpr int EW = sizeof(V) / 4;                // words per chunk
+    int* slot = (int*)ctx.scratch();                 // [kMaxBatch] first child slot, -1 = leaf
+    int* badf = slot + kMaxBatch;                    // [kMaxBatch] leaf payload mismatch
     const int lane = threadIdx.x & 31;
+    const uint32_t fan = p.fanout;
     for (int base = 0; base < n; base += kThreads) {
       const int k = base + threadIdx.x;
       const bool valid = k < n;
-      bool leaf = false, bad = false;
-      uint32_t id = 0;
-      if (valid) {
-        const uint32_t* src = (const uint32_t*)(items + (size_t)k * stride(s));
-        const uint32_t w0 = src[0];
-        id = w0 & 0xffffffu;
-        const uint32_t d = w0 >> 24;
-        if (p.fanout == 0 || d == 0) {
-          leaf = true;
-#pragma unroll 4
-          for (int i = 1; i < W; ++i) bad |= src[i] != payload(id, i);
-        } else {
-          const int slot = ctx.template reserve<s>((int)p.fanout);
-          if (slot >= 0) {
-            for (uint32_t c = 0; c < p.fanout; ++c) {
-              uint32_t* dst = (uint32_t*)ctx.template out_ptr<s>(slot + (int)c);
-              dst[0] = id | ((d - 1) << 24);
-#pragma unroll 4
-              for (int i = 1; i < W; ++i) dst[i] = src[i];
-            }
-          }
-        }
+      uint32_t w0 = valid ? *(const uint32_t*)(items + (size_t)k * stride(s)) : 0u;
+      const bool leaf = valid && (fan == 0 || (w0 >> 24) == 0);
+      const int want = (valid && !leaf) ? (int)fan : 0;
+      int incl = want;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        int v = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += v;
       }
-      // warp-aggregated sink counters: one atomic per warp per counter
+      const int total = __shfl_sync(0xffffffffu, incl, 31);
+      int wbase = 0;
+      if (lane == 0 && total > 0) wbase = ctx.template reserve<s>(total);
+      wbase = __shfl_sync(0xffffffffu, wbase, 0);
+      if (valid) {
+        slot[k] = leaf ? -1 : (wbase < 0 ? -2 : wbase + incl - want);
+        badf[k] = 0;
+      }
       const unsigned lm = __ballot_sync(0xffffffffu, leaf);
-      const unsigned bm = __ballot_sync(0xffffffffu, bad);
-      unsigned long long ids = leaf ? (unsigned long long)id : 0ull;
+      unsigned long long ids = leaf ? (unsigned long long)(w0 & 0xffffffu) : 0ull;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) ids += __shfl_xor_sync(0xffffffffu, ids, o);
       if (lane == 0 && lm) {
         atomicAdd(&p.leaves[s], (unsigned long long)__popc(lm));
         atomicAdd(&p.idsum[s], ids);
-        if (bm) atomicAdd(&p.bad[s], (unsigned long long)__popc(bm));
       }
+    }
+    worker_sync();
+    for (int e = threadIdx.x; e < n * CW; e += kThreads) {
+      const int k = e / CW, c = e - k * CW;
+      V v = ((const V*)(items + (size_t)k * stride(s)))[c];
+      uint32_t* w = (uint32_t*)&v;
+      const int sl = slot[k];
+      const uint32_t id = ((const uint32_t*)(items + (size_t)k * stride(s)))[0] & 0xffffffu;
+      if (sl == -1) {
+        bool bad = false;
+#pragma unroll
+        for (int j = 0; j < EW; ++j)
+          if (c * EW + j > 0) bad |= w[j] != payload(id, c * EW + j);
+        if (bad) badf[k] = 1;
+      } else if (sl >= 0) {
+        if (c == 0) w[0] = id | (((w[0] >> 24) - 1) << 24);
+        for (uint32_t ch = 0; ch < fan; ++ch) ((V*)ctx.template out_ptr<s>(sl + (int)ch))[c] = v;
+      }
+    }
+    worker_sync();
+    for (int base = 0; base < n; base += kThreads) {
+      const int k = base + threadIdx.x;
+      const unsigned bm = __ballot_sync(0xffffffffu, k < n && badf[k] != 0);
+      if (lane == 0 && bm) atomicAdd(&p.bad[s], (unsigned long long)__popc(bm));
     }
   }
   static cudaError_t init_run(const Params& p, cudaStream_t st) {

@@ -197,6 +197,7 @@ __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, lo
 // Scratch of the fused [Dice, Shade] chain.
 struct ChainScratch {
   float4 M[kWarpsW][4];        // per-warp copy of the patch's frame matrix (rows)
+  float B[kWarpsW][36];        // per-warp Bernstein table B_b(j/8), [9][4]
   uint8_t list[kWarpsW][64];   // per-warp compacted list of pixel-covering micropolygons
 };
 
@@ -378,16 +379,23 @@ struct ReyesF {
   // separable Bernstein form, the 36 u-curve points C_a(v_j) staged in the (not yet
   // written) screen rows of `out`, then the 81 surface points, projection and Q8 snap.
   // Ms: the frame matrix rows in shared memory (fused chain), else read from p.M.
+  // Bt (fused chain): the Bernstein weights B_b(j/8) as a [9][4] shared-memory table,
+  // computed by bernstein() itself (bit-identical to evaluating it per point).
   template <bool kSmemM = false>
   static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
-                                                    const float4* Ms = nullptr) {
+                                                    const float4* Ms = nullptr, const float* Bt = nullptr) {
     uint32_t frame = P->id >> 12;
     if (frame >= (uint32_t)p.n_frames) frame = 0;
     const float* M = p.M + 16 * (size_t)frame;
     for (int e = lane; e < 4 * kNG; e += 32) {  // C_a(v_j), e = 9a + j
       const int a = e / kNG, j = e - a * kNG;
       float Bv[4];
-      bernstein((float)j * 0.125f, Bv);
+      if constexpr (kSmemM) {
+#pragma unroll
+        for (int b = 0; b < 4; ++b) Bv[b] = Bt[4 * j + b];
+      } else {
+        bernstein((float)j * 0.125f, Bv);
+      }
       float cx = 0.0f, cy = 0.0f, cz = 0.0f;
 #pragma unroll
       for (int b = 0; b < 4; ++b) {
@@ -401,14 +409,20 @@ struct ReyesF {
       out->g[5][e] = cz;
     }
     __syncwarp();
-    float xs[3], ys[3], zs_[3];
+    // S(u_i, v_j): object-space rows 0..2 are written at once (the C rows 3..5 are still
+    // being read by other lanes, so the screen rows wait for the next __syncwarp)
 #pragma unroll
     for (int r = 0; r < 3; ++r) {
       const int g = lane + 32 * r;
       if (g < kNP) {
         const int i = g / kNG, j = g - i * kNG;
         float Bu[4];
-        bernstein((float)i * 0.125f, Bu);
+        if constexpr (kSmemM) {
+#pragma unroll
+          for (int a = 0; a < 4; ++a) Bu[a] = Bt[4 * i + a];
+        } else {
+          bernstein((float)i * 0.125f, Bu);
+        }
         float x = 0.0f, y = 0.0f, z = 0.0f;
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
@@ -416,9 +430,9 @@ struct ReyesF {
           y = y + Bu[a] * out->g[4][a * kNG + j];
           z = z + Bu[a] * out->g[5][a * kNG + j];
         }
-        xs[r] = x;
-        ys[r] = y;
-        zs_[r] = z;
+        out->g[0][g] = x;
+        out->g[1][g] = y;
+        out->g[2][g] = z;
       }
     }
     __syncwarp();  // every C read before the screen rows are written
@@ -426,7 +440,7 @@ struct ReyesF {
     for (int r = 0; r < 3; ++r) {
       const int g = lane + 32 * r;
       if (g < kNP) {
-        const float x = xs[r], y = ys[r], z = zs_[r];
+        const float x = out->g[0][g], y = out->g[1][g], z = out->g[2][g];  // this lane's own writes
         float4 c;
         if constexpr (kSmemM) {
           float cc[4];
@@ -445,9 +459,6 @@ struct ReyesF {
         }
         float sx, sy, zs;
         screen(p, c, sx, sy, zs);
-        out->g[0][g] = x;
-        out->g[1][g] = y;
-        out->g[2][g] = z;
         // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
         const float X = sx * 256.0f, Y = sy * 256.0f;
         const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
@@ -622,6 +633,12 @@ struct ReyesF {
     // screen, so a static warp -> patch map leaves warps idle at the round barrier.
     int* next = ctx.work_counter();
     if (threadIdx.x == 0) ctx.template note_local_count<SHADE>(n);  // Dice emits one grid per patch
+    float* Bt = cs.B[warp];
+    for (int e = lane; e < 36; e += 32) {
+      float B4[4];
+      bernstein((float)(e >> 2) * 0.125f, B4);
+      Bt[e] = B4[e & 3];
+    }
     for (;;) {
       int k = 0;
       if (lane == 0) k = atomicAdd(next, 1);
@@ -632,7 +649,7 @@ struct ReyesF {
       if (frame >= (uint32_t)p.n_frames) frame = 0;
       if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
       __syncwarp();
-      dice_patch<true>(p, P, g, lane, cs.M[warp]);
+      dice_patch<true>(p, P, g, lane, cs.M[warp], Bt);
       __syncwarp();
       if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
       const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);

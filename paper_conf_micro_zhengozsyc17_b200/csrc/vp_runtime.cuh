@@ -168,6 +168,9 @@ __device__ __forceinline__ void mbar_init(unsigned long long* m, uint32_t count)
 __device__ __forceinline__ void mbar_arrive_expect_tx(unsigned long long* m, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(m)), "r"(bytes) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(unsigned long long* m) {
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_u32(m)) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(unsigned long long* m, uint32_t parity) {
   uint32_t done = 0;
   while (!done) {
@@ -322,7 +325,10 @@ struct BlockShared {
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
   unsigned long long mbar[2];          // bulk-copy completion, one per in buffer
   uint32_t mbar_phase[2];
-  int work_next;                       // per-round work counter (dynamic hand-out within a batch)
+  int work[2];                         // per in buffer work counter (dynamic hand-out within a batch)
+  // sink groups (no ring outputs): buffer hand-over without the round barrier
+  unsigned long long full[2], empty[2];  // mbarriers: fetcher -> workers, workers -> fetcher
+  int bn[2], bstage[2];                // items (-1: stop) and stage of each in buffer
 };
 
 __device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
@@ -352,7 +358,7 @@ struct Ctx {
   __device__ __forceinline__ uint8_t* scratch() { return smem + kScratch; }
   // Zero at the start of every round: worker warps may hand out the batch's items among
   // themselves with atomicAdd on it (dynamic load balance inside a batch).
-  __device__ __forceinline__ int* work_counter() { return &sh.work_next; }
+  __device__ __forceinline__ int* work_counter() { return &sh.work[ob]; }
 
   template <int T>
   __device__ __forceinline__ uint8_t* out_ptr(int slot) {
@@ -945,7 +951,7 @@ struct Runner {
       }
       sh.acc_neg = 0;
       sh.done = 0;
-      sh.work_next = 0;
+      sh.work[0] = sh.work[1] = 0;
       sh.nx_n = 0;
       sh.nx_stage = -1;
       if (g.mode == MODE_WAVE) {
@@ -986,11 +992,93 @@ struct Runner {
     }
   }
 
+  // A sink group emits nothing to any ring (every successor of its stages is a later
+  // stage of the same RTC chain, or none): it needs no publisher, so worker warps and the
+  // fetcher hand the two in buffers over through mbarriers instead of a block barrier
+  // per round.  A worker warp that finishes its share of batch i starts batch i+1 as
+  // soon as the fetcher staged it, instead of waiting for the slowest warp of batch i.
+  static constexpr bool sink_group() {
+    for (int s = LO; s <= HI; ++s)
+      for (int t = 0; t < S; ++t)
+        if (F::fanout(s, t) > 0 && !(RTC && t > LO && t <= HI)) return false;
+    return true;
+  }
+
+  static __device__ void run_sink(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, uint8_t* smem) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (warp < kWarpsW) {
+      for (int it = 0;; ++it) {
+        const int b = it & 1;
+        mbar_wait(&sh.full[b], (uint32_t)((it >> 1) & 1));
+        const int n = sh.bn[b];
+        if (n < 0) break;
+        ctx.ob = b;
+        execute(a, ctx, sh, sh.bstage[b], in_buf(smem, b), n);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sh.empty[b]);
+      }
+    } else if (warp == W_FETCH) {
+      int last[2] = {0, 0};  // items of each buffer's last use, retired once it drains
+      for (int it = 0;; ++it) {
+        const int b = it & 1;
+        if (it >= 2) {
+          mbar_wait(&sh.empty[b], (uint32_t)(((it >> 1) - 1) & 1));
+          if (lane == 0) sh.acc_neg -= last[b];
+          last[b] = 0;
+        }
+        bool other_drained = it == 0;
+        for (;;) {
+          fetch(a, sh, smem, b, other_drained, lane);
+          __syncwarp();
+          if (sh.nx_n > 0 || sh.done) break;
+          if (!other_drained) {
+            // the block may be idle: the other buffer's batch must drain (and be retired)
+            // before the termination test
+            mbar_wait(&sh.empty[b ^ 1], (uint32_t)(((it - 1) >> 1) & 1));
+            if (lane == 0) sh.acc_neg -= last[b ^ 1];
+            last[b ^ 1] = 0;
+            other_drained = true;
+          }
+        }
+        const bool stop = sh.done && sh.nx_n == 0;
+        last[b] = stop ? 0 : sh.nx_n;
+        if (lane == 0) {
+          sh.bn[b] = stop ? -1 : sh.nx_n;
+          sh.bstage[b] = sh.nx_stage;
+          sh.work[b] = 0;
+          sh.rounds++;
+          mbar_arrive(&sh.full[b]);
+        }
+        __syncwarp();
+        if (stop) break;
+      }
+      // still-staged batches (abort path) are executed by the workers before they reach
+      // the stop marker; they are retired here and flushed after the final block barrier
+      if (lane == 0) sh.acc_neg -= last[0] + last[1];
+    }
+  }
+
   static __device__ void run(const KArgs<F>& a) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ BlockShared sh;
     if (!admit(a, sh)) return;
     CtxT ctx(a, smem, sh);
+    if constexpr (sink_group()) {
+      if (threadIdx.x == 0) {
+        for (int b = 0; b < 2; ++b) {
+          mbar_init(&sh.full[b], 1);
+          mbar_init(&sh.empty[b], kWarpsW);
+        }
+      }
+      if constexpr (F::scratch_bytes(LO, HI) > 0) {
+        for (int i = threadIdx.x; i < F::scratch_bytes(LO, HI) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+      }
+      __syncthreads();
+      run_sink(a, ctx, sh, smem);
+      __syncthreads();
+      flush_stats(a, sh);
+      return;
+    }
     if constexpr (F::scratch_bytes(LO, HI) > 0) {  // family scratch starts zeroed
       for (int i = threadIdx.x; i < F::scratch_bytes(LO, HI) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
     }
@@ -1001,9 +1089,9 @@ struct Runner {
     int b = 0, prev_s = -1, prev_n = 0;
     for (;;) {
       const int done = sh.done, cur_s = sh.nx_stage, cur_n = sh.nx_n;
-      // the previous round's users of work_next finished at its end barrier; this round's
-      // start after the next one
-      if (threadIdx.x == 0) sh.work_next = 0;
+      // the previous round's users of the work counters finished at its end barrier; this
+      // round's start after the next one
+      if (threadIdx.x == 0) sh.work[0] = sh.work[1] = 0;
       __syncthreads();  // everyone has read the round's batch; the fetcher may overwrite it
       if (done) break;
       if (warp < kWarpsW) {
