@@ -212,6 +212,8 @@ struct ReyesF {
   // Dice batches above 8 only in the fused RTC [Dice, Shade] kernel, whose grids stay in
   // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
   static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
+    // block-local [Bound, Split]: the first stack pass takes the whole claimed batch
+    if (!rtc && lo == BOUND && hi == SPLIT && (s == BOUND || s == SPLIT)) return 16;
     return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
   }
   static constexpr int fused_local_cap(int, int, int) { return kThreads / 32; }
@@ -222,7 +224,9 @@ struct ReyesF {
   static constexpr bool rtc_ok(int, int) { return true; }
   // every kernel whose range ends in [Dice, Shade] may run the fused chain (an RTC
   // kernel [Split..Shade] fuses its Dice batches too), so each reserves the chain scratch
-  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0; }
+  static constexpr int scratch_bytes(int lo, int hi) {
+    return (lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : (lo == BOUND && hi == SPLIT) ? (int)sizeof(LocalStack) : 0;
+  }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
   static constexpr int min_blocks(int, int, bool) { return VP_REYES_MINB; }
@@ -248,6 +252,67 @@ struct ReyesF {
   }
 
   // -------------------------------------------------------------- Bound (16 thr/patch)
+  // Bound of patch P by one 16-thread group (lane = its control point; both groups of a
+  // warp call together, `valid` may differ): returns 0 cull, 1 split, 2 dice (readings
+  // R-R2..R-R5), the split direction, and this thread's control point q.
+  static __device__ __forceinline__ int bound_patch(const Params& p, const RPatch* P, int lane, bool valid, int& dir,
+                                                    float4& q) {
+    const uint32_t id = P->id, depth = P->depth;
+    uint32_t frame = id >> 12;
+    if (frame >= (uint32_t)p.n_frames) frame = 0;
+    const float* M = p.M + 16 * (size_t)frame;
+    q = P->cp[lane];
+    float4 c = project(M, q.x, q.y, q.z, q.w);
+    const bool behind = !(c.w > p.near_w);
+    const unsigned bal = __ballot_sync(0xffffffffu, behind);
+    const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
+    float sx, sy, zs;
+    screen(p, c, sx, sy, zs);
+    // screen-space split metric (reading R-R5)
+    float sx12 = __shfl_sync(0xffffffffu, sx, (lane & 3) + 12, 16), sy12 = __shfl_sync(0xffffffffu, sy, (lane & 3) + 12, 16);
+    float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
+    float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
+    float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
+    // object-space metric (near-plane straddle, R-R4)
+    float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16), oy12 = __shfl_sync(0xffffffffu, q.y, (lane & 3) + 12, 16),
+          oz12 = __shfl_sync(0xffffffffu, q.z, (lane & 3) + 12, 16);
+    float ox3 = __shfl_down_sync(0xffffffffu, q.x, 3, 16), oy3 = __shfl_down_sync(0xffffffffu, q.y, 3, 16),
+          oz3 = __shfl_down_sync(0xffffffffu, q.z, 3, 16);
+    float olu = 0.0f, olv = 0.0f;
+    if (lane < 4) {
+      olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
+      olu = olu + fabsf(oz12 - q.z);
+    }
+    if ((lane & 3) == 0) {
+      olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
+      olv = olv + fabsf(oz3 - q.z);
+    }
+    float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
+    lu = red16_max(lu);
+    lv = red16_max(lv);
+    olu = red16_max(olu);
+    olv = red16_max(olv);
+    int cls;  // 0 cull, 1 split, 2 dice
+    dir = 0;
+    if (nbehind == 16) {
+      cls = 0;
+    } else if (nbehind > 0) {
+      cls = ((int)depth >= p.max_depth) ? 0 : 1;
+      dir = (olu >= olv) ? 0 : 1;
+    } else if (xmax < 0.0f || xmin >= (float)p.W || ymax < 0.0f || ymin >= (float)p.H) {
+      cls = 0;
+    } else {
+      float bw = xmax - xmin, bh = ymax - ymin;
+      float ext = bw > bh ? bw : bh;
+      if ((int)depth >= p.max_depth || ext <= p.t_dice) cls = 2;
+      else {
+        cls = 1;
+        dir = (lu >= lv) ? 0 : 1;
+      }
+    }
+    return valid ? cls : 0;
+  }
+
   template <class Ctx>
   static __device__ void bound(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
@@ -256,60 +321,10 @@ struct ReyesF {
       const int k = r0 + (threadIdx.x >> 4);
       const bool valid = k < n;
       const RPatch* P = (const RPatch*)(items + (size_t)(valid ? k : 0) * sizeof(RPatch));
-      const uint32_t id = P->id, depth = P->depth;
-      uint32_t frame = id >> 12;
-      if (frame >= (uint32_t)p.n_frames) frame = 0;
-      const float* M = p.M + 16 * (size_t)frame;
-      const float4 q = P->cp[lane];
-      float4 c = project(M, q.x, q.y, q.z, q.w);
-      const bool behind = !(c.w > p.near_w);
-      const unsigned bal = __ballot_sync(0xffffffffu, behind);
-      const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
-      float sx, sy, zs;
-      screen(p, c, sx, sy, zs);
-      // screen-space split metric (reading R-R5)
-      float sx12 = __shfl_sync(0xffffffffu, sx, (lane & 3) + 12, 16), sy12 = __shfl_sync(0xffffffffu, sy, (lane & 3) + 12, 16);
-      float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
-      float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
-      float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
-      // object-space metric (near-plane straddle, R-R4)
-      float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16), oy12 = __shfl_sync(0xffffffffu, q.y, (lane & 3) + 12, 16),
-            oz12 = __shfl_sync(0xffffffffu, q.z, (lane & 3) + 12, 16);
-      float ox3 = __shfl_down_sync(0xffffffffu, q.x, 3, 16), oy3 = __shfl_down_sync(0xffffffffu, q.y, 3, 16),
-            oz3 = __shfl_down_sync(0xffffffffu, q.z, 3, 16);
-      float olu = 0.0f, olv = 0.0f;
-      if (lane < 4) {
-        olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
-        olu = olu + fabsf(oz12 - q.z);
-      }
-      if ((lane & 3) == 0) {
-        olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
-        olv = olv + fabsf(oz3 - q.z);
-      }
-      float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
-      lu = red16_max(lu);
-      lv = red16_max(lv);
-      olu = red16_max(olu);
-      olv = red16_max(olv);
-      int cls;  // 0 cull, 1 split, 2 dice
-      int dir = 0;
-      if (nbehind == 16) {
-        cls = 0;
-      } else if (nbehind > 0) {
-        cls = ((int)depth >= p.max_depth) ? 0 : 1;
-        dir = (olu >= olv) ? 0 : 1;
-      } else if (xmax < 0.0f || xmin >= (float)p.W || ymax < 0.0f || ymin >= (float)p.H) {
-        cls = 0;
-      } else {
-        float bw = xmax - xmin, bh = ymax - ymin;
-        float ext = bw > bh ? bw : bh;
-        if ((int)depth >= p.max_depth || ext <= p.t_dice) cls = 2;
-        else {
-          cls = 1;
-          dir = (lu >= lv) ? 0 : 1;
-        }
-      }
-      if (!valid) cls = 0;
+      int dir;
+      float4 q;
+      const int cls = bound_patch(p, P, lane, valid, dir, q);
+      const uint32_t depth = P->depth;
       int slot = -1;
       if (lane == 0 && cls == 1) slot = ctx.template reserve<SPLIT>();
       if (lane == 0 && cls == 2) slot = ctx.template reserve<DICE>();
@@ -318,7 +333,7 @@ struct ReyesF {
         RPatch* out = (RPatch*)(cls == 1 ? ctx.template out_ptr<SPLIT>(slot) : ctx.template out_ptr<DICE>(slot));
         out->cp[lane] = q;
         if (lane == 0) {
-          out->id = id;
+          out->id = P->id;
           out->path = P->path;
           out->dirs = (cls == 1) ? ((P->dirs & ~(1u << depth)) | ((uint32_t)dir << depth)) : P->dirs;
           out->depth = depth;
@@ -328,22 +343,15 @@ struct ReyesF {
   }
 
   // -------------------------------------------------------------- Split (16 thr/patch)
-  template <class Ctx>
-  static __device__ void split(Ctx& ctx, const uint8_t* items, int n) {
-    const int lane = threadIdx.x & 15;
+  // de Casteljau at t = 1/2 (reading R-R6) of the curve through this thread's control point
+  // (thread `lane` of a 16-thread group): L / R are child control point `my` of the two halves.
+  static __device__ __forceinline__ void split_cp(const RPatch* P, int dir, int lane, float4& L, float4& R, int& my) {
     const int line = lane >> 2, t = lane & 3;
-    for (int r0 = 0; r0 < n; r0 += kThreads / 16) {
-      const int k = r0 + (threadIdx.x >> 4);
-      const bool valid = k < n;
-      const RPatch* P = (const RPatch*)(items + (size_t)(valid ? k : 0) * sizeof(RPatch));
-      const uint32_t depth = P->depth;
-      const int dir = (int)((P->dirs >> depth) & 1u);
-      // control point u of this thread's curve: (u, line) for a u-split, (line, u) for v
-      const int base = dir == 0 ? line : 4 * line, step = dir == 0 ? 4 : 1;
-      const int my = base + step * t;
-      float4 a = P->cp[base], b = P->cp[base + step], c = P->cp[base + 2 * step], d = P->cp[base + 3 * step];
-      float4 L, R;
-      // de Casteljau at t = 1/2 (reading R-R6), per component, exactly this order
+    // control point u of this thread's curve: (u, line) for a u-split, (line, u) for v
+    const int base = dir == 0 ? line : 4 * line, step = dir == 0 ? 4 : 1;
+    my = base + step * t;
+    float4 a = P->cp[base], b = P->cp[base + step], c = P->cp[base + 2 * step], d = P->cp[base + 3 * step];
+    // per component, exactly this order
 #define VP_CASTELJAU(comp)                                                   \
   {                                                                          \
     float ab = (a.comp + b.comp) * 0.5f, bc = (b.comp + c.comp) * 0.5f;      \
@@ -353,8 +361,31 @@ struct ReyesF {
     L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
     R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
   }
-      VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+    VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
 #undef VP_CASTELJAU
+  }
+  // children headers (split tree: path bit `depth` = 0 left / 1 right, dirs bit = direction)
+  static __device__ __forceinline__ void split_headers(RPatch* l, RPatch* r, uint32_t id, uint32_t path, uint32_t dirs,
+                                                       uint32_t depth, int dir) {
+    l->id = r->id = id;
+    l->dirs = r->dirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
+    l->depth = r->depth = depth + 1;
+    l->path = path & ~(1u << depth);
+    r->path = path | (1u << depth);
+  }
+
+  template <class Ctx>
+  static __device__ void split(Ctx& ctx, const uint8_t* items, int n) {
+    const int lane = threadIdx.x & 15;
+    for (int r0 = 0; r0 < n; r0 += kThreads / 16) {
+      const int k = r0 + (threadIdx.x >> 4);
+      const bool valid = k < n;
+      const RPatch* P = (const RPatch*)(items + (size_t)(valid ? k : 0) * sizeof(RPatch));
+      const uint32_t depth = P->depth;
+      const int dir = (int)((P->dirs >> depth) & 1u);
+      float4 L, R;
+      int my;
+      split_cp(P, dir, lane, L, R, my);
       int slot = -1;
       if (lane == 0 && valid) slot = ctx.template reserve<BOUND>(2);
       slot = __shfl_sync(0xffffffffu, slot, 0, 16);
@@ -363,14 +394,125 @@ struct ReyesF {
         RPatch* r = (RPatch*)ctx.template out_ptr<BOUND>(slot + 1);
         l->cp[my] = L;
         r->cp[my] = R;
-        if (lane == 0) {
-          l->id = r->id = P->id;
-          l->dirs = r->dirs = (P->dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
-          l->depth = r->depth = depth + 1;
-          l->path = P->path & ~(1u << depth);
-          r->path = P->path | (1u << depth);
+        if (lane == 0) split_headers(l, r, P->id, P->path, P->dirs, depth, dir);
+      }
+    }
+  }
+
+  // -------------------------------------------------------------- [Bound, Split] locally
+  // Block-local recursion (the paper fuses Bound into Split, L55): a batch
+  // of Bound (or Split) items is worked off from a shared-memory stack.  Each pass pops up
+  // to 16 patches (16 threads each), bounds them, culls, appends diceable ones to the Dice
+  // out buffer and splits the others in place, pushing both children back.  Only what is
+  // left when the stack or the Dice buffer would overflow goes back to the Bound ring, so
+  // Split items never travel through a ring.  Same arithmetic as bound() / split().
+  static constexpr int kStack = 48, kLocalDice = 48;
+  struct LocalStack {
+    RPatch st[kStack];
+    int top, nchild, nbound, nsplit, dump;
+  };
+  static constexpr bool local_recursion(int lo, int hi) { return lo == BOUND && hi == SPLIT; }
+  static constexpr int local_out_cap(int, int, int t) { return t == BOUND ? kStack : t == DICE ? kLocalDice : 0; }
+
+  template <int SS, int LO, int HI, class Ctx>
+  static __device__ void exec_local(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    LocalStack& ls = *(LocalStack*)ctx.scratch();
+    const int lane = threadIdx.x & 15, grp = threadIdx.x >> 4;
+    if constexpr (SS == BOUND) {
+      for (int e = threadIdx.x; e < n * 17; e += kThreads) ((uint4*)ls.st)[e] = ((const uint4*)items)[e];
+      if (threadIdx.x == 0) ls.top = n;
+    } else {
+      for (int r0 = 0; r0 < n; r0 += kThreads / 16) {  // Split items: their Bound already chose the direction
+        const int k = r0 + grp;
+        if (k < n) {
+          const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
+          const uint32_t depth = P->depth;
+          const int dir = (int)((P->dirs >> depth) & 1u);
+          float4 L, R;
+          int my;
+          split_cp(P, dir, lane, L, R, my);
+          ls.st[2 * k].cp[my] = L;
+          ls.st[2 * k + 1].cp[my] = R;
+          if (lane == 0) split_headers(&ls.st[2 * k], &ls.st[2 * k + 1], P->id, P->path, P->dirs, depth, dir);
         }
       }
+      if (threadIdx.x == 0) ls.top = 2 * n;
+    }
+    if (threadIdx.x == 0) ls.nchild = ls.nbound = ls.nsplit = 0;
+    worker_sync();
+    bool first = SS == BOUND;  // the first pass pops exactly the claimed Bound items (n <= 16)
+    for (;;) {
+      const int top = ls.top;
+      const int dice_room = Ctx::template cap<DICE>() - ctx.sh.out_cnt[ctx.ob][DICE];
+      const int m = min(min(kThreads / 16, top), min(kStack - top, dice_room));
+      if (m <= 0) break;
+      const int base = top - m;
+      const bool mine = grp < m;
+      const RPatch* P = &ls.st[base + (mine ? grp : 0)];
+      int dir;
+      float4 q;
+      const int cls = bound_patch(p, P, lane, mine, dir, q);
+      const uint32_t id = P->id, path = P->path, dirs = P->dirs, depth = P->depth;
+      float4 L, R;
+      int my = 0;
+      if (cls == 1) split_cp(P, dir, lane, L, R, my);
+      if (lane == 0 && mine) {
+        if (!first) ctx.template trace_local<BOUND>((const uint8_t*)P);
+        if (cls == 1) ctx.template trace_local<SPLIT>((const uint8_t*)P);
+      }
+      if (cls == 2) {
+        int slot = 0;
+        if (lane == 0) slot = ctx.template reserve<DICE>();
+        slot = __shfl_sync(0xFFFFu << (threadIdx.x & 16), slot, threadIdx.x & 16, 32);
+        if (slot >= 0) {
+          RPatch* out = (RPatch*)ctx.template out_ptr<DICE>(slot);
+          out->cp[lane] = q;
+          if (lane == 0) {
+            out->id = id;
+            out->path = path;
+            out->dirs = dirs;
+            out->depth = depth;
+          }
+        }
+      }
+      worker_sync();  // every read of the popped patches is done
+      if (cls == 1) {
+        int c = 0;
+        if (lane == 0) {
+          c = atomicAdd(&ls.nchild, 2);
+          atomicAdd(&ls.nsplit, 1);
+        }
+        c = __shfl_sync(0xFFFFu << (threadIdx.x & 16), c, threadIdx.x & 16, 32);
+        RPatch* l = &ls.st[base + c];
+        RPatch* r = &ls.st[base + c + 1];
+        l->cp[my] = L;
+        r->cp[my] = R;
+        if (lane == 0) split_headers(l, r, id, path, dirs, depth, dir);
+      }
+      worker_sync();
+      if (threadIdx.x == 0) {
+        ls.top = base + ls.nchild;
+        ls.nchild = 0;
+        if (!first) ls.nbound += m;
+      }
+      worker_sync();
+      first = false;
+    }
+    // what is left goes back to the Bound ring (unbounded children: no work is repeated)
+    const int left = ls.top;
+    if (left > 0) {
+      if (threadIdx.x == 0) ls.dump = ctx.template reserve<BOUND>(left);
+      worker_sync();
+      const int d = ls.dump;
+      if (d >= 0) {
+        uint4* dst = (uint4*)ctx.template out_ptr<BOUND>(d);
+        for (int e = threadIdx.x; e < left * 17; e += kThreads) dst[e] = ((const uint4*)ls.st)[e];
+      }
+    }
+    if (threadIdx.x == 0) {
+      ctx.template note_local_count<BOUND>(ls.nbound);
+      ctx.template note_local_count<SPLIT>(ls.nsplit);
     }
   }
 

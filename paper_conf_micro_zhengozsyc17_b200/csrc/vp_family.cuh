@@ -33,6 +33,8 @@ struct FamilyOps {
   virtual int default_batch(int s) const = 0;
   virtual int threads_per_item(int s) const = 0;
   virtual int fanout(int s, int t) const = 0;
+  virtual int out_cap(int lo, int hi, bool rtc, int t) const = 0;  // items a kernel publishes to t per batch
+  virtual bool local_rec(int lo, int hi, bool rtc) const = 0;        // block-local recursion kernel
   virtual bool rtc_legal(int lo, int hi) const = 0;
   virtual bool latched(int lo, int hi) const = 0;
   virtual int default_cap_log2(int s) const = 0;
@@ -90,6 +92,20 @@ struct FamilyImpl final : FamilyOps {
   int default_batch(int s) const override { return F::default_batch(s); }
   int threads_per_item(int s) const override { return F::threads_per_item(s); }
   int fanout(int s, int t) const override { return F::fanout(s, t); }
+  template <int LO, int HI>
+  int out_cap_of(int lo, int hi, bool rtc, int t) const {
+    if constexpr (LO < F::S) {
+      if constexpr (HI < F::S) {
+        if (lo == LO && hi == HI) return G::out_cap(LO, HI, rtc && G::rtc_legal(LO, HI), t);
+        return out_cap_of<LO, HI + 1>(lo, hi, rtc, t);
+      } else {
+        return out_cap_of<LO + 1, LO + 1>(lo, hi, rtc, t);
+      }
+    }
+    return 0;
+  }
+  int out_cap(int lo, int hi, bool rtc, int t) const override { return out_cap_of<0, 0>(lo, hi, rtc, t); }
+  bool local_rec(int lo, int hi, bool rtc) const override { return local_recursion<F>(lo, hi, rtc); }
   bool rtc_legal(int lo, int hi) const override { return fn[lo][hi][1] != nullptr; }
   bool latched(int lo, int hi) const override { return !F::rtc_ok(lo, hi); }
   int default_cap_log2(int s) const override { return F::default_cap_log2(s); }

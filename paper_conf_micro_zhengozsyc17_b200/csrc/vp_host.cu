@@ -583,6 +583,8 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       long long blocks = (long long)per * mask_count(k.mask, N);
       long long mx = 0;
       for (int s = k.lo; s <= k.hi; ++s) mx = std::max(mx, (long long)pl.batch[s] * p->fam->fanout(s, t));
+      // block-local recursion publishes up to its out-buffer capacity per batch
+      if (p->fam->local_rec(k.lo, k.hi, k.rtc)) mx = std::max(mx, (long long)p->fam->out_cap(k.lo, k.hi, false, t));
       need += 2 * blocks * mx;
     }
     int lg = 12;

@@ -255,6 +255,38 @@ constexpr int fused_local_cap(int lo, int hi, int t) {
   else return 0;
 }
 
+// A family may run the batches of a persistent (non-RTC) kernel [lo, hi] with block-local
+// recursion (F::local_recursion(lo, hi), F::exec_local<s, LO, HI>): children that would go
+// back to a ring of the same kernel are processed in the block from a shared-memory work
+// stack, and only what does not fit is published.  Its out-buffer capacities are then
+// F::local_out_cap(lo, hi, t).
+template <class F, class = void>
+struct HasLocalRec : std::false_type {};
+template <class F>
+struct HasLocalRec<F, std::void_t<decltype(F::local_recursion(0, 0))>> : std::true_type {};
+template <class F>
+constexpr bool local_recursion(int lo, int hi, bool rtc) {
+  if constexpr (HasLocalRec<F>::value) return !rtc && F::local_recursion(lo, hi);
+  else return false;
+}
+template <class F>
+constexpr int local_out_cap(int lo, int hi, int t) {
+  if constexpr (HasLocalRec<F>::value) return F::local_out_cap(lo, hi, t);
+  else return 0;
+}
+template <class F, bool kHas = HasLocalRec<F>::value>
+struct LocalRec {
+  template <int SS, int LO, int HI, class C>
+  static __device__ __forceinline__ void run(C&, const uint8_t*, int) {}
+};
+template <class F>
+struct LocalRec<F, true> {
+  template <int SS, int LO, int HI, class C>
+  static __device__ __forceinline__ void run(C& ctx, const uint8_t* items, int n) {
+    F::template exec_local<SS, LO, HI>(ctx, items, n);
+  }
+};
+
 // ------------------------------------------------------------------ constexpr graph helpers
 template <class F>
 struct Graph {
@@ -280,6 +312,7 @@ struct Graph {
   // out-buffer capacity (items) for target t in a kernel [lo,hi]
   static constexpr int out_cap(int lo, int hi, bool rtc, int t) {
     if (rtc && lo < t && t <= hi && fused_chain<F>(lo, hi)) return fused_local_cap<F>(lo, hi, t);
+    if (local_recursion<F>(lo, hi, rtc)) return local_out_cap<F>(lo, hi, t);
     int c = 0;
     for (int s = lo; s <= hi; ++s) {
       if (fan(s, t) == 0) continue;
@@ -383,6 +416,7 @@ struct Ctx {
   template <int T>
   __device__ __forceinline__ void note_local_count(int n) {
     sh.deq[T] += (unsigned long long)n;
+    sh.enq[T] += (unsigned long long)n;  // entered stage T block-locally (sum enq == sum deq holds)
   }
   // ... and, with FLAG_TRACE, the trace record of one of them (one thread per item).
   template <int T>
@@ -872,6 +906,8 @@ struct Runner {
         if (threadIdx.x == 0) sh.deq[SS] += n;
         if constexpr (RTC && SS < HI && fused_chain<F>(SS, HI)) {
           FusedChain<F>::template run<SS, HI>(ctx, items, n);
+        } else if constexpr (local_recursion<F>(LO, HI, RTC)) {
+          LocalRec<F>::template run<SS, LO, HI>(ctx, items, n);
         } else {
         F::template exec<SS>(ctx, items, n);
         if constexpr (RTC && SS < HI) {

@@ -18,6 +18,8 @@ ap.add_argument("--frames", type=int, default=512)
 ap.add_argument("--reps", type=int, default=3)
 ap.add_argument("--configs", default="mega,kbk,h37,h50,h74,h100,fine_h")
 ap.add_argument("--batch", type=int, default=0)
+ap.add_argument("--bats", default="", help="per-stage batch sets for hybrid configs, e.g. 32,16,8,4;32,16,64,4")
+ap.add_argument("--no-timers", action="store_true")
 args = ap.parse_args()
 
 scene = inputs.reyes_config5(n_frames=args.frames)
@@ -34,14 +36,16 @@ def cfgs(name):
     if name == "fine":
         return vp.FINE, None
     if name.startswith("h"):
-        s = int(name[1:])
-        return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, s), (2, 3, vp.GROUP_RTC, s, nsm)], nsm)
+        s, _, bat = name[1:].partition("b")
+        s = int(s)
+        batch = [int(x) for x in bat.split("_")] if bat else None
+        return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, s), (2, 3, vp.GROUP_RTC, s, nsm)], nsm, batch=batch)
     if name.startswith("fine_h"):
         return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_FINE, 0, 40), (2, 3, vp.GROUP_RTC, 40, nsm)], nsm)
     raise ValueError(name)
 
 
-for timers in (False, True):
+for timers in ((False,) if args.no_timers else (False, True)):
     rp = ReyesPipeline(scene, flags=vp.FLAG_TIMERS if timers else 0)
     for name in args.configs.split(","):
         model, b = cfgs(name)
