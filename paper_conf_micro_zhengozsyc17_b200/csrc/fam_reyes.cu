@@ -213,7 +213,7 @@ struct ReyesF {
   // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
   static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
     // block-local [Bound, Split]: the first stack pass takes the whole claimed batch
-    if (!rtc && lo == BOUND && hi == SPLIT && (s == BOUND || s == SPLIT)) return 16;
+    if (!rtc && lo == BOUND && hi >= SPLIT && (s == BOUND || s == SPLIT)) return 16;
     return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
   }
   static constexpr int fused_local_cap(int, int, int) { return kThreads / 32; }
@@ -225,7 +225,8 @@ struct ReyesF {
   // every kernel whose range ends in [Dice, Shade] may run the fused chain (an RTC
   // kernel [Split..Shade] fuses its Dice batches too), so each reserves the chain scratch
   static constexpr int scratch_bytes(int lo, int hi) {
-    return (lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : (lo == BOUND && hi == SPLIT) ? (int)sizeof(LocalStack) : 0;
+    return ((lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
+           ((lo == BOUND && hi >= SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
   }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
@@ -257,8 +258,8 @@ struct ReyesF {
   // R-R2..R-R5), the split direction, and this thread's control point q.
   static __device__ __forceinline__ int bound_patch(const Params& p, const RPatch* P, int lane, bool valid, int& dir,
                                                     float4& q) {
-    const uint32_t id = P->id, depth = P->depth;
-    uint32_t frame = id >> 12;
+    const uint32_t depth = P->depth;
+    uint32_t frame = P->id >> 12;
     if (frame >= (uint32_t)p.n_frames) frame = 0;
     const float* M = p.M + 16 * (size_t)frame;
     q = P->cp[lane];
@@ -268,49 +269,60 @@ struct ReyesF {
     const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
     float sx, sy, zs;
     screen(p, c, sx, sy, zs);
-    // screen-space split metric (reading R-R5)
-    float sx12 = __shfl_sync(0xffffffffu, sx, (lane & 3) + 12, 16), sy12 = __shfl_sync(0xffffffffu, sy, (lane & 3) + 12, 16);
-    float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
-    float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
-    float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
-    // object-space metric (near-plane straddle, R-R4)
-    float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16), oy12 = __shfl_sync(0xffffffffu, q.y, (lane & 3) + 12, 16),
-          oz12 = __shfl_sync(0xffffffffu, q.z, (lane & 3) + 12, 16);
-    float ox3 = __shfl_down_sync(0xffffffffu, q.x, 3, 16), oy3 = __shfl_down_sync(0xffffffffu, q.y, 3, 16),
-          oz3 = __shfl_down_sync(0xffffffffu, q.z, 3, 16);
-    float olu = 0.0f, olv = 0.0f;
-    if (lane < 4) {
-      olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
-      olu = olu + fabsf(oz12 - q.z);
-    }
-    if ((lane & 3) == 0) {
-      olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
-      olv = olv + fabsf(oz3 - q.z);
-    }
-    float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
-    lu = red16_max(lu);
-    lv = red16_max(lv);
-    olu = red16_max(olu);
-    olv = red16_max(olv);
+    const float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
+    // The split metrics are computed only where a split needs them (the branch is uniform
+    // per 16-thread group; the group's shuffles use its own half-warp mask).  max over
+    // non-negative values is exact in any order, so the results equal a full evaluation.
+    const unsigned gm = 0xFFFFu << (threadIdx.x & 16);
     int cls;  // 0 cull, 1 split, 2 dice
     dir = 0;
-    if (nbehind == 16) {
+    if (!valid || nbehind == 16) {
       cls = 0;
     } else if (nbehind > 0) {
       cls = ((int)depth >= p.max_depth) ? 0 : 1;
-      dir = (olu >= olv) ? 0 : 1;
+      if (cls == 1) {  // object-space metric (near-plane straddle, R-R4)
+        const float ox12 = __shfl_sync(gm, q.x, (lane & 3) + 12, 16), oy12 = __shfl_sync(gm, q.y, (lane & 3) + 12, 16),
+                    oz12 = __shfl_sync(gm, q.z, (lane & 3) + 12, 16);
+        const float ox3 = __shfl_down_sync(gm, q.x, 3, 16), oy3 = __shfl_down_sync(gm, q.y, 3, 16),
+                    oz3 = __shfl_down_sync(gm, q.z, 3, 16);
+        float olu = 0.0f, olv = 0.0f;
+        if (lane < 4) {
+          olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
+          olu = olu + fabsf(oz12 - q.z);
+        }
+        if ((lane & 3) == 0) {
+          olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
+          olv = olv + fabsf(oz3 - q.z);
+        }
+#pragma unroll
+        for (int o = 8; o >= 1; o >>= 1) {
+          olu = fmaxf(olu, __shfl_xor_sync(gm, olu, o, 16));
+          olv = fmaxf(olv, __shfl_xor_sync(gm, olv, o, 16));
+        }
+        dir = (olu >= olv) ? 0 : 1;
+      }
     } else if (xmax < 0.0f || xmin >= (float)p.W || ymax < 0.0f || ymin >= (float)p.H) {
       cls = 0;
     } else {
-      float bw = xmax - xmin, bh = ymax - ymin;
-      float ext = bw > bh ? bw : bh;
-      if ((int)depth >= p.max_depth || ext <= p.t_dice) cls = 2;
-      else {
+      const float bw = xmax - xmin, bh = ymax - ymin;
+      const float ext = bw > bh ? bw : bh;
+      if ((int)depth >= p.max_depth || ext <= p.t_dice) {
+        cls = 2;
+      } else {  // screen-space split metric (reading R-R5)
         cls = 1;
+        const float sx12 = __shfl_sync(gm, sx, (lane & 3) + 12, 16), sy12 = __shfl_sync(gm, sy, (lane & 3) + 12, 16);
+        const float sx3 = __shfl_down_sync(gm, sx, 3, 16), sy3 = __shfl_down_sync(gm, sy, 3, 16);
+        float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
+        float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
+#pragma unroll
+        for (int o = 8; o >= 1; o >>= 1) {
+          lu = fmaxf(lu, __shfl_xor_sync(gm, lu, o, 16));
+          lv = fmaxf(lv, __shfl_xor_sync(gm, lv, o, 16));
+        }
         dir = (lu >= lv) ? 0 : 1;
       }
     }
-    return valid ? cls : 0;
+    return cls;
   }
 
   template <class Ctx>
@@ -409,19 +421,24 @@ struct ReyesF {
   static constexpr int kStack = 48, kLocalDice = 48;
   struct LocalStack {
     RPatch st[kStack];
-    int top, nchild, nbound, nsplit, dump;
+    int nchild[2], nsplit, dump;
   };
-  static constexpr bool local_recursion(int lo, int hi) { return lo == BOUND && hi == SPLIT; }
-  static constexpr int local_out_cap(int, int, int t) { return t == BOUND ? kStack : t == DICE ? kLocalDice : 0; }
+  static constexpr bool local_recursion(int lo, int hi) { return lo == BOUND && hi >= SPLIT; }
+  static constexpr int local_out_cap(int, int hi, int t) {
+    return t == BOUND ? kStack : t == DICE ? kLocalDice : (t == SHADE && hi >= DICE) ? 8 : 0;
+  }
 
   template <int SS, int LO, int HI, class Ctx>
   static __device__ void exec_local(Ctx& ctx, const uint8_t* items, int n) {
+    if constexpr (SS == DICE || SS == SHADE) {  // a megakernel's later stages run as usual
+      exec<SS>(ctx, items, n);
+      return;
+    }
     const Params& p = ctx.params();
     LocalStack& ls = *(LocalStack*)ctx.scratch();
     const int lane = threadIdx.x & 15, grp = threadIdx.x >> 4;
     if constexpr (SS == BOUND) {
       for (int e = threadIdx.x; e < n * 17; e += kThreads) ((uint4*)ls.st)[e] = ((const uint4*)items)[e];
-      if (threadIdx.x == 0) ls.top = n;
     } else {
       for (int r0 = 0; r0 < n; r0 += kThreads / 16) {  // Split items: their Bound already chose the direction
         const int k = r0 + grp;
@@ -437,13 +454,12 @@ struct ReyesF {
           if (lane == 0) split_headers(&ls.st[2 * k], &ls.st[2 * k + 1], P->id, P->path, P->dirs, depth, dir);
         }
       }
-      if (threadIdx.x == 0) ls.top = 2 * n;
     }
-    if (threadIdx.x == 0) ls.nchild = ls.nbound = ls.nsplit = 0;
+    if (threadIdx.x == 0) ls.nchild[0] = ls.nchild[1] = ls.nsplit = 0;
     worker_sync();
+    int top = (SS == BOUND) ? n : 2 * n, nbound = 0;
     bool first = SS == BOUND;  // the first pass pops exactly the claimed Bound items (n <= 16)
-    for (;;) {
-      const int top = ls.top;
+    for (int pass = 0;; ++pass) {
       const int dice_room = Ctx::template cap<DICE>() - ctx.sh.out_cnt[ctx.ob][DICE];
       const int m = min(min(kThreads / 16, top), min(kStack - top, dice_room));
       if (m <= 0) break;
@@ -461,10 +477,11 @@ struct ReyesF {
         if (!first) ctx.template trace_local<BOUND>((const uint8_t*)P);
         if (cls == 1) ctx.template trace_local<SPLIT>((const uint8_t*)P);
       }
+      const unsigned gm = 0xFFFFu << (threadIdx.x & 16);
       if (cls == 2) {
         int slot = 0;
         if (lane == 0) slot = ctx.template reserve<DICE>();
-        slot = __shfl_sync(0xFFFFu << (threadIdx.x & 16), slot, threadIdx.x & 16, 32);
+        slot = __shfl_sync(gm, slot, threadIdx.x & 16, 32);
         if (slot >= 0) {
           RPatch* out = (RPatch*)ctx.template out_ptr<DICE>(slot);
           out->cp[lane] = q;
@@ -477,30 +494,29 @@ struct ReyesF {
         }
       }
       worker_sync();  // every read of the popped patches is done
+      int* nchild = &ls.nchild[pass & 1];
       if (cls == 1) {
         int c = 0;
         if (lane == 0) {
-          c = atomicAdd(&ls.nchild, 2);
+          c = atomicAdd(nchild, 2);
           atomicAdd(&ls.nsplit, 1);
         }
-        c = __shfl_sync(0xFFFFu << (threadIdx.x & 16), c, threadIdx.x & 16, 32);
+        c = __shfl_sync(gm, c, threadIdx.x & 16, 32);
         RPatch* l = &ls.st[base + c];
         RPatch* r = &ls.st[base + c + 1];
         l->cp[my] = L;
         r->cp[my] = R;
         if (lane == 0) split_headers(l, r, id, path, dirs, depth, dir);
       }
-      worker_sync();
-      if (threadIdx.x == 0) {
-        ls.top = base + ls.nchild;
-        ls.nchild = 0;
-        if (!first) ls.nbound += m;
-      }
-      worker_sync();
+      worker_sync();  // children written, nchild final
+      top = base + *nchild;
+      // the other counter was last read before this pass's first barrier
+      if (threadIdx.x == 0) ls.nchild[(pass + 1) & 1] = 0;
+      if (!first) nbound += m;
       first = false;
     }
     // what is left goes back to the Bound ring (unbounded children: no work is repeated)
-    const int left = ls.top;
+    const int left = top;
     if (left > 0) {
       if (threadIdx.x == 0) ls.dump = ctx.template reserve<BOUND>(left);
       worker_sync();
@@ -511,7 +527,7 @@ struct ReyesF {
       }
     }
     if (threadIdx.x == 0) {
-      ctx.template note_local_count<BOUND>(ls.nbound);
+      ctx.template note_local_count<BOUND>(nbound);
       ctx.template note_local_count<SPLIT>(ls.nsplit);
     }
   }

@@ -5,6 +5,7 @@ so co-running persistent groups cannot be captured together).
   rtc_dice  : the [Dice,Shade] RTC kernel alone: every seed patch is inserted into the
               Dice queue, the [Bound,Split] group is an (idle) KBK group
   kbk       : one launch per stage per wave
+  bs_mega   : the block-local [Bound,Split] megakernel alone (Dice items left in a full ring)
   rtc_leaf  : the [Dice,Shade] RTC kernel alone on representative leaf patches
               (tools/reyes_leaves.py: numpy approximation of the Bound/Split recursion)
 """
@@ -30,6 +31,9 @@ if args.target.startswith("raster"):
     from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
     scene = inputs.raster_scene()
     rp = RasterPipeline(scene)
+elif args.target == "bs_mega":
+    scene = inputs.reyes_config5(n_frames=args.frames)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_FULL_RINGS)
 else:
     scene = inputs.reyes_config5(n_frames=args.frames)
     rp = ReyesPipeline(scene)
@@ -41,6 +45,10 @@ elif args.target == "mega":
     rp.configure(vp.MEGAKERNEL)
 elif args.target == "kbk":
     rp.configure(vp.KBK)
+elif args.target == "bs_mega":
+    # the block-local [Bound, Split] kernel alone (its Dice items wait in a full-size ring
+    # for the KBK [Dice, Shade] waves that run after it under ncu's serialisation)
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm - 8), (2, 3, vp.GROUP_KBK, nsm - 8, nsm)], nsm))
 elif args.target == "rtc_dice":
     rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
     rp.p.insert(2, rp.seeds_dev, n=scene.seeds.size)
