@@ -355,8 +355,18 @@ def main():
     achieved = dom_flop / (kmean[dom] / 1e3) / 1e12
     b = main_cfg.binding
     is_rtc = bool(main_cfg.has_binding and b.group_model[b.group_of_stage[lo]] == vp.GROUP_RTC)
+    # traffic: dram bytes per leaf from the committed ncu --set full capture of this kernel
+    # (profiles/r1_rtc_leaf_traffic.json), times the leaves this launch processed
+    traffic = None
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "r1_rtc_leaf_traffic.json")))
+        if (lo, hi) == (2, 3):
+            traffic = tr["bytes_per_leaf"] * d[2]
+    except Exception:
+        pass
     roofline = {"bound": "alu", "achieved": achieved, "peak": alu_peak, "unit": "TFLOP/s",
-                "frac": achieved / alu_peak, "traffic": None,
+                "frac": achieved / alu_peak, "traffic": traffic,
+                "traffic_source": "ncu dram__bytes_read+write per leaf (profiles/r1_rtc_leaf_traffic.json) x leaves",
                 "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if is_rtc else 'MEGA'}>",
                 "peak_source": "derived: SMs x 128 fp32 lanes x clocks.max.sm (MEASURED_PEAKS sm_max_mhz), non-FMA",
                 "kernel_ms": float(kmean[dom]), "kernel_share_of_step": float(kmean[dom] / ms_per_step)}
