@@ -102,6 +102,11 @@ typedef enum vp_stage_kind {
 #define VP_FLAG_QUEUE_DEPTH 0x2u    /* track max ring depth per stage (one extra read/flush) */
 #define VP_FLAG_STRICT_BINDING 0x4u /* vp_run fails with VP_ERR_BINDING on quota shortfall   */
 #define VP_FLAG_TIMERS 0x8u         /* in-kernel %globaltimer accumulators per stage/kernel  */
+#define VP_FLAG_ONLINE 0x20u        /* online adaptation (L41-L45): a persistent group whose  */
+                                    /* stages can get no more items retires and the host      */
+                                    /* relaunches the next group downstream on its SMs         */
+                                    /* (persistent plans only; extra grids appear in           */
+                                    /* vp_run_stats.kernel_* after the planned ones)           */
 #define VP_FLAG_FULL_RINGS 0x10u    /* persistent plans keep every ring at its registered     */
                                     /* capacity instead of shrinking it to what the producer  */
                                     /* blocks can hold (needed when a recursive stage's live   */

@@ -59,6 +59,7 @@ struct RunInit {
   long long pending;
   unsigned long long watchdog_ns;
   unsigned long long seeds[kMaxStages];
+  long long gpend[kMaxKernels];  // online adaptation: seeds of each group's stages
 };
 
 __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
@@ -79,6 +80,9 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
   if (t < kMaxKernels) {
     c->arrivals[t].v = 0;
     c->admitted[t].v = 0;
+    c->gpend[t].v = (unsigned long long)ri.gpend[t];
+    c->retired[t] = 0;
+    c->exits[t] = 0;
   }
   if (t < kMaxStages) c->wave_n[t] = 0;
   if (t == 0) {
@@ -185,6 +189,11 @@ struct KernelPlan {
   int grid;
   bool coop;
   int kslot;
+  // online adaptation
+  int group = -1;        // = kslot of the group's primary kernel
+  bool can_retire = false;
+  uint32_t feeders = 0;  // groups emitting into this kernel's stages
+  int refill = -1;       // kernel whose group gets this kernel's SMs when it retires
 };
 
 struct Plan {
@@ -193,6 +202,8 @@ struct Plan {
   std::vector<int> kbk_stages;         // stages driven by the host wave loop
   bool wave_rtc = false;               // standalone RTC: waves of the [0,S-1] RTC kernel
   bool kbk_graph = false;              // KBK waves driven on the device by a CUDA-graph while loop
+  bool online = false;                 // online adaptation (VP_FLAG_ONLINE): retire + refill
+  int8_t stage_group[kMaxStages] = {};
   int batch[kMaxStages] = {};
   int cap_log2[kMaxStages] = {};       // effective ring size this plan runs with
   vp_config cfg{};
@@ -219,6 +230,8 @@ struct vp_pipeline_s {
   uint32_t* h_blk = nullptr;
   volatile uint32_t* h_arrive = nullptr;  // mapped pinned: per-kernel dispatch-complete flags
   uint32_t* d_arrive = nullptr;
+  volatile uint32_t* h_retire = nullptr;  // mapped pinned: per-kernel "retired, SMs free" flags
+  uint32_t* d_retire = nullptr;
   uint32_t epoch = 0;
   cudaStream_t streams[kMaxKernels] = {};
   cudaEvent_t ev_fork = nullptr, ev_start = nullptr, ev_end = nullptr, ev_join[kMaxKernels] = {};
@@ -227,6 +240,7 @@ struct vp_pipeline_s {
   int kernel_occ_cache[kMaxStages][kMaxStages][2] = {};
   double timeout_ms = 30000;
   // device-driven KBK: instantiated graph and the launch arguments it was captured with
+  int refill_lo[kMaxKernels] = {}, refill_hi[kMaxKernels] = {}, refill_quota[kMaxKernels] = {};
   cudaGraph_t kg_graph = nullptr;
   cudaGraphExec_t kg_exec = nullptr;
   std::vector<uint8_t> kg_key;
@@ -346,7 +360,9 @@ Common make_common(vp_pipeline_s* p) {
             ((p->desc.flags & VP_FLAG_TIMERS) ? FLAG_TIMERS : 0u);
   c.n_stages = (int)p->st.size();
   c.host_arrive = p->d_arrive;
+  c.host_retire = p->d_retire;
   c.epoch = p->epoch;
+  for (int s = 0; s < kMaxStages; ++s) c.stage_group[s] = p->plan.online ? p->plan.stage_group[s] : (int8_t)-1;
   return c;
 }
 
@@ -599,6 +615,31 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
         return fail(p, VP_ERR_INVALID, "queue_capacity of stage %d (%lld) < 2 x batch(%d) x fanout(%d) of stage %d", t,
                     1ll << pl.cap_log2[t], pl.batch[s], f, s);
     }
+  // Online adaptation (VP_FLAG_ONLINE; "online tuner ... adjusting SM
+  // mappings"): each persistent kernel is a group; a group may retire once nothing can
+  // reach its stages (all its feeders are persistent groups that retired), and its SMs go
+  // to the first persistent group downstream of it.  KBK stages never retire.
+  for (int s = 0; s < kMaxStages; ++s) pl.stage_group[s] = -1;
+  pl.online = (p->desc.flags & VP_FLAG_ONLINE) && pl.kbk_stages.empty() && !pl.wave_rtc && pl.kernels.size() > 1;
+  if (pl.online) {
+    for (KernelPlan& k : pl.kernels) {
+      k.group = k.kslot;
+      for (int s = k.lo; s <= k.hi; ++s) pl.stage_group[s] = (int8_t)k.kslot;
+    }
+    for (KernelPlan& k : pl.kernels) {
+      k.can_retire = !k.coop;
+      for (int s = 0; s < S; ++s) {
+        if (s >= k.lo && s <= k.hi) continue;
+        bool feeds = false;
+        for (int t = k.lo; t <= k.hi; ++t) feeds |= p->fam->fanout(s, t) > 0;
+        if (feeds) k.feeders |= 1u << pl.stage_group[s];
+      }
+      int best = -1;
+      for (const KernelPlan& j : pl.kernels)
+        if (j.lo > k.hi && !j.coop && (best < 0 || j.lo < pl.kernels[best].lo)) best = j.kslot;
+      k.refill = best;
+    }
+  }
   pl.cfg.model = model;
   pl.cfg.has_binding = b ? 1 : 0;
   if (b) pl.cfg.binding = *b;
@@ -862,6 +903,11 @@ vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) 
     memset(ha, 0, sizeof(uint32_t) * kMaxKernels);
     p->h_arrive = (volatile uint32_t*)ha;
     if (bad(cudaHostGetDevicePointer((void**)&p->d_arrive, ha, 0))) return VP_ERR_CUDA;
+    void* hr = nullptr;
+    if (bad(cudaHostAlloc(&hr, sizeof(uint32_t) * kMaxKernels, cudaHostAllocMapped))) return VP_ERR_OOM;
+    memset(hr, 0, sizeof(uint32_t) * kMaxKernels);
+    p->h_retire = (volatile uint32_t*)hr;
+    if (bad(cudaHostGetDevicePointer((void**)&p->d_retire, hr, 0))) return VP_ERR_CUDA;
   }
   if (p->desc.flags & VP_FLAG_TRACE)
     if (bad(cudaMalloc(&p->trace, sizeof(TraceRec) * (size_t)p->desc.trace_capacity))) return VP_ERR_OOM;
@@ -892,6 +938,7 @@ vp_status vp_pipeline_destroy(void* h) {
   cudaFreeHost(p->h_ctrl);
   cudaFreeHost(p->h_blk);
   cudaFreeHost((void*)p->h_arrive);
+  cudaFreeHost((void*)p->h_retire);
   for (int i = 0; i < kMaxKernels; ++i) {
     cudaStreamDestroy(p->streams[i]);
     cudaEventDestroy(p->ev_join[i]);
@@ -1046,6 +1093,7 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   for (int s = 0; s < S; ++s) {
     ri.seeds[s] = p->st[s].n_seeds;
     ri.pending += (long long)p->st[s].n_seeds;
+    if (p->plan.online && p->plan.stage_group[s] >= 0) ri.gpend[p->plan.stage_group[s]] += (long long)p->st[s].n_seeds;
   }
   ri.watchdog_ns = (unsigned long long)(p->timeout_ms * 1e6);
   p->epoch++;
@@ -1070,6 +1118,9 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       g.kslot = k.kslot;
       g.mode = MODE_PERSISTENT;
       for (int s = 0; s < kMaxStages; ++s) g.batch[s] = pl.batch[s] ? pl.batch[s] : 1;
+      g.group = pl.online ? k.group : -1;
+      g.can_retire = pl.online && k.can_retire;
+      g.feeders = k.feeders;
       occupancy(p, k.lo, k.hi, k.rtc);
       CUDA_TRY(p, cudaEventRecord(p->ev_kbeg[i], ks));
       CUDA_TRY(p, p->fam->launch(k.lo, k.hi, k.rtc, c, g, p->params.data(), k.grid, k.coop, ks));
@@ -1085,6 +1136,48 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       }
     }
   }
+  int nk_total = nk;
+  if (pl.online) {
+    // Online adaptation: when a group retires (its last block left: mapped flag), launch
+    // a refill grid of its downstream group restricted to the freed SMs.
+    bool handled[kMaxKernels] = {};
+    for (;;) {
+      bool running = false;
+      for (int i = 0; i < nk_total; ++i) {
+        cudaError_t q = cudaEventQuery(p->ev_join[i]);
+        if (q == cudaErrorNotReady) running = true;
+        else if (q != cudaSuccess) CUDA_TRY(p, q);
+      }
+      if (!running) break;
+      for (int i = 0; i < nk; ++i) {
+        const KernelPlan& k = pl.kernels[i];
+        if (handled[i] || k.refill < 0 || p->h_retire[i] != p->epoch || nk_total >= kMaxKernels) continue;
+        handled[i] = true;
+        const KernelPlan& t = pl.kernels[k.refill];
+        const int slot = nk_total++;
+        GroupArgs g;
+        memset(&g, 0, sizeof(g));
+        memcpy(g.sm_mask, k.mask, sizeof(g.sm_mask));  // the retired group's SMs
+        g.quota = t.quota;
+        g.kslot = slot;
+        g.mode = MODE_PERSISTENT;
+        for (int s = 0; s < kMaxStages; ++s) g.batch[s] = pl.batch[s] ? pl.batch[s] : 1;
+        g.group = t.group;
+        g.can_retire = t.can_retire;
+        g.feeders = t.feeders;
+        const int per = t.quota > 0 ? t.quota : std::max(1, occupancy(p, t.lo, t.hi, t.rtc));
+        const int grid = per * std::max(1, mask_count(k.mask, p->num_sms));
+        cudaStream_t ks = p->streams[slot];
+        CUDA_TRY(p, cudaEventRecord(p->ev_kbeg[slot], ks));
+        CUDA_TRY(p, p->fam->launch(t.lo, t.hi, t.rtc, c, g, p->params.data(), grid, false, ks));
+        CUDA_TRY(p, cudaEventRecord(p->ev_join[slot], ks));
+        p->refill_lo[slot] = t.lo;
+        p->refill_hi[slot] = t.hi;
+        p->refill_quota[slot] = t.quota;
+      }
+      std::this_thread::yield();
+    }
+  }
   uint64_t launches = 0;
   if (pl.kbk_graph) {
     vp_status rc = graph_wave_run(p, c, st, &launches);
@@ -1093,7 +1186,7 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
     vp_status rc = host_wave_loop(p, c, st, &launches);
     if (rc != VP_OK) return rc;
   }
-  for (int i = 0; i < nk; ++i) CUDA_TRY(p, cudaStreamWaitEvent(st, p->ev_join[i], 0));
+  for (int i = 0; i < nk_total; ++i) CUDA_TRY(p, cudaStreamWaitEvent(st, p->ev_join[i], 0));
   CUDA_TRY(p, p->fam->finalize(p->params.data(), st));
   CUDA_TRY(p, cudaEventRecord(p->ev_end, st));
   CUDA_TRY(p, cudaMemcpyAsync(p->h_ctrl, p->ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, st));
@@ -1110,11 +1203,11 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       stats->enqueued[s] = hc.enq[s];
       stats->max_depth[s] = hc.max_depth[s];
     }
-    stats->num_kernels = nk;
-    for (int i = 0; i < nk && i < 16; ++i) {
-      stats->kernel_lo[i] = pl.kernels[i].lo;
-      stats->kernel_hi[i] = pl.kernels[i].hi;
-      stats->kernel_quota[i] = pl.kernels[i].quota;
+    stats->num_kernels = nk_total;  // + refill grids of the online adaptation
+    for (int i = 0; i < nk_total && i < 16; ++i) {
+      stats->kernel_lo[i] = i < nk ? pl.kernels[i].lo : p->refill_lo[i];
+      stats->kernel_hi[i] = i < nk ? pl.kernels[i].hi : p->refill_hi[i];
+      stats->kernel_quota[i] = i < nk ? pl.kernels[i].quota : p->refill_quota[i];
       float kms = 0;
       cudaEventElapsedTime(&kms, p->ev_kbeg[i], p->ev_join[i]);
       stats->kernel_ms[i] = kms;

@@ -68,6 +68,9 @@ struct Ctrl {
   unsigned long long flush_ns[kMaxStages];  // FLAG_TIMERS: publish (queue overhead) per stage
   unsigned long long idle_ns[kMaxKernels];  // FLAG_TIMERS: blocks finding no work, per kernel
   unsigned long long rounds[kMaxKernels];   // persistent-loop rounds, summed over blocks, per kernel
+  Line gpend[kMaxKernels];                  // online adaptation: items alive in each group's stages
+  unsigned long long retired[kMaxKernels];  // online adaptation: group drained for good, its blocks exit
+  unsigned long long exits[kMaxKernels];    // admitted blocks of each kernel slot that have exited
   unsigned long long graph_iters;           // device-driven KBK: iterations of the graph's while loop
   long long wave_n[kMaxStages];             // device-driven KBK: size of each stage's current wave
 };
@@ -97,7 +100,9 @@ struct Common {
   uint32_t flags;
   int n_stages;
   volatile uint32_t* host_arrive;  // mapped pinned host words: grid of kernel k fully dispatched
-  uint32_t epoch;                  // run counter written into host_arrive
+  volatile uint32_t* host_retire;  // mapped pinned host words: every block of kernel k exited on retirement
+  uint32_t epoch;                  // run counter written into host_arrive / host_retire
+  int8_t stage_group[kMaxStages];  // online adaptation: group of each stage (-1: none / KBK)
 };
 
 enum : int { MODE_PERSISTENT = 0, MODE_WAVE = 1 };
@@ -113,6 +118,12 @@ struct GroupArgs {
   const long long* wave_n_dev;   // WAVE, device-driven KBK: wave size written by the planner
                                  // kernel just before this launch (overrides wave_n/chunk)
   int batch[kMaxStages];         // items per claim, per stage
+  // online adaptation (the online tuner adjusts SM mappings at run time):
+  // a group whose stages can receive no more items (its feeders retired, gpend == 0)
+  // retires, and the host gives its SMs to another group
+  int group;                     // group id of this kernel (-1: no adaptation)
+  int can_retire;
+  uint32_t feeders;              // bitmask of the groups that emit into this group's stages
 };
 
 template <class F>
@@ -651,11 +662,20 @@ struct Runner {
     // Termination accounting: children are counted in `pending` before they become
     // visible (the release stores below order this reduction before them); completions
     // may be deferred (pending only stays conservatively high).
+    // per-group alive counts (online adaptation): children into this kernel's own group and
+    // its completions go in ONE atomic, so the group's count never dips to 0 transiently
+    const int tg = (myn > 0) ? (int)a.c.stage_group[lane] : -1;
+    int own = (tg >= 0 && tg == a.g.group) ? myn : 0;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) own += __shfl_xor_sync(0xffffffffu, own, o);
     if (lane == 0) {
       const long long d = children - completed + sh.acc_neg;
       if (d != 0) red_add(&c->pending.v, d);
+      const long long dg = own - completed + sh.acc_neg;
+      if (a.g.group >= 0 && dg != 0) red_add(&c->gpend[a.g.group].v, dg);
       sh.acc_neg = 0;
     }
+    if (tg >= 0 && tg != a.g.group) red_add(&c->gpend[tg].v, myn);
     unsigned long long mybase = 0;
     if (myn > 0) {
       mybase = atom_add(&c->tail[lane].v, myn);
@@ -757,6 +777,8 @@ struct Runner {
       sh.done = 0;
       if (aborted(c)) {
         sh.done = 1;
+      } else if (a.g.group >= 0 && *(volatile unsigned long long*)&c->retired[a.g.group]) {
+        sh.done = 1;  // another block of this group retired it (nothing is left for it)
       } else if (globaltimer() > c->deadline.v) {
         // watchdog, checked every round even by busy blocks (the tuner's timeoutexec)
         atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
@@ -797,9 +819,15 @@ struct Runner {
           // idle: retire deferred completions first, then test for termination
           if (sh.acc_neg != 0) {
             atom_add(&c->pending.v, sh.acc_neg);
+            if (a.g.group >= 0) atom_add(&c->gpend[a.g.group].v, sh.acc_neg);
             sh.acc_neg = 0;
           }
           if ((long long)ld_acquire(&c->pending.v) <= 0) {
+            sh.done = 1;
+          } else if (a.g.can_retire && group_drained(a)) {
+            // nothing can reach this group's stages any more: retire it (its SMs go to
+            // another group, the host launches the refill)
+            atomicExch(&c->retired[a.g.group], 1ull);
             sh.done = 1;
           } else if (globaltimer() > c->deadline.v) {
             atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
@@ -970,6 +998,14 @@ struct Runner {
           atomicAdd(&c->admitted[g.kslot].v, 1ull);
           atomicAdd(&c->fallback_admits, 1ull);
         }
+        // online adaptation: the grid's last block arrives after every admitted block of a
+        // retired group already left -> it tells the host instead of them
+        if (!good && t == (unsigned long long)gridDim.x - 1 && g.group >= 0 && a.c.host_retire &&
+            *(volatile unsigned long long*)&c->retired[g.group] &&
+            *(volatile unsigned long long*)&c->exits[g.kslot] == ld_relaxed(&c->admitted[g.kslot].v)) {
+          a.c.host_retire[g.kslot] = a.c.epoch;
+          __threadfence_system();
+        }
       } else if (sm < (uint32_t)kMaxSM) {
         atomicAdd(&a.c.blk[g.kslot * kMaxSM + sm], 1u);
       }
@@ -1016,6 +1052,7 @@ struct Runner {
     if (threadIdx.x == 0) {
       Ctrl* c = a.c.ctrl;
       if (sh.acc_neg != 0) atom_add(&c->pending.v, sh.acc_neg);
+      if (sh.acc_neg != 0 && a.g.group >= 0) atom_add(&c->gpend[a.g.group].v, sh.acc_neg);
       sh.acc_neg = 0;
       for (int s = 0; s < S; ++s) {
         if (sh.deq[s]) atomicAdd(&c->deq[s], sh.deq[s]);
@@ -1025,7 +1062,30 @@ struct Runner {
       }
       if (sh.t_idle) atomicAdd(&c->idle_ns[a.g.kslot], sh.t_idle);
       atomicAdd(&c->rounds[a.g.kslot], sh.rounds);
+      if (a.g.group >= 0 && a.c.host_retire && a.g.mode == MODE_PERSISTENT) {
+        // the last admitted block of a retired group's kernel to leave tells the host
+        // that the kernel's SMs are free (the grid is fully dispatched: every block that
+        // will ever be admitted has been)
+        __threadfence();
+        const unsigned long long e = atomicAdd(&c->exits[a.g.kslot], 1ull) + 1;
+        if (*(volatile unsigned long long*)&c->retired[a.g.group] &&
+            ld_relaxed(&c->arrivals[a.g.kslot].v) == (unsigned long long)gridDim.x &&
+            e == ld_relaxed(&c->admitted[a.g.kslot].v)) {
+          a.c.host_retire[a.g.kslot] = a.c.epoch;
+          __threadfence_system();
+        }
+      }
     }
+  }
+
+  // every feeder group retired and no item alive in this group's stages (seeds included)
+  static __device__ __forceinline__ bool group_drained(const KArgs<F>& a) {
+    Ctrl* c = a.c.ctrl;
+    for (uint32_t f = a.g.feeders; f; f &= f - 1) {
+      const int g = __ffs(f) - 1;
+      if (!*(volatile unsigned long long*)&c->retired[g]) return false;
+    }
+    return (long long)ld_acquire(&c->gpend[a.g.group].v) <= 0;
   }
 
   // A sink group emits nothing to any ring (every successor of its stages is a later

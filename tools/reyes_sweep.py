@@ -20,6 +20,7 @@ ap.add_argument("--configs", default="mega,kbk,h37,h50,h74,h100,fine_h")
 ap.add_argument("--batch", type=int, default=0)
 ap.add_argument("--bats", default="", help="per-stage batch sets for hybrid configs, e.g. 32,16,8,4;32,16,64,4")
 ap.add_argument("--no-timers", action="store_true")
+ap.add_argument("--online", action="store_true", help="VP_FLAG_ONLINE (retire + refill)")
 args = ap.parse_args()
 
 scene = inputs.reyes_config5(n_frames=args.frames)
@@ -46,7 +47,7 @@ def cfgs(name):
 
 
 for timers in ((False,) if args.no_timers else (False, True)):
-    rp = ReyesPipeline(scene, flags=vp.FLAG_TIMERS if timers else 0)
+    rp = ReyesPipeline(scene, flags=(vp.FLAG_TIMERS if timers else 0) | (vp.FLAG_ONLINE if args.online else 0))
     for name in args.configs.split(","):
         model, b = cfgs(name)
         try:
