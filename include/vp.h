@@ -107,6 +107,9 @@ typedef enum vp_stage_kind {
                                     /* relaunches the next group downstream on its SMs         */
                                     /* (persistent plans only; extra grids appear in           */
                                     /* vp_run_stats.kernel_* after the planned ones)           */
+#define VP_FLAG_L2_PERSIST 0x40u    /* an L2 access-policy window (persisting) over */
+                                    /* every ring's sequence words on the run stream and the  */
+                                    /* group streams (sets cudaLimitPersistingL2CacheSize)    */
 #define VP_FLAG_FULL_RINGS 0x10u    /* persistent plans keep every ring at its registered     */
                                     /* capacity instead of shrinking it to what the producer  */
                                     /* blocks can hold (needed when a recursive stage's live   */

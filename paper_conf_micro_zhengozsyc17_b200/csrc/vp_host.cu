@@ -241,6 +241,10 @@ struct vp_pipeline_s {
   double timeout_ms = 30000;
   // device-driven KBK: instantiated graph and the launch arguments it was captured with
   int refill_lo[kMaxKernels] = {}, refill_hi[kMaxKernels] = {}, refill_quota[kMaxKernels] = {};
+  bool launched[kMaxKernels] = {};  // planned kernels launched by the last vp_run
+  void* seq_arena = nullptr;  // every ring's sequence words (one L2 persisting window)
+  size_t seq_arena_bytes = 0;
+  bool l2_window_set = false;
   cudaGraph_t kg_graph = nullptr;
   cudaGraphExec_t kg_exec = nullptr;
   std::vector<uint8_t> kg_key;
@@ -314,11 +318,19 @@ int mask_count(const uint32_t* m, int nsm) {
 
 vp_status ensure_queues(vp_pipeline_s* p) {
   if (p->queues_ready) return VP_OK;
+  // All sequence-word arrays live in one arena, so one L2 access-policy window can pin
+  // them (VP_FLAG_L2_PERSIST); each array starts on a 256-B boundary.
+  size_t seq_bytes = 0;
+  for (size_t s = 0; s < p->st.size(); ++s) seq_bytes += ((1ull << p->st[s].cap_log2) * 8 + 255) / 256 * 256;
+  CUDA_TRY(p, cudaMalloc(&p->seq_arena, seq_bytes));
+  p->seq_arena_bytes = seq_bytes;
+  size_t off = 0;
   for (size_t s = 0; s < p->st.size(); ++s) {
     StageRec& r = p->st[s];
     size_t cap = 1ull << r.cap_log2;
     CUDA_TRY(p, cudaMalloc(&r.slots, cap * (size_t)p->fam->stride((int)s)));
-    CUDA_TRY(p, cudaMalloc(&r.seq, cap * sizeof(unsigned long long)));
+    r.seq = (unsigned long long*)((uint8_t*)p->seq_arena + off);
+    off += (cap * 8 + 255) / 256 * 256;
     k_init_seq<<<256, 256>>>(r.seq, cap, 0);
     p->run_cap_log2[s] = r.cap_log2;
     CUDA_TRY(p, cudaGetLastError());
@@ -929,9 +941,9 @@ vp_status vp_pipeline_destroy(void* h) {
   cudaDeviceSynchronize();
   for (StageRec& r : p->st) {
     cudaFree(r.slots);
-    cudaFree(r.seq);
     cudaFree(r.seeds);
   }
+  cudaFree(p->seq_arena);
   cudaFree(p->ctrl);
   cudaFree(p->blk);
   cudaFree(p->trace);
@@ -1099,18 +1111,59 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   p->epoch++;
   if (p->epoch == 0) p->epoch = 1;
   Common c = make_common(p);
+  if ((p->desc.flags & VP_FLAG_L2_PERSIST) && !p->l2_window_set) {
+    // keep the claim/publish sequence words in a persisting L2 carve-out
+    // (the ring counters are atomics, which execute in L2 anyway)
+    int max_persist = 0, max_window = 0;
+    cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, p->device);
+    cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, p->device);
+    const size_t win = std::min(p->seq_arena_bytes, (size_t)std::max(0, max_window));
+    if (max_persist > 0 && win > 0) {
+      CUDA_TRY(p, cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(win, (size_t)max_persist)));
+      cudaStreamAttrValue av;
+      memset(&av, 0, sizeof(av));
+      av.accessPolicyWindow.base_ptr = p->seq_arena;
+      av.accessPolicyWindow.num_bytes = win;
+      av.accessPolicyWindow.hitRatio = std::min(1.0f, (float)max_persist / (float)win);
+      av.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      av.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      CUDA_TRY(p, cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &av));
+      for (int i = 0; i < kMaxKernels; ++i)
+        CUDA_TRY(p, cudaStreamSetAttribute(p->streams[i], cudaStreamAttributeAccessPolicyWindow, &av));
+    }
+    p->l2_window_set = true;
+  }
   CUDA_TRY(p, cudaEventRecord(p->ev_start, st));
   k_run_init<<<1, 256, 0, st>>>(p->ctrl, p->blk, ri);
   CUDA_TRY(p, cudaGetLastError());
   CUDA_TRY(p, p->fam->init_run(p->params.data(), st));
   const Plan& pl = p->plan;
   int nk = (int)pl.kernels.size();
+  // Stages no seed can reach (through the fan-out graph) never get an item: their
+  // persistent kernels are not launched (they would only hold SMs, and their resident
+  // idle blocks can keep a later kernel's grid from being dispatched).
+  bool reach[kMaxStages] = {};
+  for (int s = 0; s < S; ++s) reach[s] = p->st[s].n_seeds > 0;
+  for (bool grew = true; grew;) {
+    grew = false;
+    for (int s = 0; s < S; ++s)
+      for (int t = 0; t < S; ++t)
+        if (reach[s] && !reach[t] && p->fam->fanout(s, t) > 0) reach[t] = grew = true;
+  }
   if (nk > 0) {
     CUDA_TRY(p, cudaEventRecord(p->ev_fork, st));
     for (int i = 0; i < nk; ++i) {
       const KernelPlan& k = pl.kernels[i];
       cudaStream_t ks = p->streams[i];
       CUDA_TRY(p, cudaStreamWaitEvent(ks, p->ev_fork, 0));
+      bool live = false;
+      for (int s = k.lo; s <= k.hi; ++s) live |= reach[s];
+      p->launched[i] = live;
+      if (!live) {
+        CUDA_TRY(p, cudaEventRecord(p->ev_kbeg[i], ks));
+        CUDA_TRY(p, cudaEventRecord(p->ev_join[i], ks));
+        continue;
+      }
       GroupArgs g;
       memset(&g, 0, sizeof(g));
       memcpy(g.sm_mask, k.mask, sizeof(g.sm_mask));
@@ -1255,7 +1308,7 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   if (p->desc.flags & VP_FLAG_STRICT_BINDING) {
     for (int i = 0; i < nk; ++i) {
       const KernelPlan& k = pl.kernels[i];
-      if (k.quota <= 0) continue;
+      if (k.quota <= 0 || !p->launched[i]) continue;
       for (int sm = 0; sm < p->num_sms; ++sm)
         if ((k.mask[sm >> 5] >> (sm & 31)) & 1u)
           if ((int)p->h_blk[i * kMaxSM + sm] < k.quota)

@@ -164,19 +164,22 @@ def default_light() -> np.ndarray:
 
 
 def reyes_config1(seed: int = seed_for(1), W: int = 256, H: int = 256, n_side: int = 4,
-                  max_depth: int = 8) -> ReyesScene:
+                  max_depth: int = 8, n_frames: int = 1) -> ReyesScene:
     """BASELINE config 1: 16 bicubic Bezier patches, 256x256, max split depth 8.
 
     4x4 patches tile a height field over [-1,1]^2 (13x13 lattice, z ~ U(-0.25,0.25));
     camera eye (0,-1.6,1.2) -> origin, up +z, fovy 50 deg, near 0.1.
+    n_frames > 1: the same frame replicated (SURVEY §8(d) throughput mode, R frames in
+    flight in one run).
     """
     lat = heightfield_lattice(n_side, seed, 0.25)
     cps = lattice_patches(lat, n_side)
     M = look_at_perspective((0.0, -1.6, 1.2), aspect=W / H).astype(np.float32).reshape(1, 16)
+    M = np.repeat(M, n_frames, axis=0)
     alb = np.zeros((n_side * n_side, 4), np.float32)
     alb[:, :3] = uniform01(seed + 1, n_side * n_side * 3).reshape(-1, 3)
-    return ReyesScene(W=W, H=H, n_frames=1, patches_per_frame=n_side * n_side, M=M, albedo=alb,
-                      light=default_light(), seeds=make_patch_items(cps, 1), max_depth=max_depth)
+    return ReyesScene(W=W, H=H, n_frames=n_frames, patches_per_frame=n_side * n_side, M=M, albedo=alb,
+                      light=default_light(), seeds=make_patch_items(cps, n_frames), max_depth=max_depth)
 
 
 def reyes_frame_camera(f: int, n_frames_orbit: int = 512, W: int = 256, H: int = 256) -> np.ndarray:

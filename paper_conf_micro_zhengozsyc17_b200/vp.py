@@ -38,7 +38,8 @@ PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
 FD_GRAY, FD_CDF, FD_MAP, FD_RESIZE, FD_LBP, FD_SCAN = 60, 61, 62, 63, 64, 65
 QB_ITEM4, QB_ITEM16, QB_ITEM272 = 70, 71, 72
-FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS, FLAG_ONLINE = 1, 2, 4, 8, 16, 32
+FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS, FLAG_ONLINE, FLAG_L2_PERSIST = (
+    1, 2, 4, 8, 16, 32, 64)
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
 P = C.c_void_p

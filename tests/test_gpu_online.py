@@ -89,3 +89,21 @@ def test_latched_workloads_online_parity(vpm, orc, model):
             st = fp.run()
             check(orc, fs, fp, st)
     assert st["pending"] == 0 and st["abort_reason"] == 0
+
+
+@pytest.mark.parametrize("model", ["hybrid", "megakernel", "kbk_graph"])
+def test_reyes_l2_persist_parity(vpm, orc, model):
+    """VP_FLAG_L2_PERSIST: the persisting window over the sequence words changes
+    only cache residency, never results."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    from test_gpu_reyes import check_against_oracle
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    scene = inputs.reyes_config5(n_frames=8, n_side=16)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_L2_PERSIST)
+    if model == "hybrid":
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 60), (2, 3, vp.GROUP_RTC, 60, nsm)], nsm))
+    else:
+        rp.configure({"megakernel": vp.MEGAKERNEL, "kbk_graph": vp.KBK_GRAPH}[model])
+    for _ in range(2):
+        check_against_oracle(orc, scene, rp, rp.run())

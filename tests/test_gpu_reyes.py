@@ -176,3 +176,13 @@ def test_reyes_full_config5_sampled_frames(vpm, orc):
     # whole-shard conservation (any size): Bound = seeds + 2 Split; Shade = Dice
     d = st["dequeued"]
     assert d[0] == scene.seeds.size + 2 * d[1] and d[3] == d[2]
+
+
+def test_reyes_config1_throughput_mode_replicas(vpm, orc):
+    """SURVEY §8(d) throughput mode: R replicated config-1 frames in one run; every frame
+    equals the single-frame oracle result."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    scene = inputs.reyes_config1(n_frames=4)
+    rp = ReyesPipeline(scene)
+    configure(vpm, rp, "hybrid_mega_rtc")
+    check_against_oracle(orc, scene, rp, rp.run())

@@ -21,6 +21,7 @@ ap.add_argument("--batch", type=int, default=0)
 ap.add_argument("--bats", default="", help="per-stage batch sets for hybrid configs, e.g. 32,16,8,4;32,16,64,4")
 ap.add_argument("--no-timers", action="store_true")
 ap.add_argument("--online", action="store_true", help="VP_FLAG_ONLINE (retire + refill)")
+ap.add_argument("--l2", action="store_true", help="VP_FLAG_L2_PERSIST (persisting window over the sequence words)")
 args = ap.parse_args()
 
 scene = inputs.reyes_config5(n_frames=args.frames)
@@ -47,7 +48,8 @@ def cfgs(name):
 
 
 for timers in ((False,) if args.no_timers else (False, True)):
-    rp = ReyesPipeline(scene, flags=(vp.FLAG_TIMERS if timers else 0) | (vp.FLAG_ONLINE if args.online else 0))
+    rp = ReyesPipeline(scene, flags=(vp.FLAG_TIMERS if timers else 0) | (vp.FLAG_ONLINE if args.online else 0)
+                       | (vp.FLAG_L2_PERSIST if args.l2 else 0))
     for name in args.configs.split(","):
         model, b = cfgs(name)
         try:
