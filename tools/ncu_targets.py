@@ -24,6 +24,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("target")
 ap.add_argument("--frames", type=int, default=64)
 ap.add_argument("--runs", type=int, default=2)
+ap.add_argument("--l2", action="store_true", help="VP_FLAG_L2_PERSIST")
 args = ap.parse_args()
 
 nsm, _ = vp.device_info(0)
@@ -36,7 +37,7 @@ elif args.target == "bs_mega":
     rp = ReyesPipeline(scene, flags=vp.FLAG_FULL_RINGS)
 else:
     scene = inputs.reyes_config5(n_frames=args.frames)
-    rp = ReyesPipeline(scene)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_L2_PERSIST if args.l2 else 0)
 if args.target == "raster_mega":
     rp.configure(vp.MEGAKERNEL)
 elif args.target == "raster_kbk":
