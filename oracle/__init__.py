@@ -75,6 +75,8 @@ def _declare(L):
     L.orc_toy_definition.argtypes = [P, C.c_size_t, C.c_int32, P, P]
     L.orc_toy_pipeline.argtypes = [P, C.c_size_t, C.c_int32, P, P, P]
     L.orc_qbench_pipeline.argtypes = [P, C.c_size_t, C.c_size_t, C.c_uint32, P, P, P, P]
+    L.orc_ldpc_definition.argtypes = [P, P, P]
+    L.orc_ldpc_pipeline.argtypes = [P, P, P, P]
     L.orc_collatz_definition.argtypes = [P, C.c_size_t, P]
     L.orc_collatz_pipeline.argtypes = [P, C.c_size_t, C.c_uint32, P, P, P]
     L.orc_reyes_definition.argtypes = [P, P, C.c_size_t, P]
@@ -123,6 +125,40 @@ def qbench_pipeline(seeds: np.ndarray, item_bytes: int, fanout: int):
                                    C.byref(st))
     assert rc == 0
     return lv.value, ids.value, bad.value, int(st.deq[0])
+
+
+class LdpcC(C.Structure):
+    _fields_ = [("N", C.c_int32), ("M", C.c_int32), ("dv", C.c_int32), ("dc", C.c_int32), ("n_frames", C.c_int32),
+                ("n_iter", C.c_int32), ("alpha", C.c_float), ("pad", C.c_int32), ("check_vars", P),
+                ("var_edges", P), ("llr", P)]
+
+
+def _ldpc_run(fn, sc, llr=None, n_iter=None, alpha=None):
+    llr = np.ascontiguousarray(sc.llr if llr is None else llr, np.float32)
+    cv = np.ascontiguousarray(sc.check_vars, np.int32)
+    ve = np.ascontiguousarray(sc.var_edges, np.int32)
+    nf = llr.shape[0]
+    it = sc.n_iter if n_iter is None else n_iter
+    d = LdpcC(N=sc.N, M=sc.M, dv=sc.dv, dc=sc.dc, n_frames=nf, n_iter=it,
+              alpha=sc.alpha if alpha is None else alpha, check_vars=_ptr(cv), var_edges=_ptr(ve), llr=_ptr(llr))
+    post = np.zeros((nf, sc.N), np.float32)
+    err = np.zeros((nf, it), np.int32)
+    if fn == "orc_ldpc_pipeline":
+        st = Stats()
+        assert lib().orc_ldpc_pipeline(C.byref(d), _ptr(post), _ptr(err), C.byref(st)) == 0
+        return dict(post=post, errors=err, deq=list(st.deq[:4]), enq=list(st.enq[:4]))
+    assert lib().orc_ldpc_definition(C.byref(d), _ptr(post), _ptr(err)) == 0
+    return dict(post=post, errors=err)
+
+
+def ldpc_definition(sc, **kw):
+    """LDPC min-sum decoder, definition layer (ldpc.c): posterior LLRs after the last
+    iteration and bit errors per (frame, iteration)."""
+    return _ldpc_run("orc_ldpc_definition", sc, **kw)
+
+
+def ldpc_pipeline(sc, **kw):
+    return _ldpc_run("orc_ldpc_pipeline", sc, **kw)
 
 
 def collatz_definition(seeds: np.ndarray):

@@ -62,6 +62,17 @@ typedef struct orc_stats { uint64_t deq[ORC_MAX_STAGES], enq[ORC_MAX_STAGES]; } 
 int orc_toy_definition(const int32_t* in, size_t n, int32_t threshold, int32_t* out, uint64_t* s1_passes);
 int orc_toy_pipeline(const int32_t* in, size_t n, int32_t threshold, int32_t* out, size_t* n_out,
                      orc_stats* st);
+/* ldpc.c: LDPC decoder, Fig. 17; H as data, edges in check-major order */
+typedef struct orc_ldpc {
+  int32_t N, M, dv, dc, n_frames, n_iter;
+  float alpha;            /* min-sum normalisation                               */
+  int32_t pad;
+  const int32_t* check_vars; /* [M*dc] variable node of each edge (check-major)  */
+  const int32_t* var_edges;  /* [N*dv] edges of each variable node, ascending    */
+  const float* llr;          /* [n_frames*N] channel LLRs                        */
+} orc_ldpc;
+int orc_ldpc_definition(const orc_ldpc* d, float* post, int32_t* errors);
+int orc_ldpc_pipeline(const orc_ldpc* d, float* post, int32_t* errors, orc_stats* st);
 /* qbench.c: queue microbenchmark */
 int orc_qbench_pipeline(const void* seeds, size_t n, size_t item_bytes, uint32_t fanout, uint64_t* leaves,
                         uint64_t* idsum, uint64_t* bad, orc_stats* st);

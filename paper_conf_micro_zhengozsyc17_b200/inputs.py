@@ -428,3 +428,75 @@ def reyes_planar(S_px: float, W: int = 64, H: int = 64, x0: float = 8.0, y0: flo
     return ReyesScene(W=W, H=H, n_frames=1, patches_per_frame=1, M=M.astype(np.float32).reshape(1, 16),
                       albedo=alb, light=np.array([0.0, 0.0, 1.0, 0.0], np.float32),
                       seeds=make_patch_items(cps, 1), max_depth=max_depth)
+
+
+# ----------------------------------------------------------------------------------------
+# LDPC decoder (Fig. 17, L59; 100 frames x 100 iterations, L53)
+# ----------------------------------------------------------------------------------------
+@dataclass
+class LdpcScene:
+    """A (dv, dc)-regular parity-check matrix as edge lists (check-major edge order) and
+    per-frame channel LLRs of the all-zero codeword (readings R-L1..R-L6)."""
+    N: int
+    M: int
+    dv: int
+    dc: int
+    check_vars: np.ndarray   # [M*dc] int32: variable node of edge e = m*dc + k
+    var_edges: np.ndarray    # [N*dv] int32: the dv edges of variable n, ascending
+    llr: np.ndarray          # [n_frames, N] float32
+    n_iter: int = 100
+    alpha: float = 0.75
+
+    @property
+    def n_frames(self) -> int:
+        return self.llr.shape[0]
+
+
+def ldpc_regular_h(N: int, dv: int, dc: int, seed: int) -> np.ndarray:
+    """Socket-permutation (configuration-model) construction of a (dv, dc)-regular H:
+    check-major edge list check_vars[M*dc]; a check never holds the same variable twice
+    (colliding sockets are swapped with random partners until none is left)."""
+    assert (N * dv) % dc == 0
+    E = N * dv
+    M = E // dc
+    sockets = np.repeat(np.arange(N, dtype=np.int64), dv)
+    key = splitmix64(seed, E)
+    cv = sockets[np.argsort(key, kind="stable")].copy()
+    r = 0
+    while True:
+        rows = cv.reshape(M, dc)
+        srt = np.sort(rows, axis=1)
+        bad_rows = np.nonzero((srt[:, 1:] == srt[:, :-1]).any(axis=1))[0]
+        if bad_rows.size == 0:
+            break
+        r += 1
+        pick = splitmix64(seed + 7919 * r, 2 * bad_rows.size)
+        for i, m in enumerate(bad_rows):
+            a = m * dc + int(pick[2 * i] % np.uint64(dc))
+            b = int(pick[2 * i + 1] % np.uint64(E))
+            cv[a], cv[b] = cv[b], cv[a]
+    return cv.astype(np.int32)
+
+
+def ldpc_var_edges(check_vars: np.ndarray, N: int, dv: int) -> np.ndarray:
+    order = np.argsort(check_vars, kind="stable")      # edges grouped by variable, ascending
+    ve = order.astype(np.int32).reshape(N, dv)
+    assert np.all(check_vars[ve] == np.arange(N)[:, None])
+    return ve.reshape(-1)
+
+
+def ldpc_scene(n_frames: int = 100, N: int = 2048, dv: int = 3, dc: int = 6, ebn0_db: float = 2.0,
+               n_iter: int = 100, seed: int = seed_for(6), alpha: float = 0.75) -> LdpcScene:
+    """Rate-(1 - dv/dc) regular code, BPSK over AWGN at Eb/N0 = ebn0_db, all-zero codeword:
+    y = 1 + sigma*z (Box-Muller in float64 from SplitMix64), LLR = 2y/sigma^2 as float32."""
+    cv = ldpc_regular_h(N, dv, dc, seed)
+    ve = ldpc_var_edges(cv, N, dv)
+    rate = 1.0 - dv / dc
+    sigma2 = 1.0 / (2.0 * rate * 10.0 ** (ebn0_db / 10.0))
+    u1 = np.maximum(uniform01(seed + 1, n_frames * N).astype(np.float64), 2.0 ** -25)
+    u2 = uniform01(seed + 2, n_frames * N).astype(np.float64)
+    z = np.sqrt(-2.0 * np.log(u1)) * np.cos(2.0 * np.pi * u2)
+    y = 1.0 + np.sqrt(sigma2) * z
+    llr = (2.0 * y / sigma2).astype(np.float32).reshape(n_frames, N)
+    return LdpcScene(N=N, M=N * dv // dc, dv=dv, dc=dc, check_vars=cv, var_edges=ve, llr=llr,
+                     n_iter=n_iter, alpha=alpha)
