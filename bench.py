@@ -225,7 +225,7 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
     workload is HBM-bound."""
     from paper_conf_micro_zhengozsyc17_b200 import inputs
     from paper_conf_micro_zhengozsyc17_b200.workloads import (CfdPipeline, FaceDetPipeline, PyramidPipeline,
-                                                              RasterPipeline, ReyesPipeline)
+                                                              RasterPipeline, ReyesPipeline)  # noqa: F401
 
     def measure(pipe, frames, alg_bytes=None, reps=3):
         best, rep = pipe.p.autotune(time_budget_s=tune_s, sm_granularity=4, batch_choices=(1, 2))
@@ -282,6 +282,11 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
     cs = inputs.cfd_scene(G=4096, n_outer=10)
     out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
     out["cfd_config3"]["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (out["cfd_config3"]["ms"] / 1e3)
+    # the LDPC decoder (Fig. 17), 100 frames x 100 iterations (L53)
+    from paper_conf_micro_zhengozsyc17_b200.workloads import LdpcPipeline
+    ls = inputs.ldpc_scene()
+    out["ldpc_f3"] = measure(LdpcPipeline(ls), ls.n_frames)
+    out["ldpc_f3"]["decoder_iterations_per_s"] = ls.n_frames * ls.n_iter / (out["ldpc_f3"]["ms"] / 1e3)
     rs = inputs.raster_scene()
     out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
     out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)

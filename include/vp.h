@@ -91,7 +91,10 @@ typedef enum vp_stage_kind {
   /* Queue microbenchmark (not a paper workload): three independent
    * self-recursive stages with 4-, 16- and 272-B items (Fig. 9's int; Table 2's window /
    * tile items; the Reyes patch, L61 §8.5).  See vp_qbench_params. */
-  VP_QB_ITEM4 = 70, VP_QB_ITEM16 = 71, VP_QB_ITEM272 = 72
+  VP_QB_ITEM4 = 70, VP_QB_ITEM16 = 71, VP_QB_ITEM272 = 72,
+  /* LDPC decoder (Fig. 17, L59): Initialize, C2V, V2C, ProbVar (loops back to C2V for the
+   * next of n_iter iterations); items {frame, iteration}; see vp_ldpc_params */
+  VP_LDPC_INIT = 80, VP_LDPC_C2V = 81, VP_LDPC_V2C = 82, VP_LDPC_PROBVAR = 83
 } vp_stage_kind;
 
 #define VP_MAX_STAGES 8
@@ -228,6 +231,23 @@ typedef struct vp_qbench_params {
   unsigned long long* idsum;   /* [3] sum of leaf ids per stage                            */
   unsigned long long* bad;     /* [3] leaves whose payload was corrupted                   */
 } vp_qbench_params;
+
+/* LDPC decoder (Fig. 17; readings R-L1..R-L6): normalised min-sum on a
+ * (dv, dc)-regular parity-check matrix given as edge arrays in check-major order
+ * (edge e = m*dc + k joins check m and variable check_vars[e]). */
+typedef struct vp_ldpc_params {
+  int32_t N, M, dv, dc;        /* variables, checks, degrees (N*dv == M*dc, dc <= 32, dv <= 8) */
+  int32_t n_frames, n_iter;    /* frames decoded in one run; iterations per frame              */
+  float alpha;                 /* min-sum normalisation                                        */
+  int32_t pad;
+  const int32_t* check_vars;   /* [M*dc] variable of each edge                                 */
+  const int32_t* var_edges;    /* [N*dv] edges of each variable, ascending                     */
+  const float* llr;            /* [n_frames*N] channel LLRs                                    */
+  float* v2c;                  /* [n_frames*M*dc] work: variable-to-check messages             */
+  float* c2v;                  /* [n_frames*M*dc] work: check-to-variable messages             */
+  float* post;                 /* [n_frames*N] posterior LLRs after the last iteration         */
+  int32_t* errors;             /* [n_frames*n_iter] bits decided 1 per iteration (reset by run) */
+} vp_ldpc_params;
 
 typedef struct vp_collatz_params {
   uint32_t* steps_out;       /* [n ids] stopping time per id                               */

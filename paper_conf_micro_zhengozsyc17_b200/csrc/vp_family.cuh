@@ -146,5 +146,6 @@ const FamilyOps* family_pyramid();
 const FamilyOps* family_cfd();
 const FamilyOps* family_facedet();
 const FamilyOps* family_qbench();
+const FamilyOps* family_ldpc();
 
 }  // namespace vp

@@ -21,9 +21,10 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
+    all_families[8] = family_ldpc();
     all_families[7] = family_qbench();
     all_families[5] = family_cfd();
     all_families[6] = family_facedet();
@@ -489,7 +490,12 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
     memcpy(k.mask, mask, sizeof(k.mask));
     k.coop = coop;
     int per = quota > 0 ? quota : occ;
-    k.grid = coop ? per * N : occ * N;  // filling-retreating: enough blocks to fill every SM (L27)
+    // filling-retreating (L27): enough blocks to fill every SM.  A kernel with a block
+    // quota (fine groups) launches exactly quota x (its SMs) blocks: its quotas and its
+    // co-resident kernels' fill the SMs, so surplus blocks would have no SM to retreat
+    // through and would stall the dispatch of every later grid (seen with 4 fine LDPC
+    // stage kernels at 1 block/SM each).
+    k.grid = coop ? per * N : (quota > 0 ? quota * std::max(1, mask_count(mask, N)) : occ * N);
     k.kslot = (int)pl.kernels.size();
     if (k.kslot >= kMaxKernels) return fail(p, VP_ERR_INVALID, "too many kernels");
     pl.kernels.push_back(k);

@@ -38,6 +38,7 @@ PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
 FD_GRAY, FD_CDF, FD_MAP, FD_RESIZE, FD_LBP, FD_SCAN = 60, 61, 62, 63, 64, 65
 QB_ITEM4, QB_ITEM16, QB_ITEM272 = 70, 71, 72
+LDPC_INIT, LDPC_C2V, LDPC_V2C, LDPC_PROBVAR = 80, 81, 82, 83
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS, FLAG_ONLINE, FLAG_L2_PERSIST = (
     1, 2, 4, 8, 16, 32, 64)
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
@@ -93,6 +94,12 @@ class TuneReport(C.Structure):
 
 class ToyParams(C.Structure):
     _fields_ = [("threshold", C.c_int32), ("pad", C.c_int32), ("out", P), ("n_out", P)]
+
+
+class LdpcParams(C.Structure):
+    _fields_ = [("N", C.c_int32), ("M", C.c_int32), ("dv", C.c_int32), ("dc", C.c_int32), ("n_frames", C.c_int32),
+                ("n_iter", C.c_int32), ("alpha", C.c_float), ("pad", C.c_int32), ("check_vars", P), ("var_edges", P),
+                ("llr", P), ("v2c", P), ("c2v", P), ("post", P), ("errors", P)]
 
 
 class QBenchParams(C.Structure):

@@ -74,6 +74,42 @@ class QBenchPipeline:
         return {"leaves": int(c[self.stage]), "idsum": int(c[3 + self.stage]), "bad": int(c[6 + self.stage])}, st
 
 
+class LdpcPipeline:
+    """LDPC decoder (Fig. 17, L59): Initialize -> C2V -> V2C -> ProbVar, looping back to C2V
+    for n_iter iterations, one item per (frame, iteration)."""
+
+    def __init__(self, scene: inputs.LdpcScene, device: int = 0, **kw):
+        dev = _dev(device)
+        self.scene = scene
+        nf, E = scene.n_frames, scene.N * scene.dv
+        self.cv = torch.from_numpy(np.ascontiguousarray(scene.check_vars, np.int32)).to(dev)
+        self.ve = torch.from_numpy(np.ascontiguousarray(scene.var_edges, np.int32)).to(dev)
+        self.llr = torch.from_numpy(np.ascontiguousarray(scene.llr, np.float32)).to(dev)
+        self.v2c = torch.empty((nf, E), dtype=torch.float32, device=dev)
+        self.c2v = torch.empty((nf, E), dtype=torch.float32, device=dev)
+        self.post = torch.empty((nf, scene.N), dtype=torch.float32, device=dev)
+        self.errors = torch.zeros((nf, scene.n_iter), dtype=torch.int32, device=dev)
+        self.prm = vp.LdpcParams(N=scene.N, M=scene.M, dv=scene.dv, dc=scene.dc, n_frames=nf, n_iter=scene.n_iter,
+                                 alpha=scene.alpha, check_vars=self.cv.data_ptr(), var_edges=self.ve.data_ptr(),
+                                 llr=self.llr.data_ptr(), v2c=self.v2c.data_ptr(), c2v=self.c2v.data_ptr(),
+                                 post=self.post.data_ptr(), errors=self.errors.data_ptr())
+        self.p = vp.Pipeline(device, **kw)
+        for kind in (vp.LDPC_INIT, vp.LDPC_C2V, vp.LDPC_V2C, vp.LDPC_PROBVAR):
+            self.p.register(kind, 16, self.prm)
+        seeds = np.zeros((nf, 4), np.uint32)
+        seeds[:, 0] = np.arange(nf, dtype=np.uint32)
+        self.p.insert(0, seeds, n=nf)
+
+    def configure(self, model, binding=None, batch=0):
+        self.p.configure(model, binding, batch)
+
+    def run(self, stream=None):
+        return self.p.run(stream)
+
+    def results(self):
+        return dict(post=self.post.cpu().numpy(), errors=self.errors.cpu().numpy())
+
+
 class CollatzPipeline:
     def __init__(self, seeds: np.ndarray, max_steps: int = 1000, device: int = 0, **kw):
         n = int(seeds.size)
