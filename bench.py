@@ -259,37 +259,60 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         return r
 
     out = {}
-    sc1 = inputs.reyes_config1()
-    out["reyes_config1"] = measure(ReyesPipeline(sc1), 1)
-    # SURVEY §8(d) throughput mode: R = 256 independent config-1 frames in one run
-    sc1r = inputs.reyes_config1(n_frames=256)
-    out["reyes_config1_x256"] = measure(ReyesPipeline(sc1r), 256)
-    fs = inputs.face_scene()
-    fp = FaceDetPipeline(fs)
-    out["facedet_config2"] = measure(fp, fs.n_frames)
-    out["facedet_config2"]["windows_per_s"] = fp.results()["windows"] / (out["facedet_config2"]["ms"] / 1e3)
-    fs8 = inputs.face_scene(n_frames=8)  # throughput mode, R = 8 frames
-    fp8 = FaceDetPipeline(fs8)
-    out["facedet_config2_x8"] = measure(fp8, fs8.n_frames)
-    out["facedet_config2_x8"]["windows_per_s"] = fp8.results()["windows"] / (out["facedet_config2_x8"]["ms"] / 1e3)
-    del fp8
-    n_img, S = 32, 4096
-    rgb = inputs.pyramid_images(n_img, S)
-    # Gray: RGB read; Map: RGB read + level-0 write; Resize: read + write per level; hist negligible
-    per_img = 3 * S * S + (3 * S * S + S * S) + sum(((S >> l) ** 2) * 5 for l in range(1, 13))
-    out["pyramid_config3"] = measure(PyramidPipeline(rgb), n_img, alg_bytes=n_img * per_img)
-    del rgb
-    cs = inputs.cfd_scene(G=4096, n_outer=10)
-    out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
-    out["cfd_config3"]["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (out["cfd_config3"]["ms"] / 1e3)
-    # the LDPC decoder (Fig. 17), 100 frames x 100 iterations (L53)
-    from paper_conf_micro_zhengozsyc17_b200.workloads import LdpcPipeline
-    ls = inputs.ldpc_scene()
-    out["ldpc_f3"] = measure(LdpcPipeline(ls), ls.n_frames)
-    out["ldpc_f3"]["decoder_iterations_per_s"] = ls.n_frames * ls.n_iter / (out["ldpc_f3"]["ms"] / 1e3)
-    rs = inputs.raster_scene()
-    out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
-    out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)
+
+    def guarded(name, fn):
+        try:
+            fn()
+        except Exception as ex:  # one workload's failure must not hide the others
+            out[name] = {"error": repr(ex)}
+
+    def w_reyes1():
+        out["reyes_config1"] = measure(ReyesPipeline(inputs.reyes_config1()), 1)
+
+    def w_reyes1x():
+        # SURVEY §8(d) throughput mode: R = 256 independent config-1 frames in one run
+        out["reyes_config1_x256"] = measure(ReyesPipeline(inputs.reyes_config1(n_frames=256)), 256)
+
+    def w_face():
+        fs = inputs.face_scene()
+        fp = FaceDetPipeline(fs)
+        out["facedet_config2"] = measure(fp, fs.n_frames)
+        out["facedet_config2"]["windows_per_s"] = fp.results()["windows"] / (out["facedet_config2"]["ms"] / 1e3)
+
+    def w_face8():
+        fs8 = inputs.face_scene(n_frames=8)  # throughput mode, R = 8 frames
+        fp8 = FaceDetPipeline(fs8)
+        out["facedet_config2_x8"] = measure(fp8, fs8.n_frames)
+        out["facedet_config2_x8"]["windows_per_s"] = fp8.results()["windows"] / (out["facedet_config2_x8"]["ms"] / 1e3)
+
+    def w_pyr():
+        n_img, S = 32, 4096
+        rgb = inputs.pyramid_images(n_img, S)
+        # Gray: RGB read; Map: RGB read + level-0 write; Resize: read + write per level; hist negligible
+        per_img = 3 * S * S + (3 * S * S + S * S) + sum(((S >> l) ** 2) * 5 for l in range(1, 13))
+        out["pyramid_config3"] = measure(PyramidPipeline(rgb), n_img, alg_bytes=n_img * per_img)
+
+    def w_cfd():
+        cs = inputs.cfd_scene(G=4096, n_outer=10)
+        out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
+        out["cfd_config3"]["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (out["cfd_config3"]["ms"] / 1e3)
+
+    def w_ldpc():
+        # the LDPC decoder (Fig. 17), 100 frames x 100 iterations (L53)
+        from paper_conf_micro_zhengozsyc17_b200.workloads import LdpcPipeline
+        ls = inputs.ldpc_scene()
+        out["ldpc_f3"] = measure(LdpcPipeline(ls), ls.n_frames)
+        out["ldpc_f3"]["decoder_iterations_per_s"] = ls.n_frames * ls.n_iter / (out["ldpc_f3"]["ms"] / 1e3)
+
+    def w_raster():
+        rs = inputs.raster_scene()
+        out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
+        out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)
+
+    for name, fn in (("reyes_config1", w_reyes1), ("reyes_config1_x256", w_reyes1x), ("facedet_config2", w_face),
+                     ("facedet_config2_x8", w_face8), ("pyramid_config3", w_pyr), ("cfd_config3", w_cfd),
+                     ("ldpc_f3", w_ldpc), ("raster_config4", w_raster)):
+        guarded(name, fn)
     return out
 
 

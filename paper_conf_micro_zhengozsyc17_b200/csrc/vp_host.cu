@@ -611,6 +611,16 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       pl.cap_log2[t] = full;
       continue;
     }
+    // The recursive stages of a block-local-recursion kernel hold its stack overflow: a
+    // breadth of deep trees (many seeds recursing at once) can need far more than the
+    // producers' batches, so they keep the registered capacity.
+    bool rec_target = false;
+    for (const KernelPlan& k : pl.kernels)
+      if (p->fam->local_rec(k.lo, k.hi, k.rtc) && t >= k.lo && t <= k.hi) rec_target = true;
+    if (rec_target) {
+      pl.cap_log2[t] = full;
+      continue;
+    }
     long long need = 0;
     for (const KernelPlan& k : pl.kernels) {
       int per = k.quota > 0 ? k.quota : occupancy(p, k.lo, k.hi, k.rtc);

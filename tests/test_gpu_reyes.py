@@ -186,3 +186,22 @@ def test_reyes_config1_throughput_mode_replicas(vpm, orc):
     rp = ReyesPipeline(scene)
     configure(vpm, rp, "hybrid_mega_rtc")
     check_against_oracle(orc, scene, rp, rp.run())
+
+
+@pytest.mark.parametrize("model", ["megakernel", "hybrid_mega_rtc", "kbk_graph"])
+def test_reyes_config1_x256_wide_recursion(vpm, orc, model):
+    """256 replicas of config 1 recurse all at once (a frontier of thousands of deep split
+    trees): the recursive rings of the block-local [Bound, Split] kernel must hold it (no
+    VP_ERR_QUEUE_OVERFLOW), and every replica equals the single-frame oracle."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    one = inputs.reyes_config1()
+    ref = orc.reyes_pipeline(one)
+    scene = inputs.reyes_config1(n_frames=256)
+    rp = ReyesPipeline(scene)
+    configure(vpm, rp, model)
+    st = rp.run()
+    assert st["dequeued"][:4] == [256 * ref["n_bound"], 256 * ref["n_split"], 256 * ref["n_dice"], 256 * ref["n_shade"]]
+    key, _ = rp.keys()
+    col = rp.colours()
+    for f in (0, 1, 77, 255):
+        assert np.array_equal(key[f], ref["key"][0]) and np.array_equal(col[f], ref["colour"][0])
