@@ -22,6 +22,15 @@ namespace vp {
 #ifndef VP_REYES_MINB
 #define VP_REYES_MINB 3
 #endif
+#ifndef VP_BS_MINB          // resident blocks/SM the block-local [Bound, Split] kernel is built for
+#define VP_BS_MINB 3
+#endif
+#ifndef VP_BS_STACK         // its shared-memory work stack (patches) = its Bound dump capacity
+#define VP_BS_STACK 48
+#endif
+#ifndef VP_BS_DICE          // its Dice out-buffer capacity per round
+#define VP_BS_DICE 48
+#endif
 
 struct RPatch {           // 272 B
   float4 cp[16];          // P[a][b] at cp[4a+b]; a = u index, b = v index
@@ -230,7 +239,9 @@ struct ReyesF {
   }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
-  static constexpr int min_blocks(int, int, bool) { return VP_REYES_MINB; }
+  static constexpr int min_blocks(int lo, int hi, bool rtc) {
+    return (!rtc && lo == BOUND && hi == SPLIT) ? VP_BS_MINB : VP_REYES_MINB;
+  }
 
   template <int s>
   static __device__ unsigned long long item_id(const uint8_t* it) {
@@ -418,7 +429,7 @@ struct ReyesF {
   // out buffer and splits the others in place, pushing both children back.  Only what is
   // left when the stack or the Dice buffer would overflow goes back to the Bound ring, so
   // Split items never travel through a ring.  Same arithmetic as bound() / split().
-  static constexpr int kStack = 48, kLocalDice = 48;
+  static constexpr int kStack = VP_BS_STACK, kLocalDice = VP_BS_DICE;
   struct LocalStack {
     RPatch st[kStack];
     int nchild[2], nsplit, dump;

@@ -194,6 +194,21 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* m, uint32_t parity
         : "memory");
   }
 }
+// Worker-side wait on a buffer hand-over: the warp is suspended in the barrier (up to the
+// time hint) instead of re-issuing try_wait, so idle workers leave the issue slots to the
+// warps that still execute.
+__device__ __forceinline__ void mbar_wait_sleep(unsigned long long* m, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(m)), "r"(parity), "r"(20000u)
+        : "memory");
+  }
+}
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* m) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
                    smem_u32(dst)),
@@ -1105,7 +1120,7 @@ struct Runner {
     if (warp < kWarpsW) {
       for (int it = 0;; ++it) {
         const int b = it & 1;
-        mbar_wait(&sh.full[b], (uint32_t)((it >> 1) & 1));
+        mbar_wait_sleep(&sh.full[b], (uint32_t)((it >> 1) & 1));
         const int n = sh.bn[b];
         if (n < 0) break;
         ctx.ob = b;
