@@ -15,6 +15,9 @@
 #include "../../include/vp.h"
 #include "vp_family.cuh"
 
+#ifndef VP_PYR_PREFETCH  // Gray: load the next tile while converting this one
+#define VP_PYR_PREFETCH 0  // measured: +16% time in the megakernel (register pressure), off
+#endif
 #ifndef VP_PYR_MINB
 #define VP_PYR_MINB 3
 #endif
@@ -85,7 +88,10 @@ struct PyramidF {
   }
   // CDF's fan-out must not be expanded block-locally from a batch of latch-fired items
   static constexpr bool rtc_ok(int lo, int hi) { return !(lo < CDF && hi >= CDF); }
-  static constexpr int scratch_bytes(int, int) { return kWarpsW * 256 * 4; }  // sub-histograms / CDF / LUT staging
+  // sub-histograms / CDF / LUT staging, then the Map LUT-cache tag (image + 1, 0 = none)
+  static constexpr int kLutTag = kWarpsW * 256 * 4;
+  static constexpr int scratch_bytes(int, int) { return kLutTag + 16; }
+  static __device__ __forceinline__ uint32_t* lut_tag(uint8_t* scratch) { return (uint32_t*)(scratch + kLutTag); }
   static constexpr int default_cap_log2(int s) { return s == MAP ? 16 : 15; }
   static constexpr int min_blocks(int, int, bool) { return VP_PYR_MINB; }
 
@@ -99,6 +105,8 @@ struct PyramidF {
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
     if constexpr (s == GRAY) {
       gray_batch(ctx, (const PyrItem*)items, n);
+    } else if constexpr (s == MAP) {
+      map_batch(ctx, (const PyrItem*)items, n);
     } else if constexpr (s == RESIZE) {
       resize_batch(ctx, (const PyrItem*)items, n);
     } else {
@@ -121,19 +129,37 @@ struct PyramidF {
     const Params& p = ctx.params();
     uint32_t* hs = (uint32_t*)ctx.scratch();  // [kWarpsW][256]
     const int t = threadIdx.x, w = t >> 5;
+    if (t == 0) *lut_tag(ctx.scratch()) = 0u;  // the sub-histograms overwrite Map's cached LUT
     for (int i = t; i < kWarpsW * 256; i += kThreads) hs[i] = 0;
     worker_sync();
     const size_t npx = (size_t)p.S * p.S;
     const int y = t >> 2, x0 = (t & 3) * 16;  // thread t: 16 consecutive pixels of tile row t/4
-    int k0 = 0;
-    for (int k = 0; k < n; ++k) {
+    // the next tile's 48 B per thread are loaded while this tile is converted (two tiles
+    // of loads in flight per block instead of one)
+    auto load = [&](int k, uint4* v) {
       const PyrItem it = items[k];
       if (it.img < (uint32_t)p.n_img) {
         const size_t row = (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + x0;
         const uint4* src = (const uint4*)(p.rgb + ((size_t)it.img * npx + row) * 3);
-        uint4 v[3];
 #pragma unroll
         for (int q = 0; q < 3; ++q) v[q] = __ldg(src + q);
+      }
+    };
+    uint4 vn[3];
+    if (VP_PYR_PREFETCH && n > 0) load(0, vn);
+    int k0 = 0;
+    for (int k = 0; k < n; ++k) {
+      const PyrItem it = items[k];
+      uint4 v[3];
+      if (VP_PYR_PREFETCH) {
+#pragma unroll
+        for (int q = 0; q < 3; ++q) v[q] = vn[q];
+        if (k + 1 < n) load(k + 1, vn);
+      } else {
+        load(k, v);
+      }
+      if (it.img < (uint32_t)p.n_img) {
+        const size_t row = (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + x0;
         const uint8_t* b = (const uint8_t*)v;
         __align__(16) uint8_t g[16];
 #pragma unroll
@@ -183,6 +209,7 @@ struct PyramidF {
     uint32_t* cs = (uint32_t*)ctx.scratch();
     uint8_t* lut = ctx.scratch() + 256 * 4;
     const int t = threadIdx.x;
+    if (t == 0) *lut_tag(ctx.scratch()) = 0u;  // lut below is this image's, but staged before it is final
     const uint32_t h = __ldcg(&p.hist[(size_t)it.img * 256 + t]);
     cs[t] = h;
     worker_sync();
@@ -218,56 +245,74 @@ struct PyramidF {
   }
 
   // ------------------------------------------------------------ Map (level 0 = LUT[gray])
+  // A batch of row segments: the LUT is staged in shared memory once per image (tagged,
+  // so consecutive items and rounds of the same image reuse it), every segment's loads are
+  // in flight before its lookups and stores, and the level-1 latch arrivals of the whole
+  // batch happen together after one barrier (their fences and atomics overlap).
   template <class Ctx>
-  static __device__ void map(Ctx& ctx, const PyrItem& it) {
+  static __device__ void map_batch(Ctx& ctx, const PyrItem* items, int n) {
     const Params& p = ctx.params();
-    if (it.img >= (uint32_t)p.n_img) return;
     uint8_t* lut = ctx.scratch() + 256 * 4;
+    uint32_t* tag = lut_tag(ctx.scratch());
     const int t = threadIdx.x;
-    lut[t] = __ldcg(p.lut + (size_t)it.img * 256 + t);
-    worker_sync();
     const int nt = pyr_tiles(p.S, 0);
-    const int tx1 = min((int)it.tx + kMapSeg, nt);
-    const int wpx = (tx1 - (int)it.tx) * kPT;              // segment width in pixels
     const size_t npx = (size_t)p.S * p.S, total = pyr_img_stride(p.S);
-    const uint8_t* g = p.gray + (size_t)it.img * npx;
-    uint8_t* dst = p.pyr + (size_t)it.img * total;
-    const int vec_per_row = wpx / 16, nvec = kPT * vec_per_row;
-    // up to 8 vectors per thread, all loads in flight before the lookups and stores
-    constexpr int kV = kMapSeg * kPT * kPT / 16 / kThreads;
-    uint4 v[kV];
-#pragma unroll
-    for (int u = 0; u < kV; ++u) {
-      const int i = t + u * kThreads;
-      if (i < nvec) {
-        const int y = i / vec_per_row, xv = i - y * vec_per_row;
-        v[u] = *(const uint4*)(g + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16);
+    for (int k = 0; k < n; ++k) {
+      const PyrItem it = items[k];
+      if (it.img >= (uint32_t)p.n_img) continue;  // block-uniform
+      if (*tag != it.img + 1u) {  // block-uniform: everyone read the same tag
+        worker_sync();            // nobody still reads the previous LUT
+        lut[t] = __ldcg(p.lut + (size_t)it.img * 256 + t);
+        worker_sync();
+        if (t == 0) *tag = it.img + 1u;
       }
-    }
+      const int tx1 = min((int)it.tx + kMapSeg, nt);
+      const int wpx = (tx1 - (int)it.tx) * kPT;              // segment width in pixels
+      const uint8_t* g = p.gray + (size_t)it.img * npx;
+      uint8_t* dst = p.pyr + (size_t)it.img * total;
+      const int vec_per_row = wpx / 16, nvec = kPT * vec_per_row;
+      // up to 8 vectors per thread, all loads in flight before the lookups and stores
+      constexpr int kV = kMapSeg * kPT * kPT / 16 / kThreads;
+      uint4 v[kV];
 #pragma unroll
-    for (int u = 0; u < kV; ++u) {
-      const int i = t + u * kThreads;
-      if (i < nvec) {
-        const int y = i / vec_per_row, xv = i - y * vec_per_row;
-        uint8_t* b = (uint8_t*)&v[u];
-#pragma unroll
-        for (int q = 0; q < 16; ++q) b[q] = lut[b[q]];
-        *(uint4*)(dst + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16) = v[u];
+      for (int u = 0; u < kV; ++u) {
+        const int i = t + u * kThreads;
+        if (i < nvec) {
+          const int y = i / vec_per_row, xv = i - y * vec_per_row;
+          v[u] = *(const uint4*)(g + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16);
+        }
       }
+#pragma unroll
+      for (int u = 0; u < kV; ++u) {
+        const int i = t + u * kThreads;
+        if (i < nvec) {
+          const int y = i / vec_per_row, xv = i - y * vec_per_row;
+          uint8_t* b = (uint8_t*)&v[u];
+#pragma unroll
+          for (int q = 0; q < 16; ++q) b[q] = lut[b[q]];
+          *(uint4*)(dst + (size_t)(it.ty * kPT + y) * p.S + (size_t)it.tx * kPT + xv * 16) = v[u];
+        }
+      }
+      worker_sync();  // the tag may be read again only after every thread read it for this item
     }
-    worker_sync();
     // latch arrivals on level 1: each level-1 tile gets one count per source tile
-    if (pyr_levels(p.S) > 1 && t < kMapSeg / 2 + 1) {
-      const int a = (int)it.tx / 2 + t;                       // level-1 tile column
-      const int c0 = max((int)it.tx, 2 * a), c1 = min(tx1, 2 * a + 2);
-      const int k = c1 - c0;
-      const int nt1 = pyr_tiles(p.S, 1);
-      if (k > 0) {  // k > 0 implies a < nt1
-        const int by = (int)it.ty / 2, bx = a;
-        int* lat = p.latch + (size_t)it.img * pyr_latches_per_img(p.S) + pyr_latch_off(p.S, 1) + (size_t)by * nt1 + bx;
-        if (latch_arrive(lat, k)) {
-          PyrItem r{it.img, 1, (uint32_t)by, (uint32_t)bx};
-          ctx.template emit<RESIZE>(&r);
+    constexpr int kA = kMapSeg / 2 + 1;  // level-1 tiles a segment can touch
+    if (pyr_levels(p.S) > 1 && t < n * kA) {
+      const PyrItem it = items[t / kA];
+      const int j = t % kA;
+      if (it.img < (uint32_t)p.n_img) {
+        const int tx1 = min((int)it.tx + kMapSeg, nt);
+        const int a = (int)it.tx / 2 + j;                       // level-1 tile column
+        const int c0 = max((int)it.tx, 2 * a), c1 = min(tx1, 2 * a + 2);
+        const int k = c1 - c0;
+        const int nt1 = pyr_tiles(p.S, 1);
+        if (k > 0) {  // k > 0 implies a < nt1
+          const int by = (int)it.ty / 2, bx = a;
+          int* lat = p.latch + (size_t)it.img * pyr_latches_per_img(p.S) + pyr_latch_off(p.S, 1) + (size_t)by * nt1 + bx;
+          if (latch_arrive(lat, k)) {
+            PyrItem r{it.img, 1, (uint32_t)by, (uint32_t)bx};
+            ctx.template emit<RESIZE>(&r);
+          }
         }
       }
     }
