@@ -1133,7 +1133,7 @@ struct Runner {
       for (int it = 0;; ++it) {
         const int b = it & 1;
         if (it >= 2) {
-          mbar_wait(&sh.empty[b], (uint32_t)(((it >> 1) - 1) & 1));
+          mbar_wait_sleep(&sh.empty[b], (uint32_t)(((it >> 1) - 1) & 1));
           if (lane == 0) sh.acc_neg -= last[b];
           last[b] = 0;
         }
@@ -1145,7 +1145,7 @@ struct Runner {
           if (!other_drained) {
             // the block may be idle: the other buffer's batch must drain (and be retired)
             // before the termination test
-            mbar_wait(&sh.empty[b ^ 1], (uint32_t)(((it - 1) >> 1) & 1));
+            mbar_wait_sleep(&sh.empty[b ^ 1], (uint32_t)(((it - 1) >> 1) & 1));
             if (lane == 0) sh.acc_neg -= last[b ^ 1];
             last[b ^ 1] = 0;
             other_drained = true;

@@ -1,4 +1,5 @@
-"""Multi-GPU frame sharding for the Reyes batch (BASELINE config 5).
+"""Multi-GPU sharding: frames of the Reyes batch (BASELINE config 5) and
+triangles of one raster frame (one exchange step, a MIN of z-keys).
 
 Frames are independent, so rank r of P renders frames [r*F/P, (r+1)*F/P) with a complete
 pipeline of its own and no inter-GPU traffic during the run.  The only exchange steps
@@ -53,3 +54,30 @@ def gather_frames(local: torch.Tensor, total: int) -> torch.Tensor:
     parts = [torch.empty_like(pad) for _ in range(world)]
     dist.all_gather(parts, pad)
     return torch.cat([parts[r][: sizes[r]] for r in range(world)], 0)
+
+
+_SIGN = -(1 << 63)  # int64 bit pattern 0x8000000000000000
+
+
+def ukey_to_ordered(keys: torch.Tensor) -> torch.Tensor:
+    """uint64 z-keys stored in an int64 tensor -> int64 values with the same order under
+    signed comparison (flip the top bit), so MIN reductions (which are signed) work."""
+    return keys ^ _SIGN
+
+
+def raster_merge(keys: torch.Tensor, colour: torch.Tensor):
+    """Triangle-sharded rasterisation: every rank rendered the triangles
+    of its shard_range into keys [H, W] (uint64 bits in int64: zkey << 32 | global tri id,
+    UINT64_MAX = empty) and colour [H, W, 4].  One exchange step: all_reduce(MIN) of the
+    order-preserving keys, then the colour of the winning triangle -- held by exactly one
+    rank, because triangle ids are unique across shards -- by an all_reduce(SUM) of the
+    colours masked to the pixels each rank won (exact: one addend per pixel is nonzero).
+    Returns (keys, colour) of the whole frame on every rank."""
+    k = ukey_to_ordered(keys.clone())
+    if dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(k, op=dist.ReduceOp.MIN)
+    won = ukey_to_ordered(keys) == k
+    c = torch.where(won.unsqueeze(-1), colour, torch.zeros_like(colour))
+    if dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(c, op=dist.ReduceOp.SUM)
+    return ukey_to_ordered(k), c

@@ -133,7 +133,9 @@ class CollatzPipeline:
 class RasterPipeline:
     """Vertex -> Clip -> Raster -> Fragment (+ colour resolve) over a RasterScene (Fig. 16, L59)."""
 
-    def __init__(self, scene: inputs.RasterScene, device: int = 0, **kw):
+    def __init__(self, scene: inputs.RasterScene, device: int = 0, tri_range=None, **kw):
+        """tri_range = (lo, hi): seed only triangles [lo, hi) (a rank's shard, SURVEY §8(f-4));
+        keys keep the global triangle ids."""
         dev = _dev(device)
         self.scene = scene
         n = scene.n_tris
@@ -149,8 +151,9 @@ class RasterPipeline:
         self.p = vp.Pipeline(device, **kw)
         for kind, stride in zip((vp.RASTER_VERTEX, vp.RASTER_CLIP, vp.RASTER_RASTER, vp.RASTER_FRAGMENT), (4, 4, 4, 8)):
             self.p.register(kind, stride, self.prm)
-        self.ids = torch.arange(n, dtype=torch.int32, device=dev)
-        self.p.insert(0, self.ids, n=n)
+        lo, hi = tri_range if tri_range is not None else (0, n)
+        self.ids = torch.arange(lo, hi, dtype=torch.int32, device=dev)
+        self.p.insert(0, self.ids, n=hi - lo)
 
     def configure(self, model, binding=None, batch=0):
         self.p.configure(model, binding, batch)

@@ -94,3 +94,46 @@ def test_raster_full_config4_sampled(vpm, orc):
     rp = RasterPipeline(scene)
     configure(vpm, rp, "hybrid_rtc_mega")
     check(orc, scene, rp, rp.run())
+
+
+def _merge_local(parts):
+    """raster_merge's exchange step on one device: MIN of the order-preserving keys, then
+    the colour of the rank that holds the winning key."""
+    import torch
+    from paper_conf_micro_zhengozsyc17_b200 import shard
+    ks = [shard.ukey_to_ordered(k) for k, _ in parts]
+    kmin = ks[0]
+    for k in ks[1:]:
+        kmin = torch.minimum(kmin, k)
+    col = sum(torch.where((k == kmin).unsqueeze(-1), c, torch.zeros_like(c)) for k, (_, c) in zip(ks, parts))
+    return shard.ukey_to_ordered(kmin), col
+
+
+@pytest.mark.parametrize("shards", [2, 4])
+def test_raster_triangle_shards_merge_bit_exact(vpm, orc, shards):
+    """the frame rendered as `shards` triangle shards (each a pipeline run
+    over its id range, as one rank would) and merged by the MIN-key exchange equals the
+    oracle (reduced scene) and the unsharded GPU frame (full 1M-triangle config 4)."""
+    from paper_conf_micro_zhengozsyc17_b200 import shard
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    vp = vpm
+    for sc, ref_fn in ((inputs.raster_scene(n=10_000, W=320, H=180), "oracle"), (inputs.raster_scene(), "gpu")):
+        parts = []
+        for r in range(shards):
+            lo, hi = shard.shard_range(r, shards, sc.n_tris)
+            rp = RasterPipeline(sc, tri_range=(lo, hi))
+            rp.configure(vp.MEGAKERNEL)
+            rp.run()
+            parts.append((rp.fb.clone(), rp.colour.clone()))
+            del rp
+        k, c = _merge_local(parts)
+        if ref_fn == "oracle":
+            ref = orc.raster_definition(sc)
+            rk, rc = ref["key"], ref["colour"]
+        else:
+            full = RasterPipeline(sc)
+            full.configure(vp.MEGAKERNEL)
+            full.run()
+            rk, rc = full.keys(), full.colour.cpu().numpy()
+        assert np.array_equal(k.cpu().numpy().view(np.uint64), rk.reshape(k.shape))
+        assert np.array_equal(c.cpu().numpy(), rc.reshape(c.shape))

@@ -68,3 +68,62 @@ def test_sharded_render_equals_single_process(orc, world):
     assert np.array_equal(full, ref["colour"])
     assert counts == [ref["n_bound"], ref["n_split"], ref["n_dice"], ref["n_shade"]]
     assert t == float(world)
+
+
+# ---------------------------------------------------------------- raster triangle sharding
+def collapse_outside(scene, lo, hi):
+    """The shard's scene: triangles outside [lo, hi) collapsed to a point (zero area, culled
+    by Clip), so every surviving key keeps its global triangle id."""
+    import dataclasses
+    pos = scene.pos.copy()
+    keep = np.zeros(scene.n_tris, bool)
+    keep[lo:hi] = True
+    pos[~keep, 1] = pos[~keep, 0]
+    pos[~keep, 2] = pos[~keep, 0]
+    return dataclasses.replace(scene, pos=pos)
+
+
+def test_ordered_key_transform_preserves_uint64_order():
+    rng = np.random.default_rng(5)
+    u = np.concatenate([rng.integers(0, 2**64 - 1, 2000, dtype=np.uint64),
+                        np.array([0, 1, 2**63 - 1, 2**63, 2**63 + 1, 2**64 - 1], np.uint64)])
+    o = shard.ukey_to_ordered(torch.from_numpy(u.view(np.int64))).numpy()
+    assert np.array_equal(np.argsort(o, kind="stable"), np.argsort(u, kind="stable"))
+    assert np.array_equal(shard.ukey_to_ordered(torch.from_numpy(o)).numpy().view(np.uint64), u)
+
+
+def _raster_worker(rank, world, port, q):
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        from paper_conf_micro_zhengozsyc17_b200 import inputs
+        sc = inputs.raster_scene(n=3000, W=96, H=64)
+        lo, hi = shard.shard_range(rank, world, sc.n_tris)
+        r = oracle.raster_definition(collapse_outside(sc, lo, hi))
+        k, c = shard.raster_merge(torch.from_numpy(r["key"].view(np.int64).copy()), torch.from_numpy(r["colour"].copy()))
+        if rank == 0:
+            q.put((k.numpy().view(np.uint64), c.numpy()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_triangle_sharded_raster_equals_single_frame(orc, world):
+    """each rank rasterises a shard of the triangles (the CPU oracle stands
+    in for the GPU here); one MIN all-reduce of the z-keys plus the winner's colour
+    reproduces the single-process frame bit for bit."""
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_raster_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    k, c = q.get(timeout=120)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    ref = orc.raster_definition(inputs.raster_scene(n=3000, W=96, H=64))
+    assert np.array_equal(k, ref["key"]) and np.array_equal(c, ref["colour"])

@@ -1,2 +1,4 @@
 mkdir -p gpurun_out
-for lib in libvp.so libvp_nopf.so libvp_m2.so; do echo "== $lib"; VP_LIB_NAME=$lib timeout 300 python tools/pyr_time.py; done > gpurun_out/pyr_time2.log 2>&1
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 600 python tools/reyes_sweep.py --reps 3 --no-timers --configs h56b16_16_64_4,h60b16_16_64_4,h64b16_16_64_4 > gpurun_out/sweep11.log 2>&1
+timeout 600 python -m pytest tests/test_gpu_reyes.py tests/test_gpu_raster.py tests/test_gpu_basic.py -q > gpurun_out/pr.log 2>&1
