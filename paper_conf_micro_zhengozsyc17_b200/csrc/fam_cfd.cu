@@ -311,7 +311,8 @@ struct CfdF {
 #pragma unroll
           for (int q = 0; q < 5; ++q) __stcg((float4*)(p.old + (size_t)q * N + i0 + i), v[q]);
         }
-        worker_sync();
+        // the emitted item becomes visible only through the publisher, after the round
+        // barrier: no barrier is needed here
         if (threadIdx.x == 0) ctx.template emit<STEP>(&ci);
       } else if constexpr (s == STEP) {
         for (int i = threadIdx.x * 4; i < p.T; i += kThreads * 4) {
@@ -333,8 +334,6 @@ struct CfdF {
           }
           __stcg((float4*)(p.sf + c), r);
         }
-        worker_sync();
-        if (threadIdx.x == 0) arrive(ctx, p, ci.tile, k);
       } else if constexpr (s == FLUX) {
         flux_item(ctx, p, ci);
         if (threadIdx.x == 0) ctx.template emit<TIME>(&ci);
@@ -368,14 +367,31 @@ struct CfdF {
             __stcg((float4*)(nxt + (size_t)v * N + c), r);
           }
         }
-        worker_sync();
-        // latch arrivals: thread j < m arrives on neighbour j, thread m on the tile itself
-        // (or emits the next outer iteration's Copy) -- the fences and atomics of one item
-        // overlap instead of running back to back on one thread
-        if (threadIdx.x < 5 && outer + (rk == kRK - 1 ? 1u : 0u) < (uint32_t)p.n_outer) {
+      }
+      // (Flux ends with a barrier of its own; Copy / StepFactor / TimeStep items write
+      // disjoint tiles, so the next item's loads overlap this item's stores)
+    }
+    // Latch arrivals of the whole batch after ONE barrier (every thread's writes of every
+    // item precede them), all in parallel: their fences and atomics overlap.
+    if constexpr (s == STEP) {
+      worker_sync();
+      if ((int)threadIdx.x < n) {
+        const CfdItem ci = ((const CfdItem*)items)[threadIdx.x];
+        arrive(ctx, p, ci.tile, ci.k);
+      }
+    } else if constexpr (s == TIME) {
+      worker_sync();
+      // per item: thread j < m arrives on neighbour j, thread m on the tile itself (or
+      // emits the next outer iteration's Copy)
+      if ((int)threadIdx.x < 5 * n) {
+        const CfdItem ci = ((const CfdItem*)items)[threadIdx.x / 5];
+        const int j = threadIdx.x % 5;
+        const uint32_t k = ci.k;
+        const int rk = (int)(k % kRK);
+        const uint32_t outer = k / kRK;
+        if (outer + (rk == kRK - 1 ? 1u : 0u) < (uint32_t)p.n_outer) {
           uint32_t nbt[4];
           const int m = tile_neighbours(p, ci.tile, nbt);
-          const int j = threadIdx.x;
           if (j < m) {
             arrive(ctx, p, nbt[j], k + 1);
           } else if (j == m) {
@@ -388,7 +404,6 @@ struct CfdF {
           }
         }
       }
-      worker_sync();
     }
   }
 

@@ -1,4 +1,3 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 600 python tools/reyes_sweep.py --reps 3 --no-timers --configs h56b16_16_64_4,h60b16_16_64_4,h64b16_16_64_4 > gpurun_out/sweep11.log 2>&1
-timeout 600 python -m pytest tests/test_gpu_reyes.py tests/test_gpu_raster.py tests/test_gpu_basic.py -q > gpurun_out/pr.log 2>&1
+timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__warps_active.avg.pct_of_peak_sustained_active --clock-control none --csv --log-file gpurun_out/cfd_kbk_launches2.csv python tools/ncu_wl.py cfd kbk --outer 1 > /dev/null 2>&1
