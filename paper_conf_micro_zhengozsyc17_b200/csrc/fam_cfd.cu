@@ -94,7 +94,7 @@ struct CfdF {
   using Params = vp_cfd_params;
   static constexpr int stride(int) { return 16; }
   static constexpr int threads_per_item(int) { return 256; }
-  static constexpr int max_batch(int s) { return s == FLUX ? 2 : 4; }
+  static constexpr int max_batch(int s) { return s == FLUX ? 2 : 8; }
   static constexpr int default_batch(int s) { return max_batch(s); }
   static constexpr int fanout(int s, int t) {
     return (s == COPY && t == STEP) || (s == STEP && t == FLUX) || (s == FLUX && t == TIME) || (s == TIME && t == COPY) ? 1
