@@ -329,9 +329,17 @@ def main():
     from paper_conf_micro_zhengozsyc17_b200 import inputs, vp
     from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
 
+    # VP_BENCH_ONE_GPU=1 (dev only): every rank on cuda:0 with gloo, to exercise the N > 1
+    # code path (sharding, reductions, gather) on a one-GPU box; the driver never sets it
+    one_gpu = os.environ.get("VP_BENCH_ONE_GPU") == "1"
+    if one_gpu:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if one_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     nsm, cc = vp.device_info(local)
     # ---- shard: rank r renders frames [r*F/P, (r+1)*F/P) of the orbit
     from paper_conf_micro_zhengozsyc17_b200 import shard
