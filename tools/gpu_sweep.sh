@@ -1,3 +1,2 @@
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,smsp__issue_active.avg.pct_of_peak_sustained_active,sm__warps_active.avg.pct_of_peak_sustained_active --clock-control none --csv --log-file gpurun_out/cfd_kbk_launches2.csv python tools/ncu_wl.py cfd kbk --outer 1 > /dev/null 2>&1
+for lib in libvp.so libvp_p4.so libvp_p5.so; do echo "== $lib"; VP_LIB_NAME=$lib timeout 300 python tools/pyr_time.py; done > gpurun_out/pyr_time3.log 2>&1
