@@ -242,7 +242,7 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
 
         ms, st = t_run()
         pipe.configure(vp.KBK)
-        kbk_ms, _ = t_run()
+        kbk_ms, kst = t_run()
         pipe.configure(vp.KBK_GRAPH)
         kbkg_ms, _ = t_run()
         pipe.configure(vp.MEGAKERNEL)
@@ -253,6 +253,13 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
              "items": items, "kbk_ms": kbk_ms, "kbk_graph_ms": kbkg_ms, "megakernel_ms": mega_ms,
              "speedup_vs_kbk": kbk_ms / ms, "speedup_vs_kbk_graph": kbkg_ms / ms,
              "speedup_vs_megakernel": mega_ms / ms, "tuned": tuned_cfg.split(" mask")[0]}
+        # Table 2 analog (L51): the longest stage run in isolation (its KBK waves, whole GPU)
+        # vs the pipeline; the difference is queue / runtime overhead and stage imbalance
+        sw = [x for x in kst["stage_wave_ms"] if x > 0]
+        if sw:
+            r["stage_wave_ms"] = [round(x, 4) for x in kst["stage_wave_ms"][:len(st["dequeued"])]]
+            r["longest_stage_ms"] = max(sw)
+            r["overhead_vs_longest_stage_pct"] = 100.0 * (ms - max(sw)) / ms
         if alg_bytes:
             gbs = alg_bytes / (ms / 1e3) / 1e9
             r.update({"alg_bytes": alg_bytes, "achieved_gbs": gbs, "pct_hbm_measured": 100 * gbs / hbm_gbs})

@@ -188,6 +188,9 @@ typedef struct vp_run_stats {
   uint64_t seed_head[VP_MAX_STAGES];
   int64_t pending;
   uint64_t kernel_rounds[16];               /* persistent-loop rounds summed over blocks  */
+  /* host-driven KBK: summed device time of each stage's wave kernels (every wave uses the
+   * whole GPU), i.e. each stage run in isolation -- Table 2's "longest stage" analog (L51) */
+  float stage_wave_ms[VP_MAX_STAGES];
 } vp_run_stats;
 
 typedef struct vp_autotune_opts {

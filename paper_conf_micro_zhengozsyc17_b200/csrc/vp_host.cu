@@ -243,6 +243,9 @@ struct vp_pipeline_s {
   // device-driven KBK: instantiated graph and the launch arguments it was captured with
   int refill_lo[kMaxKernels] = {}, refill_hi[kMaxKernels] = {}, refill_quota[kMaxKernels] = {};
   bool launched[kMaxKernels] = {};  // planned kernels launched by the last vp_run
+  // host-driven KBK: per-wave event pairs (pooled) and the stage of each wave of the last run
+  std::vector<cudaEvent_t> wave_ev;
+  std::vector<int> wave_stage;
   void* seq_arena = nullptr;  // every ring's sequence words (one L2 persisting window)
   size_t seq_arena_bytes = 0;
   bool l2_window_set = false;
@@ -749,12 +752,30 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
       return VP_OK;
     }
     bool launched = false;
+    // one event pair per wave (from a pool), read back after the run for stage_wave_ms
+    auto wave_begin = [&](int s) -> vp_status {
+      const size_t i = p->wave_stage.size();
+      while (p->wave_ev.size() < 2 * (i + 1)) {
+        cudaEvent_t e;
+        CUDA_TRY(p, cudaEventCreate(&e));
+        p->wave_ev.push_back(e);
+      }
+      p->wave_stage.push_back(s);
+      CUDA_TRY(p, cudaEventRecord(p->wave_ev[2 * i], st));
+      return VP_OK;
+    };
+    auto wave_end = [&]() -> vp_status {
+      CUDA_TRY(p, cudaEventRecord(p->wave_ev[2 * (p->wave_stage.size() - 1) + 1], st));
+      return VP_OK;
+    };
     if (p->plan.wave_rtc) {
       for (int s = 0; s < S && !launched; ++s) {
         long long n = wave_n(s, a);
         if (n > 0) {
+          if ((rc = wave_begin(s)) != VP_OK) return rc;
           rc = launch_wave(p, c, 0, S - 1, true, s, n, st, 0);
           if (rc != VP_OK) return rc;
+          if ((rc = wave_end()) != VP_OK) return rc;
           launched = true;
         }
       }
@@ -763,8 +784,10 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
         int s = ks[i];
         long long n = wave_n(s, a);
         if (n > 0) {
+          if ((rc = wave_begin(s)) != VP_OK) return rc;
           rc = launch_wave(p, c, s, s, false, s, n, st, 0);
           if (rc != VP_OK) return rc;
+          if ((rc = wave_end()) != VP_OK) return rc;
           launched = true;
         }
       }
@@ -974,6 +997,7 @@ vp_status vp_pipeline_destroy(void* h) {
   }
   if (p->kg_exec) cudaGraphExecDestroy(p->kg_exec);
   if (p->kg_graph) cudaGraphDestroy(p->kg_graph);
+  for (cudaEvent_t e : p->wave_ev) cudaEventDestroy(e);
   cudaEventDestroy(p->ev_fork);
   cudaEventDestroy(p->ev_start);
   cudaEventDestroy(p->ev_end);
@@ -1248,6 +1272,7 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
     }
   }
   uint64_t launches = 0;
+  p->wave_stage.clear();
   if (pl.kbk_graph) {
     vp_status rc = graph_wave_run(p, c, st, &launches);
     if (rc != VP_OK) return rc;
@@ -1298,6 +1323,11 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
     for (int i = 0; i < kMaxKernels; ++i) {
       stats->kernel_idle_ns[i] = hc.idle_ns[i];
       stats->kernel_rounds[i] = hc.rounds[i];
+    }
+    for (size_t w = 0; w < p->wave_stage.size(); ++w) {
+      float ms_w = 0.0f;
+      if (cudaEventElapsedTime(&ms_w, p->wave_ev[2 * w], p->wave_ev[2 * w + 1]) == cudaSuccess)
+        stats->stage_wave_ms[p->wave_stage[w]] += ms_w;
     }
     for (int s = 0; s < S; ++s) {
       stats->ring_tail[s] = hc.tail[s].v;

@@ -77,7 +77,8 @@ class RunStats(C.Structure):
                 ("stage_exec_ns", C.c_uint64 * MAX_STAGES), ("stage_flush_ns", C.c_uint64 * MAX_STAGES),
                 ("kernel_idle_ns", C.c_uint64 * 16), ("ring_tail", C.c_uint64 * MAX_STAGES),
                 ("ring_head", C.c_uint64 * MAX_STAGES), ("ring_count", C.c_int64 * MAX_STAGES),
-                ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16)]
+                ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16),
+                ("stage_wave_ms", C.c_float * MAX_STAGES)]
 
 
 class AutotuneOpts(C.Structure):
@@ -338,7 +339,8 @@ def stats_dict(st: RunStats):
                 num_sms=st.num_sms, stage_exec_ns=list(st.stage_exec_ns), stage_flush_ns=list(st.stage_flush_ns),
                 kernel_idle_ns=list(st.kernel_idle_ns[:max(nk, 1)]), ring_tail=list(st.ring_tail),
                 ring_head=list(st.ring_head), ring_count=list(st.ring_count), seed_head=list(st.seed_head),
-                pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]))
+                pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]),
+                stage_wave_ms=list(st.stage_wave_ms))
 
 
 def config_to_string(cfg: Config) -> str:

@@ -171,3 +171,16 @@ def test_configure_validation(vpm, bad):
     with pytest.raises(vp.VPError) as e:
         tp.configure(vp.HYBRID, b)
     assert e.value.status == vp.VP_ERR_INVALID
+
+
+def test_kbk_stage_wave_times(vpm, orc):
+    """Host-driven KBK reports each stage's summed wave time (Table 2's longest-stage
+    analog); stages that ran have > 0, the others 0, and their sum fits in the run."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ToyPipeline
+    vp = vpm
+    tp = ToyPipeline(inputs.toy_seeds(100_000))
+    tp.configure(vp.KBK)
+    _, st = tp.run()
+    w = st["stage_wave_ms"]
+    assert all(x > 0 for x in w[:3]) and all(x == 0 for x in w[3:])
+    assert sum(w[:3]) <= st["device_ms"] * 1.05
