@@ -104,7 +104,8 @@ typedef enum vp_stage_kind {
 #define VP_FLAG_TRACE 0x1u          /* record (stage, item id, smid) of every task           */
 #define VP_FLAG_QUEUE_DEPTH 0x2u    /* track max ring depth per stage (one extra read/flush) */
 #define VP_FLAG_STRICT_BINDING 0x4u /* vp_run fails with VP_ERR_BINDING on quota shortfall   */
-#define VP_FLAG_TIMERS 0x8u         /* in-kernel %globaltimer accumulators per stage/kernel  */
+#define VP_FLAG_TIMERS 0x8u         /* in-kernel %globaltimer accumulators per stage/kernel, */
+                                    /* and KBK wave times per stage (stage_wave_ms)         */
 #define VP_FLAG_ONLINE 0x20u        /* online adaptation (L41-L45): a persistent group whose  */
                                     /* stages can get no more items retires and the host      */
                                     /* relaunches the next group downstream on its SMs         */
@@ -376,6 +377,11 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best, vp_tu
 
 /* Profiling component (L13, L45): max resident blocks per SM of each single-stage kernel. */
 vp_status vp_profile(void* p, int* max_blocks_per_sm, int* regs_per_thread, int* smem_per_block);
+
+/* Change the run-time diagnostics flags of a pipeline (VP_FLAG_QUEUE_DEPTH,
+ * VP_FLAG_STRICT_BINDING, VP_FLAG_TIMERS; the others are fixed at create and rejected with
+ * VP_ERR_INVALID).  old_flags (optional) receives all flags before the change. */
+vp_status vp_set_flags(void* p, uint32_t flags, uint32_t* old_flags);
 
 /* Library-owned / borrowed outputs of the family (sink results). index 0 = primary. */
 vp_status vp_get_output(void* p, int index, void** dev_ptr, size_t* bytes);

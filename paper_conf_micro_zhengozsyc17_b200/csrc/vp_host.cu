@@ -752,8 +752,11 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
       return VP_OK;
     }
     bool launched = false;
-    // one event pair per wave (from a pool), read back after the run for stage_wave_ms
+    // VP_FLAG_TIMERS: one event pair per wave (from a pool), read back after the run for
+    // stage_wave_ms (off by default: the records would slow the KBK baseline down)
+    const bool wave_times = (p->desc.flags & VP_FLAG_TIMERS) != 0;
     auto wave_begin = [&](int s) -> vp_status {
+      if (!wave_times) return VP_OK;
       const size_t i = p->wave_stage.size();
       while (p->wave_ev.size() < 2 * (i + 1)) {
         cudaEvent_t e;
@@ -765,6 +768,7 @@ vp_status host_wave_loop(vp_pipeline_s* p, const Common& c, cudaStream_t st, uin
       return VP_OK;
     };
     auto wave_end = [&]() -> vp_status {
+      if (!wave_times) return VP_OK;
       CUDA_TRY(p, cudaEventRecord(p->wave_ev[2 * (p->wave_stage.size() - 1) + 1], st));
       return VP_OK;
     };
@@ -1382,6 +1386,16 @@ int vpi_rtc_legal(void* h, int lo, int hi) {
   return p && p->fam && p->fam->rtc_legal(lo, hi) ? 1 : 0;
 }
 int vpi_default_batch(void* h, int s) { return ((vp_pipeline_s*)h)->fam->default_batch(s); }
+vp_status vp_set_flags(void* h, uint32_t flags, uint32_t* old_flags) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  const uint32_t mutable_bits = VP_FLAG_QUEUE_DEPTH | VP_FLAG_STRICT_BINDING | VP_FLAG_TIMERS;
+  if (flags & ~mutable_bits) return fail(p, VP_ERR_INVALID, "vp_set_flags: only QUEUE_DEPTH, STRICT_BINDING, TIMERS change after create");
+  if (old_flags) *old_flags = p->desc.flags;
+  p->desc.flags = (p->desc.flags & ~mutable_bits) | flags;
+  return VP_OK;
+}
+
 uint32_t vpi_swap_flags(void* h, uint32_t flags) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;
   uint32_t old = p->desc.flags;

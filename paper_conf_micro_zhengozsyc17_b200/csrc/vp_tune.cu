@@ -119,6 +119,11 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
   const auto t0 = std::chrono::steady_clock::now();
   auto elapsed = [&] { return std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count(); };
 
+  struct Cand {
+    double ms;
+    vp_config c;
+  };
+  std::vector<Cand> fastest;  // fastest candidates seen (single-run times are noisy)
   double mintime = 1e30;
   vp_config best;
   memset(&best, 0, sizeof(best));
@@ -146,6 +151,11 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
       mintime = t;
       best = c;
       have_best = true;
+    }
+    if (t > 0) {  // keep the fastest few for the final re-timing
+      fastest.push_back({t, c});
+      std::sort(fastest.begin(), fastest.end(), [](const Cand& a, const Cand& b) { return a.ms < b.ms; });
+      if (fastest.size() > 4) fastest.pop_back();
     }
     return t;
   };
@@ -290,6 +300,22 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
     }
   }
 
+  // Final re-timing: the fastest few candidates (the baselines included) run again
+  // with more repeats; the search's single-run times decide only which ones get here.
+  if (fatal == VP_OK && fastest.size() > 1) {
+    double best_ms = 1e30;
+    for (const Cand& k : fastest) {
+      bool to = false;
+      const double t = timeoutexec(p, k.c, 2.0 * k.ms, std::max(3, reps), &to, &fatal);
+      R.candidates_run++;
+      if (fatal != VP_OK) break;
+      if (t > 0 && t < best_ms) {
+        best_ms = t;
+        best = k.c;
+      }
+    }
+    if (best_ms < 1e30) mintime = best_ms;
+  }
   vp_set_timeout(p, saved_timeout);
   if (fatal != VP_OK) return fatal;  // vp_last_error holds the CUDA message
   if (!have_best) {

@@ -168,11 +168,12 @@ vp_config_to_string = _decl("vp_config_to_string", [C.POINTER(Config), C.c_char_
 vp_config_from_string = _decl("vp_config_from_string", [C.c_char_p, C.POINTER(Config)])
 vp_device_info = _decl("vp_device_info", [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)])
 vp_memcpy = _decl("vp_memcpy", [P, P, C.c_size_t, C.c_int, P])
+vp_set_flags = _decl("vp_set_flags", [P, C.c_uint32, C.POINTER(C.c_uint32)])
 
 EXPORTED = ["vp_status_string", "vp_last_error", "vp_pipeline_create", "vp_pipeline_destroy", "vp_stage_register",
             "vp_insert", "vp_insert_async", "vp_configure", "vp_configure_config", "vp_get_config", "vp_run",
             "vp_set_timeout", "vp_get_trace", "vp_autotune", "vp_profile", "vp_get_output", "vp_config_to_string", "vp_config_from_string",
-            "vp_device_info", "vp_memcpy"]
+            "vp_device_info", "vp_memcpy", "vp_set_flags"]
 
 
 class VPError(RuntimeError):
@@ -288,6 +289,13 @@ class Pipeline:
         ptr, n = P(), C.c_size_t()
         self._check(vp_get_trace(self.h, C.byref(ptr), C.byref(n)), "vp_get_trace")
         return ptr.value
+
+    def set_flags(self, flags):
+        """Run-time diagnostics flags (FLAG_QUEUE_DEPTH | FLAG_STRICT_BINDING | FLAG_TIMERS);
+        returns the previous flags."""
+        old = C.c_uint32()
+        self._check(vp_set_flags(self.h, flags, C.byref(old)), "vp_set_flags")
+        return old.value
 
     def set_timeout_ms(self, ms):
         self._check(vp_set_timeout(self.h, float(ms)), "vp_set_timeout")

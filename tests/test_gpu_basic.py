@@ -181,6 +181,9 @@ def test_kbk_stage_wave_times(vpm, orc):
     tp = ToyPipeline(inputs.toy_seeds(100_000))
     tp.configure(vp.KBK)
     _, st = tp.run()
+    assert not any(st["stage_wave_ms"])          # only with VP_FLAG_TIMERS
+    assert tp.p.set_flags(vp.FLAG_TIMERS) == 0
+    _, st = tp.run()
     w = st["stage_wave_ms"]
     assert all(x > 0 for x in w[:3]) and all(x == 0 for x in w[3:])
     assert sum(w[:3]) <= st["device_ms"] * 1.05
