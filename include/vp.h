@@ -243,6 +243,8 @@ typedef struct vp_ldpc_params {
   int32_t N, M, dv, dc;        /* variables, checks, degrees (N*dv == M*dc, dc <= 32, dv <= 8) */
   int32_t n_frames, n_iter;    /* frames decoded in one run; iterations per frame              */
   float alpha;                 /* min-sum normalisation                                        */
+  int32_t nc_chk, nc_var;      /* items: C2V chunks of the checks, V2C / ProbVar chunks of the */
+                               /* variables (1..16 each; reading R-L6)                         */
   int32_t pad;
   const int32_t* check_vars;   /* [M*dc] variable of each edge                                 */
   const int32_t* var_edges;    /* [N*dv] edges of each variable, ascending                     */
@@ -251,6 +253,7 @@ typedef struct vp_ldpc_params {
   float* c2v;                  /* [n_frames*M*dc] work: check-to-variable messages             */
   float* post;                 /* [n_frames*N] posterior LLRs after the last iteration         */
   int32_t* errors;             /* [n_frames*n_iter] bits decided 1 per iteration (reset by run) */
+  int32_t* latch;              /* [n_frames*2] work: the chunk-join latches (reset by run)      */
 } vp_ldpc_params;
 
 typedef struct vp_collatz_params {

@@ -129,8 +129,8 @@ def qbench_pipeline(seeds: np.ndarray, item_bytes: int, fanout: int):
 
 class LdpcC(C.Structure):
     _fields_ = [("N", C.c_int32), ("M", C.c_int32), ("dv", C.c_int32), ("dc", C.c_int32), ("n_frames", C.c_int32),
-                ("n_iter", C.c_int32), ("alpha", C.c_float), ("pad", C.c_int32), ("check_vars", P),
-                ("var_edges", P), ("llr", P)]
+                ("n_iter", C.c_int32), ("alpha", C.c_float), ("nc_chk", C.c_int32), ("nc_var", C.c_int32),
+                ("pad", C.c_int32), ("check_vars", P), ("var_edges", P), ("llr", P)]
 
 
 def _ldpc_run(fn, sc, llr=None, n_iter=None, alpha=None):
@@ -140,13 +140,15 @@ def _ldpc_run(fn, sc, llr=None, n_iter=None, alpha=None):
     nf = llr.shape[0]
     it = sc.n_iter if n_iter is None else n_iter
     d = LdpcC(N=sc.N, M=sc.M, dv=sc.dv, dc=sc.dc, n_frames=nf, n_iter=it,
-              alpha=sc.alpha if alpha is None else alpha, check_vars=_ptr(cv), var_edges=_ptr(ve), llr=_ptr(llr))
+              alpha=sc.alpha if alpha is None else alpha, nc_chk=sc.nc_chk, nc_var=sc.nc_var, check_vars=_ptr(cv),
+              var_edges=_ptr(ve), llr=_ptr(llr))
     post = np.zeros((nf, sc.N), np.float32)
     err = np.zeros((nf, it), np.int32)
     if fn == "orc_ldpc_pipeline":
         st = Stats()
         assert lib().orc_ldpc_pipeline(C.byref(d), _ptr(post), _ptr(err), C.byref(st)) == 0
         return dict(post=post, errors=err, deq=list(st.deq[:4]), enq=list(st.enq[:4]))
+    assert fn == "orc_ldpc_definition"
     assert lib().orc_ldpc_definition(C.byref(d), _ptr(post), _ptr(err)) == 0
     return dict(post=post, errors=err)
 

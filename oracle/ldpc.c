@@ -92,12 +92,18 @@ int orc_ldpc_definition(const orc_ldpc* d, float* post, int32_t* errors) {
   return 0;
 }
 
-/* Pipeline: items {frame, iteration} through the four stages (Fig. 17). */
-typedef struct ldpc_item { uint32_t frame, iter, pad0, pad1; } ldpc_item;
+/* Pipeline (reading R-L6): items {frame, iteration, chunk}.  Initialize(f) emits the
+ * nc_chk C2V chunks of iteration 0; the last C2V chunk of (f, it) to finish (a dependency
+ * latch) emits the nc_var V2C and nc_var ProbVar chunks of (f, it); the last of those 2*nc_var
+ * chunks emits the C2V chunks of (f, it + 1) -- ProbVar(it) must read c2v before C2V(it+1)
+ * overwrites it.  Chunk c of n covers [c*K/n, (c+1)*K/n) of the K checks or variables. */
+typedef struct ldpc_item { uint32_t frame, iter, chunk, pad; } ldpc_item;
 typedef struct ldpc_user {
   const orc_ldpc* d;
   float *v2c, *c2v, *post;
   int32_t* errors;
+  int32_t* latch_c;  /* [frames] C2V chunks of the current iteration still to finish   */
+  int32_t* latch_v;  /* [frames] V2C + ProbVar chunks still to finish                  */
 } ldpc_user;
 
 static void ldpc_exec(orc_engine* eng, int stage, const void* p) {
@@ -109,38 +115,62 @@ static void ldpc_exec(orc_engine* eng, int stage, const void* p) {
   float* v2c = u->v2c + (size_t)it.frame * E;
   float* c2v = u->c2v + (size_t)it.frame * E;
   const float* L = d->llr + (size_t)it.frame * d->N;
-  orc_record(eng, stage, ((uint64_t)it.frame << 32) | it.iter);
+  orc_record(eng, stage, ((uint64_t)it.frame << 32) | ((uint64_t)it.iter << 8) | it.chunk);
   if (stage == 0) {          /* Initialize */
     for (size_t e = 0; e < E; ++e) v2c[e] = L[d->check_vars[e]];
-    orc_push(eng, 1, &it);
-  } else if (stage == 1) {   /* C2V */
-    for (int m = 0; m < d->M; ++m) c2v_check(d, v2c, c2v, m);
-    orc_push(eng, 2, &it);
-  } else if (stage == 2) {   /* V2C */
-    for (int n = 0; n < d->N; ++n) v2c_var(d, L, c2v, v2c, n);
-    orc_push(eng, 3, &it);
-  } else {                   /* ProbVar */
-    int err = 0;
-    for (int n = 0; n < d->N; ++n) {
-      const float P = posterior(d, L, c2v, n);
-      err += P < 0.0f;
-      if ((int)it.iter == d->n_iter - 1) u->post[(size_t)it.frame * d->N + n] = P;
+    for (int c = 0; c < d->nc_chk; ++c) {
+      ldpc_item x = {it.frame, 0u, (uint32_t)c, 0u};
+      orc_push(eng, 1, &x);
     }
-    u->errors[(size_t)it.frame * d->n_iter + it.iter] = err;
-    if ((int)it.iter + 1 < d->n_iter) {
-      ldpc_item nx = it;
-      nx.iter++;
-      orc_push(eng, 1, &nx);  /* inner loop back to C2V */
+  } else if (stage == 1) {   /* C2V chunk */
+    const int m0 = (int)((long long)it.chunk * d->M / d->nc_chk), m1 = (int)((long long)(it.chunk + 1) * d->M / d->nc_chk);
+    for (int m = m0; m < m1; ++m) c2v_check(d, v2c, c2v, m);
+    if (--u->latch_c[it.frame] == 0) {
+      u->latch_c[it.frame] = d->nc_chk;
+      for (int c = 0; c < d->nc_var; ++c) {
+        ldpc_item x = {it.frame, it.iter, (uint32_t)c, 0u};
+        orc_push(eng, 2, &x);
+        orc_push(eng, 3, &x);
+      }
+    }
+  } else {                   /* V2C / ProbVar chunk */
+    const int n0 = (int)((long long)it.chunk * d->N / d->nc_var), n1 = (int)((long long)(it.chunk + 1) * d->N / d->nc_var);
+    if (stage == 2) {
+      for (int n = n0; n < n1; ++n) v2c_var(d, L, c2v, v2c, n);
+    } else {
+      int err = 0;
+      for (int n = n0; n < n1; ++n) {
+        const float P = posterior(d, L, c2v, n);
+        err += P < 0.0f;
+        if ((int)it.iter == d->n_iter - 1) u->post[(size_t)it.frame * d->N + n] = P;
+      }
+      u->errors[(size_t)it.frame * d->n_iter + it.iter] += err;
+    }
+    if (--u->latch_v[it.frame] == 0) {
+      u->latch_v[it.frame] = 2 * d->nc_var;
+      if ((int)it.iter + 1 < d->n_iter)
+        for (int c = 0; c < d->nc_chk; ++c) {
+          ldpc_item x = {it.frame, it.iter + 1u, (uint32_t)c, 0u};
+          orc_push(eng, 1, &x);  /* inner loop back to C2V */
+        }
     }
   }
 }
 
 int orc_ldpc_pipeline(const orc_ldpc* d, float* post, int32_t* errors, orc_stats* st) {
-  if (check_desc(d)) return 1;
+  if (check_desc(d) || d->nc_chk < 1 || d->nc_var < 1 || d->nc_chk > d->M || d->nc_var > d->N) return 1;
   const size_t E = (size_t)d->N * d->dv;
   ldpc_user u = {d, (float*)malloc(E * d->n_frames * sizeof(float)), (float*)malloc(E * d->n_frames * sizeof(float)),
-                 post, errors};
-  if (!u.v2c || !u.c2v) { free(u.v2c); free(u.c2v); return 1; }
+                 post, errors, (int32_t*)malloc(sizeof(int32_t) * d->n_frames), (int32_t*)malloc(sizeof(int32_t) * d->n_frames)};
+  if (!u.v2c || !u.c2v || !u.latch_c || !u.latch_v) {
+    free(u.v2c); free(u.c2v); free(u.latch_c); free(u.latch_v);
+    return 1;
+  }
+  memset(errors, 0, sizeof(int32_t) * (size_t)d->n_frames * d->n_iter);
+  for (int f = 0; f < d->n_frames; ++f) {
+    u.latch_c[f] = d->nc_chk;
+    u.latch_v[f] = 2 * d->nc_var;
+  }
   size_t strides[4] = {16, 16, 16, 16};
   orc_engine e;
   orc_engine_init(&e, 4, strides, ldpc_exec, &u);
@@ -156,5 +186,7 @@ int orc_ldpc_pipeline(const orc_ldpc* d, float* post, int32_t* errors, orc_stats
   orc_engine_free(&e);
   free(u.v2c);
   free(u.c2v);
+  free(u.latch_c);
+  free(u.latch_v);
   return rc;
 }

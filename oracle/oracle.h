@@ -66,6 +66,7 @@ int orc_toy_pipeline(const int32_t* in, size_t n, int32_t threshold, int32_t* ou
 typedef struct orc_ldpc {
   int32_t N, M, dv, dc, n_frames, n_iter;
   float alpha;            /* min-sum normalisation                               */
+  int32_t nc_chk, nc_var;   /* pipeline items: check chunks, variable chunks (R-L6) */
   int32_t pad;
   const int32_t* check_vars; /* [M*dc] variable node of each edge (check-major)  */
   const int32_t* var_edges;  /* [N*dv] edges of each variable node, ascending    */

@@ -451,6 +451,15 @@ class LdpcScene:
     def n_frames(self) -> int:
         return self.llr.shape[0]
 
+    # pipeline decomposition (reading R-L6): chunks of <= 256 checks / variables, <= 16 each
+    @property
+    def nc_chk(self) -> int:
+        return min(16, (self.M + 255) // 256)
+
+    @property
+    def nc_var(self) -> int:
+        return min(16, (self.N + 255) // 256)
+
 
 def ldpc_regular_h(N: int, dv: int, dc: int, seed: int) -> np.ndarray:
     """Socket-permutation (configuration-model) construction of a (dv, dc)-regular H:

@@ -99,8 +99,9 @@ class ToyParams(C.Structure):
 
 class LdpcParams(C.Structure):
     _fields_ = [("N", C.c_int32), ("M", C.c_int32), ("dv", C.c_int32), ("dc", C.c_int32), ("n_frames", C.c_int32),
-                ("n_iter", C.c_int32), ("alpha", C.c_float), ("pad", C.c_int32), ("check_vars", P), ("var_edges", P),
-                ("llr", P), ("v2c", P), ("c2v", P), ("post", P), ("errors", P)]
+                ("n_iter", C.c_int32), ("alpha", C.c_float), ("nc_chk", C.c_int32), ("nc_var", C.c_int32),
+                ("pad", C.c_int32), ("check_vars", P), ("var_edges", P), ("llr", P), ("v2c", P), ("c2v", P), ("post", P),
+                ("errors", P), ("latch", P)]
 
 
 class QBenchParams(C.Structure):

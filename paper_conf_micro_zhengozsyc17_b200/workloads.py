@@ -89,10 +89,12 @@ class LdpcPipeline:
         self.c2v = torch.empty((nf, E), dtype=torch.float32, device=dev)
         self.post = torch.empty((nf, scene.N), dtype=torch.float32, device=dev)
         self.errors = torch.zeros((nf, scene.n_iter), dtype=torch.int32, device=dev)
+        self.latch = torch.zeros((nf, 2), dtype=torch.int32, device=dev)
         self.prm = vp.LdpcParams(N=scene.N, M=scene.M, dv=scene.dv, dc=scene.dc, n_frames=nf, n_iter=scene.n_iter,
-                                 alpha=scene.alpha, check_vars=self.cv.data_ptr(), var_edges=self.ve.data_ptr(),
+                                 alpha=scene.alpha, nc_chk=scene.nc_chk, nc_var=scene.nc_var,
+                                 check_vars=self.cv.data_ptr(), var_edges=self.ve.data_ptr(),
                                  llr=self.llr.data_ptr(), v2c=self.v2c.data_ptr(), c2v=self.c2v.data_ptr(),
-                                 post=self.post.data_ptr(), errors=self.errors.data_ptr())
+                                 post=self.post.data_ptr(), errors=self.errors.data_ptr(), latch=self.latch.data_ptr())
         self.p = vp.Pipeline(device, **kw)
         for kind in (vp.LDPC_INIT, vp.LDPC_C2V, vp.LDPC_V2C, vp.LDPC_PROBVAR):
             self.p.register(kind, 16, self.prm)

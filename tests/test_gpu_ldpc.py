@@ -1,7 +1,7 @@
 """GPU parity for the LDPC decoder (Fig. 17, L59): posteriors,
-per-iteration bit-error counts and stage counts bit-exact against the CPU oracle under
-every execution model, including the paper's hybrid ([Initialize, C2V] fine | [V2C] |
-[ProbVar]) and the full 100 frames x 100 iterations."""
+per-iteration bit-error counts and stage counts (chunked items, reading R-L6) bit-exact
+against the CPU oracle under every execution model, including the paper's hybrid
+([Initialize, C2V] fine | [V2C] | [ProbVar]) and the full 100 frames x 100 iterations."""
 import numpy as np
 import pytest
 
@@ -27,8 +27,8 @@ def configure(vp, lp, model):
     elif model == "hybrid_paper":   # L59: Initialize and C2V in a fine group, V2C and ProbVar megakernels
         lp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_FINE, 0, 60), (2, 2, vp.GROUP_MEGA, 60, 104),
                                                  (3, 3, vp.GROUP_MEGA, 104, nsm)], nsm))
-    elif model == "hybrid_rtc":     # [Initialize, C2V, V2C] RTC (linear inside) | [ProbVar] megakernel
-        lp.configure(vp.HYBRID, vp.make_binding([(0, 2, vp.GROUP_RTC, 0, 100), (3, 3, vp.GROUP_MEGA, 100, nsm)], nsm))
+    elif model == "hybrid_rtc":     # [Initialize] RTC | [C2V, V2C, ProbVar] megakernel
+        lp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_RTC, 0, 20), (1, 3, vp.GROUP_MEGA, 20, nsm)], nsm))
     else:
         raise ValueError(model)
 

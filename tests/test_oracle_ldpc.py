@@ -105,11 +105,24 @@ def test_noiseless_closed_form_recursion():
         assert np.all(r["post"] == np.float32(P)) and not r["errors"].any()
 
 
+@pytest.mark.parametrize("N", [1024, 2048])
+def test_pipeline_chunking_is_exact(N):
+    """Chunked items with latches reproduce the per-frame definition for every chunking."""
+    sc = inputs.ldpc_scene(n_frames=3, N=N, n_iter=6)
+    a = oracle.ldpc_definition(sc)
+    b = oracle.ldpc_pipeline(sc)
+    assert np.array_equal(a["post"], b["post"]) and np.array_equal(a["errors"], b["errors"])
+    assert b["deq"] == [3, 3 * 6 * sc.nc_chk, 3 * 6 * sc.nc_var, 3 * 6 * sc.nc_var]
+
+
 def test_definition_equals_pipeline_and_counts():
     sc = inputs.ldpc_scene(n_frames=5, N=1024, n_iter=15)
     a = oracle.ldpc_definition(sc)
     b = oracle.ldpc_pipeline(sc)
     assert np.array_equal(a["post"], b["post"]) and np.array_equal(a["errors"], b["errors"])
-    assert b["deq"] == [5, 5 * 15, 5 * 15, 5 * 15]
+    # items (reading R-L6): Initialize per frame, then per iteration nc_chk C2V chunks and
+    # nc_var V2C + nc_var ProbVar chunks (chunks of <= 256 checks / variables)
+    assert (sc.nc_chk, sc.nc_var) == (2, 4)
+    assert b["deq"] == [5, 5 * 15 * 2, 5 * 15 * 4, 5 * 15 * 4]
     # the decoder converges on this channel (errors reach 0 for every frame)
     assert not a["errors"][:, -1].any() and a["errors"][:, 0].sum() > 0
