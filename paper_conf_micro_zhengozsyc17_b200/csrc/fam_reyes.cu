@@ -267,14 +267,31 @@ struct ReyesF {
   // Bound of patch P by one 16-thread group (lane = its control point; both groups of a
   // warp call together, `valid` may differ): returns 0 cull, 1 split, 2 dice (readings
   // R-R2..R-R5), the split direction, and this thread's control point q.
+  // Mc / mframe: a shared-memory copy of one frame's matrix (block-local recursion: the
+  // patches of a batch and their children almost always share the frame)
   static __device__ __forceinline__ int bound_patch(const Params& p, const RPatch* P, int lane, bool valid, int& dir,
-                                                    float4& q) {
+                                                    float4& q, const float4* Mc = nullptr, uint32_t mframe = ~0u) {
     const uint32_t depth = P->depth;
     uint32_t frame = P->id >> 12;
     if (frame >= (uint32_t)p.n_frames) frame = 0;
     const float* M = p.M + 16 * (size_t)frame;
     q = P->cp[lane];
-    float4 c = project(M, q.x, q.y, q.z, q.w);
+    float4 c;
+    if (Mc && frame == mframe) {
+      float cc[4];
+#pragma unroll
+      for (int r = 0; r < 4; ++r) {  // project() with the rows from shared memory (same op order)
+        const float4 m = Mc[r];
+        float acc = m.x * q.x;
+        acc = acc + m.y * q.y;
+        acc = acc + m.z * q.z;
+        acc = acc + m.w * q.w;
+        cc[r] = acc;
+      }
+      c = make_float4(cc[0], cc[1], cc[2], cc[3]);
+    } else {
+      c = project(M, q.x, q.y, q.z, q.w);
+    }
     const bool behind = !(c.w > p.near_w);
     const unsigned bal = __ballot_sync(0xffffffffu, behind);
     const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
@@ -432,7 +449,9 @@ struct ReyesF {
   static constexpr int kStack = VP_BS_STACK, kLocalDice = VP_BS_DICE;
   struct LocalStack {
     RPatch st[kStack];
+    float4 M[4];        // the batch's frame matrix rows
     int nchild[2], nsplit, dump;
+    uint32_t mframe;
   };
   static constexpr bool local_recursion(int lo, int hi) { return lo == BOUND && hi >= SPLIT; }
   static constexpr int local_out_cap(int, int hi, int t) {
@@ -467,6 +486,12 @@ struct ReyesF {
       }
     }
     if (threadIdx.x == 0) ls.nchild[0] = ls.nchild[1] = ls.nsplit = 0;
+    {
+      uint32_t frame = ((const RPatch*)items)->id >> 12;
+      if (frame >= (uint32_t)p.n_frames) frame = 0;
+      if (threadIdx.x < 16) ((float*)ls.M)[threadIdx.x] = __ldg(p.M + 16 * (size_t)frame + threadIdx.x);
+      if (threadIdx.x == 0) ls.mframe = frame;
+    }
     worker_sync();
     int top = (SS == BOUND) ? n : 2 * n, nbound = 0;
     bool first = SS == BOUND;  // the first pass pops exactly the claimed Bound items (n <= 16)
@@ -479,7 +504,7 @@ struct ReyesF {
       const RPatch* P = &ls.st[base + (mine ? grp : 0)];
       int dir;
       float4 q;
-      const int cls = bound_patch(p, P, lane, mine, dir, q);
+      const int cls = bound_patch(p, P, lane, mine, dir, q, ls.M, ls.mframe);
       const uint32_t id = P->id, path = P->path, dirs = P->dirs, depth = P->depth;
       float4 L, R;
       int my = 0;

@@ -1,4 +1,4 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 600 python -m pytest tests/test_gpu_tuner.py tests/test_gpu_basic.py -q > gpurun_out/pt.log 2>&1
-timeout 1200 python tools/suite_only.py > gpurun_out/suite.json 2> gpurun_out/suite.err
+timeout 600 python tools/reyes_sweep.py --reps 3 --no-timers --configs h52b16_16_64_4,h56b16_16_64_4,h60b16_16_64_4 > gpurun_out/sweep12.log 2>&1
+timeout 600 python -m pytest tests/test_gpu_reyes.py -q > gpurun_out/pr.log 2>&1
