@@ -1,3 +1,2 @@
 mkdir -p gpurun_out
-python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-timeout 900 python tools/reyes_sweep.py --reps 3 --no-timers --configs h56b16_16_64_4,h57b16_16_64_4,h58b16_16_64_4,h59b16_16_64_4,h60b16_16_64_4,h58b16_16_48_4,h58b16_16_32_4,h58b8_16_64_4,h58b16_8_64_4 > gpurun_out/sweep13.log 2>&1
+for lib in libvp.so libvp_r2.so; do echo "== $lib"; VP_LIB_NAME=$lib timeout 600 python tools/reyes_sweep.py --reps 3 --no-timers --configs h50b16_16_64_4,h54b16_16_64_4,h58b16_16_64_4,h62b16_16_64_4; done > gpurun_out/sweep14.log 2>&1
