@@ -207,7 +207,7 @@ __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, lo
 struct ChainScratch {
   float4 M[kWarpsW][4];        // per-warp copy of the patch's frame matrix (rows)
   float B[kWarpsW][36];        // per-warp Bernstein table B_b(j/8), [9][4]
-  uint8_t list[kWarpsW][64];   // per-warp compacted list of pixel-covering micropolygons
+  uint8_t list[kWarpsW][128];  // per-warp compacted list of pixel-covering micropolygons (q | grid << 6)
 };
 
 struct ReyesF {
@@ -820,7 +820,6 @@ struct ReyesF {
     const Params& p = ctx.params();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     ChainScratch& cs = *(ChainScratch*)ctx.scratch();
-    RGrid* g = (RGrid*)ctx.template out_ptr<SHADE>(warp);
     float* Mw = (float*)cs.M[warp];
     uint8_t* list = cs.list[warp];
     // Patches are handed out dynamically: shade work per patch varies with its size on
@@ -833,28 +832,47 @@ struct ReyesF {
       bernstein((float)(e >> 2) * 0.125f, B4);
       Bt[e] = B4[e & 3];
     }
+    // Two grids per warp: its grid slot in both out buffers (no other warp uses slot
+    // `warp`, and the publisher never reads Shade slots of a fused chain).  Patches are
+    // diced in pairs and the pixel-covering micropolygons of both are shaded in one pass:
+    // at config 5 about a quarter of a grid's 64 micropolygons cover a pixel centre, so one
+    // grid alone fills only half of the warp's shading lanes.
+    RGrid* const g0 = (RGrid*)ctx.template out_ptr_in<SHADE>(0, warp);
+    RGrid* const g1 = (RGrid*)ctx.template out_ptr_in<SHADE>(1, warp);
     for (;;) {
       int k = 0;
-      if (lane == 0) k = atomicAdd(next, 1);
+      if (lane == 0) k = atomicAdd(next, 2);
       k = __shfl_sync(0xffffffffu, k, 0);
       if (k >= n) break;
-      const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
-      uint32_t frame = P->id >> 12;
-      if (frame >= (uint32_t)p.n_frames) frame = 0;
-      if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+      const int np = min(2, n - k);
+      int tot = 0;
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        if (j >= np) break;
+        RGrid* g = j ? g1 : g0;
+        const RPatch* P = (const RPatch*)(items + (size_t)(k + j) * sizeof(RPatch));
+        uint32_t frame = P->id >> 12;
+        if (frame >= (uint32_t)p.n_frames) frame = 0;
+        __syncwarp();  // the previous patch's dice is done with the matrix
+        if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+        __syncwarp();
+        dice_patch<true>(p, P, g, lane, cs.M[warp], Bt);
+        __syncwarp();
+        if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
+        const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
+        const unsigned m0 = __ballot_sync(0xffffffffu, a0), m1 = __ballot_sync(0xffffffffu, a1);
+        const unsigned lt = (1u << lane) - 1u;
+        const int c0 = __popc(m0);
+        if (a0) list[tot + __popc(m0 & lt)] = (uint8_t)(lane | (j << 6));
+        if (a1) list[tot + c0 + __popc(m1 & lt)] = (uint8_t)((lane + 32) | (j << 6));
+        tot += c0 + __popc(m1);
+      }
       __syncwarp();
-      dice_patch<true>(p, P, g, lane, cs.M[warp], Bt);
-      __syncwarp();
-      if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
-      const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
-      const unsigned m0 = __ballot_sync(0xffffffffu, a0), m1 = __ballot_sync(0xffffffffu, a1);
-      const unsigned lt = (1u << lane) - 1u;
-      const int c0 = __popc(m0), tot = c0 + __popc(m1);
-      if (a0) list[__popc(m0 & lt)] = (uint8_t)lane;
-      if (a1) list[c0 + __popc(m1 & lt)] = (uint8_t)(lane + 32);
-      __syncwarp();
-      for (int t = lane; t < tot; t += 32) shade_mp(p, g, list[t]);
-      __syncwarp();  // the slot, the matrix and the list are rewritten next
+      for (int t = lane; t < tot; t += 32) {
+        const int e = list[t];
+        shade_mp(p, (e >> 6) ? g1 : g0, e & 63);
+      }
+      __syncwarp();  // the slots, the matrix and the list are rewritten next
     }
   }
 

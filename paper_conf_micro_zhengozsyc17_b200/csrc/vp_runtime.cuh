@@ -425,6 +425,11 @@ struct Ctx {
   }
   template <int T>
   static constexpr int cap() { return OutT<T>::cap; }
+  // out slot of target T in out buffer b (either buffer, independent of the current one)
+  template <int T>
+  __device__ __forceinline__ uint8_t* out_ptr_in(int b, int slot) {
+    return smem + kOutBase0 + b * kOutRegion + OutT<T>::off + slot * F::stride(T);
+  }
 
   // Reserve k consecutive out slots for target T (one thread).  The declared fan-out
   // bounds guarantee capacity; exceeding it aborts the run (ABORT_FANOUT).
