@@ -233,9 +233,13 @@ struct ReyesF {
   static constexpr bool rtc_ok(int, int) { return true; }
   // every kernel whose range ends in [Dice, Shade] may run the fused chain (an RTC
   // kernel [Split..Shade] fuses its Dice batches too), so each reserves the chain scratch
-  static constexpr int scratch_bytes(int lo, int hi) {
-    return ((lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
-           ((lo == BOUND && hi >= SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
+  static constexpr int scratch_bytes(int lo, int hi) { return scratch_bytes_k(lo, hi, true); }
+  // the fused [Dice, Shade] chain runs only in RTC kernels; block-local recursion only in
+  // non-RTC ones (a megakernel [Bound..Shade] must not pay for the chain's scratch: it sits
+  // at the edge of 2 blocks per SM)
+  static constexpr int scratch_bytes_k(int lo, int hi, bool rtc) {
+    return ((rtc && lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
+           ((!rtc && lo == BOUND && hi >= SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
   }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM

@@ -275,6 +275,18 @@ constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
   if constexpr (HasKernelMaxBatch<F>::value) return F::kernel_max_batch(lo, hi, rtc, s);
   else return F::max_batch(s);
 }
+// A family may size its shared-memory scratch per kernel kind (F::scratch_bytes_k(lo, hi,
+// rtc)), e.g. scratch only an RTC chain uses; default F::scratch_bytes(lo, hi).
+template <class F, class = void>
+struct HasScratchK : std::false_type {};
+template <class F>
+struct HasScratchK<F, std::void_t<decltype(F::scratch_bytes_k(0, 0, false))>> : std::true_type {};
+template <class F>
+constexpr int scratch_of(int lo, int hi, bool rtc) {
+  if constexpr (HasScratchK<F>::value) return F::scratch_bytes_k(lo, hi, rtc);
+  else return F::scratch_bytes(lo, hi);
+}
+
 template <class F>
 constexpr int fused_local_cap(int lo, int hi, int t) {
   if constexpr (HasFusedRtc<F>::value) return F::fused_local_cap(lo, hi, t);
@@ -368,7 +380,7 @@ struct Graph {
   static constexpr int in_base(int lo, int hi, bool rtc, int b) { return b * in_region(lo, hi, rtc); }
   static constexpr int out_base(int lo, int hi, bool rtc, int b) { return 2 * in_region(lo, hi, rtc) + b * out_region(lo, hi, rtc); }
   static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_base(lo, hi, rtc, 2); }
-  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + F::scratch_bytes(lo, hi); }
+  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + scratch_of<F>(lo, hi, rtc); }
 };
 
 // ------------------------------------------------------------------ per-block context
@@ -1186,8 +1198,8 @@ struct Runner {
           mbar_init(&sh.empty[b], kWarpsW);
         }
       }
-      if constexpr (F::scratch_bytes(LO, HI) > 0) {
-        for (int i = threadIdx.x; i < F::scratch_bytes(LO, HI) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+      if constexpr (scratch_of<F>(LO, HI, RTC) > 0) {
+        for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
       }
       __syncthreads();
       run_sink(a, ctx, sh, smem);
@@ -1195,8 +1207,8 @@ struct Runner {
       flush_stats(a, sh);
       return;
     }
-    if constexpr (F::scratch_bytes(LO, HI) > 0) {  // family scratch starts zeroed
-      for (int i = threadIdx.x; i < F::scratch_bytes(LO, HI) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+    if constexpr (scratch_of<F>(LO, HI, RTC) > 0) {  // family scratch starts zeroed
+      for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // prologue: stage the first batch into in[0]
