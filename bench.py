@@ -91,6 +91,19 @@ class Clocks:
         except Exception:
             self.p = None
 
+    def wait_ready(self, timeout_s=3.0):
+        """Block until nvidia-smi has written its first sample, so the timed region that
+        follows is actually sampled (the tool takes ~100 ms to start)."""
+        t0 = time.time()
+        while self.p and time.time() - t0 < timeout_s:
+            self.f.flush()
+            try:
+                if os.path.getsize(self.path) > 0:
+                    return
+            except OSError:
+                pass
+            time.sleep(0.01)
+
     def stop(self):
         if not self.p:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
@@ -382,6 +395,7 @@ def main():
     # ---- timed region: inputs resident in HBM (seeds 4096 x 272 B per frame > L2)
     barrier()
     clk = Clocks(local)
+    clk.wait_ready()
     t_ms, st, kms = time_steps(torch, rp, args.steps, stream)
     barrier()
     clocks = clk.stop()
