@@ -458,8 +458,11 @@ def main():
                 dist.all_reduce(bt_t, op=dist.ReduceOp.MAX)
             extra[name] = {"ms_per_step": float(bt_t.item()) / max(1, min(args.steps, 3)),
                            "launches_per_step": int(bst["kbk_launches"])}
-            if name == "kbk_graph":  # + one planner per wave and one loop-condition kernel per iteration
-                extra[name]["launches_per_step"] = int(bst["kbk_launches"]) * 2 + int(bst["kbk_launches"]) // 4
+            if name == "kbk_graph":
+                # kbk_launches = graph iterations x S wave kernels; each iteration also runs S
+                # planner kernels and one loop-condition kernel
+                n_st = 4  # Reyes stages
+                extra[name]["launches_per_step"] = 2 * int(bst["kbk_launches"]) + int(bst["kbk_launches"]) // n_st
         rp.p.configure_config(main_cfg)
 
     # ---- e2e through the public API with HOST buffers: H2D seeds + run + D2H colours
