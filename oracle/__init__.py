@@ -284,7 +284,8 @@ REYES_CULL, REYES_SPLIT, REYES_DICE = 0, 1, 2
 
 # ------------------------------------------------------------------ Rasterization
 class RasterSceneC(C.Structure):
-    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P)]
+    _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P),
+                ("near_clip", C.c_int32)]
 
 
 class RasterOutC(C.Structure):
@@ -301,7 +302,7 @@ def _raster_run(fname, scene, trace_cap=0):
     pos = np.ascontiguousarray(scene.pos, np.float32)
     col = np.ascontiguousarray(scene.col, np.float32)
     sc = RasterSceneC(W=scene.W, H=scene.H, n_tris=pos.shape[0], M=M.ctypes.data, pos=pos.ctypes.data,
-                      col=col.ctypes.data)
+                      col=col.ctypes.data, near_clip=int(getattr(scene, "near_clip", 0)))
     npix = scene.W * scene.H
     key = np.empty(npix, np.uint64)
     colour = np.empty((npix, 4), np.float32)

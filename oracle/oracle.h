@@ -134,6 +134,7 @@ typedef struct orc_raster_scene {
   const float* M;   /* [16] row-major                                   */
   const float* pos; /* [n_tris][3][4] (x_px, y_px, z, 1)                 */
   const float* col; /* [n_tris][3][4] (r, g, b, 0)                       */
+  int32_t near_clip; /* 1: clip against z = 0, keys carry sub-ids 2 tri + j (R-S9) */
 } orc_raster_scene;
 
 typedef struct orc_raster_out {

@@ -20,6 +20,14 @@
  *                 l1 = E(v2,v0,P)/area2, l2 = E(v0,v1,P)/area2; z = (l0 z0 + l1 z1) + l2 z2;
  *                 discard unless 0 <= z <= 1; keep min key (zkey(z) << 32 | tri).
  *  Resolve:       colour = (l0 c0 + l1 c1) + l2 c2 of the winning triangle, alpha 1.
+ *
+ *  Near-plane clipping (sc->near_clip != 0, reading R-S9 of DESIGN.md
+ *  §2): after the trivial reject, a triangle with a vertex at z < 0 is clipped against
+ *  the plane z = 0 by Sutherland-Hodgman (edges v0v1, v1v2, v2v0 in order: keep a vertex
+ *  with z >= 0; where an edge changes side, t = za / (za - zb) and every clip coordinate
+ *  and colour channel is a + t (b - a), z set to exactly 0).  The 3- or 4-gon (p0..pn-1)
+ *  fans into triangles (p0, p(j+1), p(j+2)), j = 0..n-3, each set up as above under the
+ *  sub-triangle id 2 tri + j, which replaces tri in the depth key.  Clip's fan-out is 0..2.
  */
 #include <math.h>
 #include <stdlib.h>
@@ -33,6 +41,7 @@ typedef struct rsetup {
   int32_t vi[3]; /* vertex order after orientation normalisation */
   int64_t area;
   int32_t px0, px1, py0, py1;
+  float c[3][4]; /* near-clip mode: vertex colours in setup order */
 } rsetup;
 
 static uint32_t r_zkey(float z) {
@@ -130,6 +139,60 @@ static int clip_setup(const orc_raster_scene* sc, const float clip[3][4], rsetup
   return 1;
 }
 
+/* Near-plane clip (R-S9): polygon of the triangle clipped against z >= 0, fanned into
+ * sub-triangles 2 tri + j.  Returns the number of surviving sub-triangles; alive[j] set. */
+static int near_clip_setup(const orc_raster_scene* sc, uint32_t tri, const float clip[3][4], rsetup s[2],
+                           int alive[2]) {
+  alive[0] = alive[1] = 0;
+  int out[6] = {1, 1, 1, 1, 1, 1};
+  for (int k = 0; k < 3; ++k) {
+    float x = clip[k][0], y = clip[k][1], z = clip[k][2], w = clip[k][3];
+    out[0] &= x < -w;
+    out[1] &= x > w;
+    out[2] &= y < -w;
+    out[3] &= y > w;
+    out[4] &= z < 0.0f;
+    out[5] &= z > w;
+  }
+  for (int i = 0; i < 6; ++i)
+    if (out[i]) return 0;
+  const float* col = sc->col + 12 * (size_t)tri;
+  float P[4][4], C[4][4];
+  int n = 0;
+  for (int k = 0; k < 3; ++k) {
+    const float* a = clip[k];
+    const float* b = clip[(k + 1) % 3];
+    const float* ca = col + 4 * k;
+    const float* cb = col + 4 * ((k + 1) % 3);
+    int ina = a[2] >= 0.0f, inb = b[2] >= 0.0f;
+    if (ina) {
+      memcpy(P[n], a, sizeof(float[4]));
+      memcpy(C[n], ca, sizeof(float[4]));
+      ++n;
+    }
+    if (ina != inb) {
+      float t = a[2] / (a[2] - b[2]);
+      for (int r = 0; r < 4; ++r) {
+        P[n][r] = a[r] + t * (b[r] - a[r]);
+        C[n][r] = ca[r] + t * (cb[r] - ca[r]);
+      }
+      P[n][2] = 0.0f;
+      ++n;
+    }
+  }
+  int m = 0;
+  for (int j = 0; j + 2 < n; ++j) {
+    int idx[3] = {0, j + 1, j + 2};
+    float v[3][4];
+    for (int k = 0; k < 3; ++k) memcpy(v[k], P[idx[k]], sizeof(float[4]));
+    if (!clip_setup(sc, (const float(*)[4])v, &s[j])) continue;
+    for (int k = 0; k < 3; ++k) memcpy(s[j].c[k], C[idx[s[j].vi[k]]], sizeof(float[4]));
+    alive[j] = 1;
+    ++m;
+  }
+  return m;
+}
+
 /* Raster stage: does any edge reject the tile (all 4 corner samples strictly outside)? */
 static int tile_rejected(const rsetup* s, int tx, int ty) {
   int64_t x0 = tx * 8, x1 = tx * 8 + 7, y0 = ty * 8, y1 = ty * 8 + 7;
@@ -194,17 +257,20 @@ static void raster_resolve(const orc_raster_scene* sc, const rsetup* setups, con
         c[0] = c[1] = c[2] = c[3] = 0.0f;
         continue;
       }
-      uint32_t tri = (uint32_t)(out->key[p] & 0xFFFFFFFFu);
+      uint32_t tri = (uint32_t)(out->key[p] & 0xFFFFFFFFu); /* sub-triangle id in near-clip mode */
       const rsetup* s = &setups[tri];
       float l[3] = {0, 0, 0};
       if (!alive[tri] || !frag_weights(s, px, py, l)) { /* cannot happen */
         c[0] = c[1] = c[2] = c[3] = -1.0f;
         continue;
       }
-      const float* col = sc->col + 12 * (size_t)tri;
+      float cv[3][4];
+      for (int k = 0; k < 3; ++k)
+        for (int ch = 0; ch < 4; ++ch)
+          cv[k][ch] = sc->near_clip ? s->c[k][ch] : sc->col[12 * (size_t)tri + 4 * s->vi[k] + ch];
       for (int ch = 0; ch < 3; ++ch) {
-        float v = l[0] * col[4 * s->vi[0] + ch] + l[1] * col[4 * s->vi[1] + ch];
-        v = v + l[2] * col[4 * s->vi[2] + ch];
+        float v = l[0] * cv[0][ch] + l[1] * cv[1][ch];
+        v = v + l[2] * cv[2][ch];
         c[ch] = v;
       }
       c[3] = 1.0f;
@@ -220,24 +286,36 @@ static void raster_out_reset(const orc_raster_scene* sc, orc_raster_out* out) {
 /* ---------- definition oracle: per-triangle loop into a z-buffer ---------- */
 int orc_raster_definition(const orc_raster_scene* sc, orc_raster_out* out) {
   raster_out_reset(sc, out);
-  rsetup* setups = (rsetup*)calloc((size_t)sc->n_tris, sizeof(rsetup));
-  uint8_t* alive = (uint8_t*)calloc((size_t)sc->n_tris, 1);
+  const size_t nsub = (size_t)sc->n_tris * (sc->near_clip ? 2 : 1);
+  rsetup* setups = (rsetup*)calloc(nsub, sizeof(rsetup));
+  uint8_t* alive = (uint8_t*)calloc(nsub, 1);
   if (!setups || !alive) return 1;
   for (int64_t t = 0; t < sc->n_tris; ++t) {
     float clip[3][4];
     out->n_vertex++;
     orc_raster_vertex(sc, (uint32_t)t, clip);
     out->n_clip++;
-    if (!clip_setup(sc, clip, &setups[t])) continue;
-    alive[t] = 1;
-    out->n_raster++;
-    const rsetup* s = &setups[t];
-    for (int ty = s->py0 >> 3; ty <= s->py1 >> 3; ++ty)
-      for (int tx = s->px0 >> 3; tx <= s->px1 >> 3; ++tx) {
-        if (tile_rejected(s, tx, ty)) continue;
-        out->n_fragment++;
-        fragment_tile(sc, (uint32_t)t, s, tx, ty, out);
-      }
+    uint32_t ids[2];
+    int m = 0;
+    if (sc->near_clip) {
+      int al[2];
+      near_clip_setup(sc, (uint32_t)t, clip, &setups[2 * t], al);
+      for (int j = 0; j < 2; ++j)
+        if (al[j]) alive[2 * t + j] = 1, ids[m++] = (uint32_t)(2 * t + j);
+    } else if (clip_setup(sc, clip, &setups[t])) {
+      alive[t] = 1;
+      ids[m++] = (uint32_t)t;
+    }
+    for (int i = 0; i < m; ++i) {
+      out->n_raster++;
+      const rsetup* s = &setups[ids[i]];
+      for (int ty = s->py0 >> 3; ty <= s->py1 >> 3; ++ty)
+        for (int tx = s->px0 >> 3; tx <= s->px1 >> 3; ++tx) {
+          if (tile_rejected(s, tx, ty)) continue;
+          out->n_fragment++;
+          fragment_tile(sc, ids[i], s, tx, ty, out);
+        }
+    }
   }
   raster_resolve(sc, setups, alive, out);
   free(setups);
@@ -264,7 +342,16 @@ static void raster_exec(orc_engine* e, int stage, const void* item) {
       orc_raster_vertex(u->sc, tri, u->clip[tri]);
       orc_push(e, 1, &tri);
     } else if (stage == 1) {
-      if (clip_setup(u->sc, (const float(*)[4])u->clip[tri], &u->setups[tri])) {
+      if (u->sc->near_clip) {
+        int al[2];
+        near_clip_setup(u->sc, tri, (const float(*)[4])u->clip[tri], &u->setups[2 * (size_t)tri], al);
+        for (int j = 0; j < 2; ++j)
+          if (al[j]) {
+            uint32_t sub = 2 * tri + (uint32_t)j;
+            u->alive[sub] = 1;
+            orc_push(e, 2, &sub);
+          }
+      } else if (clip_setup(u->sc, (const float(*)[4])u->clip[tri], &u->setups[tri])) {
         u->alive[tri] = 1;
         orc_push(e, 2, &tri);
       }
@@ -291,8 +378,9 @@ int orc_raster_pipeline(const orc_raster_scene* sc, orc_raster_out* out) {
   u.sc = sc;
   u.out = out;
   u.clip = (float(*)[3][4])calloc((size_t)sc->n_tris, sizeof(float[3][4]));
-  u.setups = (rsetup*)calloc((size_t)sc->n_tris, sizeof(rsetup));
-  u.alive = (uint8_t*)calloc((size_t)sc->n_tris, 1);
+  const size_t nsub = (size_t)sc->n_tris * (sc->near_clip ? 2 : 1);
+  u.setups = (rsetup*)calloc(nsub, sizeof(rsetup));
+  u.alive = (uint8_t*)calloc(nsub, 1);
   if (!u.clip || !u.setups || !u.alive) return 1;
   size_t strides[4] = {4, 4, 4, 8};
   orc_engine e;

@@ -215,6 +215,7 @@ class RasterScene:
     M: np.ndarray      # [16] float32 pixel -> NDC, w = 1
     pos: np.ndarray    # [n, 3, 4] float32 (x_px, y_px, z, 1)
     col: np.ndarray    # [n, 3, 4] float32 (r, g, b, 0)
+    near_clip: int = 0  # 1: clip against z = 0 (Clip fan-out 0..2, keys carry 2 tri + j; R-S9)
 
     @property
     def n_tris(self):
@@ -256,6 +257,18 @@ def raster_scene(n: int = 1 << 20, W: int = 1920, H: int = 1080, seed: int = see
     col = np.zeros((n, 3, 4), np.float32)
     col[:, :, :3] = u[:, 8:17].reshape(n, 3, 3)
     return RasterScene(W=W, H=H, M=pixel_to_ndc(W, H), pos=pos, col=col)
+
+
+def raster_near_scene(n: int = 4096, W: int = 256, H: int = 192, seed: int = seed_for(4) + 17,
+                      z_range=(-0.6, 0.95), area_range=(4.0, 2048.0)) -> RasterScene:
+    """Near-plane clipping workload (DESIGN R-S9): the config-4 recipe with
+    per-vertex z ~ U(z_range), so about half the triangles straddle z = 0 (one or two
+    vertices behind the near plane) and a few lie wholly behind it; near_clip = 1."""
+    sc = raster_scene(n=n, W=W, H=H, seed=seed, area_range=area_range)
+    u = uniform01(seed ^ 0x5A5A, n * 3).reshape(n, 3)
+    sc.pos[:, :, 2] = (z_range[0] + (z_range[1] - z_range[0]) * u).astype(np.float32)
+    sc.near_clip = 1
+    return sc
 
 
 def raster_quad_mesh(W: int, H: int, cell: int = 8, z: float = 0.5) -> RasterScene:
