@@ -283,6 +283,13 @@ typedef struct vp_raster_params {
   void* setup;               /* [n_tris] x 128 B scratch (per-triangle setup), 128-B aligned */
   unsigned long long* fb;    /* [H*W] depth keys (zkey(z) << 32 | tri), reset by vp_run    */
   float* colour;             /* [H*W][4] resolved colour, written by vp_run                */
+  int32_t near_clip;         /* 0: cull triangles with a vertex at w <= 1e-6 (keys carry tri);  */
+                             /* 1: clip against z = 0 first (DESIGN R-S9):      */
+                             /*    Clip emits 0..2 sub-triangles 2 tri + j, keys carry that id, */
+                             /*    setup must hold 2 n_tris records                              */
+  int32_t pad0;
+  float* ccol;               /* near_clip: [2 n_tris][3][4] sub-triangle vertex colours (scratch, */
+                             /* 16-B aligned, written by Clip); ignored when near_clip == 0      */
 } vp_raster_params;
 
 typedef struct vp_pyramid_params {

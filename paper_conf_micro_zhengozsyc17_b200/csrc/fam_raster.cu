@@ -88,6 +88,9 @@ __device__ __forceinline__ bool frag_weights(const RSetup& s, int px, int py, fl
 
 struct RasterF {
   static constexpr int S = 4;
+  static __host__ __device__ __forceinline__ unsigned long long n_setups(const vp_raster_params& p) {
+    return (unsigned long long)p.n_tris << (p.near_clip ? 1 : 0);
+  }
   static constexpr int VERTEX = 0, CLIP = 1, RASTER = 2, FRAGMENT = 3;
   static constexpr int kMaxTiles = 128;  // declared fan-out of Raster (10 x 10 for the generator's triangles)
   static constexpr int kinds[S] = {VP_RASTER_VERTEX, VP_RASTER_CLIP, VP_RASTER_RASTER, VP_RASTER_FRAGMENT};
@@ -96,7 +99,9 @@ struct RasterF {
   static constexpr int threads_per_item(int s) { return s == RASTER ? 32 : s == FRAGMENT ? 64 : 1; }
   static constexpr int max_batch(int s) { return s <= CLIP ? 256 : s == RASTER ? 32 : 32; }
   static constexpr int default_batch(int s) { return max_batch(s); }
-  static constexpr int fanout(int s, int t) { return (t == s + 1) ? (s == RASTER ? kMaxTiles : 1) : 0; }
+  static constexpr int fanout(int s, int t) {
+    return (t == s + 1) ? (s == RASTER ? kMaxTiles : s == CLIP ? 2 : 1) : 0;  // Clip: 0..2 (near clip)
+  }
   // RTC groups must not expand Raster's fan-out block-locally from more than one claimed
   // batch: Raster may only be the first stage of an RTC group.
   static constexpr bool rtc_ok(int lo, int hi) { return !(lo < RASTER && hi >= RASTER); }
@@ -143,10 +148,75 @@ struct RasterF {
           acc = acc + __ldg(p.M + 4 * r + 3) * x.w;
           c[r] = acc;
         }
-        setup[tri].clip[q] = make_float4(c[0], c[1], c[2], c[3]);
+        setup[p.near_clip ? 2 * (size_t)tri : tri].clip[q] = make_float4(c[0], c[1], c[2], c[3]);
       }
       ctx.template emit<CLIP>(&tri);
     }
+  }
+
+  // Setup of one (sub-)triangle from its clip coordinates (R-S2..R-S4): trivial reject,
+  // w cull, Q4 snap, orientation, pixel range.  Returns false if it is culled.
+  static __device__ __forceinline__ bool setup_one(const Params& p, const float4 c[3], RSetup& s) {
+    bool o0 = true, o1 = true, o2 = true, o3 = true, o4 = true, o5 = true;
+#pragma unroll
+    for (int q = 0; q < 3; ++q) {
+      o0 &= c[q].x < -c[q].w;
+      o1 &= c[q].x > c[q].w;
+      o2 &= c[q].y < -c[q].w;
+      o3 &= c[q].y > c[q].w;
+      o4 &= c[q].z < 0.0f;
+      o5 &= c[q].z > c[q].w;
+    }
+    if (o0 || o1 || o2 || o3 || o4 || o5) return false;  // trivial reject
+    if (!(c[0].w > 1e-6f) || !(c[1].w > 1e-6f) || !(c[2].w > 1e-6f)) return false;
+    long long X[3], Y[3];
+    float Z[3];
+    bool ok = true;
+#pragma unroll
+    for (int q = 0; q < 3; ++q) {
+      const float w = c[q].w;
+      const float sx = ((c[q].x / w) * 0.5f + 0.5f) * (float)p.W;
+      const float sy = ((c[q].y / w) * 0.5f + 0.5f) * (float)p.H;
+      const float fx = sx * 16.0f, fy = sy * 16.0f;
+      if (!(fabsf(fx) < 1073741824.0f) || !(fabsf(fy) < 1073741824.0f)) ok = false;
+      X[q] = __float2ll_rn(fx);
+      Y[q] = __float2ll_rn(fy);
+      Z[q] = c[q].z / w;
+    }
+    if (!ok) return false;
+    long long area = r_edge(X[0], Y[0], X[1], Y[1], X[2], Y[2]);
+    if (area == 0) return false;
+    int o[3] = {0, 1, 2};
+    if (area < 0) {
+      o[1] = 2;
+      o[2] = 1;
+      area = -area;
+    }
+    long long xmin = min(X[0], min(X[1], X[2])), xmax = max(X[0], max(X[1], X[2]));
+    long long ymin = min(Y[0], min(Y[1], Y[2])), ymax = max(Y[0], max(Y[1], Y[2]));
+    long long px0 = -((-(xmin - 8)) >> 4), px1 = (xmax - 8) >> 4;  // ceil / floor of (v - 8) / 16
+    long long py0 = -((-(ymin - 8)) >> 4), py1 = (ymax - 8) >> 4;
+    px0 = max(px0, 0ll);
+    py0 = max(py0, 0ll);
+    px1 = min(px1, (long long)p.W - 1);
+    py1 = min(py1, (long long)p.H - 1);
+    if (px0 > px1 || py0 > py1) return false;
+    int vi = 0;
+#pragma unroll
+    for (int q = 0; q < 3; ++q) {
+      const int src = q == 0 ? o[0] : q == 1 ? o[1] : o[2];
+      s.X[q] = (int)(src == 0 ? X[0] : src == 1 ? X[1] : X[2]);
+      s.Y[q] = (int)(src == 0 ? Y[0] : src == 1 ? Y[1] : Y[2]);
+      s.z[q] = src == 0 ? Z[0] : src == 1 ? Z[1] : Z[2];
+      vi |= src << (2 * q);
+    }
+    s.px0 = (int)px0;
+    s.px1 = (int)px1;
+    s.py0 = (int)py0;
+    s.py1 = (int)py1;
+    s.area = area;
+    s.vi = vi;
+    return true;
   }
 
   // ------------------------------------------------------------ Clip (1 thread/tri)
@@ -157,68 +227,60 @@ struct RasterF {
     for (int k = threadIdx.x; k < n; k += kThreads) {
       const uint32_t tri = ((const uint32_t*)items)[k];
       if (tri >= (uint32_t)p.n_tris) continue;
-      RSetup& s = setup[tri];
-      float4 c[3] = {s.clip[0], s.clip[1], s.clip[2]};
-      bool o0 = true, o1 = true, o2 = true, o3 = true, o4 = true, o5 = true;
+      if (!p.near_clip) {
+        RSetup& s = setup[tri];
+        const float4 c[3] = {s.clip[0], s.clip[1], s.clip[2]};
+        if (setup_one(p, c, s)) ctx.template emit<RASTER>(&tri);
+        continue;
+      }
+      // Near-plane clip (R-S9): Sutherland-Hodgman against z >= 0, fan into sub-triangles
+      // 2 tri + j.  Clip coordinates were left in setup[2 tri] by Vertex.
+      const float4 c[3] = {setup[2 * tri].clip[0], setup[2 * tri].clip[1], setup[2 * tri].clip[2]};
+      {
+        bool o0 = true, o1 = true, o2 = true, o3 = true, o4 = true, o5 = true;
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+          o0 &= c[q].x < -c[q].w;
+          o1 &= c[q].x > c[q].w;
+          o2 &= c[q].y < -c[q].w;
+          o3 &= c[q].y > c[q].w;
+          o4 &= c[q].z < 0.0f;
+          o5 &= c[q].z > c[q].w;
+        }
+        if (o0 || o1 || o2 || o3 || o4 || o5) continue;
+      }
+      const float4* col = (const float4*)p.col + 3 * (size_t)tri;
+      float4 P[4], Cc[4];
+      int np = 0;
 #pragma unroll
       for (int q = 0; q < 3; ++q) {
-        o0 &= c[q].x < -c[q].w;
-        o1 &= c[q].x > c[q].w;
-        o2 &= c[q].y < -c[q].w;
-        o3 &= c[q].y > c[q].w;
-        o4 &= c[q].z < 0.0f;
-        o5 &= c[q].z > c[q].w;
+        const float4 a = c[q], b = c[(q + 1) % 3];
+        const float4 ca = __ldg(col + q), cb = __ldg(col + (q + 1) % 3);
+        const bool ina = a.z >= 0.0f, inb = b.z >= 0.0f;
+        if (ina) {
+          P[np] = a;
+          Cc[np] = ca;
+          ++np;
+        }
+        if (ina != inb) {
+          const float t = a.z / (a.z - b.z);
+          P[np] = make_float4(a.x + t * (b.x - a.x), a.y + t * (b.y - a.y), 0.0f, a.w + t * (b.w - a.w));
+          Cc[np] = make_float4(ca.x + t * (cb.x - ca.x), ca.y + t * (cb.y - ca.y), ca.z + t * (cb.z - ca.z),
+                               ca.w + t * (cb.w - ca.w));
+          ++np;
+        }
       }
-      if (o0 || o1 || o2 || o3 || o4 || o5) continue;  // trivial reject
-      if (!(c[0].w > 1e-6f) || !(c[1].w > 1e-6f) || !(c[2].w > 1e-6f)) continue;
-      long long X[3], Y[3];
-      float Z[3];
-      bool ok = true;
+      float4* ccol = (float4*)p.ccol;
+      for (int j = 0; j + 2 < np; ++j) {
+        const int idx[3] = {0, j + 1, j + 2};
+        const float4 v[3] = {P[idx[0]], P[idx[1]], P[idx[2]]};
+        const uint32_t sub = 2 * tri + (uint32_t)j;
+        RSetup& s = setup[sub];
+        if (!setup_one(p, v, s)) continue;
 #pragma unroll
-      for (int q = 0; q < 3; ++q) {
-        const float w = c[q].w;
-        const float sx = ((c[q].x / w) * 0.5f + 0.5f) * (float)p.W;
-        const float sy = ((c[q].y / w) * 0.5f + 0.5f) * (float)p.H;
-        const float fx = sx * 16.0f, fy = sy * 16.0f;
-        if (!(fabsf(fx) < 1073741824.0f) || !(fabsf(fy) < 1073741824.0f)) ok = false;
-        X[q] = __float2ll_rn(fx);
-        Y[q] = __float2ll_rn(fy);
-        Z[q] = c[q].z / w;
+        for (int q = 0; q < 3; ++q) ccol[3 * (size_t)sub + q] = Cc[idx[(s.vi >> (2 * q)) & 3]];
+        ctx.template emit<RASTER>(&sub);
       }
-      if (!ok) continue;
-      long long area = r_edge(X[0], Y[0], X[1], Y[1], X[2], Y[2]);
-      if (area == 0) continue;
-      int o[3] = {0, 1, 2};
-      if (area < 0) {
-        o[1] = 2;
-        o[2] = 1;
-        area = -area;
-      }
-      long long xmin = min(X[0], min(X[1], X[2])), xmax = max(X[0], max(X[1], X[2]));
-      long long ymin = min(Y[0], min(Y[1], Y[2])), ymax = max(Y[0], max(Y[1], Y[2]));
-      long long px0 = -((-(xmin - 8)) >> 4), px1 = (xmax - 8) >> 4;  // ceil / floor of (v - 8) / 16
-      long long py0 = -((-(ymin - 8)) >> 4), py1 = (ymax - 8) >> 4;
-      px0 = max(px0, 0ll);
-      py0 = max(py0, 0ll);
-      px1 = min(px1, (long long)p.W - 1);
-      py1 = min(py1, (long long)p.H - 1);
-      if (px0 > px1 || py0 > py1) continue;
-      int vi = 0;
-#pragma unroll
-      for (int q = 0; q < 3; ++q) {
-        const int src = q == 0 ? o[0] : q == 1 ? o[1] : o[2];
-        s.X[q] = (int)(src == 0 ? X[0] : src == 1 ? X[1] : X[2]);
-        s.Y[q] = (int)(src == 0 ? Y[0] : src == 1 ? Y[1] : Y[2]);
-        s.z[q] = src == 0 ? Z[0] : src == 1 ? Z[1] : Z[2];
-        vi |= src << (2 * q);
-      }
-      s.px0 = (int)px0;
-      s.px1 = (int)px1;
-      s.py0 = (int)py0;
-      s.py1 = (int)py1;
-      s.area = area;
-      s.vi = vi;
-      ctx.template emit<RASTER>(&tri);
     }
   }
 
@@ -231,8 +293,8 @@ struct RasterF {
     for (int r0 = 0; r0 < n; r0 += kWarpsW) {
       const int k = r0 + (threadIdx.x >> 5);
       if (k >= n) break;  // warp-uniform
-      const uint32_t tri = ((const uint32_t*)items)[k];
-      if (tri >= (uint32_t)p.n_tris) continue;
+      const uint32_t tri = ((const uint32_t*)items)[k];  // sub-triangle id in near-clip mode
+      if ((unsigned long long)tri >= n_setups(p)) continue;
       const RSetup& s = setup[tri];
       const int tx0 = s.px0 >> 3, tx1 = s.px1 >> 3, ty0 = s.py0 >> 3, ty1 = s.py1 >> 3;
       const int ntx = tx1 - tx0 + 1, nt = ntx * (ty1 - ty0 + 1);
@@ -286,7 +348,7 @@ struct RasterF {
       const int k = r0 + (threadIdx.x >> 6);
       if (k >= n) break;
       const FragItem f = ((const FragItem*)items)[k];
-      if (f.tri >= (uint32_t)p.n_tris) continue;
+      if ((unsigned long long)f.tri >= n_setups(p)) continue;
       const RSetup& s = setup[f.tri];
       const int px = (int)(f.tile & 0xFFFFu) * 8 + (q & 7), py = (int)(f.tile >> 16) * 8 + (q >> 3);
       if (px < s.px0 || px > s.px1 || py < s.py0 || py > s.py1) continue;
@@ -312,6 +374,8 @@ struct RasterF {
     if (p.W <= 0 || p.H <= 0 || p.W > 65535 || p.H > 65535) return "vp_raster_params: bad W/H";
     if (p.n_tris <= 0 || p.n_tris > (1ll << 31)) return "vp_raster_params: bad n_tris";
     if (!p.M || !p.pos || !p.col || !p.setup || !p.fb || !p.colour) return "vp_raster_params: M, pos, col, setup, fb, colour required";
+    if (p.near_clip != 0 && p.near_clip != 1) return "vp_raster_params: near_clip must be 0 or 1";
+    if (p.near_clip && (!p.ccol || ((uintptr_t)p.ccol & 15))) return "vp_raster_params: near_clip needs a 16-B aligned ccol";
     if (((uintptr_t)p.setup & 127) || ((uintptr_t)p.pos & 15) || ((uintptr_t)p.colour & 15))
       return "vp_raster_params: setup must be 128-B aligned; pos, colour 16-B aligned";
     return nullptr;
@@ -335,8 +399,14 @@ __global__ void k_raster_resolve(vp_raster_params p) {
       const RSetup& s = setup[tri];
       float l[3];
       if (frag_weights(s, (int)(i % p.W), (int)(i / p.W), l)) {
-        const float4* col = (const float4*)p.col + 3 * (size_t)tri;
-        const float4 c0 = col[s.vi & 3], c1 = col[(s.vi >> 2) & 3], c2 = col[(s.vi >> 4) & 3];
+        float4 c0, c1, c2;
+        if (p.near_clip) {  // sub-triangle colours, already in setup order
+          const float4* cc = (const float4*)p.ccol + 3 * (size_t)tri;
+          c0 = cc[0], c1 = cc[1], c2 = cc[2];
+        } else {
+          const float4* col = (const float4*)p.col + 3 * (size_t)tri;
+          c0 = col[s.vi & 3], c1 = col[(s.vi >> 2) & 3], c2 = col[(s.vi >> 4) & 3];
+        }
         float r = l[0] * c0.x + l[1] * c1.x;
         r = r + l[2] * c2.x;
         float g = l[0] * c0.y + l[1] * c1.y;

@@ -120,7 +120,8 @@ class ReyesParams(C.Structure):
 
 class RasterParams(C.Structure):
     _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_tris", C.c_int64), ("M", P), ("pos", P), ("col", P),
-                ("setup", P), ("fb", P), ("colour", P)]
+                ("setup", P), ("fb", P), ("colour", P), ("near_clip", C.c_int32), ("pad0", C.c_int32),
+                ("ccol", P)]
 
 
 class PyramidParams(C.Structure):

@@ -144,12 +144,16 @@ class RasterPipeline:
         self.M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).to(dev)
         self.pos = torch.from_numpy(np.ascontiguousarray(scene.pos, np.float32)).to(dev)
         self.col = torch.from_numpy(np.ascontiguousarray(scene.col, np.float32)).to(dev)
-        self.setup = torch.empty((n, 32), dtype=torch.float32, device=dev)          # 128 B per triangle
+        near = int(getattr(scene, "near_clip", 0))
+        nsub = n * (2 if near else 1)                                                 # sub-triangles 2 tri + j
+        self.setup = torch.empty((nsub, 32), dtype=torch.float32, device=dev)       # 128 B per (sub-)triangle
+        self.ccol = torch.empty((nsub if near else 1, 12), dtype=torch.float32, device=dev)
         self.fb = torch.empty((scene.H, scene.W), dtype=torch.int64, device=dev)
         self.colour = torch.empty((scene.H, scene.W, 4), dtype=torch.float32, device=dev)
         self.prm = vp.RasterParams(W=scene.W, H=scene.H, n_tris=n, M=self.M.data_ptr(), pos=self.pos.data_ptr(),
                                    col=self.col.data_ptr(), setup=self.setup.data_ptr(), fb=self.fb.data_ptr(),
-                                   colour=self.colour.data_ptr())
+                                   colour=self.colour.data_ptr(), near_clip=near,
+                                   ccol=self.ccol.data_ptr())
         self.p = vp.Pipeline(device, **kw)
         for kind, stride in zip((vp.RASTER_VERTEX, vp.RASTER_CLIP, vp.RASTER_RASTER, vp.RASTER_FRAGMENT), (4, 4, 4, 8)):
             self.p.register(kind, stride, self.prm)

@@ -137,3 +137,36 @@ def test_raster_triangle_shards_merge_bit_exact(vpm, orc, shards):
             rk, rc = full.keys(), full.colour.cpu().numpy()
         assert np.array_equal(k.cpu().numpy().view(np.uint64), rk.reshape(k.shape))
         assert np.array_equal(c.cpu().numpy(), rc.reshape(c.shape))
+
+
+@pytest.mark.parametrize("model", MODELS)
+def test_raster_near_clip(vpm, orc, model):
+    """Near-plane clipping (SURVEY §8(f-4), DESIGN R-S9): Clip fans out 0..2 sub-triangles;
+    keys (sub-ids 2 tri + j), colours and per-stage counts bit-exact with the oracle."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_near_scene(4096, W=256, H=192)
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, model)
+    for _ in range(2):
+        ref = check(orc, scene, rp, rp.run())
+    assert ref["n_raster"] > ref["n_clip"] // 2  # sub-triangles were emitted
+
+
+def test_raster_near_clip_off_matches_default(vpm, orc):
+    """near_clip = 1 on a scene with no vertex behind z = 0 renders the default image with
+    every key's id doubled (the clip is the identity there)."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_scene(3000, W=256, H=192)
+    a = RasterPipeline(scene)
+    a.configure(vpm.MEGAKERNEL)
+    a.run()
+    scene.near_clip = 1
+    b = RasterPipeline(scene)
+    b.configure(vpm.MEGAKERNEL)
+    b.run()
+    ka, kb = a.keys(), b.keys()
+    hit = ka != np.uint64(0xFFFFFFFFFFFFFFFF)
+    assert np.array_equal(hit, kb != np.uint64(0xFFFFFFFFFFFFFFFF))
+    assert np.array_equal(ka[hit] >> np.uint64(32), kb[hit] >> np.uint64(32))
+    assert np.array_equal((ka[hit] & np.uint64(0xFFFFFFFF)) * np.uint64(2), kb[hit] & np.uint64(0xFFFFFFFF))
+    assert np.array_equal(a.colours(), b.colours())
