@@ -260,14 +260,21 @@ def raster_scene(n: int = 1 << 20, W: int = 1920, H: int = 1080, seed: int = see
 
 
 def raster_near_scene(n: int = 4096, W: int = 256, H: int = 192, seed: int = seed_for(4) + 17,
-                      z_range=(-0.6, 0.95), area_range=(4.0, 2048.0)) -> RasterScene:
+                      z_range=(-0.6, 0.95), area_range=(4.0, 2048.0), perspective: bool = False) -> RasterScene:
     """Near-plane clipping workload (DESIGN R-S9): the config-4 recipe with
     per-vertex z ~ U(z_range), so about half the triangles straddle z = 0 (one or two
-    vertices behind the near plane) and a few lie wholly behind it; near_clip = 1."""
+    vertices behind the near plane) and a few lie wholly behind it; near_clip = 1.
+    perspective: w = z + 0.5 (rows 0, 1 as pixel_to_ndc, row 3 = (0, 0, 1, 0.5)), so
+    vertices with z <= -0.5 have w <= 0 -- the default mode culls their triangles whole,
+    the clip keeps the part in front (w = 0.5 on the plane)."""
     sc = raster_scene(n=n, W=W, H=H, seed=seed, area_range=area_range)
     u = uniform01(seed ^ 0x5A5A, n * 3).reshape(n, 3)
     sc.pos[:, :, 2] = (z_range[0] + (z_range[1] - z_range[0]) * u).astype(np.float32)
     sc.near_clip = 1
+    if perspective:
+        M = sc.M.reshape(4, 4).copy()
+        M[3] = (0.0, 0.0, 1.0, 0.5)
+        sc.M = M.reshape(16)
     return sc
 
 

@@ -152,6 +152,17 @@ def test_raster_near_clip(vpm, orc, model):
     assert ref["n_raster"] > ref["n_clip"] // 2  # sub-triangles were emitted
 
 
+@pytest.mark.parametrize("model", ["kbk", "megakernel", "hybrid_rtc_mega"])
+def test_raster_near_clip_perspective(vpm, orc, model):
+    """Perspective scene (w = z + 0.5, some vertices at w <= 0): the clipped sub-triangles
+    have interpolated w; bit-exact with the oracle."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_near_scene(4096, W=256, H=192, z_range=(-0.9, 0.95), perspective=True)
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, model)
+    check(orc, scene, rp, rp.run())
+
+
 def test_raster_near_clip_off_matches_default(vpm, orc):
     """near_clip = 1 on a scene with no vertex behind z = 0 renders the default image with
     every key's id doubled (the clip is the identity there)."""

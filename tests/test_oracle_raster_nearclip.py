@@ -123,3 +123,18 @@ def test_near_definition_equals_pipeline(orc):
     assert sc.n_tris < b["n_raster"] <= 2 * sc.n_tris
     ids = b["trace"]["id"][b["trace"]["stage"] == 2]
     assert np.unique(ids).size == ids.size and (ids < 2 * sc.n_tris).all()
+
+
+def test_perspective_clip_keeps_what_the_w_cull_drops(orc):
+    """Perspective (w = z + 0.5): triangles with a vertex at w <= 0 are culled whole by
+    the default mode; the clip keeps their front part, so it rasterises strictly more
+    (sub-)triangles, and every pixel it shares with the default image at a triangle the
+    default mode kept has the same depth within the snap bound."""
+    sc = inputs.raster_near_scene(120, W=160, H=120, z_range=(-0.9, 0.95), perspective=True)
+    b = orc.raster_definition(sc)
+    sc0 = copy.deepcopy(sc)
+    sc0.near_clip = 0
+    a = orc.raster_definition(sc0)
+    assert b["n_raster"] > a["n_raster"]
+    assert int((b["key"] != U64MAX).sum()) > int((a["key"] != U64MAX).sum())
+    assert (_z_of_key(b["key"][b["key"] != U64MAX]) >= 0).all()
