@@ -333,9 +333,16 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
         out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)
 
+    def w_raster_near():
+        # SURVEY §8(f-4), DESIGN R-S9: config-4 triangles with per-vertex z ~ U(-0.6, 0.95),
+        # so about half straddle the near plane and Clip fans out 0..2 sub-triangles
+        rs = inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
+        out["raster_near_clip"] = measure(RasterPipeline(rs), 1)
+        out["raster_near_clip"]["triangles_per_s"] = rs.n_tris / (out["raster_near_clip"]["ms"] / 1e3)
+
     for name, fn in (("reyes_config1", w_reyes1), ("reyes_config1_x256", w_reyes1x), ("facedet_config2", w_face),
                      ("facedet_config2_x8", w_face8), ("pyramid_config3", w_pyr), ("cfd_config3", w_cfd),
-                     ("ldpc_f3", w_ldpc), ("raster_config4", w_raster)):
+                     ("ldpc_f3", w_ldpc), ("raster_config4", w_raster), ("raster_near_clip", w_raster_near)):
         guarded(name, fn)
     return out
 
