@@ -181,3 +181,33 @@ def test_raster_near_clip_off_matches_default(vpm, orc):
     assert np.array_equal(ka[hit] >> np.uint64(32), kb[hit] >> np.uint64(32))
     assert np.array_equal((ka[hit] & np.uint64(0xFFFFFFFF)) * np.uint64(2), kb[hit] & np.uint64(0xFFFFFFFF))
     assert np.array_equal(a.colours(), b.colours())
+
+
+@pytest.mark.parametrize("model", ["hybrid_rtc_rtc", "megakernel"])
+def test_raster_near_clip_full_size(vpm, orc, model):
+    """The bench's near-clip workload at full size (1M triangles, 1920x1080, about half
+    straddling z = 0) against the whole-frame oracle (~5 s), bit-exact."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    scene = inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, model)
+    check(orc, scene, rp, rp.run())
+
+
+def test_raster_near_clip_shards_merge_bit_exact(vpm, orc):
+    """Triangle shards with near clipping: sub-ids 2 tri + j stay global,
+    so the MIN-key merge of 3 shards equals the oracle's frame."""
+    from paper_conf_micro_zhengozsyc17_b200 import shard
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    sc = inputs.raster_near_scene(4096, W=256, H=192, z_range=(-0.9, 0.95), perspective=True)
+    parts = []
+    for r in range(3):
+        lo, hi = shard.shard_range(r, 3, sc.n_tris)
+        rp = RasterPipeline(sc, tri_range=(lo, hi))
+        rp.configure(vpm.MEGAKERNEL)
+        rp.run()
+        parts.append((rp.fb.clone(), rp.colour.clone()))
+    k, c = _merge_local(parts)
+    ref = orc.raster_definition(sc)
+    assert np.array_equal(k.cpu().numpy().view(np.uint64), ref["key"].reshape(k.shape))
+    assert np.array_equal(c.cpu().numpy(), ref["colour"].reshape(c.shape))
