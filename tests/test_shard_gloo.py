@@ -92,14 +92,21 @@ def test_ordered_key_transform_preserves_uint64_order():
     assert np.array_equal(shard.ukey_to_ordered(torch.from_numpy(o)).numpy().view(np.uint64), u)
 
 
-def _raster_worker(rank, world, port, q):
+def _raster_scene(near):
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    if near:
+        return inputs.raster_near_scene(1500, W=96, H=64, area_range=(2.0, 600.0), z_range=(-0.9, 0.95), perspective=True)
+    return inputs.raster_scene(n=3000, W=96, H=64)
+
+
+def _raster_worker(rank, world, port, q, near=False):
     import torch.distributed as dist
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         import oracle
         from paper_conf_micro_zhengozsyc17_b200 import inputs
-        sc = inputs.raster_scene(n=3000, W=96, H=64)
+        sc = _raster_scene(near)
         lo, hi = shard.shard_range(rank, world, sc.n_tris)
         r = oracle.raster_definition(collapse_outside(sc, lo, hi))
         k, c = shard.raster_merge(torch.from_numpy(r["key"].view(np.int64).copy()), torch.from_numpy(r["colour"].copy()))
@@ -109,8 +116,8 @@ def _raster_worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_triangle_sharded_raster_equals_single_frame(orc, world):
+@pytest.mark.parametrize("world,near", [(2, False), (3, False), (2, True)])
+def test_triangle_sharded_raster_equals_single_frame(orc, world, near):
     """each rank rasterises a shard of the triangles (the CPU oracle stands
     in for the GPU here); one MIN all-reduce of the z-keys plus the winner's colour
     reproduces the single-process frame bit for bit."""
@@ -118,12 +125,12 @@ def test_triangle_sharded_raster_equals_single_frame(orc, world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_raster_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_raster_worker, args=(r, world, port, q, near)) for r in range(world)]
     for p in procs:
         p.start()
     k, c = q.get(timeout=120)
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    ref = orc.raster_definition(inputs.raster_scene(n=3000, W=96, H=64))
+    ref = orc.raster_definition(_raster_scene(near))
     assert np.array_equal(k, ref["key"]) and np.array_equal(c, ref["colour"])
