@@ -5,6 +5,7 @@ so co-running persistent groups cannot be captured together).
   rtc_dice  : the [Dice,Shade] RTC kernel alone: every seed patch is inserted into the
               Dice queue, the [Bound,Split] group is an (idle) KBK group
   kbk       : one launch per stage per wave
+  raster_{mega,kbk}, raster_near_{mega,kbk} : config 4 / the near-clip raster workload
   bs_mega   : the block-local [Bound,Split] megakernel alone (Dice items left in a full ring)
   rtc_leaf  : the [Dice,Shade] RTC kernel alone on representative leaf patches
               (tools/reyes_leaves.py: numpy approximation of the Bound/Split recursion)
@@ -30,7 +31,8 @@ args = ap.parse_args()
 nsm, _ = vp.device_info(0)
 if args.target.startswith("raster"):
     from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
-    scene = inputs.raster_scene()
+    scene = (inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
+             if args.target.startswith("raster_near") else inputs.raster_scene())
     rp = RasterPipeline(scene)
 elif args.target == "bs_mega":
     scene = inputs.reyes_config5(n_frames=args.frames)
@@ -38,9 +40,9 @@ elif args.target == "bs_mega":
 else:
     scene = inputs.reyes_config5(n_frames=args.frames)
     rp = ReyesPipeline(scene, flags=vp.FLAG_L2_PERSIST if args.l2 else 0)
-if args.target == "raster_mega":
+if args.target in ("raster_mega", "raster_near_mega"):
     rp.configure(vp.MEGAKERNEL)
-elif args.target == "raster_kbk":
+elif args.target in ("raster_kbk", "raster_near_kbk"):
     rp.configure(vp.KBK)
 elif args.target == "mega":
     rp.configure(vp.MEGAKERNEL)
