@@ -249,36 +249,66 @@ struct RasterF {
         }
         if (o0 || o1 || o2 || o3 || o4 || o5) continue;
       }
-      const float4* col = (const float4*)p.col + 3 * (size_t)tri;
-      float4 P[4], Cc[4];
+      // The polygon is kept as up to 4 (source edge q, t) pairs -- t < 0: vertex q itself,
+      // else the point a + t (b - a) on edge q (a = vertex q, b = vertex q+1) -- written by
+      // select into fixed slots, so it stays in 8 registers (no local-memory array).
+      int pe0 = 0, pe1 = 0, pe2 = 0, pe3 = 0;
+      float pt0 = -1.f, pt1 = -1.f, pt2 = -1.f, pt3 = -1.f;
       int np = 0;
 #pragma unroll
       for (int q = 0; q < 3; ++q) {
         const float4 a = c[q], b = c[(q + 1) % 3];
-        const float4 ca = __ldg(col + q), cb = __ldg(col + (q + 1) % 3);
         const bool ina = a.z >= 0.0f, inb = b.z >= 0.0f;
         if (ina) {
-          P[np] = a;
-          Cc[np] = ca;
+          if (np == 0) pe0 = q, pt0 = -1.f;
+          if (np == 1) pe1 = q, pt1 = -1.f;
+          if (np == 2) pe2 = q, pt2 = -1.f;
+          if (np == 3) pe3 = q, pt3 = -1.f;  // v0 in, v1 out, v2 in: v2 is the 4th vertex
           ++np;
         }
         if (ina != inb) {
           const float t = a.z / (a.z - b.z);
-          P[np] = make_float4(a.x + t * (b.x - a.x), a.y + t * (b.y - a.y), 0.0f, a.w + t * (b.w - a.w));
-          Cc[np] = make_float4(ca.x + t * (cb.x - ca.x), ca.y + t * (cb.y - ca.y), ca.z + t * (cb.z - ca.z),
-                               ca.w + t * (cb.w - ca.w));
+          if (np == 0) pe0 = q, pt0 = t;
+          if (np == 1) pe1 = q, pt1 = t;
+          if (np == 2) pe2 = q, pt2 = t;
+          if (np == 3) pe3 = q, pt3 = t;
           ++np;
         }
       }
+      const float4* col = (const float4*)p.col + 3 * (size_t)tri;
       float4* ccol = (float4*)p.ccol;
-      for (int j = 0; j + 2 < np; ++j) {
-        const int idx[3] = {0, j + 1, j + 2};
-        const float4 v[3] = {P[idx[0]], P[idx[1]], P[idx[2]]};
+      // polygon vertex (q, t): clip coordinates and colour
+      auto vert = [&](int q, float t, float4& v, float4& cv) {
+        const float4 a = q == 0 ? c[0] : q == 1 ? c[1] : c[2];
+        const int qb = q == 2 ? 0 : q + 1;
+        const float4 ca = __ldg(col + q);
+        if (t < 0.0f) {
+          v = a;
+          cv = ca;
+        } else {
+          const float4 b = qb == 0 ? c[0] : qb == 1 ? c[1] : c[2];
+          const float4 cb = __ldg(col + qb);
+          v = make_float4(a.x + t * (b.x - a.x), a.y + t * (b.y - a.y), 0.0f, a.w + t * (b.w - a.w));
+          cv = make_float4(ca.x + t * (cb.x - ca.x), ca.y + t * (cb.y - ca.y), ca.z + t * (cb.z - ca.z),
+                           ca.w + t * (cb.w - ca.w));
+        }
+      };
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        if (j + 2 >= np) break;
+        // fan triangle (p0, p(j+1), p(j+2))
+        float4 v[3], cv[3];
+        vert(pe0, pt0, v[0], cv[0]);
+        vert(j == 0 ? pe1 : pe2, j == 0 ? pt1 : pt2, v[1], cv[1]);
+        vert(j == 0 ? pe2 : pe3, j == 0 ? pt2 : pt3, v[2], cv[2]);
         const uint32_t sub = 2 * tri + (uint32_t)j;
         RSetup& s = setup[sub];
         if (!setup_one(p, v, s)) continue;
 #pragma unroll
-        for (int q = 0; q < 3; ++q) ccol[3 * (size_t)sub + q] = Cc[idx[(s.vi >> (2 * q)) & 3]];
+        for (int q = 0; q < 3; ++q) {
+          const int src = (s.vi >> (2 * q)) & 3;
+          ccol[3 * (size_t)sub + q] = src == 0 ? cv[0] : src == 1 ? cv[1] : cv[2];
+        }
         ctx.template emit<RASTER>(&sub);
       }
     }
