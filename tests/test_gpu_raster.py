@@ -211,3 +211,22 @@ def test_raster_near_clip_shards_merge_bit_exact(vpm, orc):
     ref = orc.raster_definition(sc)
     assert np.array_equal(k.cpu().numpy().view(np.uint64), ref["key"].reshape(k.shape))
     assert np.array_equal(c.cpu().numpy(), ref["colour"].reshape(c.shape))
+
+
+@pytest.mark.parametrize("zs", [(-0.2, 0.3, 0.4), (0.2, -0.3, 0.4), (0.2, 0.3, -0.4), (-0.2, -0.3, 0.4),
+                                (0.2, -0.3, -0.4), (-0.2, 0.3, -0.4), (0.2, 0.3, 0.4)])
+def test_raster_near_clip_every_side_pattern(vpm, orc, zs):
+    """One triangle per in/out pattern of its vertices (the polygon's 4th vertex is an
+    original vertex only for in-out-in), under both vertex orders, bit-exact."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    for order in ((0, 1, 2), (0, 2, 1)):
+        xy = [(8, 8), (56, 10), (30, 56)]
+        pos = np.zeros((1, 3, 4), np.float32)
+        col = np.zeros((1, 3, 4), np.float32)
+        for k, o in enumerate(order):
+            pos[0, k] = (*xy[o], zs[o], 1.0)
+            col[0, k, :3] = np.eye(3)[o]
+        scene = inputs.RasterScene(W=64, H=64, M=inputs.pixel_to_ndc(64, 64), pos=pos, col=col, near_clip=1)
+        rp = RasterPipeline(scene)
+        rp.configure(vpm.MEGAKERNEL)
+        check(orc, scene, rp, rp.run())

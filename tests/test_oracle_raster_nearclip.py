@@ -82,7 +82,9 @@ def test_orthographic_equivalence_single_triangle(orc, seed):
 
 
 @pytest.mark.parametrize("zs,n_sub", [((0.2, 0.3, 0.4), 1), ((-0.2, 0.3, 0.4), 2), ((-0.2, -0.3, 0.4), 1),
-                                      ((-0.2, -0.3, -0.4), 0), ((0.0, 0.3, 0.4), 1), ((-0.2, 0.0, 0.4), 1)])
+                                      ((-0.2, -0.3, -0.4), 0), ((0.0, 0.3, 0.4), 1), ((-0.2, 0.0, 0.4), 1),
+                                      ((0.2, -0.3, 0.4), 2), ((0.2, 0.3, -0.4), 2), ((0.2, -0.3, -0.4), 1),
+                                      ((-0.2, 0.3, -0.4), 1)])
 def test_subtriangle_count_by_case(orc, zs, n_sub):
     v = [(8, 8, zs[0]), (56, 10, zs[1]), (30, 56, zs[2])]
     r = orc.raster_pipeline(_tri_scene(v))
