@@ -150,55 +150,108 @@ def time_steps(torch, rp, steps, stream):
     return ev0.elapsed_time(ev1), st, kms
 
 
-def cpu_oracle_sample(frames_total, seconds, frame0=0):
-    """The CPU oracle as it stands (single-threaded C per frame), frames spread over the
-    host cores with a process pool; returns (frames/s, items/s, cores, sample text)."""
-    import multiprocessing as mp
-    t0 = time.perf_counter()
-    _oracle_frame(frame0)  # one frame first, to size the sample
-    one = time.perf_counter() - t0
-    cores = os.cpu_count() or 1
-    n = int(max(cores, min(frames_total, seconds * cores / max(one, 1e-3))))
-    n = max(1, min(n, frames_total))
-    t0 = time.perf_counter()
-    with mp.get_context("fork").Pool(cores) as pool:
-        res = pool.map(_oracle_frame, [(frame0 + f) % TOTAL_FRAMES for f in range(n)])
-    dt = time.perf_counter() - t0
-    items = sum(r for r in res)
-    return n / dt, items / dt, cores, f"{n} of {frames_total} frames (config 5, 4096 patches each), oracle per frame on {cores} processes, {dt:.1f} s"
+# Parity frames of the timed run: spread over the orbit; the camera is nearest (deepest
+# recursion, depth-8 leaves) at f = 32 mod 64 and farthest at f = 0 mod 64.
+PARITY_FRAMES = (0, 32, 75, 96, 160, 224, 288, 352, 416, 480, 511)
 
 
-def _oracle_frame(f):
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
+def oracle_frames(frames, threads):
+    """The C oracle as it stands (single-threaded per frame) on the given config-5 frames,
+    one frame per host thread at a time (ctypes releases the GIL, so the threads run the
+    C code in parallel).  Input generation happens before the timer starts."""
+    import concurrent.futures as cf
     import oracle
     from paper_conf_micro_zhengozsyc17_b200 import inputs
-    sc = inputs.reyes_config5(n_frames=1, n_side=PATCH_SIDE, frame0=f)
-    r = oracle.reyes_pipeline(sc)
-    return r["n_bound"] + r["n_split"] + r["n_dice"] + r["n_shade"]
+    scenes = [inputs.reyes_config5(n_frames=1, n_side=PATCH_SIDE, frame0=f % TOTAL_FRAMES) for f in frames]
+    t0 = time.perf_counter()
+    with cf.ThreadPoolExecutor(max(1, threads)) as ex:
+        res = list(ex.map(oracle.reyes_pipeline, scenes))
+    return time.perf_counter() - t0, res
+
+
+def cpu_oracle_sample(frames_total, seconds, must=()):
+    """cpu_baseline: the oracle on a bounded sample of the same workload (about `seconds`
+    of CPU time over all host cores).  The sample always contains the `must` frames (the
+    parity frames), then frames spread evenly over the shard.  Returns (record, per-frame
+    oracle results)."""
+    import oracle
+    oracle.build()
+    cores = os.cpu_count() or 1
+    one, _ = oracle_frames([32], 1)   # the nearest-camera frame bounds the per-frame cost
+    n = int(min(frames_total, max(cores, len(must), seconds * cores / max(one, 1e-3))))
+    frames = list(dict.fromkeys(must))
+    for f in np.linspace(0, frames_total - 1, n).astype(int).tolist():
+        if len(frames) >= n:
+            break
+        if f not in frames:
+            frames.append(f)
+    dt, res = oracle_frames(frames, cores)
+    items = sum(r["n_bound"] + r["n_split"] + r["n_dice"] + r["n_shade"] for r in res)
+    hist = np.sum([r["depth_hist"][:9] for r in res], axis=0).tolist()
+    rec = {"value": len(frames) / dt, "unit": "frames/s", "cores": cores, "threads": cores, "kind": "oracle",
+           "cpu_model": cpu_model(), "items_per_sec": items / dt, "seconds": dt, "frames": len(frames),
+           "sample": f"{len(frames)} of {frames_total} config-5 frames (4096 patches each, parity frames included), "
+                     f"C oracle one frame per thread on {cores} threads, input generation excluded, {dt:.1f} s",
+           "leaf_depth_hist_sample": hist}
+    return rec, dict(zip(frames, res))
+
+
+def parity_check(snap, ref):
+    """The timed configuration's outputs (snapshotted right after the timed region) vs the
+    oracle, per sampled frame: depth keys and shade factors bit-exact, colours within
+    north_star's 1e-4 (bit-exact expected)."""
+    keys_bad, s_bad, err = 0, 0, 0.0
+    for f, (k, sf, c) in snap.items():
+        r = ref[f]
+        keys_bad += int(np.count_nonzero(k != r["key"][0]))
+        s_bad += int(np.count_nonzero(sf != r["s"][0]))
+        err = max(err, float(np.max(np.abs(c - r["colour"][0]))))
+    return {"pass": keys_bad == 0 and s_bad == 0 and err <= 1e-4, "frames": sorted(snap), "keys_differing": keys_bad,
+            "s_differing": s_bad, "max_abs_err": err, "tolerance": 1e-4,
+            "checked": "outputs of the last timed step (timed configuration) vs the CPU oracle"}
 
 
 def run_reference(args, rank, world):
-    """--impl reference: the CPU oracle, rank 0 only (other ranks exit without work)."""
+    """--impl reference: the CPU oracle, rank 0 only (other ranks exit without work).
+    Each step renders a bounded sample of the config-5 frames; ms_per_step is that
+    step's measured wall time, so steps x ms_per_step is what ran."""
     if rank != 0:
         return
     import oracle
     oracle.build()
-    vals, items = [], []
+    cores = os.cpu_count() or 1
+    one, _ = oracle_frames([32], 1)
+    per_step = int(max(cores, min(args.frames, args.cpu_seconds / max(args.steps, 1) * cores / max(one, 1e-3))))
+    frames = np.linspace(0, args.frames - 1, per_step).astype(int).tolist()
     for _ in range(args.warmup):
-        _oracle_frame(0)
-    info = None
+        oracle_frames(frames[:cores], cores)
+    secs, items = [], []
     for _ in range(args.steps):
-        fps, ips, cores, sample = cpu_oracle_sample(args.frames, max(1.0, args.cpu_seconds / max(args.steps, 1)))
-        vals.append(fps)
-        items.append(ips)
-        info = (cores, sample)
-    v = float(np.median(vals))
+        dt, res = oracle_frames(frames, cores)
+        secs.append(dt)
+        items.append(sum(r["n_bound"] + r["n_split"] + r["n_dice"] + r["n_shade"] for r in res) / dt)
+    ms = 1000.0 * float(np.median(secs))
+    v = per_step / (ms / 1000.0)
+    sample = (f"{per_step} of {args.frames} config-5 frames per step (spread over the orbit), C oracle one frame per "
+              f"thread on {cores} threads, input generation excluded")
     line = {"impl": "reference", "metric": "frames/sec", "value": v, "unit": "frames/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * args.frames / v,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
-            "data": "synthetic", "items_per_sec": float(np.median(items)),
+            "data": "synthetic", "items_per_sec": float(np.median(items)), "frames_per_step": per_step,
             "config": {"workload": "reyes_batch_config5", "frames": args.frames, "patches_per_frame": 4096,
-                       "image": "256x256", "max_depth": 8},
-            "cpu_baseline": {"value": v, "unit": "frames/s", "cores": info[0], "kind": "oracle", "sample": info[1]},
+                       "image": "256x256", "max_depth": 8, "sample_frames_per_step": per_step},
+            "cpu_baseline": {"value": v, "unit": "frames/s", "cores": cores, "kind": "oracle", "sample": sample,
+                             "cpu_model": cpu_model()},
             "e2e": {"value": v, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -406,6 +459,16 @@ def main():
     t_ms, st, kms = time_steps(torch, rp, args.steps, stream)
     barrier()
     clocks = clk.stop()
+    # outputs of the last timed step, for the parity check against the oracle (the
+    # baselines below re-render the same buffers)
+    npf = scene.W * scene.H
+    snap = {}
+    for f in PARITY_FRAMES:
+        if f0 <= f < f1:
+            lf = f - f0
+            fbf = rp.fb[lf * npf:(lf + 1) * npf].cpu().numpy()
+            snap[f] = (fbf[:, :2].copy().view(np.uint64).reshape(scene.H, scene.W),
+                       fbf[:, 2].copy().view(np.float32).reshape(scene.H, scene.W), rp.colour[lf].cpu().numpy())
     t_ms = shard.max_over_ranks(t_ms, "cuda")
     items_all, frames_all = shard.sum_over_ranks([sum(st["dequeued"][:4]), f1 - f0], "cuda")
     ms_per_step = t_ms / args.steps
@@ -525,14 +588,15 @@ def main():
             qbench = {"error": repr(ex)}
 
     cpu = None
+    parity = {"pass": None, "checked": "only at N=1 (the oracle runs on rank 0 at N=1)"}
     if rank == 0 and world == 1:
         try:
-            cfps, cips, cores, sample = cpu_oracle_sample(args.frames, args.cpu_seconds)
-            cpu = {"value": cfps, "unit": "frames/s", "cores": cores, "kind": "oracle", "sample": sample,
-                   "items_per_sec": cips}
+            cpu, ref = cpu_oracle_sample(args.frames, args.cpu_seconds, must=sorted(snap))
+            parity = parity_check(snap, ref)
         except Exception as ex:  # the oracle is a reported baseline only
             cpu = {"value": None, "unit": "frames/s", "cores": os.cpu_count(), "kind": "oracle",
                    "sample": f"failed: {ex}"}
+            parity = {"pass": False, "error": repr(ex)}
 
     launches = 3 + nk + int(st["kbk_launches"])   # run-init, fb clear, resolve + kernels + waves
     line = {
@@ -553,7 +617,8 @@ def main():
         "speedup_vs_kbk": (extra["kbk"]["ms_per_step"] / ms_per_step) if "kbk" in extra else None,
         "speedup_vs_kbk_graph": (extra["kbk_graph"]["ms_per_step"] / ms_per_step) if "kbk_graph" in extra else None,
         "baselines": extra, "e2e": e2e, "gather_ms": gather_ms, "clocks": clocks, "gpu_launches": launches * args.steps,
-        "cpu_baseline": cpu, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune, "workloads": suite,
+        "cpu_baseline": cpu, "parity": parity, "device": f"sm_{cc[0]}{cc[1]} x{nsm} SMs", "autotune": tune,
+        "workloads": suite,
         "queue_microbench": qbench,
         "config_string": vp.config_to_string(main_cfg),
     }

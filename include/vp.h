@@ -114,6 +114,15 @@ typedef enum vp_stage_kind {
 #define VP_FLAG_L2_PERSIST 0x40u    /* an L2 access-policy window (persisting) over */
                                     /* every ring's sequence words on the run stream and the  */
                                     /* group streams (sets cudaLimitPersistingL2CacheSize)    */
+#define VP_FLAG_SERIALIZE_GROUPS 0x80u /* test hook: each persistent group's grid starts only */
+                                      /* after the previous group's grid finished, i.e. what a */
+                                      /* profiler's kernel serialisation (or MPS / a co-tenant) */
+                                      /* can do to separately launched groups  */
+#define VP_FLAG_NO_RERUN 0x100u       /* when the groups of a coarse/fine/hybrid plan cannot all */
+                                      /* be resident (a group stalled >= 20 ms on a planned grid */
+                                      /* with no resident block), vp_run returns                 */
+                                      /* VP_ERR_UNSUPPORTED instead of repeating the run as one  */
+                                      /* cooperative megakernel (vp_run_stats.model_rerun)        */
 #define VP_FLAG_FULL_RINGS 0x10u    /* persistent plans keep every ring at its registered     */
                                     /* capacity instead of shrinking it to what the producer  */
                                     /* blocks can hold (needed when a recursive stage's live   */
@@ -174,7 +183,8 @@ typedef struct vp_run_stats {
   uint64_t fallback_admits;                 /* progress-guarantee admissions              */
   uint64_t kbk_launches;                    /* wave launches (KBK / RTC)                   */
   uint64_t trace_records;                   /* with VP_FLAG_TRACE                          */
-  int abort_reason;                         /* 0 none, 1 timeout, 2 overflow, 3 fan-out   */
+  int abort_reason;                         /* 0 none, 1 timeout, 2 overflow, 3 fan-out,  */
+                                            /* 4 guard, 5 groups not co-resident          */
   int num_sms;
   /* VP_FLAG_TIMERS: block-time (ns, summed over blocks) spent executing each stage     */
   /* (stage-in + execute), publishing its outputs (queue overhead, §8.5), and idle per  */
@@ -192,6 +202,12 @@ typedef struct vp_run_stats {
   /* host-driven KBK: summed device time of each stage's wave kernels (every wave uses the
    * whole GPU), i.e. each stage run in isolation -- Table 2's "longest stage" analog (L51) */
   float stage_wave_ms[VP_MAX_STAGES];
+  /* the host waited > 2 s for a group's grid to be fully dispatched before launching the
+   * next group (SM binding is then not deterministic), per run */
+  int dispatch_timeouts;
+  /* 1: the planned groups were not co-resident (ABORT_NOT_CORESIDENT), so the run was
+   * repeated from its seeds as one cooperative megakernel; device_ms covers both attempts */
+  int model_rerun;
 } vp_run_stats;
 
 typedef struct vp_autotune_opts {
@@ -388,16 +404,17 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best, vp_tu
 /* Profiling component (L13, L45): max resident blocks per SM of each single-stage kernel. */
 vp_status vp_profile(void* p, int* max_blocks_per_sm, int* regs_per_thread, int* smem_per_block);
 
-/* Change the run-time diagnostics flags of a pipeline (VP_FLAG_QUEUE_DEPTH,
- * VP_FLAG_STRICT_BINDING, VP_FLAG_TIMERS; the others are fixed at create and rejected with
- * VP_ERR_INVALID).  old_flags (optional) receives all flags before the change. */
+/* Change the run-time flags of a pipeline (VP_FLAG_QUEUE_DEPTH, VP_FLAG_STRICT_BINDING,
+ * VP_FLAG_TIMERS, VP_FLAG_SERIALIZE_GROUPS, VP_FLAG_NO_RERUN; the others are fixed at create
+ * and rejected with VP_ERR_INVALID).  old_flags (optional) receives all flags before the change. */
 vp_status vp_set_flags(void* p, uint32_t flags, uint32_t* old_flags);
 
 /* Library-owned / borrowed outputs of the family (sink results). index 0 = primary. */
 vp_status vp_get_output(void* p, int index, void** dev_ptr, size_t* bytes);
 
-/* The task trace of the last run (VP_FLAG_TRACE): library-owned device array of
- * {u64 item id, u32 stage, u32 smid} records, valid until the next vp_run. */
+/* The task trace of the last run (VP_FLAG_TRACE): library-owned device array of 24-B
+ * {u64 item id, u32 stage, u32 smid, u32 kernel slot, u32 blockIdx.x} records (the kernel
+ * slot indexes vp_run_stats.kernel_*), valid until the next vp_run. */
 vp_status vp_get_trace(void* p, void** dev_ptr, size_t* n_records);
 
 vp_status vp_config_to_string(const vp_config* c, char* buf, size_t buf_len);

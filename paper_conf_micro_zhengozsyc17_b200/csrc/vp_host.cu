@@ -925,6 +925,35 @@ vp_status vp_memcpy(void* dst, const void* src, size_t bytes, int kind, void* st
   return VP_OK;
 }
 
+// Frees everything a pipeline owns; safe on a partially constructed object (every handle
+// starts null), so vp_pipeline_create's error paths and vp_pipeline_destroy share it.
+static void free_pipeline(vp_pipeline_s* p) {
+  for (StageRec& r : p->st) {
+    cudaFree(r.slots);
+    cudaFree(r.seeds);
+  }
+  if (p->seq_arena) cudaFree(p->seq_arena);
+  if (p->ctrl) cudaFree(p->ctrl);
+  if (p->blk) cudaFree(p->blk);
+  if (p->trace) cudaFree(p->trace);
+  if (p->h_ctrl) cudaFreeHost(p->h_ctrl);
+  if (p->h_blk) cudaFreeHost(p->h_blk);
+  if (p->h_arrive) cudaFreeHost((void*)p->h_arrive);
+  if (p->h_retire) cudaFreeHost((void*)p->h_retire);
+  for (int i = 0; i < kMaxKernels; ++i) {
+    if (p->streams[i]) cudaStreamDestroy(p->streams[i]);
+    if (p->ev_join[i]) cudaEventDestroy(p->ev_join[i]);
+    if (p->ev_kbeg[i]) cudaEventDestroy(p->ev_kbeg[i]);
+  }
+  if (p->kg_exec) cudaGraphExecDestroy(p->kg_exec);
+  if (p->kg_graph) cudaGraphDestroy(p->kg_graph);
+  for (cudaEvent_t e : p->wave_ev) cudaEventDestroy(e);
+  if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+  if (p->ev_start) cudaEventDestroy(p->ev_start);
+  if (p->ev_end) cudaEventDestroy(p->ev_end);
+  delete p;
+}
+
 vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) {
   if (!out) return VP_ERR_INVALID;
   *out = nullptr;
@@ -944,7 +973,7 @@ vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) 
   if ((p->desc.flags & VP_FLAG_TRACE) && p->desc.trace_capacity <= 0) p->desc.trace_capacity = 1 << 20;
   auto bad = [&](cudaError_t e) {
     if (e == cudaSuccess) return false;
-    delete p;
+    free_pipeline(p);
     return true;
   };
   if (bad(cudaMalloc(&p->ctrl, sizeof(Ctrl)))) return VP_ERR_OOM;
@@ -954,8 +983,8 @@ vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) 
   if (bad(cudaMallocHost(&p->h_blk, sizeof(uint32_t) * kMaxKernels * kMaxSM))) return VP_ERR_OOM;
   {
     void* ha = nullptr;
-    if (bad(cudaHostAlloc(&ha, sizeof(uint32_t) * kMaxKernels, cudaHostAllocMapped))) return VP_ERR_OOM;
-    memset(ha, 0, sizeof(uint32_t) * kMaxKernels);
+    if (bad(cudaHostAlloc(&ha, sizeof(uint32_t) * (kMaxKernels + 1), cudaHostAllocMapped))) return VP_ERR_OOM;
+    memset(ha, 0, sizeof(uint32_t) * (kMaxKernels + 1));
     p->h_arrive = (volatile uint32_t*)ha;
     if (bad(cudaHostGetDevicePointer((void**)&p->d_arrive, ha, 0))) return VP_ERR_CUDA;
     void* hr = nullptr;
@@ -982,30 +1011,7 @@ vp_status vp_pipeline_destroy(void* h) {
   if (!p) return VP_ERR_INVALID;
   DeviceGuard dg(p->device);
   cudaDeviceSynchronize();
-  for (StageRec& r : p->st) {
-    cudaFree(r.slots);
-    cudaFree(r.seeds);
-  }
-  cudaFree(p->seq_arena);
-  cudaFree(p->ctrl);
-  cudaFree(p->blk);
-  cudaFree(p->trace);
-  cudaFreeHost(p->h_ctrl);
-  cudaFreeHost(p->h_blk);
-  cudaFreeHost((void*)p->h_arrive);
-  cudaFreeHost((void*)p->h_retire);
-  for (int i = 0; i < kMaxKernels; ++i) {
-    cudaStreamDestroy(p->streams[i]);
-    cudaEventDestroy(p->ev_join[i]);
-    cudaEventDestroy(p->ev_kbeg[i]);
-  }
-  if (p->kg_exec) cudaGraphExecDestroy(p->kg_exec);
-  if (p->kg_graph) cudaGraphDestroy(p->kg_graph);
-  for (cudaEvent_t e : p->wave_ev) cudaEventDestroy(e);
-  cudaEventDestroy(p->ev_fork);
-  cudaEventDestroy(p->ev_start);
-  cudaEventDestroy(p->ev_end);
-  delete p;
+  free_pipeline(p);
   return VP_OK;
 }
 
@@ -1131,12 +1137,7 @@ vp_status vp_get_output(void* h, int index, void** dev_ptr, size_t* bytes) {
   return VP_OK;
 }
 
-vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
-  vp_pipeline_s* p = (vp_pipeline_s*)h;
-  if (!p) return VP_ERR_INVALID;
-  if (!p->configured) return fail(p, VP_ERR_INVALID, "vp_run before vp_configure/vp_autotune");
-  DeviceGuard dg(p->device);
-  cudaStream_t st = (cudaStream_t)stream;
+static vp_status run_once(vp_pipeline_s* p, cudaStream_t st, vp_run_stats* stats) {
   const int S = (int)p->st.size();
   for (int s = 0; s < S; ++s)
     if (p->run_cap_log2[s] != (p->plan.cap_log2[s] ? p->plan.cap_log2[s] : p->st[s].cap_log2)) p->dirty_queues = true;
@@ -1154,7 +1155,30 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   ri.watchdog_ns = (unsigned long long)(p->timeout_ms * 1e6);
   p->epoch++;
   if (p->epoch == 0) p->epoch = 1;
+  const Plan& pl = p->plan;
+  int nk = (int)pl.kernels.size();
+  // Stages no seed can reach (through the fan-out graph) never get an item: their
+  // persistent kernels are not launched (they would only hold SMs, and their resident
+  // idle blocks can keep a later kernel's grid from being dispatched).
+  bool reach[kMaxStages] = {};
+  for (int s = 0; s < S; ++s) reach[s] = p->st[s].n_seeds > 0;
+  for (bool grew = true; grew;) {
+    grew = false;
+    for (int s = 0; s < S; ++s)
+      for (int t = 0; t < S; ++t)
+        if (reach[s] && !reach[t] && p->fam->fanout(s, t) > 0) reach[t] = grew = true;
+  }
+  uint32_t live_mask = 0;
+  for (int i = 0; i < nk; ++i) {
+    bool live = false;
+    for (int s = pl.kernels[i].lo; s <= pl.kernels[i].hi; ++s) live |= reach[s];
+    p->launched[i] = live;
+    if (live) live_mask |= 1u << i;
+  }
   Common c = make_common(p);
+  // co-residency check only where groups depend on each other's grids being resident
+  c.peer_mask = __builtin_popcount(live_mask) >= 2 ? live_mask : 0u;
+  int dispatch_timeouts = 0;
   if ((p->desc.flags & VP_FLAG_L2_PERSIST) && !p->l2_window_set) {
     // keep the claim/publish sequence words in a persisting L2 carve-out
     // (the ring counters are atomics, which execute in L2 anyway)
@@ -1181,28 +1205,17 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
   k_run_init<<<1, 256, 0, st>>>(p->ctrl, p->blk, ri);
   CUDA_TRY(p, cudaGetLastError());
   CUDA_TRY(p, p->fam->init_run(p->params.data(), st));
-  const Plan& pl = p->plan;
-  int nk = (int)pl.kernels.size();
-  // Stages no seed can reach (through the fan-out graph) never get an item: their
-  // persistent kernels are not launched (they would only hold SMs, and their resident
-  // idle blocks can keep a later kernel's grid from being dispatched).
-  bool reach[kMaxStages] = {};
-  for (int s = 0; s < S; ++s) reach[s] = p->st[s].n_seeds > 0;
-  for (bool grew = true; grew;) {
-    grew = false;
-    for (int s = 0; s < S; ++s)
-      for (int t = 0; t < S; ++t)
-        if (reach[s] && !reach[t] && p->fam->fanout(s, t) > 0) reach[t] = grew = true;
-  }
+  const bool serialize = (p->desc.flags & VP_FLAG_SERIALIZE_GROUPS) != 0;
   if (nk > 0) {
     CUDA_TRY(p, cudaEventRecord(p->ev_fork, st));
     for (int i = 0; i < nk; ++i) {
       const KernelPlan& k = pl.kernels[i];
       cudaStream_t ks = p->streams[i];
       CUDA_TRY(p, cudaStreamWaitEvent(ks, p->ev_fork, 0));
-      bool live = false;
-      for (int s = k.lo; s <= k.hi; ++s) live |= reach[s];
-      p->launched[i] = live;
+      // test hook: each group's grid starts only after the previous one finished (what a
+      // profiler's kernel serialisation does to concurrently launched groups)
+      if (serialize && i > 0) CUDA_TRY(p, cudaStreamWaitEvent(ks, p->ev_join[i - 1], 0));
+      const bool live = p->launched[i];
       if (!live) {
         CUDA_TRY(p, cudaEventRecord(p->ev_kbeg[i], ks));
         CUDA_TRY(p, cudaEventRecord(p->ev_join[i], ks));
@@ -1228,7 +1241,13 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
         // kernel's blocks arrive (deterministic filling-retreating, L27 §5).
         auto t0 = std::chrono::steady_clock::now();
         while (p->h_arrive[i] != p->epoch) {
-          if (std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(2000)) break;
+          if (p->h_arrive[kMaxKernels] == p->epoch) break;  // aborted: groups not co-resident
+          if (std::chrono::steady_clock::now() - t0 > std::chrono::milliseconds(2000)) {
+            // binding is then no longer deterministic (the next grid may take SMs this one
+            // wanted); recorded in vp_run_stats.dispatch_timeouts
+            ++dispatch_timeouts;
+            break;
+          }
         }
       }
     }
@@ -1340,6 +1359,8 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       stats->seed_head[s] = hc.seed_head[s].v;
     }
     stats->pending = (int64_t)hc.pending.v;
+    stats->dispatch_timeouts = dispatch_timeouts;
+    stats->model_rerun = 0;
   }
   if (hc.abort.v != ABORT_NONE) {
     p->dirty_queues = true;
@@ -1348,6 +1369,9 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
       case ABORT_OVERFLOW: return fail(p, VP_ERR_QUEUE_OVERFLOW, "a ring stayed full for > 200 ms (raise queue_capacity)");
       case ABORT_FANOUT: return fail(p, VP_ERR_FANOUT, "a stage exceeded its declared fan-out");
       case ABORT_GUARD: return fail(p, VP_ERR_INVALID, "a stage's recursion guard fired (input outside the domain)");
+      case ABORT_NOT_CORESIDENT:
+        return fail(p, VP_ERR_UNSUPPORTED, "a planned group's grid never became resident while another group waited on it "
+                                           "(non-concurrent kernel scheduling: profiler, MPS or a co-tenant)");
       default: return fail(p, VP_ERR_CUDA, "unknown abort reason %llu", (unsigned long long)hc.abort.v);
     }
   }
@@ -1366,6 +1390,35 @@ vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
     }
   }
   return VP_OK;
+}
+
+vp_status vp_run(void* h, void* stream, vp_run_stats* stats) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p) return VP_ERR_INVALID;
+  if (!p->configured) return fail(p, VP_ERR_INVALID, "vp_run before vp_configure/vp_autotune");
+  DeviceGuard dg(p->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  vp_status rc = run_once(p, st, stats);
+  if (rc != VP_ERR_UNSUPPORTED || p->h_ctrl->abort.v != ABORT_NOT_CORESIDENT || (p->desc.flags & VP_FLAG_NO_RERUN))
+    return rc;
+  // The groups of this plan could not all be resident at once: the run is
+  // repeated from its seeds as one cooperative megakernel, which the driver co-schedules by
+  // construction; every model computes the same result (SURVEY §8(c-6) model equivalence).
+  const double first_ms = stats ? stats->device_ms : 0.0;
+  Plan saved = p->plan;
+  Plan mega;
+  rc = build_plan(p, VP_MEGAKERNEL, nullptr, saved.cfg.batch, mega);
+  if (rc != VP_OK) return rc;
+  p->plan = mega;
+  p->dirty_queues = true;  // the aborted run's rings are reset before the rerun
+  rc = run_once(p, st, stats);
+  p->plan = saved;
+  p->dirty_queues = true;
+  if (stats) {
+    stats->device_ms += first_ms;
+    stats->model_rerun = 1;
+  }
+  return rc;
 }
 
 vp_status vp_get_trace(void* h, void** dev_ptr, size_t* n) {
@@ -1389,8 +1442,10 @@ int vpi_default_batch(void* h, int s) { return ((vp_pipeline_s*)h)->fam->default
 vp_status vp_set_flags(void* h, uint32_t flags, uint32_t* old_flags) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;
   if (!p) return VP_ERR_INVALID;
-  const uint32_t mutable_bits = VP_FLAG_QUEUE_DEPTH | VP_FLAG_STRICT_BINDING | VP_FLAG_TIMERS;
-  if (flags & ~mutable_bits) return fail(p, VP_ERR_INVALID, "vp_set_flags: only QUEUE_DEPTH, STRICT_BINDING, TIMERS change after create");
+  const uint32_t mutable_bits =
+      VP_FLAG_QUEUE_DEPTH | VP_FLAG_STRICT_BINDING | VP_FLAG_TIMERS | VP_FLAG_SERIALIZE_GROUPS | VP_FLAG_NO_RERUN;
+  if (flags & ~mutable_bits)
+    return fail(p, VP_ERR_INVALID, "vp_set_flags: only QUEUE_DEPTH, STRICT_BINDING, TIMERS, SERIALIZE_GROUPS, NO_RERUN change after create");
   if (old_flags) *old_flags = p->desc.flags;
   p->desc.flags = (p->desc.flags & ~mutable_bits) | flags;
   return VP_OK;

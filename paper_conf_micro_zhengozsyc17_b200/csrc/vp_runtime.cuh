@@ -41,6 +41,8 @@ enum Abort : unsigned long long {
   ABORT_OVERFLOW = 2,  // a producer could not get a free ring slot (VP_ERR_QUEUE_OVERFLOW)
   ABORT_FANOUT = 3,    // a stage emitted more items than its declared fan-out
   ABORT_GUARD = 4,     // a stage's own recursion guard fired (invalid input)
+  ABORT_NOT_CORESIDENT = 5,  // a group waited on a planned group whose grid never became
+                             // resident (non-concurrent scheduling: profiler, MPS, co-tenant)
 };
 
 // Each hot counter on its own 128-B line (no false sharing between L2 atomics).
@@ -87,6 +89,7 @@ struct QueueDesc {
 struct TraceRec {
   unsigned long long id;
   uint32_t stage, smid;
+  uint32_t kslot, block;  // kernel slot and blockIdx.x of the executing block (binding checks)
 };
 
 enum : uint32_t { FLAG_TRACE = 1u, FLAG_DEPTH = 2u, FLAG_TIMERS = 4u };
@@ -99,11 +102,16 @@ struct Common {
   unsigned long long trace_cap;
   uint32_t flags;
   int n_stages;
-  volatile uint32_t* host_arrive;  // mapped pinned host words: grid of kernel k fully dispatched
+  volatile uint32_t* host_arrive;  // mapped pinned host words: grid of kernel k fully dispatched;
+                                   // [kMaxKernels]: the run aborted as not co-resident
   volatile uint32_t* host_retire;  // mapped pinned host words: every block of kernel k exited on retirement
   uint32_t epoch;                  // run counter written into host_arrive / host_retire
   int8_t stage_group[kMaxStages];  // online adaptation: group of each stage (-1: none / KBK)
+  uint32_t peer_mask;              // planned persistent kernel slots of this run: a block stalled
+                                   // for > kCoresidentNs while one of them has no block resident
+                                   // aborts with ABORT_NOT_CORESIDENT
 };
+constexpr unsigned long long kCoresidentNs = 20000000ull;  // 20 ms
 
 enum : int { MODE_PERSISTENT = 0, MODE_WAVE = 1 };
 
@@ -391,6 +399,7 @@ struct BlockShared {
   unsigned long long nx_base;
   long long acc_neg;                   // completions not yet subtracted from `pending` (<= 0)
   long long wave_rem;                  // WAVE: items of this block's chunk not yet claimed
+  unsigned long long idle_since;       // %globaltimer when the fetcher last started idling (0: busy)
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
@@ -470,6 +479,8 @@ struct Ctx {
         a.c.trace[idx].id = F::template item_id<T>(item);
         a.c.trace[idx].stage = T;
         a.c.trace[idx].smid = smid();
+        a.c.trace[idx].kslot = (uint32_t)a.g.kslot;
+        a.c.trace[idx].block = blockIdx.x;
       }
     }
   }
@@ -492,6 +503,29 @@ struct Ctx {
 // ------------------------------------------------------------------ queue operations
 __device__ __forceinline__ bool aborted(const Ctrl* c) {
   return *(volatile const unsigned long long*)&c->abort.v != 0ull;
+}
+
+// Non-concurrent scheduling (a profiler serialising kernels, MPS, a co-tenant): CUDA does
+// not guarantee that separately launched grids run concurrently, and a coarse/fine/hybrid
+// plan needs every group resident.  A block that has been stalled for kCoresidentNs checks
+// whether some planned kernel still has no block that ran its prologue; if so the run
+// aborts (the host reruns it as one cooperative megakernel, vp_run_stats.model_rerun).
+__device__ __forceinline__ bool peers_missing(const Common& c) {
+  for (uint32_t m = c.peer_mask; m; m &= m - 1) {
+    const int k = __ffs(m) - 1;
+    if (ld_relaxed(&c.ctrl->arrivals[k].v) == 0ull) return true;
+  }
+  return false;
+}
+__device__ __forceinline__ bool check_coresident(const Common& c, unsigned long long stalled_ns) {
+  if (stalled_ns < kCoresidentNs || !c.peer_mask || !peers_missing(c)) return false;
+  if (atomicCAS((unsigned long long*)&c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_NOT_CORESIDENT) == 0ull &&
+      c.host_arrive) {
+    // tell the host thread, which may be waiting for a grid that cannot be dispatched
+    c.host_arrive[kMaxKernels] = c.epoch;
+    __threadfence_system();
+  }
+  return true;
 }
 
 // One thread: claim up to k published items of stage s from its ring.
@@ -545,6 +579,7 @@ __device__ __forceinline__ void wait_slots(const Common& c, const QueueDesc& q, 
       if (ns < 1024) ns <<= 1;
       if (aborted(c.ctrl)) return;
       unsigned long long now = globaltimer();
+      if (mode == 1 && check_coresident(c, now - t0)) return;  // the consumer group never started
       // a producer stuck > 200 ms on a full ring is a capacity failure, not progress
       if (mode == 1 && now - t0 > 200000000ull) {
         atomicCAS((unsigned long long*)&c.ctrl->abort.v, 0ull, (unsigned long long)ABORT_OVERFLOW);
@@ -700,6 +735,15 @@ struct Runner {
     int own = (tg >= 0 && tg == a.g.group) ? myn : 0;
 #pragma unroll
     for (int o = 16; o; o >>= 1) own += __shfl_xor_sync(0xffffffffu, own, o);
+    if (a.g.group >= 0) {
+      // online adaptation: children counted in their target groups BEFORE this group's
+      // completions are subtracted, so no observer can see this group drained (gpend 0)
+      // while its children are not yet counted downstream (the target could otherwise
+      // retire with items in its ring)
+      if (tg >= 0 && tg != a.g.group) red_add(&c->gpend[tg].v, myn);
+      __syncwarp();
+      fence_acq_rel_gpu();
+    }
     if (lane == 0) {
       const long long d = children - completed + sh.acc_neg;
       if (d != 0) red_add(&c->pending.v, d);
@@ -707,7 +751,6 @@ struct Runner {
       if (a.g.group >= 0 && dg != 0) red_add(&c->gpend[a.g.group].v, dg);
       sh.acc_neg = 0;
     }
-    if (tg >= 0 && tg != a.g.group) red_add(&c->gpend[tg].v, myn);
     unsigned long long mybase = 0;
     if (myn > 0) {
       mybase = atom_add(&c->tail[lane].v, myn);
@@ -865,10 +908,14 @@ struct Runner {
             atomicCAS((unsigned long long*)&c->abort.v, 0ull, (unsigned long long)ABORT_TIMEOUT);
             sh.done = 1;
           } else {
-            __nanosleep(256);
+            const unsigned long long now = globaltimer();
+            if (!sh.idle_since) sh.idle_since = now;
+            if (check_coresident(a.c, now - sh.idle_since)) sh.done = 1;
+            else __nanosleep(256);
           }
         }
       }
+      if (got) sh.idle_since = 0;
       sh.nx_stage = st;
       sh.nx_n = got;
       sh.nx_base = base;
@@ -948,6 +995,8 @@ struct Runner {
             a.c.trace[idx].id = F::template item_id<SS>(items + k * F::stride(SS));
             a.c.trace[idx].stage = SS;
             a.c.trace[idx].smid = sm;
+            a.c.trace[idx].kslot = (uint32_t)a.g.kslot;
+            a.c.trace[idx].block = blockIdx.x;
           }
         }
       }
@@ -1054,6 +1103,7 @@ struct Runner {
         sh.mbar_phase[b] = 0;
       }
       sh.acc_neg = 0;
+      sh.idle_since = 0;
       sh.done = 0;
       sh.work[0] = sh.work[1] = 0;
       sh.nx_n = 0;

@@ -41,6 +41,7 @@ QB_ITEM4, QB_ITEM16, QB_ITEM272 = 70, 71, 72
 LDPC_INIT, LDPC_C2V, LDPC_V2C, LDPC_PROBVAR = 80, 81, 82, 83
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS, FLAG_ONLINE, FLAG_L2_PERSIST = (
     1, 2, 4, 8, 16, 32, 64)
+FLAG_SERIALIZE_GROUPS, FLAG_NO_RERUN = 0x80, 0x100
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
 P = C.c_void_p
@@ -78,7 +79,7 @@ class RunStats(C.Structure):
                 ("kernel_idle_ns", C.c_uint64 * 16), ("ring_tail", C.c_uint64 * MAX_STAGES),
                 ("ring_head", C.c_uint64 * MAX_STAGES), ("ring_count", C.c_int64 * MAX_STAGES),
                 ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16),
-                ("stage_wave_ms", C.c_float * MAX_STAGES)]
+                ("stage_wave_ms", C.c_float * MAX_STAGES), ("dispatch_timeouts", C.c_int), ("model_rerun", C.c_int)]
 
 
 class AutotuneOpts(C.Structure):
@@ -239,6 +240,7 @@ class Pipeline:
             raise VPError(rc, f"vp_pipeline_create(device={device})")
         self.h = h
         self.device = device
+        self.trace_capacity = trace_capacity if trace_capacity > 0 else (1 << 20)
         self._keep = []
 
     def _check(self, rc, what):
@@ -292,8 +294,21 @@ class Pipeline:
         self._check(vp_get_trace(self.h, C.byref(ptr), C.byref(n)), "vp_get_trace")
         return ptr.value
 
+    TRACE_DTYPE = np.dtype([("id", "<u8"), ("stage", "<u4"), ("smid", "<u4"), ("kslot", "<u4"), ("block", "<u4")])
+
+    def trace(self, stats):
+        """The last run's task trace (VP_FLAG_TRACE) copied to the host: one record per
+        task {id, stage, smid, kslot, block} (vp.h vp_get_trace)."""
+        n = min(int(stats["trace_records"]), int(self.trace_capacity))
+        host = np.zeros(n, self.TRACE_DTYPE)
+        if n:
+            rc = vp_memcpy(C.c_void_p(host.ctypes.data), C.c_void_p(self.trace_ptr()), host.nbytes, 1, None)
+            self._check(rc, "vp_memcpy(trace)")
+        return host
+
     def set_flags(self, flags):
-        """Run-time diagnostics flags (FLAG_QUEUE_DEPTH | FLAG_STRICT_BINDING | FLAG_TIMERS);
+        """Run-time flags (FLAG_QUEUE_DEPTH | FLAG_STRICT_BINDING | FLAG_TIMERS | FLAG_SERIALIZE_GROUPS |
+        FLAG_NO_RERUN);
         returns the previous flags."""
         old = C.c_uint32()
         self._check(vp_set_flags(self.h, flags, C.byref(old)), "vp_set_flags")
@@ -350,7 +365,8 @@ def stats_dict(st: RunStats):
                 kernel_idle_ns=list(st.kernel_idle_ns[:max(nk, 1)]), ring_tail=list(st.ring_tail),
                 ring_head=list(st.ring_head), ring_count=list(st.ring_count), seed_head=list(st.seed_head),
                 pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]),
-                stage_wave_ms=list(st.stage_wave_ms))
+                stage_wave_ms=list(st.stage_wave_ms), dispatch_timeouts=st.dispatch_timeouts,
+                model_rerun=st.model_rerun)
 
 
 def config_to_string(cfg: Config) -> str:

@@ -110,16 +110,8 @@ def test_reyes_trace_multiset(vpm, orc, model):
 
 
 def trace_array(rp, st):
-    """Read the library trace buffer (device) through the binding's memcpy."""
-    import ctypes
-    from paper_conf_micro_zhengozsyc17_b200 import vp
-    n = st["trace_records"]
-    ptr = rp.p.trace_ptr()
-    host = np.zeros(n, np.dtype([("id", "<u8"), ("stage", "<u4"), ("smid", "<u4")]))
-    if n:
-        rc = vp.vp_memcpy(ctypes.c_void_p(host.ctypes.data), ctypes.c_void_p(ptr), host.nbytes, 1, None)
-        assert rc == 0
-    return host
+    """The library trace buffer (device) through the binding's memcpy."""
+    return rp.p.trace(st)
 
 
 @pytest.mark.parametrize("batch", [1, 3, 8])

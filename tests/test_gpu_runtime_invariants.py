@@ -1,0 +1,181 @@
+"""GPU: runtime invariants of SURVEY §8(c-6) checked task by task, the timed configuration
+checked at full size, and the hybrid model under non-concurrent scheduling.
+
+* Binding (Fig. 5, L21: check_sm / check_sm_blk): every traced task ran on an SM of its
+  kernel's mask, inside its kernel's stage range, and no (kernel, SM) hosted more distinct
+  blocks than its quota.
+* The exact configuration bench.py times (the auto-tuner's pick, committed as
+  tests/data/reyes_config5_tuned.cfg) on the full 512-frame config-5 batch: keys, shade
+  factors and colours of frames spread over the orbit (nearest-camera frames included)
+  equal the oracle's, and the conservation identities hold for the whole batch.
+* Groups that cannot be co-resident (VP_FLAG_SERIALIZE_GROUPS reproduces a profiler's
+  kernel serialisation) are detected within a bound and the run is repeated as one
+  cooperative megakernel (or fails fast with VP_FLAG_NO_RERUN).
+* The online adaptation's group counters under repetition (publish order).
+"""
+import os
+import time
+
+import numpy as np
+import pytest
+
+from paper_conf_micro_zhengozsyc17_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+@pytest.fixture(scope="module")
+def vpm():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a GPU")
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    return vp
+
+
+def mask_sms(binding, g, nsm):
+    return {sm for sm in range(nsm) if (binding.group_sm_mask[g][sm >> 5] >> (sm & 31)) & 1}
+
+
+def check_trace_binding(vp, tr, st, kernel_sms, nsm):
+    """Every record: smid in its kernel's SM set, stage in its kernel's range; per (kernel,
+    SM) the distinct blocks are <= the quota (or the kernel's resident limit)."""
+    assert tr.size == st["trace_records"] and tr.size > 0
+    ks = tr["kslot"].astype(np.int64)
+    assert ks.max() < st["num_kernels"]
+    for k, (lo, hi, quota) in enumerate(st["kernels"]):
+        sel = tr[ks == k]
+        if sel.size == 0:
+            continue
+        assert np.all((sel["stage"] >= lo) & (sel["stage"] <= hi)), f"kernel {k} ran a stage outside [{lo},{hi}]"
+        bad = set(np.unique(sel["smid"]).tolist()) - kernel_sms[k]
+        assert not bad, f"kernel {k} ran tasks on SMs {sorted(bad)[:8]} outside its mask"
+        pairs = np.unique(np.stack([sel["smid"].astype(np.int64), sel["block"].astype(np.int64)], 1), axis=0)
+        per_sm = np.bincount(pairs[:, 0], minlength=nsm)
+        cap = quota if quota > 0 else max(st["blocks_on_sm"][k])
+        assert per_sm.max() <= cap + st["fallback_admits"], (k, per_sm.max(), cap)
+
+
+def test_trace_binding_hybrid_reyes(vpm, orc):
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    scene = inputs.reyes_config5(n_frames=8, n_side=16)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_TRACE, trace_capacity=1 << 22)
+    split = 40
+    b = vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, split), (2, 3, vp.GROUP_RTC, split, nsm)], nsm,
+                        blocks_per_sm=[2, 0, 2, 0])
+    rp.configure(vp.HYBRID, b)
+    st = rp.run()
+    tr = rp.p.trace(st)
+    check_trace_binding(vp, tr, st, {0: mask_sms(b, 0, nsm), 1: mask_sms(b, 1, nsm)}, nsm)
+    ref = orc.reyes_pipeline(scene)
+    key, _ = rp.keys()
+    assert np.array_equal(key, ref["key"])
+
+
+def test_trace_binding_fine_collatz(vpm, orc):
+    """Fine pipeline (Fig. 5): two stage kernels share SMs with per-(stage, SM) quotas."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import CollatzPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    cp = CollatzPipeline(inputs.collatz_seeds(50_000), flags=vp.FLAG_TRACE, trace_capacity=1 << 24)
+    b = vp.make_binding([(0, 0, vp.GROUP_FINE, 0, nsm // 2), (1, 1, vp.GROUP_FINE, nsm // 2, nsm)], nsm,
+                        blocks_per_sm=[2, 1])
+    cp.configure(vp.HYBRID, b)
+    steps, seen, st = cp.run()
+    assert np.all(seen == 1)
+    tr = cp.p.trace(st)
+    sms = {}
+    for k, (lo, _, _) in enumerate(st["kernels"]):
+        sms[k] = mask_sms(b, 0 if lo == 0 else 1, nsm)
+    check_trace_binding(vp, tr, st, sms, nsm)
+
+
+def test_bench_tuned_config_full_batch(vpm, orc):
+    """The configuration bench.py times, on the full 512-frame x 4096-patch batch."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    cfg = open(os.path.join(HERE, "data", "reyes_config5_tuned.cfg")).read().strip()
+    if nsm != 148:
+        pytest.skip("the committed tuned config is for a 148-SM B200")
+    scene = inputs.reyes_config5(n_frames=512)
+    rp = ReyesPipeline(scene)
+    rp.p.configure_config(vp.config_from_string(cfg))
+    st = rp.run()
+    st = rp.run()            # the bench times repeated runs of one pipeline
+    d = st["dequeued"]
+    assert d[0] == scene.seeds.size + 2 * d[1] and d[3] == d[2]
+    key, s = rp.keys()
+    col = rp.colours()
+    # nearest camera at f = 32 mod 64 (distance 1.3), farthest at 0 mod 64 (2.5)
+    for f in (0, 32, 75, 96, 160, 224, 288, 352, 416, 480, 511):
+        ref = orc.reyes_pipeline(inputs.reyes_config5(n_frames=1, frame0=f))
+        assert np.array_equal(key[f], ref["key"][0]), f"frame {f}: {(key[f] != ref['key'][0]).sum()} keys differ"
+        assert np.array_equal(s[f], ref["s"][0])
+        assert np.array_equal(col[f], ref["colour"][0])
+
+
+@pytest.mark.parametrize("model", ["hybrid_mega_rtc", "coarse"])
+def test_noncoresident_groups_rerun(vpm, orc, model):
+    """Serialised group grids (what ncu does): detected and rerun as a megakernel, exact."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    scene = inputs.reyes_config1()
+    rp = ReyesPipeline(scene)
+    if model == "coarse":
+        rp.configure(vp.COARSE)
+    else:
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm // 2),
+                                                 (2, 3, vp.GROUP_RTC, nsm // 2, nsm)], nsm))
+    rp.run()
+    assert rp.run()["model_rerun"] == 0
+    rp.p.set_flags(vp.FLAG_SERIALIZE_GROUPS)
+    t0 = time.perf_counter()
+    st = rp.run()
+    wall = time.perf_counter() - t0
+    assert st["model_rerun"] == 1 and wall < 5.0, (st["model_rerun"], wall)
+    ref = orc.reyes_pipeline(scene)
+    key, s = rp.keys()
+    assert np.array_equal(key, ref["key"]) and np.array_equal(rp.colours(), ref["colour"])
+    assert st["dequeued"][:4] == [ref["n_bound"], ref["n_split"], ref["n_dice"], ref["n_shade"]]
+    # fail fast instead of rerunning
+    rp.p.set_flags(vp.FLAG_SERIALIZE_GROUPS | vp.FLAG_NO_RERUN)
+    t0 = time.perf_counter()
+    rc, st, msg = rp.p.run_status()
+    wall = time.perf_counter() - t0
+    assert rc == vp.VP_ERR_UNSUPPORTED and st["abort_reason"] == 5 and wall < 1.0, (rc, st["abort_reason"], wall, msg)
+    # and the planned model works again afterwards
+    rp.p.set_flags(0)
+    st = rp.run()
+    assert st["model_rerun"] == 0
+    key, _ = rp.keys()
+    assert np.array_equal(key, ref["key"])
+
+
+def test_online_adaptation_repeated(vpm, orc):
+    """Online retire/refill (VP_FLAG_ONLINE) run many times: never ends with items left
+    (the group counters are updated children-first)."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline, ToyPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    seeds = inputs.toy_seeds(20_000)
+    tp = ToyPipeline(seeds, flags=vp.FLAG_ONLINE)
+    tp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, 8), (1, 1, vp.GROUP_MEGA, 8, 40),
+                                             (2, 2, vp.GROUP_MEGA, 40, nsm)], nsm))
+    ref_out, ref_deq, _ = orc.toy_pipeline(seeds, inputs.TOY_THRESHOLD)
+    ref_sorted = np.sort(ref_out)
+    for _ in range(40):
+        out, st = tp.run()
+        assert st["dequeued"][:3] == ref_deq and np.array_equal(np.sort(out), ref_sorted)
+    scene = inputs.reyes_config5(n_frames=4, n_side=16)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_ONLINE)
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 16), (2, 3, vp.GROUP_RTC, 16, nsm)], nsm))
+    ref = orc.reyes_pipeline(scene)
+    for _ in range(20):
+        rp.run()
+        key, _ = rp.keys()
+        assert np.array_equal(key, ref["key"])

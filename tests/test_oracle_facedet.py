@@ -100,3 +100,22 @@ def test_planted_templates_detected_and_constant_invariants(orc):
     assert np.array_equal(rc["lut"][0], np.arange(256))                 # N == cmin: identity
     lb = rc["lbp"][0][: 64 * 48].reshape(48, 64)
     assert np.all(lb[1:-1, 1:-1] == 255) and lb[0].sum() == lb[-1].sum() == 0
+
+
+def test_grayscale_bins_against_bt601(orc):
+    """Face detection's own grayscale (oracle/facedet.c, reading R-D1) against float64
+    BT.601 luma: a constant frame of colour c puts all its pixels into one histogram bin,
+    which must be within one grey level of round(0.299 R + 0.587 G + 0.114 B)."""
+    from paper_conf_micro_zhengozsyc17_b200 import inputs
+    base = inputs.face_scene(W=24, H=24, n_frames=1, n_planted=0)
+    rng = np.random.default_rng(601)
+    cols = np.concatenate([rng.integers(0, 256, (250, 3)), [[0, 0, 0], [255, 255, 255], [255, 0, 0], [0, 255, 0],
+                                                            [0, 0, 255], [128, 128, 128]]]).astype(np.uint8)
+    rgb = np.broadcast_to(cols[:, None, None, :], (cols.shape[0], 24, 24, 3)).copy()
+    sc = inputs.FaceScene(W=24, H=24, rgb=rgb, n_weak=base.n_weak, thr=base.thr, weak=base.weak,
+                          planted=np.zeros((cols.shape[0], 0, 2), np.int32))
+    res = orc.fd_definition(sc)
+    for f, c in enumerate(cols.astype(np.float64)):
+        nz = np.nonzero(res["hist"][f])[0]
+        assert nz.size == 1 and res["hist"][f][nz[0]] == 24 * 24
+        assert abs(int(nz[0]) - int(np.rint(0.299 * c[0] + 0.587 * c[1] + 0.114 * c[2]))) <= 1, (c, nz[0])

@@ -102,3 +102,24 @@ def test_constant_image_constant_pyramid(orc):
     p = orc.pyr_pipeline(rgb)
     y = (77 * 90 + 150 * 90 + 29 * 90 + 128) >> 8
     assert np.all(p["pyr"] == y)          # LUT = identity, box filter keeps constants
+
+
+def test_grayscale_weights_against_bt601(orc):
+    """Reading R-P1's integer weights (77, 150, 29)/256 against ITU-R BT.601 luma in float64,
+    Y = 0.299 R + 0.587 G + 0.114 B: the oracle's level-0 gray image is within one grey level
+    of round(Y) for every (R, G) pair and 64 blue values (4 Mi colours, the extremes
+    included), and exact on the neutral axis R = G = B (where Y = R)."""
+    r, g = np.meshgrid(np.arange(256), np.arange(256), indexing="ij")
+    blues = np.unique(np.concatenate([np.linspace(0, 255, 63).astype(int), [128]]))
+    assert blues.size == 64 and blues[0] == 0 and blues[-1] == 255
+    rgb = np.zeros((2048, 2048, 3), np.uint8)
+    tiles = rgb.reshape(8, 256, 8, 256, 3)
+    for k, b in enumerate(blues):
+        t = tiles[k // 8, :, k % 8, :, :]
+        t[..., 0], t[..., 1], t[..., 2] = r, g, b
+    res = orc.pyr_definition(rgb[None])
+    gray = res["gray"][0].reshape(2048, 2048).astype(np.int64)
+    y = np.rint(0.299 * rgb[..., 0] + 0.587 * rgb[..., 1] + 0.114 * rgb[..., 2]).astype(np.int64)
+    assert np.max(np.abs(gray - y)) <= 1
+    neutral = (rgb[..., 0] == rgb[..., 1]) & (rgb[..., 1] == rgb[..., 2])
+    assert neutral.sum() >= 64 and np.array_equal(gray[neutral], rgb[..., 0][neutral].astype(np.int64))
