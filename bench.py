@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--tune-seconds", type=float, default=30.0)
     ap.add_argument("--split", type=int, default=44, help="SMs for the [Bound,Split] group (hybrid)")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--e2e-chunk", type=int, default=64, help="frames per chunk of the streamed e2e render")
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-suite", action="store_true", help="skip the configs 1-4 secondary measurements")
     ap.add_argument("--suite-tune-seconds", type=float, default=8.0)
@@ -369,6 +370,49 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         per_img = 3 * S * S + (3 * S * S + S * S) + sum(((S >> l) ** 2) * 5 for l in range(1, 13))
         out["pyramid_config3"] = measure(PyramidPipeline(rgb), n_img, alg_bytes=n_img * per_img)
 
+    def w_pyr_fig13():
+        # PAPER.md Fig. 13 (L53-L55): the pyramid at 1..32 images under KBK, KBK with
+        # streams (M25: images split over 8 streams, one host thread each), the megakernel
+        # and the auto-tuned pipeline
+        from paper_conf_micro_zhengozsyc17_b200.workloads import PyramidKbkStreams
+        S = 4096
+        rgb_all = torch.from_numpy(inputs.pyramid_images(32, S)).cuda()
+        rows = []
+        for n_img in (1, 2, 4, 8, 16, 32):
+            rgb = rgb_all[:n_img]
+            pp = PyramidPipeline(rgb, rgb_on_device=rgb)
+            row = {"images": n_img}
+
+            def t(fn, reps=3):
+                fn()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                ts = []
+                for _ in range(reps):
+                    torch.cuda.synchronize()
+                    e0.record(stream)
+                    fn()
+                    e1.record(stream)
+                    torch.cuda.synchronize()
+                    ts.append(e0.elapsed_time(e1))
+                return min(ts)
+
+            pp.configure(vp.KBK)
+            row["kbk_ms"] = t(lambda: pp.run(stream))
+            ks = PyramidKbkStreams(rgb, 8)
+            row["kbk_streams_ms"] = t(lambda: ks.run(stream))
+            row["kbk_streams"] = ks.n_streams
+            del ks
+            pp.configure(vp.MEGAKERNEL)
+            row["megakernel_ms"] = t(lambda: pp.run(stream))
+            best, _ = pp.p.autotune(time_budget_s=min(tune_s, 4.0), sm_granularity=8, batch_choices=(1, 2))
+            row["versapipe_ms"] = t(lambda: pp.run(stream))
+            row["versapipe_config"] = vp.config_to_string(best).split(" mask")[0]
+            row["images_per_s"] = {k[:-3]: n_img / (row[k] / 1e3) for k in ("kbk_ms", "kbk_streams_ms", "megakernel_ms",
+                                                                           "versapipe_ms")}
+            rows.append(row)
+            del pp
+        out["pyramid_fig13"] = rows
+
     def w_cfd():
         cs = inputs.cfd_scene(G=4096, n_outer=10)
         out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
@@ -395,7 +439,8 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
 
     for name, fn in (("reyes_config1", w_reyes1), ("reyes_config1_x256", w_reyes1x), ("facedet_config2", w_face),
                      ("facedet_config2_x8", w_face8), ("pyramid_config3", w_pyr), ("cfd_config3", w_cfd),
-                     ("ldpc_f3", w_ldpc), ("raster_config4", w_raster), ("raster_near_clip", w_raster_near)):
+                     ("ldpc_f3", w_ldpc), ("raster_config4", w_raster), ("raster_near_clip", w_raster_near),
+                     ("pyramid_fig13", w_pyr_fig13)):
         guarded(name, fn)
     return out
 
@@ -535,33 +580,38 @@ def main():
                 extra[name]["launches_per_step"] = 2 * int(bst["kbk_launches"]) + int(bst["kbk_launches"]) // n_st
         rp.p.configure_config(main_cfg)
 
-    # ---- e2e through the public API with HOST buffers: H2D seeds + run + D2H colours
+    # ---- e2e through the public API with HOST buffers: every step uploads all of its seed
+    # items and camera matrices from pinned host memory and downloads every colour buffer
+    # (workloads.ReyesStream: chunks of frames, copies on two copy streams overlapping the
+    # runs of the previous / next chunk, same tuned configuration)
     e2e = None
     if not args.no_e2e:
+        from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesStream
+        rs = ReyesStream(scene, chunk=args.e2e_chunk)
+        rs.configure_config(main_cfg)
         host_seeds = torch.from_numpy(scene.seeds.view(np.uint8).reshape(-1).copy()).pin_memory()
-        host_out = torch.empty(rp.colour.shape, dtype=torch.float32).pin_memory()
+        host_M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).pin_memory()
+        host_out = torch.empty((scene.n_frames, scene.H, scene.W, 4), dtype=torch.float32).pin_memory()
         e_steps = max(1, min(args.steps, 5))
-        for _ in range(2):
-            rp.p.insert(0, host_seeds.numpy(), n=scene.seeds.size, replace=True, stream=stream)
-            rp.run(stream)
-            host_out.copy_(rp.colour, non_blocking=True)
+        rs.render(host_seeds, host_M, host_out, stream=stream, steps=1)
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        for _ in range(e_steps):
-            rp.p.insert(0, host_seeds.numpy(), n=scene.seeds.size, replace=True, stream=stream)
-            rp.run(stream)
-            host_out.copy_(rp.colour, non_blocking=True)
+        rs.render(host_seeds, host_M, host_out, stream=stream, steps=e_steps)
         e1.record(stream)
         torch.cuda.synchronize()
         et = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device="cuda")
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e = {"value": frames_all * e_steps / (float(et.item()) / 1e3), "unit": "frames/s",
-               "h2d_bytes_per_step": int(host_seeds.numel()) * world,
-               "d2h_bytes_per_step": int(host_out.numel() * 4) * world}
-        # restore device-resident seeds
-        rp.p.insert(0, rp.seeds_dev, n=scene.seeds.size, replace=True)
+               "h2d_bytes_per_step": (int(host_seeds.numel()) + int(host_M.numel()) * 4) * world,
+               "d2h_bytes_per_step": int(host_out.numel() * 4) * world, "steps": e_steps,
+               "chunk_frames": args.e2e_chunk,
+               "how": "workloads.ReyesStream: pinned host seeds + matrices -> device, vp_run per chunk "
+                      "(vp_set_params), colours -> pinned host; copies overlap the neighbouring chunks' runs"}
+        # the e2e output is the same render: spot-check it against the timed run's snapshot
+        e2e["matches_timed_run"] = bool(all(np.array_equal(host_out[f - f0].numpy(), snap[f][2]) for f in snap))
+        del rs
 
     # ---- NCCL output gather (config 5), timed separately
     gather_ms = None

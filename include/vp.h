@@ -280,7 +280,11 @@ typedef struct vp_collatz_params {
 } vp_collatz_params;
 
 typedef struct vp_reyes_params {
-  int32_t W, H, n_frames, patches_per_frame, max_depth, pad0;
+  int32_t W, H, n_frames, patches_per_frame, max_depth;
+  int32_t frame_base;        /* item ids carry global frame numbers (id = frame << 12 |    */
+                             /* patch); this run renders frames [frame_base, frame_base +   */
+                             /* n_frames): M, fb and colour are indexed by frame - frame_base */
+                             /* (0 for a whole batch; vp_set_params moves it per chunk)     */
   float t_dice, near_w;
   const float* M;            /* [n_frames][16] view-projection, row-major                  */
   const float* albedo;       /* [patches_per_frame][4]                                     */
@@ -408,6 +412,12 @@ vp_status vp_profile(void* p, int* max_blocks_per_sm, int* regs_per_thread, int*
  * VP_FLAG_TIMERS, VP_FLAG_SERIALIZE_GROUPS, VP_FLAG_NO_RERUN; the others are fixed at create
  * and rejected with VP_ERR_INVALID).  old_flags (optional) receives all flags before the change. */
 vp_status vp_set_flags(void* p, uint32_t flags, uint32_t* old_flags);
+
+/* Replace the family parameter struct between runs (same family, same params_bytes; it
+ * is validated like the one given to vp_stage_register).  E.g. the next chunk of frames of
+ * a streamed batch (vp_reyes_params.frame_base, M).  VP_ERR_INVALID on a size mismatch or
+ * invalid parameters; the previous parameters then stay in force. */
+vp_status vp_set_params(void* p, const void* params, size_t params_bytes);
 
 /* Library-owned / borrowed outputs of the family (sink results). index 0 = primary. */
 vp_status vp_get_output(void* p, int index, void** dev_ptr, size_t* bytes);

@@ -222,6 +222,7 @@ struct ReyesF {
   // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
   static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
     // block-local [Bound, Split]: the first stack pass takes the whole claimed batch
+    if (!rtc && lo == BOUND && hi == SPLIT && (s == BOUND || s == SPLIT)) return s == BOUND ? 32 : 16;  // DFS kernel
     if (!rtc && lo == BOUND && hi >= SPLIT && (s == BOUND || s == SPLIT)) return 16;
     return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
   }
@@ -239,7 +240,8 @@ struct ReyesF {
   // at the edge of 2 blocks per SM)
   static constexpr int scratch_bytes_k(int lo, int hi, bool rtc) {
     return ((rtc && lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
-           ((!rtc && lo == BOUND && hi >= SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
+           ((!rtc && lo == BOUND && hi == SPLIT) ? (int)((sizeof(DfsScratch) + 127) / 128 * 128) : 0) +
+           ((!rtc && lo == BOUND && hi > SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
   }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
@@ -275,11 +277,19 @@ struct ReyesF {
   // patches of a batch and their children almost always share the frame)
   static __device__ __forceinline__ int bound_patch(const Params& p, const RPatch* P, int lane, bool valid, int& dir,
                                                     float4& q, const float4* Mc = nullptr, uint32_t mframe = ~0u) {
-    const uint32_t depth = P->depth;
-    uint32_t frame = P->id >> 12;
-    if (frame >= (uint32_t)p.n_frames) frame = 0;
-    const float* M = p.M + 16 * (size_t)frame;
+    uint32_t frame = frame_of(p, P->id);
     q = P->cp[lane];
+    return bound_q(p, q, P->depth, frame, lane, valid, dir, Mc, mframe);
+  }
+  // local frame index of an item id (frame << 12 | patch) in this run's matrices
+  static __device__ __forceinline__ uint32_t frame_of(const Params& p, uint32_t id) {
+    uint32_t frame = (id >> 12) - (uint32_t)p.frame_base;
+    return frame >= (uint32_t)p.n_frames ? 0u : frame;
+  }
+  // Bound on a patch held in registers (lane = control point q of a 16-thread group).
+  static __device__ __forceinline__ int bound_q(const Params& p, const float4 q, uint32_t depth, uint32_t frame,
+                                                int lane, bool valid, int& dir, const float4* Mc, uint32_t mframe) {
+    const float* M = p.M + 16 * (size_t)frame;
     float4 c;
     if (Mc && frame == mframe) {
       float cc[4];
@@ -462,12 +472,193 @@ struct ReyesF {
     return t == BOUND ? kStack : t == DICE ? kLocalDice : (t == SHADE && hi >= DICE) ? 8 : 0;
   }
 
+  // -------------------------------------------------------------- [Bound, Split] DFS
+  // The [Bound, Split] group's own kernel (hi == Split): each warp works
+  // claimed patches' split trees depth first, two nodes at a time (one per 16-thread group,
+  // lane = control point, the node in registers): Bound, then either stage a Dice item,
+  // cull, or split with de Casteljau over shuffles, keep the left child in registers and
+  // push the right one on the warp's shared-memory stack.  A group without a node pops the
+  // warp's stack (so both groups stay busy while either tree has pending children) and
+  // only then claims the next item of the batch.  No block barrier: the warp's Dice items
+  // are staged in shared memory and published by the warp itself (Ctx::publish_warp), and
+  // the kernel is a sink group (no publisher warp), so warps go on to the next batch as
+  // they finish.
+  static constexpr int kDfsStack = 16;  // pending right children per warp: <= 2 root paths of <= 8
+  static constexpr int kDfsStage = 8;   // Dice items a warp stages before publishing them
+  struct DfsScratch {
+    RPatch stack[kWarpsW][kDfsStack];
+    RPatch stage[kWarpsW][kDfsStage];
+    float4 M[2 * kWarpsW][4];            // each group's current frame matrix (rows)
+    uint32_t mframe[2 * kWarpsW];        // its frame + 1 (0: none; scratch starts zeroed)
+  };
+  static constexpr bool direct_publish(int lo, int hi, bool rtc) { return !rtc && lo == BOUND && hi == SPLIT; }
+  static constexpr int direct_out_cap(int, int, int t) { return t == DICE ? kWarpsW * kDfsStage : 0; }
+
+  static __device__ __forceinline__ float4 shfl4(unsigned m, float4 v, int src) {
+    return make_float4(__shfl_sync(m, v.x, src, 16), __shfl_sync(m, v.y, src, 16), __shfl_sync(m, v.z, src, 16),
+                       __shfl_sync(m, v.w, src, 16));
+  }
+
+  template <int SS, class Ctx>
+  static __device__ void exec_dfs(Ctx& ctx, const uint8_t* items, int n) {
+    const Params& p = ctx.params();
+    DfsScratch& ds = *(DfsScratch*)ctx.scratch();
+    const int lane = threadIdx.x & 15, hw = threadIdx.x >> 4, half = hw & 1, warp = threadIdx.x >> 5;
+    const unsigned hmask = 0xFFFFu << (16 * half);
+    int* next = ctx.work_counter();
+    RPatch* const stk = ds.stack[warp];
+    RPatch* const stage = ds.stage[warp];
+    int wsp = 0, wcnt = 0, nb = 0, nsp = 0;  // wsp, wcnt: warp-uniform
+    bool have = false, first = false, presplit = false, drained = false;
+    float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
+    uint32_t id = 0, path = 0, dirs = 0, depth = 0;
+    for (;;) {
+      // groups without a node: the warp's pending children first, then the batch
+      const unsigned idle = __ballot_sync(0xffffffffu, !have && lane == 0);  // bit 0 / bit 16
+      if (idle) {
+        const int nidle = __popc(idle), rank = (half && (idle & 1u)) ? 1 : 0;
+        const int from_stack = min(nidle, wsp);
+        bool failed = false;
+        if (!have) {
+          if (rank < from_stack) {
+            const RPatch* e = &stk[wsp - 1 - rank];
+            q = e->cp[lane];
+            id = e->id;
+            path = e->path;
+            dirs = e->dirs;
+            depth = e->depth;
+            have = true;
+            first = presplit = false;
+          } else if (!drained) {  // dynamic hand-out of the claimed batch
+            int k = 0;
+            if (lane == 0) k = atomicAdd(next, 1);
+            k = __shfl_sync(hmask, k, 0, 16);
+            if (k < n) {
+              const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
+              q = P->cp[lane];
+              id = P->id;
+              path = P->path;
+              dirs = P->dirs;
+              depth = P->depth;
+              have = first = true;
+              presplit = SS == SPLIT;  // a claimed Split item: its Bound already chose the direction
+            } else {
+              failed = true;
+            }
+          }
+        }
+        wsp -= from_stack;
+        drained |= __any_sync(0xffffffffu, failed);
+        __syncwarp();  // the pops' reads come before this step's pushes
+      }
+      if (!__any_sync(0xffffffffu, have)) break;
+      const uint32_t frame = frame_of(p, id);
+      if (have && ds.mframe[hw] != frame + 1) {
+        __syncwarp(hmask);  // the group's last reads of the old rows are done
+        ((float*)ds.M[hw])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+        if (lane == 0) ds.mframe[hw] = frame + 1;
+        __syncwarp(hmask);
+      }
+      int dir = 0;
+      int cls = bound_q(p, q, depth, frame, lane, have && !presplit, dir, ds.M[hw], ds.mframe[hw] - 1);
+      if (presplit) {
+        cls = 1;
+        dir = (int)((dirs >> depth) & 1u);
+      }
+      const unsigned long long node = ((unsigned long long)id << 12) | ((unsigned long long)(depth & 15u) << 8) | (path & 0xFFu);
+      if (have && !presplit && !first) {  // a Bound task that never went through a ring
+        ++nb;
+        if (lane == 0) ctx.template trace_local_id<BOUND>(node);
+      }
+      // Dice: stage the leaf in the warp's buffer (both groups may add one this step)
+      const bool leaf = have && cls == 2;
+      const unsigned lb = __ballot_sync(0xffffffffu, leaf && lane == 0);
+      if (leaf) {
+        RPatch* out = &stage[wcnt + ((half && (lb & 1u)) ? 1 : 0)];
+        out->cp[lane] = q;
+        if (lane == 0) {
+          out->id = id;
+          out->path = path;
+          out->dirs = dirs;
+          out->depth = depth;
+        }
+      }
+      wcnt += __popc(lb);
+      const bool split = have && cls == 1;
+      const unsigned sb = __ballot_sync(0xffffffffu, split && lane == 0);
+      if (split) {
+        const int slot = wsp + ((half && (sb & 1u)) ? 1 : 0);
+        if (slot >= kDfsStack) {  // deeper than max_depth allows (cannot happen for valid seeds)
+          ctx.abort(ABORT_GUARD);
+          have = false;
+        } else {
+          // de Casteljau at 1/2 (reading R-R6) of the curve through this lane's control point
+          // along the split direction; same operations as split_cp, points from shuffles
+          const int base = dir == 0 ? (lane & 3) : (lane & ~3), step = dir == 0 ? 4 : 1;
+          const int t = dir == 0 ? (lane >> 2) : (lane & 3);
+          const float4 a = shfl4(hmask, q, base), b = shfl4(hmask, q, base + step);
+          const float4 c = shfl4(hmask, q, base + 2 * step), d = shfl4(hmask, q, base + 3 * step);
+          float4 L, R;
+#define VP_CASTELJAU(comp)                                                   \
+  {                                                                          \
+    float ab = (a.comp + b.comp) * 0.5f, bc = (b.comp + c.comp) * 0.5f;      \
+    float cd = (c.comp + d.comp) * 0.5f;                                     \
+    float abc = (ab + bc) * 0.5f, bcd = (bc + cd) * 0.5f;                    \
+    float m = (abc + bcd) * 0.5f;                                            \
+    L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
+    R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
+  }
+          VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+#undef VP_CASTELJAU
+          if (!(first && presplit)) {  // a claimed Split item was counted when it was claimed
+            ++nsp;
+            if (lane == 0) ctx.template trace_local_id<SPLIT>(node);
+          }
+          const uint32_t ndirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
+          RPatch* r = &stk[slot];
+          r->cp[lane] = R;
+          if (lane == 0) {
+            r->id = id;
+            r->path = path | (1u << depth);
+            r->dirs = ndirs;
+            r->depth = depth + 1;
+          }
+          q = L;
+          path &= ~(1u << depth);
+          dirs = ndirs;
+          depth += 1;
+          first = presplit = false;
+        }
+      } else if (have) {
+        have = false;  // diced or culled: the next node comes from the stack or the batch
+      }
+      wsp = min(wsp + __popc(sb), kDfsStack);
+      if (wcnt > kDfsStage - 2) {  // warp-uniform
+        __syncwarp();
+        ctx.template publish_warp<DICE>((const uint8_t*)stage, wcnt);
+        wcnt = 0;
+      }
+    }
+    if (wcnt > 0) {
+      __syncwarp();
+      ctx.template publish_warp<DICE>((const uint8_t*)stage, wcnt);
+    }
+    if (lane == 0) {
+      ctx.template note_local_count_atomic<BOUND>(nb);
+      ctx.template note_local_count_atomic<SPLIT>(nsp);
+    }
+  }
+
   template <int SS, int LO, int HI, class Ctx>
   static __device__ void exec_local(Ctx& ctx, const uint8_t* items, int n) {
     if constexpr (SS == DICE || SS == SHADE) {  // a megakernel's later stages run as usual
       exec<SS>(ctx, items, n);
       return;
+    } else if constexpr (HI == SPLIT) {
+      exec_dfs<SS>(ctx, items, n);
+      return;
     }
+
     const Params& p = ctx.params();
     LocalStack& ls = *(LocalStack*)ctx.scratch();
     const int lane = threadIdx.x & 15, grp = threadIdx.x >> 4;
@@ -491,8 +682,7 @@ struct ReyesF {
     }
     if (threadIdx.x == 0) ls.nchild[0] = ls.nchild[1] = ls.nsplit = 0;
     {
-      uint32_t frame = ((const RPatch*)items)->id >> 12;
-      if (frame >= (uint32_t)p.n_frames) frame = 0;
+      uint32_t frame = frame_of(p, ((const RPatch*)items)->id);
       if (threadIdx.x < 16) ((float*)ls.M)[threadIdx.x] = __ldg(p.M + 16 * (size_t)frame + threadIdx.x);
       if (threadIdx.x == 0) ls.mframe = frame;
     }
@@ -582,8 +772,7 @@ struct ReyesF {
   template <bool kSmemM = false>
   static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
                                                     const float4* Ms = nullptr, const float* Bt = nullptr) {
-    uint32_t frame = P->id >> 12;
-    if (frame >= (uint32_t)p.n_frames) frame = 0;
+    const uint32_t frame = frame_of(p, P->id);
     const float* M = p.M + 16 * (size_t)frame;
     for (int e = lane; e < 4 * kNG; e += 32) {  // C_a(v_j), e = 9a + j
       const int a = e / kNG, j = e - a * kNG;
@@ -692,7 +881,7 @@ struct ReyesF {
   // Micropolygon q = 8i + j of grid Gd: the quad (i,j)..(i+1,j+1), split into the
   // triangles (v0,v1,v2), (v0,v2,v3) (reading R-R8..R-R10).
   static __device__ __forceinline__ void shade_mp(const Params& p, const RGrid* Gd, int q) {
-    const uint32_t frame = Gd->id >> 12, patch = Gd->id & 0xFFFu;
+    const uint32_t frame = (Gd->id >> 12) - (uint32_t)p.frame_base, patch = Gd->id & 0xFFFu;
     if (frame >= (uint32_t)p.n_frames) return;
     const int i = q >> 3, j = q & 7;
     const int g00 = i * kNG + j, g10 = (i + 1) * kNG + j, g01 = i * kNG + j + 1, g11 = (i + 1) * kNG + j + 1;
@@ -799,7 +988,7 @@ struct ReyesF {
 
   // shade_mp's early exit alone: does micropolygon q's box hold a pixel centre?
   static __device__ __forceinline__ bool mp_box(const Params& p, const RGrid* Gd, int q) {
-    if ((Gd->id >> 12) >= (uint32_t)p.n_frames) return false;
+    if ((Gd->id >> 12) - (uint32_t)p.frame_base >= (uint32_t)p.n_frames) return false;
     const int i = q >> 3, j = q & 7;
     const int gi[4] = {i * kNG + j, (i + 1) * kNG + j, (i + 1) * kNG + j + 1, i * kNG + j + 1};
     int vx[4], vy[4];
@@ -855,8 +1044,7 @@ struct ReyesF {
         if (j >= np) break;
         RGrid* g = j ? g1 : g0;
         const RPatch* P = (const RPatch*)(items + (size_t)(k + j) * sizeof(RPatch));
-        uint32_t frame = P->id >> 12;
-        if (frame >= (uint32_t)p.n_frames) frame = 0;
+        const uint32_t frame = frame_of(p, P->id);
         __syncwarp();  // the previous patch's dice is done with the matrix
         if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
         __syncwarp();

@@ -104,7 +104,24 @@ struct FamilyImpl final : FamilyOps {
     }
     return 0;
   }
-  int out_cap(int lo, int hi, bool rtc, int t) const override { return out_cap_of<0, 0>(lo, hi, rtc, t); }
+  template <int LO, int HI>
+  int direct_cap_of(int lo, int hi, bool rtc, int t) const {
+    if constexpr (LO < F::S) {
+      if constexpr (HI < F::S) {
+        if (lo == LO && hi == HI) return direct_out_cap<F>(LO, HI, rtc, t);
+        return direct_cap_of<LO, HI + 1>(lo, hi, rtc, t);
+      } else {
+        return direct_cap_of<LO + 1, LO + 1>(lo, hi, rtc, t);
+      }
+    }
+    return 0;
+  }
+  // items one block of kernel [lo, hi] can have in flight to t: its out buffer, or what
+  // its warps publish at once in a direct-publish kernel
+  int out_cap(int lo, int hi, bool rtc, int t) const override {
+    const int d = direct_cap_of<0, 0>(lo, hi, rtc, t);
+    return d > 0 ? d : out_cap_of<0, 0>(lo, hi, rtc, t);
+  }
   bool local_rec(int lo, int hi, bool rtc) const override { return local_recursion<F>(lo, hi, rtc); }
   bool rtc_legal(int lo, int hi) const override { return fn[lo][hi][1] != nullptr; }
   bool latched(int lo, int hi) const override { return !F::rtc_ok(lo, hi); }

@@ -1129,6 +1129,18 @@ vp_status vp_get_config(void* h, vp_config* out) {
   return VP_OK;
 }
 
+vp_status vp_set_params(void* h, const void* params, size_t params_bytes) {
+  vp_pipeline_s* p = (vp_pipeline_s*)h;
+  if (!p || !params) return VP_ERR_INVALID;
+  if (!p->fam) return fail(p, VP_ERR_INVALID, "vp_set_params before vp_stage_register");
+  if (params_bytes != p->fam->params_bytes())
+    return fail(p, VP_ERR_INVALID, "params_bytes %zu != %zu", params_bytes, p->fam->params_bytes());
+  const char* v = p->fam->validate(params);
+  if (v) return fail(p, VP_ERR_INVALID, "%s", v);
+  p->params.assign((const uint8_t*)params, (const uint8_t*)params + params_bytes);
+  return VP_OK;
+}
+
 vp_status vp_get_output(void* h, int index, void** dev_ptr, size_t* bytes) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;
   if (!p || !dev_ptr || !bytes) return VP_ERR_INVALID;

@@ -333,6 +333,26 @@ struct LocalRec<F, true> {
   }
 };
 
+// A family may let the worker warps of a kernel [lo, hi] publish their ring outputs
+// themselves (F::direct_publish(lo, hi, rtc), through Ctx::publish_warp): the kernel then
+// has no block out buffers and runs as a sink group (no publisher warp, no round
+// barrier), so warps that finish their share of a batch go on to the next one.
+// F::direct_out_cap(lo, hi, t) is what one block can have in flight to t (ring sizing).
+template <class F, class = void>
+struct HasDirect : std::false_type {};
+template <class F>
+struct HasDirect<F, std::void_t<decltype(F::direct_publish(0, 0, false))>> : std::true_type {};
+template <class F>
+constexpr bool direct_publish(int lo, int hi, bool rtc) {
+  if constexpr (HasDirect<F>::value) return F::direct_publish(lo, hi, rtc);
+  else return false;
+}
+template <class F>
+constexpr int direct_out_cap(int lo, int hi, bool rtc, int t) {
+  if constexpr (HasDirect<F>::value) return F::direct_publish(lo, hi, rtc) ? F::direct_out_cap(lo, hi, t) : 0;
+  else return 0;
+}
+
 // ------------------------------------------------------------------ constexpr graph helpers
 template <class F>
 struct Graph {
@@ -357,6 +377,7 @@ struct Graph {
   }
   // out-buffer capacity (items) for target t in a kernel [lo,hi]
   static constexpr int out_cap(int lo, int hi, bool rtc, int t) {
+    if (direct_publish<F>(lo, hi, rtc)) return 0;  // no block out buffers
     if (rtc && lo < t && t <= hi && fused_chain<F>(lo, hi)) return fused_local_cap<F>(lo, hi, t);
     if (local_recursion<F>(lo, hi, rtc)) return local_out_cap<F>(lo, hi, t);
     int c = 0;
@@ -402,6 +423,8 @@ struct BlockShared {
   unsigned long long idle_since;       // %globaltimer when the fetcher last started idling (0: busy)
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
+  uint32_t deq32[kMaxStages], enq32[kMaxStages];  // counts added by several warps at once (native
+                                                  // 32-bit shared atomics; 64-bit ones are CAS loops)
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
   unsigned long long mbar[2];          // bulk-copy completion, one per in buffer
   uint32_t mbar_phase[2];
@@ -410,6 +433,13 @@ struct BlockShared {
   unsigned long long full[2], empty[2];  // mbarriers: fetcher -> workers, workers -> fetcher
   int bn[2], bstage[2];                // items (-1: stop) and stage of each in buffer
 };
+
+// queue helpers defined below, used by Ctx::publish_warp
+__device__ __forceinline__ void wait_slots(const Common& c, const QueueDesc& q, unsigned long long base, int n,
+                                           int mode, int lane);
+template <int STRIDE>
+__device__ __forceinline__ void copy_out(uint8_t* ring, const uint8_t* src, unsigned long long base, int n,
+                                         uint32_t cap_log2, int lane);
 
 __device__ __forceinline__ void worker_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory"); }
 
@@ -470,6 +500,53 @@ struct Ctx {
     sh.deq[T] += (unsigned long long)n;
     sh.enq[T] += (unsigned long long)n;  // entered stage T block-locally (sum enq == sum deq holds)
   }
+  // As note_local_count, from any number of threads at once (direct-publish kernels,
+  // whose warps run independently).
+  template <int T>
+  __device__ __forceinline__ void note_local_count_atomic(int n) {
+    if (n) {
+      atomicAdd(&sh.deq32[T], (uint32_t)n);
+      atomicAdd(&sh.enq32[T], (uint32_t)n);
+    }
+  }
+  // Warp-cooperative enqueue<T> of n <= 32 items staged contiguously in shared memory,
+  // straight from a worker warp (direct-publish kernels; same protocol as the publisher
+  // warp's: children counted in `pending` before they are visible, tail reservation,
+  // free-slot wait, 16-B .cg payload stores, one release fence, per-slot sequence release,
+  // `count` add).  All 32 lanes call it with the same arguments.
+  template <int T>
+  __device__ void publish_warp(const uint8_t* items, int n) {
+    const int lane = threadIdx.x & 31;
+    Ctrl* c = a.c.ctrl;
+    const QueueDesc& q = a.c.q[T];
+    unsigned long long base = 0;
+    if (lane == 0) {
+      red_add(&c->pending.v, n);
+      if (a.g.group >= 0) {
+        const int tg = a.c.stage_group[T];
+        if (tg >= 0) red_add(&c->gpend[tg].v, n);
+      }
+      base = atom_add(&c->tail[T].v, n);
+      atomicAdd(&sh.enq32[T], (uint32_t)n);
+      if (a.c.flags & FLAG_DEPTH) {
+        const unsigned long long h = ld_relaxed(&c->head[T].v);
+        const unsigned long long dd = base + n - h;
+        if (dd > c->max_depth[T]) atomicMax(&c->max_depth[T], dd);
+      }
+    }
+    base = __shfl_sync(0xffffffffu, base, 0);
+    const unsigned long long mask = (1ull << q.cap_log2) - 1;
+    bool ok = true;
+    for (int k = lane; k < n; k += 32) ok &= ld_acquire(q.seq + ((base + k) & mask)) == base + k;
+    if (!__all_sync(0xffffffffu, ok)) wait_slots(a.c, q, base, n, 1, lane);
+    __syncwarp();
+    copy_out<F::stride(T)>(q.slots, items, base, n, q.cap_log2, lane);
+    __syncwarp();
+    fence_acq_rel_gpu();
+    for (int k = lane; k < n; k += 32) st_relaxed(q.seq + ((base + k) & mask), base + k + 1);
+    __syncwarp();
+    if (lane == 0) red_add(&c->count[T].v, n);
+  }
   // ... and, with FLAG_TRACE, the trace record of one of them (one thread per item).
   template <int T>
   __device__ __forceinline__ void trace_local(const uint8_t* item) {
@@ -477,6 +554,20 @@ struct Ctx {
       unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
       if (idx < a.c.trace_cap) {
         a.c.trace[idx].id = F::template item_id<T>(item);
+        a.c.trace[idx].stage = T;
+        a.c.trace[idx].smid = smid();
+        a.c.trace[idx].kslot = (uint32_t)a.g.kslot;
+        a.c.trace[idx].block = blockIdx.x;
+      }
+    }
+  }
+  // ... or given the task's item id directly (items that live only in registers).
+  template <int T>
+  __device__ __forceinline__ void trace_local_id(unsigned long long id) {
+    if (a.c.flags & FLAG_TRACE) {
+      unsigned long long idx = atomicAdd(&a.c.ctrl->trace_n.v, 1ull);
+      if (idx < a.c.trace_cap) {
+        a.c.trace[idx].id = id;
         a.c.trace[idx].stage = T;
         a.c.trace[idx].smid = smid();
         a.c.trace[idx].kslot = (uint32_t)a.g.kslot;
@@ -1012,7 +1103,7 @@ struct Runner {
       constexpr int SS = decltype(S_)::value;
       if (s == SS) {
         record_trace(a, SS, items, n);
-        if (threadIdx.x == 0) sh.deq[SS] += n;
+        if (threadIdx.x == 0) atomicAdd(&sh.deq32[SS], (uint32_t)n);  // direct-publish warps add too
         if constexpr (RTC && SS < HI && fused_chain<F>(SS, HI)) {
           FusedChain<F>::template run<SS, HI>(ctx, items, n);
         } else if constexpr (local_recursion<F>(LO, HI, RTC)) {
@@ -1094,6 +1185,7 @@ struct Runner {
       for (int s = 0; s < kMaxStages; ++s) {
         sh.out_cnt[0][s] = sh.out_cnt[1][s] = 0;
         sh.deq[s] = sh.enq[s] = 0;
+        sh.deq32[s] = sh.enq32[s] = 0;
         sh.t_exec[s] = sh.t_flush[s] = 0;
       }
       sh.t_idle = 0;
@@ -1137,8 +1229,9 @@ struct Runner {
       if (sh.acc_neg != 0 && a.g.group >= 0) atom_add(&c->gpend[a.g.group].v, sh.acc_neg);
       sh.acc_neg = 0;
       for (int s = 0; s < S; ++s) {
-        if (sh.deq[s]) atomicAdd(&c->deq[s], sh.deq[s]);
-        if (sh.enq[s]) atomicAdd(&c->enq[s], sh.enq[s]);
+        const unsigned long long dq = sh.deq[s] + sh.deq32[s], eq = sh.enq[s] + sh.enq32[s];
+        if (dq) atomicAdd(&c->deq[s], dq);
+        if (eq) atomicAdd(&c->enq[s], eq);
         if (sh.t_exec[s]) atomicAdd(&c->exec_ns[s], sh.t_exec[s]);
         if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
       }
@@ -1175,12 +1268,14 @@ struct Runner {
   // fetcher hand the two in buffers over through mbarriers instead of a block barrier
   // per round.  A worker warp that finishes its share of batch i starts batch i+1 as
   // soon as the fetcher staged it, instead of waiting for the slowest warp of batch i.
-  static constexpr bool sink_group() {
+  static constexpr bool no_ring_outputs() {
     for (int s = LO; s <= HI; ++s)
       for (int t = 0; t < S; ++t)
         if (F::fanout(s, t) > 0 && !(RTC && t > LO && t <= HI)) return false;
     return true;
   }
+  // ... or its warps publish their outputs themselves (direct-publish kernels)
+  static constexpr bool sink_group() { return direct_publish<F>(LO, HI, RTC) || no_ring_outputs(); }
 
   static __device__ void run_sink(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, uint8_t* smem) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

@@ -115,7 +115,7 @@ class CollatzParams(C.Structure):
 
 class ReyesParams(C.Structure):
     _fields_ = [("W", C.c_int32), ("H", C.c_int32), ("n_frames", C.c_int32), ("patches_per_frame", C.c_int32),
-                ("max_depth", C.c_int32), ("pad0", C.c_int32), ("t_dice", C.c_float), ("near_w", C.c_float),
+                ("max_depth", C.c_int32), ("frame_base", C.c_int32), ("t_dice", C.c_float), ("near_w", C.c_float),
                 ("M", P), ("albedo", P), ("L", C.c_float * 4), ("fb", P), ("colour", P)]
 
 
@@ -167,6 +167,7 @@ vp_get_trace = _decl("vp_get_trace", [P, C.POINTER(P), C.POINTER(C.c_size_t)])
 vp_autotune = _decl("vp_autotune", [P, C.POINTER(AutotuneOpts), C.POINTER(Config), C.POINTER(TuneReport)])
 vp_profile = _decl("vp_profile", [P, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)])
 vp_get_output = _decl("vp_get_output", [P, C.c_int, C.POINTER(P), C.POINTER(C.c_size_t)])
+vp_set_params = _decl("vp_set_params", [P, P, C.c_size_t])
 vp_config_to_string = _decl("vp_config_to_string", [C.POINTER(Config), C.c_char_p, C.c_size_t])
 vp_config_from_string = _decl("vp_config_from_string", [C.c_char_p, C.POINTER(Config)])
 vp_device_info = _decl("vp_device_info", [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)])
@@ -175,7 +176,7 @@ vp_set_flags = _decl("vp_set_flags", [P, C.c_uint32, C.POINTER(C.c_uint32)])
 
 EXPORTED = ["vp_status_string", "vp_last_error", "vp_pipeline_create", "vp_pipeline_destroy", "vp_stage_register",
             "vp_insert", "vp_insert_async", "vp_configure", "vp_configure_config", "vp_get_config", "vp_run",
-            "vp_set_timeout", "vp_get_trace", "vp_autotune", "vp_profile", "vp_get_output", "vp_config_to_string", "vp_config_from_string",
+            "vp_set_timeout", "vp_get_trace", "vp_autotune", "vp_profile", "vp_get_output", "vp_set_params", "vp_config_to_string", "vp_config_from_string",
             "vp_device_info", "vp_memcpy", "vp_set_flags"]
 
 
@@ -334,6 +335,10 @@ class Pipeline:
         rep = TuneReport()
         self._check(vp_autotune(self.h, C.byref(o), C.byref(best), C.byref(rep)), "vp_autotune")
         return best, rep
+
+    def set_params(self, params):
+        """vp_set_params: replace the family parameter struct between runs."""
+        self._check(vp_set_params(self.h, C.cast(C.byref(params), P), C.sizeof(params)), "vp_set_params")
 
     def output(self, index):
         ptr, n = P(), C.c_size_t()

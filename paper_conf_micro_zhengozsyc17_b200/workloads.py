@@ -371,3 +371,140 @@ class ReyesPipeline:
 
     def colours(self):
         return self.colour.cpu().numpy()
+
+
+class ReyesStream:
+    """End-to-end rendering of a frame batch whose inputs and outputs live in (pinned) host
+    memory: the user-facing path behind bench.py's `e2e`.
+
+    The batch is cut into chunks of `chunk` frames rendered by two pipelines in turn.  The
+    seed upload of chunk i+1 (copy stream) and the colour download of chunk i-1 (a second
+    copy stream) run while chunk i renders on the compute stream; vp_set_params moves each
+    pipeline to its chunk (vp_reyes_params.frame_base and the chunk's matrices), so the
+    seed items keep their batch-wide frame ids.  All rendering happens in libvp.so (the
+    same vp_run as a resident batch); this class only orders copies, events and runs."""
+
+    def __init__(self, scene: inputs.ReyesScene, chunk: int, config=None, device: int = 0):
+        import dataclasses
+        F, ppf = scene.n_frames, scene.patches_per_frame
+        if F % chunk:
+            raise ValueError(f"{F} frames are not a multiple of the chunk ({chunk})")
+        dev = _dev(device)
+        self.scene, self.chunk, self.n_chunks, self.dev = scene, chunk, F // chunk, dev
+        sub = dataclasses.replace(scene, n_frames=chunk, M=scene.M[:chunk], seeds=scene.seeds[:chunk * ppf])
+        self.pipes = [ReyesPipeline(sub, device) for _ in range(2)]
+        if config is not None:
+            for rp in self.pipes:
+                rp.p.configure_config(config)
+        self.seed_bytes = chunk * ppf * scene.seeds.dtype.itemsize
+        self.M_dev = torch.empty((2, F, 16), dtype=torch.float32, device=dev)  # per pass parity
+        self.staging = [torch.empty(self.seed_bytes, dtype=torch.uint8, device=dev) for _ in range(2)]
+        self.s_in, self.s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+        self.ev_in = [torch.cuda.Event() for _ in range(2)]      # chunk's seeds landed in staging[b]
+        self.ev_used = [torch.cuda.Event() for _ in range(2)]    # staging[b] copied into pipeline b
+        self.ev_out = [torch.cuda.Event() for _ in range(2)]     # pipeline b's colours downloaded
+        self.ev_M = [torch.cuda.Event() for _ in range(2)]   # a pass's last chunk has rendered
+
+    def configure(self, model, binding=None, batch=0):
+        for rp in self.pipes:
+            rp.configure(model, binding, batch)
+
+    def configure_config(self, cfg):
+        for rp in self.pipes:
+            rp.p.configure_config(cfg)
+
+    def _params(self, b, c, k):
+        rp = self.pipes[b]
+        prm = rp.prm
+        prm.frame_base = c * self.chunk
+        prm.M = self.M_dev[k & 1].data_ptr() + c * self.chunk * 16 * 4
+        rp.p.set_params(prm)
+
+    def render(self, host_seeds: torch.Tensor, host_M: torch.Tensor, host_out: torch.Tensor, stream=None,
+               steps: int = 1):
+        """`steps` passes over the batch: host_seeds (pinned uint8, every frame's seed items),
+        host_M (pinned [F, 16] float32) -> host_out (pinned [F, H, W, 4] float32).  Copies of
+        consecutive passes overlap too.  Returns the last run's stats."""
+        st = stream or torch.cuda.current_stream(self.dev)
+        nC = self.n_chunks
+        out = host_out.view(nC, -1)
+        seeds = host_seeds.view(nC, -1)
+        total = steps * nC
+        st_last = None
+
+        def upload(j):
+            b, c, k = j & 1, j % nC, j // nC
+            with torch.cuda.stream(self.s_in):
+                if c == 0:  # this pass's matrices (64 B per frame), ahead of its first chunk
+                    self.s_in.wait_event(self.ev_M[k & 1])   # pass k-2 is done with this buffer
+                    self.M_dev[k & 1].copy_(host_M, non_blocking=True)
+                self.s_in.wait_event(self.ev_used[b])
+                self.staging[b].copy_(seeds[c], non_blocking=True)
+                self.ev_in[b].record(self.s_in)
+
+        upload(0)
+        for j in range(total):
+            b, c, k = j & 1, j % nC, j // nC
+            rp = self.pipes[b]
+            if j + 1 < total:
+                upload(j + 1)
+            st.wait_event(self.ev_in[b])     # seeds (and matrices) of chunk c are on the device
+            st.wait_event(self.ev_out[b])    # pipeline b's previous colours are downloaded
+            self._params(b, c, k)
+            rp.p.insert(0, self.staging[b], n=self.seed_bytes // self.scene.seeds.dtype.itemsize, replace=True,
+                        stream=st)
+            self.ev_used[b].record(st)
+            st_last = rp.run(st)             # vp_run returns when the chunk is rendered
+            if c == nC - 1:
+                self.ev_M[k & 1].record(st)  # this pass is done with its matrices
+            with torch.cuda.stream(self.s_out):
+                self.s_out.wait_stream(st)
+                out[c].copy_(rp.colour.view(-1), non_blocking=True)
+                self.ev_out[b].record(self.s_out)
+        st.wait_stream(self.s_out)           # events recorded on `st` now cover the downloads
+        return st_last
+
+
+class PyramidKbkStreams:
+    """The paper's "KBK with Stream" baseline (Fig. 13): the images are
+    split over n_streams independent KBK pipelines, each driven by its own host thread on
+    its own CUDA stream, so kernels of different images overlap (the limited parallelism
+    of one image's KBK waves is the problem it addresses).  Same stage kernels and wave
+    loop as VP_KBK (or VP_KBK_GRAPH); no queue is shared between streams."""
+
+    def __init__(self, rgb_dev: torch.Tensor, n_streams: int, model=None, device: int = 0):
+        n = rgb_dev.shape[0]
+        self.n_streams = max(1, min(n_streams, n))
+        bounds = np.linspace(0, n, self.n_streams + 1).astype(int)
+        self.pipes = [PyramidPipeline(rgb_dev[a:b], device=device, rgb_on_device=rgb_dev[a:b])
+                      for a, b in zip(bounds[:-1], bounds[1:])]
+        for pp in self.pipes:
+            pp.configure(vp.KBK if model is None else model)
+        self.streams = [torch.cuda.Stream(_dev(device)) for _ in self.pipes]
+
+    def run(self, stream=None):
+        """One pass over every image; the caller's stream is ordered after all of them."""
+        import threading
+        st = stream or torch.cuda.current_stream()
+        for s in self.streams:
+            s.wait_stream(st)
+        errs = []
+
+        def go(pp, s):
+            try:
+                pp.run(s)
+            except Exception as ex:  # re-raised in the caller
+                errs.append(ex)
+
+        th = [threading.Thread(target=go, args=(pp, s)) for pp, s in zip(self.pipes, self.streams)]
+        for t in th:
+            t.start()
+        for t in th:
+            t.join()
+        if errs:
+            raise errs[0]
+        for s in self.streams:
+            st.wait_stream(s)
+
+    def pyramid(self):
+        return np.concatenate([pp.pyramid() for pp in self.pipes])

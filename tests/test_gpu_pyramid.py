@@ -74,3 +74,19 @@ def test_pyramid_full_size(vpm, orc):
     pp = PyramidPipeline(rgb)
     pp.configure(vpm.MEGAKERNEL)
     check(orc, rgb, pp, pp.run())
+
+
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph"])
+def test_pyramid_kbk_with_streams(vpm, orc, model):
+    """The "KBK with Stream" baseline (L53-L55, Fig. 13): images split over concurrent
+    per-stream KBK pipelines (one host thread each) give the same pyramids."""
+    import torch
+    from paper_conf_micro_zhengozsyc17_b200.workloads import PyramidKbkStreams
+    vp = vpm
+    rgb = inputs.pyramid_images(5, 256)
+    ks = PyramidKbkStreams(torch.from_numpy(rgb).cuda(), 3, model=vp.KBK if model == "kbk" else vp.KBK_GRAPH)
+    assert ks.n_streams == 3
+    for _ in range(2):
+        ks.run()
+        torch.cuda.synchronize()
+        assert np.array_equal(ks.pyramid(), orc.pyr_pipeline(rgb)["pyr"])

@@ -197,3 +197,31 @@ def test_reyes_config1_x256_wide_recursion(vpm, orc, model):
     col = rp.colours()
     for f in (0, 1, 77, 255):
         assert np.array_equal(key[f], ref["key"][0]) and np.array_equal(col[f], ref["colour"][0])
+
+
+@pytest.mark.parametrize("model", ["hybrid_mega_rtc", "megakernel"])
+def test_reyes_stream_host_buffers(vpm, orc, model):
+    """The e2e path (workloads.ReyesStream): chunks of frames re-targeted with vp_set_params
+    (frame_base, matrices) and rendered from pinned host buffers by two pipelines in turn,
+    with copies overlapping runs, twice over the batch; every frame equals the resident
+    single-pipeline render and the oracle."""
+    import torch
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline, ReyesStream
+    scene = inputs.reyes_config5(n_frames=16, n_side=16)
+    rp = ReyesPipeline(scene)
+    configure(vpm, rp, model)
+    rp.run()
+    want = rp.colours()
+    rs = ReyesStream(scene, chunk=4)
+    for p in rs.pipes:
+        configure(vpm, p, model)
+    host_seeds = torch.from_numpy(scene.seeds.view(np.uint8).reshape(-1).copy()).pin_memory()
+    host_M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).pin_memory()
+    host_out = torch.full((16, scene.H, scene.W, 4), -1.0).pin_memory()
+    rs.render(host_seeds, host_M, host_out, steps=2)
+    torch.cuda.synchronize()
+    got = host_out.numpy()
+    assert np.array_equal(got, want)
+    for f in (0, 9):
+        ref = orc.reyes_pipeline(inputs.reyes_config5(n_frames=1, n_side=16, frame0=f))
+        assert np.array_equal(got[f], ref["colour"][0])

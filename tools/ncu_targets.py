@@ -7,6 +7,11 @@ so co-running persistent groups cannot be captured together).
   kbk       : one launch per stage per wave
   raster_{mega,kbk}, raster_near_{mega,kbk} : config 4 / the near-clip raster workload
   bs_mega   : the block-local [Bound,Split] megakernel alone (Dice items left in a full ring)
+  bs_online : the tuned hybrid ([Bound,Split] block-local recursion on 60 SMs | [Dice,Shade]
+              RTC on 88) with online retirement: under ncu's serialisation the [Bound,Split]
+              grid runs alone, parks every Dice item in a full-size ring and retires, then
+              the RTC grid drains them -- so the first vp_kernel launch is the Bound/Split
+              kernel exactly as the bench runs it
   rtc_leaf  : the [Dice,Shade] RTC kernel alone on representative leaf patches
               (tools/reyes_leaves.py: numpy approximation of the Bound/Split recursion)
 """
@@ -37,6 +42,9 @@ if args.target.startswith("raster"):
 elif args.target == "bs_mega":
     scene = inputs.reyes_config5(n_frames=args.frames)
     rp = ReyesPipeline(scene, flags=vp.FLAG_FULL_RINGS)
+elif args.target == "bs_online":
+    scene = inputs.reyes_config5(n_frames=args.frames)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_FULL_RINGS | vp.FLAG_ONLINE, queue_caps=[1 << 20, 1 << 16, 1 << 21, 1 << 12])
 else:
     scene = inputs.reyes_config5(n_frames=args.frames)
     rp = ReyesPipeline(scene, flags=vp.FLAG_L2_PERSIST if args.l2 else 0)
@@ -52,6 +60,8 @@ elif args.target == "bs_mega":
     # the block-local [Bound, Split] kernel alone (its Dice items wait in a full-size ring
     # for the KBK [Dice, Shade] waves that run after it under ncu's serialisation)
     rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm - 8), (2, 3, vp.GROUP_KBK, nsm - 8, nsm)], nsm))
+elif args.target == "bs_online":
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 60), (2, 3, vp.GROUP_RTC, 60, nsm)], nsm))
 elif args.target == "rtc_dice":
     rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
     rp.p.insert(2, rp.seeds_dev, n=scene.seeds.size)
