@@ -105,7 +105,8 @@ struct RasterF {
   // RTC groups must not expand Raster's fan-out block-locally from more than one claimed
   // batch: Raster may only be the first stage of an RTC group.
   static constexpr bool rtc_ok(int lo, int hi) { return !(lo < RASTER && hi >= RASTER); }
-  static constexpr int scratch_bytes(int, int) { return 0; }
+  // kernels running Raster: a 32-item Fragment staging area per warp for big triangles
+  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= RASTER && RASTER <= hi) ? kWarpsW * 32 * 8 : 0; }
   static constexpr int default_cap_log2(int s) { return s == FRAGMENT ? 22 : 21; }
   static constexpr int min_blocks(int, int, bool) { return VP_RASTER_MINB; }
 
@@ -329,6 +330,12 @@ struct RasterF {
       const int tx0 = s.px0 >> 3, tx1 = s.px1 >> 3, ty0 = s.py0 >> 3, ty1 = s.py1 >> 3;
       const int ntx = tx1 - tx0 + 1, nt = ntx * (ty1 - ty0 + 1);
       const long long X[3] = {s.X[0], s.X[1], s.X[2]}, Y[3] = {s.Y[0], s.Y[1], s.Y[2]};
+      // A triangle with more candidate tiles than the declared fan-out (a big or near-camera
+      // triangle; reading R-S8) does not go through the block's out buffer: the warp
+      // publishes its tiles to the Fragment ring itself, 32 at a time (same items, same
+      // order-free result; the ring must hold one wave's big triangles in KBK mode).
+      const bool big = nt > kMaxTiles;  // warp-uniform
+      FragItem* const stage = (FragItem*)ctx.scratch() + 32 * (threadIdx.x >> 5);
       for (int b = 0; b < nt; b += 32) {
         const int t = b + lane;
         bool emit = false;
@@ -353,8 +360,20 @@ struct RasterF {
           }
           emit = !rejected;
         }
-        // warp-aggregated reservation of the surviving tiles (one smem atomic per warp)
         const unsigned m = __ballot_sync(0xffffffffu, emit);
+        if (big) {
+          if (emit) {
+            FragItem* out = &stage[__popc(m & ((1u << lane) - 1u))];
+            out->tri = tri;
+            out->tile = ((uint32_t)ty << 16) | (uint32_t)tx;
+          }
+          if (m) {
+            __syncwarp();
+            ctx.template publish_warp<FRAGMENT>((const uint8_t*)stage, __popc(m));
+          }
+          continue;
+        }
+        // warp-aggregated reservation of the surviving tiles (one smem atomic per warp)
         int base = 0;
         if (lane == 0 && m) base = ctx.template reserve<FRAGMENT>(__popc(m));
         base = __shfl_sync(0xffffffffu, base, 0);

@@ -367,6 +367,83 @@ struct ReyesF {
     return cls;
   }
 
+  // Bound for both 16-thread groups of a warp at once (all 32 lanes call it, converged;
+  // `valid` may differ per group), the rows of each group's frame matrix in Mr: the same
+  // operations as bound_q, with the split metrics' shuffles issued warp-uniformly (only
+  // when some group of the warp needs them, never under divergence).
+  static __device__ __forceinline__ int bound_warp(const Params& p, const float4 q, uint32_t depth, int lane,
+                                                   bool valid, int& dir, const float4* Mr) {
+    float cc[4];
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {  // project() with the rows from shared memory (same op order)
+      const float4 m = Mr[r];
+      float acc = m.x * q.x;
+      acc = acc + m.y * q.y;
+      acc = acc + m.z * q.z;
+      acc = acc + m.w * q.w;
+      cc[r] = acc;
+    }
+    const float4 c = make_float4(cc[0], cc[1], cc[2], cc[3]);
+    const bool behind = !(c.w > p.near_w);
+    const unsigned bal = __ballot_sync(0xffffffffu, behind);
+    const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
+    float sx, sy, zs;
+    screen(p, c, sx, sy, zs);
+    const float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
+    const bool deep = (int)depth >= p.max_depth;
+    int cls;  // 0 cull, 1 split, 2 dice
+    if (!valid || nbehind == 16) {
+      cls = 0;
+    } else if (nbehind > 0) {
+      cls = deep ? 0 : 1;
+    } else if (xmax < 0.0f || xmin >= (float)p.W || ymax < 0.0f || ymin >= (float)p.H) {
+      cls = 0;
+    } else {
+      const float bw = xmax - xmin, bh = ymax - ymin;
+      const float ext = bw > bh ? bw : bh;
+      cls = (deep || ext <= p.t_dice) ? 2 : 1;
+    }
+    const bool straddle = nbehind > 0;
+    dir = 0;
+    // max over non-negative values is exact in any order: the results equal bound_q's
+    if (__any_sync(0xffffffffu, cls == 1 && !straddle)) {  // screen-space split metric (R-R5)
+      const float sx12 = __shfl_sync(0xffffffffu, sx, (lane & 3) + 12, 16);
+      const float sy12 = __shfl_sync(0xffffffffu, sy, (lane & 3) + 12, 16);
+      const float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
+      float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
+      float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
+#pragma unroll
+      for (int o = 8; o >= 1; o >>= 1) {
+        lu = fmaxf(lu, __shfl_xor_sync(0xffffffffu, lu, o, 16));
+        lv = fmaxf(lv, __shfl_xor_sync(0xffffffffu, lv, o, 16));
+      }
+      if (!straddle) dir = (lu >= lv) ? 0 : 1;
+    }
+    if (__any_sync(0xffffffffu, cls == 1 && straddle)) {  // object-space metric (near-plane straddle, R-R4)
+      const float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16);
+      const float oy12 = __shfl_sync(0xffffffffu, q.y, (lane & 3) + 12, 16);
+      const float oz12 = __shfl_sync(0xffffffffu, q.z, (lane & 3) + 12, 16);
+      const float ox3 = __shfl_down_sync(0xffffffffu, q.x, 3, 16), oy3 = __shfl_down_sync(0xffffffffu, q.y, 3, 16),
+                  oz3 = __shfl_down_sync(0xffffffffu, q.z, 3, 16);
+      float olu = 0.0f, olv = 0.0f;
+      if (lane < 4) {
+        olu = fabsf(ox12 - q.x) + fabsf(oy12 - q.y);
+        olu = olu + fabsf(oz12 - q.z);
+      }
+      if ((lane & 3) == 0) {
+        olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
+        olv = olv + fabsf(oz3 - q.z);
+      }
+#pragma unroll
+      for (int o = 8; o >= 1; o >>= 1) {
+        olu = fmaxf(olu, __shfl_xor_sync(0xffffffffu, olu, o, 16));
+        olv = fmaxf(olv, __shfl_xor_sync(0xffffffffu, olv, o, 16));
+      }
+      if (straddle) dir = (olu >= olv) ? 0 : 1;
+    }
+    return cls;
+  }
+
   template <class Ctx>
   static __device__ void bound(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
@@ -513,54 +590,56 @@ struct ReyesF {
     float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
     uint32_t id = 0, path = 0, dirs = 0, depth = 0;
     for (;;) {
-      // groups without a node: the warp's pending children first, then the batch
+      // groups without a node: the warp's pending children first, then the batch (one
+      // claim atomic per warp); every decision here is warp-uniform
       const unsigned idle = __ballot_sync(0xffffffffu, !have && lane == 0);  // bit 0 / bit 16
       if (idle) {
+        __syncwarp();  // last step's pushes come before these pops
         const int nidle = __popc(idle), rank = (half && (idle & 1u)) ? 1 : 0;
         const int from_stack = min(nidle, wsp);
-        bool failed = false;
+        const int nclaim = drained ? 0 : nidle - from_stack;
+        int kb = 0;
+        if (nclaim > 0) {
+          if ((threadIdx.x & 31) == 0) kb = atomicAdd(next, nclaim);
+          kb = __shfl_sync(0xffffffffu, kb, 0);
+        }
         if (!have) {
+          const RPatch* src = nullptr;
+          bool claimed = false;
           if (rank < from_stack) {
-            const RPatch* e = &stk[wsp - 1 - rank];
-            q = e->cp[lane];
-            id = e->id;
-            path = e->path;
-            dirs = e->dirs;
-            depth = e->depth;
+            src = &stk[wsp - 1 - rank];
+          } else if (nclaim > 0 && kb + rank - from_stack < n) {
+            src = (const RPatch*)(items + (size_t)(kb + rank - from_stack) * sizeof(RPatch));
+            claimed = true;
+          }
+          if (src) {
+            q = src->cp[lane];
+            id = src->id;
+            path = src->path;
+            dirs = src->dirs;
+            depth = src->depth;
             have = true;
-            first = presplit = false;
-          } else if (!drained) {  // dynamic hand-out of the claimed batch
-            int k = 0;
-            if (lane == 0) k = atomicAdd(next, 1);
-            k = __shfl_sync(hmask, k, 0, 16);
-            if (k < n) {
-              const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
-              q = P->cp[lane];
-              id = P->id;
-              path = P->path;
-              dirs = P->dirs;
-              depth = P->depth;
-              have = first = true;
-              presplit = SS == SPLIT;  // a claimed Split item: its Bound already chose the direction
-            } else {
-              failed = true;
-            }
+            first = claimed;
+            presplit = claimed && SS == SPLIT;  // a claimed Split item: its Bound already chose the direction
           }
         }
+        if (nclaim > 0 && kb + nclaim >= n) drained = true;
         wsp -= from_stack;
-        drained |= __any_sync(0xffffffffu, failed);
         __syncwarp();  // the pops' reads come before this step's pushes
       }
       if (!__any_sync(0xffffffffu, have)) break;
       const uint32_t frame = frame_of(p, id);
-      if (have && ds.mframe[hw] != frame + 1) {
-        __syncwarp(hmask);  // the group's last reads of the old rows are done
-        ((float*)ds.M[hw])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
-        if (lane == 0) ds.mframe[hw] = frame + 1;
-        __syncwarp(hmask);
+      const bool reload = have && ds.mframe[hw] != frame + 1;
+      if (__any_sync(0xffffffffu, reload)) {
+        __syncwarp();  // every read of the old rows and tags is done
+        if (reload) {
+          ((float*)ds.M[hw])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+          if (lane == 0) ds.mframe[hw] = frame + 1;
+        }
+        __syncwarp();
       }
       int dir = 0;
-      int cls = bound_q(p, q, depth, frame, lane, have && !presplit, dir, ds.M[hw], ds.mframe[hw] - 1);
+      int cls = bound_warp(p, q, depth, lane, have && !presplit, dir, ds.M[hw]);
       if (presplit) {
         cls = 1;
         dir = (int)((dirs >> depth) & 1u);
@@ -586,19 +665,14 @@ struct ReyesF {
       wcnt += __popc(lb);
       const bool split = have && cls == 1;
       const unsigned sb = __ballot_sync(0xffffffffu, split && lane == 0);
-      if (split) {
-        const int slot = wsp + ((half && (sb & 1u)) ? 1 : 0);
-        if (slot >= kDfsStack) {  // deeper than max_depth allows (cannot happen for valid seeds)
-          ctx.abort(ABORT_GUARD);
-          have = false;
-        } else {
-          // de Casteljau at 1/2 (reading R-R6) of the curve through this lane's control point
-          // along the split direction; same operations as split_cp, points from shuffles
-          const int base = dir == 0 ? (lane & 3) : (lane & ~3), step = dir == 0 ? 4 : 1;
-          const int t = dir == 0 ? (lane >> 2) : (lane & 3);
-          const float4 a = shfl4(hmask, q, base), b = shfl4(hmask, q, base + step);
-          const float4 c = shfl4(hmask, q, base + 2 * step), d = shfl4(hmask, q, base + 3 * step);
-          float4 L, R;
+      if (sb) {  // warp-uniform: the shuffles below run converged
+        // de Casteljau at 1/2 (reading R-R6) of the curve through this lane's control point
+        // along the split direction; same operations as split_cp, points from shuffles
+        const int base = dir == 0 ? (lane & 3) : (lane & ~3), step = dir == 0 ? 4 : 1;
+        const int t = dir == 0 ? (lane >> 2) : (lane & 3);
+        const float4 a = shfl4(0xffffffffu, q, base), b = shfl4(0xffffffffu, q, base + step);
+        const float4 c = shfl4(0xffffffffu, q, base + 2 * step), d = shfl4(0xffffffffu, q, base + 3 * step);
+        float4 L, R;
 #define VP_CASTELJAU(comp)                                                   \
   {                                                                          \
     float ab = (a.comp + b.comp) * 0.5f, bc = (b.comp + c.comp) * 0.5f;      \
@@ -608,31 +682,37 @@ struct ReyesF {
     L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
     R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
   }
-          VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+        VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
 #undef VP_CASTELJAU
-          if (!(first && presplit)) {  // a claimed Split item was counted when it was claimed
-            ++nsp;
-            if (lane == 0) ctx.template trace_local_id<SPLIT>(node);
+        if (split) {
+          const int slot = wsp + ((half && (sb & 1u)) ? 1 : 0);
+          if (slot >= kDfsStack) {  // deeper than max_depth allows (cannot happen for valid seeds)
+            ctx.abort(ABORT_GUARD);
+            have = false;
+          } else {
+            if (!(first && presplit)) {  // a claimed Split item was counted when it was claimed
+              ++nsp;
+              if (lane == 0) ctx.template trace_local_id<SPLIT>(node);
+            }
+            const uint32_t ndirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
+            RPatch* r = &stk[slot];
+            r->cp[lane] = R;
+            if (lane == 0) {
+              r->id = id;
+              r->path = path | (1u << depth);
+              r->dirs = ndirs;
+              r->depth = depth + 1;
+            }
+            q = L;
+            path &= ~(1u << depth);
+            dirs = ndirs;
+            depth += 1;
+            first = presplit = false;
           }
-          const uint32_t ndirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
-          RPatch* r = &stk[slot];
-          r->cp[lane] = R;
-          if (lane == 0) {
-            r->id = id;
-            r->path = path | (1u << depth);
-            r->dirs = ndirs;
-            r->depth = depth + 1;
-          }
-          q = L;
-          path &= ~(1u << depth);
-          dirs = ndirs;
-          depth += 1;
-          first = presplit = false;
         }
-      } else if (have) {
-        have = false;  // diced or culled: the next node comes from the stack or the batch
+        wsp = min(wsp + __popc(sb), kDfsStack);
       }
-      wsp = min(wsp + __popc(sb), kDfsStack);
+      if (have && !split) have = false;  // diced or culled: the next node comes from the stack or the batch
       if (wcnt > kDfsStage - 2) {  // warp-uniform
         __syncwarp();
         ctx.template publish_warp<DICE>((const uint8_t*)stage, wcnt);
@@ -1013,7 +1093,6 @@ struct ReyesF {
     const Params& p = ctx.params();
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     ChainScratch& cs = *(ChainScratch*)ctx.scratch();
-    float* Mw = (float*)cs.M[warp];
     uint8_t* list = cs.list[warp];
     // Patches are handed out dynamically: shade work per patch varies with its size on
     // screen, so a static warp -> patch map leaves warps idle at the round barrier.
@@ -1046,7 +1125,7 @@ struct ReyesF {
         const RPatch* P = (const RPatch*)(items + (size_t)(k + j) * sizeof(RPatch));
         const uint32_t frame = frame_of(p, P->id);
         __syncwarp();  // the previous patch's dice is done with the matrix
-        if (lane < 16) Mw[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
+        if (lane < 16) ((float*)cs.M[warp])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
         __syncwarp();
         dice_patch<true>(p, P, g, lane, cs.M[warp], Bt);
         __syncwarp();

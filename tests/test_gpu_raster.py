@@ -230,3 +230,32 @@ def test_raster_near_clip_every_side_pattern(vpm, orc, zs):
         rp = RasterPipeline(scene)
         rp.configure(vpm.MEGAKERNEL)
         check(orc, scene, rp, rp.run())
+
+
+def _with_big_triangles(sc, straddle):
+    """Prepend screen-filling triangles (beyond the 128-tile fan-out): a
+    full-screen quad at z = 0.9 and a 3-screen-wide triangle; with `straddle` one vertex of
+    each lies behind the near plane (z < 0), so the clipped pieces are big as well."""
+    import dataclasses
+    W, H = sc.W, sc.H
+    zb = -0.4 if straddle else 0.3
+    big = np.array([[(0, 0, 0.9, 1), (W, 0, 0.9, 1), (W, H, 0.9, 1)],
+                    [(0, 0, 0.9, 1), (W, H, 0.9, 1), (0, H, zb, 1)],
+                    [(-W, -H, 0.8, 1), (2 * W, H / 2, zb, 1), (W / 3, 2 * H, 0.6, 1)]], np.float32)
+    col = np.array([[(1, 0, 0, 0), (0, 1, 0, 0), (0, 0, 1, 0)]] * 3, np.float32)
+    return dataclasses.replace(sc, pos=np.concatenate([big, sc.pos]), col=np.concatenate([col, sc.col]))
+
+
+@pytest.mark.parametrize("near", [False, True])
+@pytest.mark.parametrize("model", ["kbk", "megakernel", "hybrid_rtc_mega", "hybrid_rtc_rtc"])
+def test_raster_screen_filling_triangles_1080p(vpm, orc, model, near):
+    """Triangles covering tens of thousands of 8x8 tiles at 1920x1080 (no VP_ERR_FANOUT),
+    in both near-clip modes, bit-exact against the oracle."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    base = (inputs.raster_near_scene(n=2000, W=1920, H=1080, area_range=(0.5, 512.0)) if near
+            else inputs.raster_scene(2000, W=1920, H=1080))
+    scene = _with_big_triangles(base, near)
+    rp = RasterPipeline(scene)
+    configure(vpm, rp, model)
+    ref = check(orc, scene, rp, rp.run())
+    assert ref["n_fragment"] > 32_000   # the big triangles' tiles went through

@@ -73,7 +73,7 @@ def raster(model):
 def pyramid(model):
     rgb = inputs.pyramid_images(2, 256)
     p = W.PyramidPipeline(rgb, **KW)
-    conf(p, model, [(0, 0, vp.GROUP_MEGA, 0, 40), (1, 2, vp.GROUP_MEGA, 40, nsm)])
+    conf(p, model, [(0, 0, vp.GROUP_MEGA, 0, 40), (1, 3, vp.GROUP_MEGA, 40, nsm)])
     p.run()
     return np.array_equal(p.pyramid(), oracle.pyr_pipeline(rgb)["pyr"])
 
