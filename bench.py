@@ -286,6 +286,12 @@ def queue_microbench(torch, vp, stream):
     return out
 
 
+def oracle_mod():
+    import oracle
+    oracle.build()
+    return oracle
+
+
 def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
     """Secondary measurements: every BASELINE workload (configs 1-4) through the same
     runtime, auto-tuned, vs KBK; items/s, frames/s and % of measured HBM where the
@@ -319,6 +325,7 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         pipe.configure(vp.MEGAKERNEL)
         mega_ms, _ = t_run()
         pipe.p.configure_config(best)
+        pipe.run(stream)  # the outputs the parity checks read come from the tuned configuration
         items = sum(st["dequeued"][:8])
         r = {"ms": ms, "frames_per_s": frames / (ms / 1e3), "items_per_s": items / (ms / 1e3),
              "items": items, "kbk_ms": kbk_ms, "kbk_graph_ms": kbkg_ms, "megakernel_ms": mega_ms,
@@ -337,6 +344,13 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         return r
 
     out = {}
+    cores = os.cpu_count() or 1
+    alu_peak = None
+    try:
+        nsm_, _ = vp.device_info(0)
+        alu_peak = nsm_ * 128 * peaks().get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+    except Exception:
+        pass
 
     def guarded(name, fn):
         try:
@@ -344,12 +358,52 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         except Exception as ex:  # one workload's failure must not hide the others
             out[name] = {"error": repr(ex)}
 
+    def threads_run(fn, args, threads):
+        """The C oracle (as it stands) over independent units on `threads` host threads
+        (ctypes releases the GIL); inputs are built before the timer."""
+        import concurrent.futures as cf
+        t0 = time.perf_counter()
+        with cf.ThreadPoolExecutor(max(1, threads)) as ex:
+            res = list(ex.map(fn, args))
+        return time.perf_counter() - t0, res
+
+    def cpu_rec(units, unit, secs, threads, sample):
+        return {"value": units / secs, "unit": unit, "cores": cores, "threads": threads, "kind": "oracle",
+                "cpu_model": cpu_model(), "seconds": secs, "sample": sample}
+
+    def hbm_roof(alg_bytes, ms):
+        a = alg_bytes / (ms / 1e3) / 1e9
+        return {"bound": "hbm", "achieved": a, "peak": hbm_gbs, "unit": "GB/s", "frac": a / hbm_gbs,
+                "peak_source": "MEASURED_PEAKS.json hbm copy bandwidth", "alg_bytes": alg_bytes}
+
+    def reyes_roof(deq, ms):
+        fl = deq[0] * FLOP_BOUND + deq[1] * FLOP_SPLIT + deq[2] * FLOP_DICE + deq[3] * FLOP_SHADE
+        a = fl / (ms / 1e3) / 1e12
+        return {"bound": "alu", "achieved": a, "peak": alu_peak, "unit": "TFLOP/s", "frac": a / alu_peak,
+                "peak_source": "SMs x 128 fp32 lanes x sm_max_mhz (non-FMA)",
+                "note": "latency-bound at one frame: >= 10 dependent rounds of small waves"}
+
     def w_reyes1():
         out["reyes_config1"] = measure(ReyesPipeline(inputs.reyes_config1()), 1)
 
     def w_reyes1x():
         # SURVEY §8(d) throughput mode: R = 256 independent config-1 frames in one run
-        out["reyes_config1_x256"] = measure(ReyesPipeline(inputs.reyes_config1(n_frames=256)), 256)
+        rp = ReyesPipeline(inputs.reyes_config1(n_frames=256))
+        r = measure(rp, 256)
+        one = inputs.reyes_config1()
+        n = 4 * cores
+        secs, res = threads_run(oracle_mod().reyes_pipeline, [one] * n, cores)
+        r["cpu_baseline"] = cpu_rec(n, "frames/s", secs, cores, f"{n} config-1 frames, one per thread")
+        key, s_ = rp.keys()
+        col = rp.colours()
+        ref = res[0]
+        fr = (0, 1, 77, 128, 255)
+        bad = sum(int(np.count_nonzero(key[f] != ref["key"][0])) for f in fr)
+        err = max(float(np.max(np.abs(col[f] - ref["colour"][0]))) for f in fr)
+        r["parity"] = {"pass": bad == 0 and err <= 1e-4, "frames": list(fr), "keys_differing": bad, "max_abs_err": err}
+        r["roofline"] = reyes_roof(rp.run(stream)["dequeued"], r["ms"])
+        r["leaf_depth_hist"] = list(ref["depth_hist"][:9])
+        out["reyes_config1_x256"] = r
 
     def w_face():
         fs = inputs.face_scene()
@@ -358,17 +412,117 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         out["facedet_config2"]["windows_per_s"] = fp.results()["windows"] / (out["facedet_config2"]["ms"] / 1e3)
 
     def w_face8():
+        import dataclasses
         fs8 = inputs.face_scene(n_frames=8)  # throughput mode, R = 8 frames
         fp8 = FaceDetPipeline(fs8)
-        out["facedet_config2_x8"] = measure(fp8, fs8.n_frames)
-        out["facedet_config2_x8"]["windows_per_s"] = fp8.results()["windows"] / (out["facedet_config2_x8"]["ms"] / 1e3)
+        r = measure(fp8, fs8.n_frames)
+        got = fp8.results()
+        r["windows_per_s"] = got["windows"] / (r["ms"] / 1e3)
+        r["survivors_per_cascade_stage"] = got["survivors"]
+        subs = [dataclasses.replace(fs8, rgb=fs8.rgb[f:f + 1]) for f in range(fs8.n_frames)]
+        secs, res = threads_run(lambda sc: oracle_mod().fd_pipeline(sc, det_cap=1 << 20), subs, cores)
+        r["cpu_baseline"] = cpu_rec(len(subs), "frames/s", secs, min(cores, len(subs)),
+                                    f"the {len(subs)} 1920x1080 frames, one per thread")
+        want = sorted((f, *map(int, d[1:])) for f, rr in enumerate(res) for d in rr["det"])
+        have = sorted(tuple(int(v) for v in d) for d in got["det"])
+        surv = [sum(rr["survivors"][k] for rr in res) for k in range(len(res[0]["survivors"]))]
+        r["parity"] = {"pass": want == have and surv == got["survivors"], "detections": len(have),
+                       "survivors_equal": surv == got["survivors"]}
+        # ~203 MB/frame algorithmic (frame, pyramid, LBP, 16-B window items w+r)
+        r["roofline"] = hbm_roof(203e6 * fs8.n_frames, r["ms"])
+        r["roofline"]["note"] = ("issue-bound (cascade evaluation, integer ALU/LSU); see profiles/r2_suite_ncu.txt "
+                                 "for issue-slot use")
+        out["facedet_config2_x8"] = r
 
     def w_pyr():
         n_img, S = 32, 4096
         rgb = inputs.pyramid_images(n_img, S)
         # Gray: RGB read; Map: RGB read + level-0 write; Resize: read + write per level; hist negligible
         per_img = 3 * S * S + (3 * S * S + S * S) + sum(((S >> l) ** 2) * 5 for l in range(1, 13))
-        out["pyramid_config3"] = measure(PyramidPipeline(rgb), n_img, alg_bytes=n_img * per_img)
+        pp = PyramidPipeline(rgb)
+        r = measure(pp, n_img, alg_bytes=n_img * per_img)
+        r["roofline"] = hbm_roof(n_img * per_img, r["ms"])
+        got = pp.pyramid()
+        ims = [rgb[i:i + 1] for i in range(n_img)]
+        secs, res = threads_run(oracle_mod().pyr_pipeline, ims, cores)
+        r["cpu_baseline"] = cpu_rec(n_img, "images/s", secs, min(cores, n_img), f"all {n_img} 4096^2 images, one per thread")
+        bad = sum(int(np.count_nonzero(got[i] != res[i]["pyr"][0])) for i in range(n_img))
+        r["parity"] = {"pass": bad == 0, "images": n_img, "bytes_differing": bad}
+        out["pyramid_config3"] = r
+
+    def w_cfd():
+        import dataclasses
+        cs = inputs.cfd_scene(G=4096, n_outer=10)
+        cp = CfdPipeline(cs)
+        r = measure(cp, 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
+        r["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (r["ms"] / 1e3)
+        r["roofline"] = hbm_roof(572 * cs.n_cells * cs.n_outer, r["ms"])
+        r["roofline"]["note"] = ("Flux is issue-bound (~1190 thread-instructions per cell: IEEE div/sqrt, 4 faces); "
+                                 "the streaming stages are HBM-bound (profiles/r2_suite_ncu.txt)")
+        # oracle: one outer iteration of the full 4096^2 grid (a documented subset, single thread)
+        cs1 = dataclasses.replace(cs, n_outer=1)
+        t0 = time.perf_counter()
+        ref = oracle_mod().cfd_pipeline(cs1)
+        secs = time.perf_counter() - t0
+        r["cpu_baseline"] = cpu_rec(cs.n_cells * 3, "cell-updates/s", secs, 1,
+                                    "1 outer iteration (3 RK steps) of the 4096^2 grid, single-threaded C oracle")
+        cp1 = CfdPipeline(cs1)
+        cp1.p.configure_config(cp.p.get_config())
+        cp1.run(stream)
+        got = cp1.state()
+        r["parity"] = {"pass": bool(np.array_equal(got, ref["vars"])), "outer_iterations": 1,
+                       "max_abs_err": float(np.max(np.abs(got - ref["vars"])))}
+        out["cfd_config3"] = r
+
+    def w_ldpc():
+        # SURVEY §8(f-3): the LDPC decoder (Fig. 17), 100 frames x 100 iterations (L53)
+        from paper_conf_micro_zhengozsyc17_b200.workloads import LdpcPipeline
+        ls = inputs.ldpc_scene()
+        lp = LdpcPipeline(ls)
+        r = measure(lp, ls.n_frames)
+        r["decoder_iterations_per_s"] = ls.n_frames * ls.n_iter / (r["ms"] / 1e3)
+        t0 = time.perf_counter()
+        ref = oracle_mod().ldpc_pipeline(ls)
+        secs = time.perf_counter() - t0
+        r["cpu_baseline"] = cpu_rec(ls.n_frames * ls.n_iter, "decoder-iterations/s", secs, 1,
+                                    "all 100 frames x 100 iterations, single-threaded C oracle")
+        got = lp.results()
+        r["parity"] = {"pass": bool(np.array_equal(got["post"], ref["post"]) and np.array_equal(got["errors"], ref["errors"]))}
+        out["ldpc_f3"] = r
+
+    def w_raster():
+        rs = inputs.raster_scene()
+        rp = RasterPipeline(rs)
+        r = measure(rp, 1, alg_bytes=265_000_000)
+        r["triangles_per_s"] = rs.n_tris / (r["ms"] / 1e3)
+        t0 = time.perf_counter()
+        ref = oracle_mod().raster_pipeline(rs)
+        secs = time.perf_counter() - t0
+        r["cpu_baseline"] = cpu_rec(1, "frames/s", secs, 1, "the full 1M-triangle 1920x1080 frame, single-threaded")
+        key = rp.keys()
+        col = rp.colours()
+        r["parity"] = {"pass": bool(np.array_equal(key, ref["key"]) and np.array_equal(col, ref["colour"])),
+                       "keys_differing": int(np.count_nonzero(key != ref["key"]))}
+        # the L2-atomic bound of Fragment (one 64-bit RED.MIN per covered sample
+        # passing the depth range) against the measured RED.MIN.U64 rate into the same
+        # 16.6 MB key buffer; Vertex/Clip's HBM share is in profiles/r2_suite_ncu.txt
+        try:
+            peak = vp.bench_red_min_u64(rs.W * rs.H)
+            a = ref["n_frag_pixels"] / (r["ms"] / 1e3)
+            r["roofline"] = {"bound": "l2_atomic", "achieved": a / 1e9, "peak": peak / 1e9, "unit": "G atomics/s",
+                             "frac": a / peak, "atomics": int(ref["n_frag_pixels"]),
+                             "peak_source": "vp_bench_red_min_u64 (measured, same buffer size)"}
+        except Exception as ex:
+            r["roofline"] = {"error": repr(ex)}
+        r["roofline_hbm"] = hbm_roof(265_000_000, r["ms"])
+        out["raster_config4"] = r
+
+    def w_raster_near():
+        # SURVEY §8(f-4), DESIGN R-S9: config-4 triangles with per-vertex z ~ U(-0.6, 0.95),
+        # so about half straddle the near plane and Clip fans out 0..2 sub-triangles
+        rs = inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
+        out["raster_near_clip"] = measure(RasterPipeline(rs), 1)
+        out["raster_near_clip"]["triangles_per_s"] = rs.n_tris / (out["raster_near_clip"]["ms"] / 1e3)
 
     def w_pyr_fig13():
         # PAPER.md Fig. 13 (L53-L55): the pyramid at 1..32 images under KBK, KBK with
@@ -412,30 +566,6 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
             rows.append(row)
             del pp
         out["pyramid_fig13"] = rows
-
-    def w_cfd():
-        cs = inputs.cfd_scene(G=4096, n_outer=10)
-        out["cfd_config3"] = measure(CfdPipeline(cs), 1, alg_bytes=572 * cs.n_cells * cs.n_outer, reps=2)
-        out["cfd_config3"]["cell_updates_per_s"] = cs.n_cells * 3 * cs.n_outer / (out["cfd_config3"]["ms"] / 1e3)
-
-    def w_ldpc():
-        # SURVEY §8(f-3): the LDPC decoder (Fig. 17), 100 frames x 100 iterations (L53)
-        from paper_conf_micro_zhengozsyc17_b200.workloads import LdpcPipeline
-        ls = inputs.ldpc_scene()
-        out["ldpc_f3"] = measure(LdpcPipeline(ls), ls.n_frames)
-        out["ldpc_f3"]["decoder_iterations_per_s"] = ls.n_frames * ls.n_iter / (out["ldpc_f3"]["ms"] / 1e3)
-
-    def w_raster():
-        rs = inputs.raster_scene()
-        out["raster_config4"] = measure(RasterPipeline(rs), 1, alg_bytes=265_000_000)
-        out["raster_config4"]["triangles_per_s"] = rs.n_tris / (out["raster_config4"]["ms"] / 1e3)
-
-    def w_raster_near():
-        # SURVEY §8(f-4), DESIGN R-S9: config-4 triangles with per-vertex z ~ U(-0.6, 0.95),
-        # so about half straddle the near plane and Clip fans out 0..2 sub-triangles
-        rs = inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
-        out["raster_near_clip"] = measure(RasterPipeline(rs), 1)
-        out["raster_near_clip"]["triangles_per_s"] = rs.n_tris / (out["raster_near_clip"]["ms"] / 1e3)
 
     for name, fn in (("reyes_config1", w_reyes1), ("reyes_config1_x256", w_reyes1x), ("facedet_config2", w_face),
                      ("facedet_config2_x8", w_face8), ("pyramid_config3", w_pyr), ("cfd_config3", w_cfd),

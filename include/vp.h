@@ -430,6 +430,12 @@ vp_status vp_get_trace(void* p, void** dev_ptr, size_t* n_records);
 vp_status vp_config_to_string(const vp_config* c, char* buf, size_t buf_len);
 vp_status vp_config_from_string(const char* s, vp_config* out);
 
+/* Measured ceiling for the L2-atomic rooflines: fire-and-forget 64-bit
+ * atomic minimum (the raster z-buffer update) from a full grid to pseudo-random slots of a
+ * `slots` x 8-B device buffer; *ops_per_s = n_ops / best-of-3 CUDA-event time.
+ * Diagnostics only; it does not touch any pipeline. */
+vp_status vp_bench_red_min_u64(int device, unsigned long long slots, unsigned long long n_ops, double* ops_per_s);
+
 /* Device properties the binding layer needs (no torch types cross the ABI). */
 vp_status vp_device_info(int device, int* num_sms, int* cc_major, int* cc_minor);
 /* Minimal CUDA plumbing for bindings without their own CUDA runtime. kind: 0 H2D, 1 D2H, 2 D2D */

@@ -9,7 +9,7 @@ CSRC = os.path.join(HERE, "csrc")
 LIB_NAME = os.environ.get("VP_LIB_NAME", "libvp.so")
 LIB = os.path.join(HERE, LIB_NAME)
 OBJDIR = os.path.join(HERE, "build" if LIB_NAME == "libvp.so" else "build_" + LIB_NAME.split(".")[0])
-SOURCES = ["vp_host.cu", "vp_tune.cu", "fam_basic.cu", "fam_reyes.cu", "fam_raster.cu", "fam_pyramid.cu", "fam_cfd.cu", "fam_facedet.cu", "fam_qbench.cu", "fam_ldpc.cu"]
+SOURCES = ["vp_host.cu", "vp_tune.cu", "fam_basic.cu", "fam_reyes.cu", "fam_raster.cu", "fam_pyramid.cu", "fam_cfd.cu", "fam_facedet.cu", "fam_qbench.cu", "fam_ldpc.cu", "vp_microbench.cu"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
          # no FMA contraction, IEEE div/sqrt, no fast math -> bit-exact vs oracle

@@ -173,11 +173,12 @@ vp_config_from_string = _decl("vp_config_from_string", [C.c_char_p, C.POINTER(Co
 vp_device_info = _decl("vp_device_info", [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)])
 vp_memcpy = _decl("vp_memcpy", [P, P, C.c_size_t, C.c_int, P])
 vp_set_flags = _decl("vp_set_flags", [P, C.c_uint32, C.POINTER(C.c_uint32)])
+vp_bench_red_min_u64 = _decl("vp_bench_red_min_u64", [C.c_int, C.c_ulonglong, C.c_ulonglong, C.POINTER(C.c_double)])
 
 EXPORTED = ["vp_status_string", "vp_last_error", "vp_pipeline_create", "vp_pipeline_destroy", "vp_stage_register",
             "vp_insert", "vp_insert_async", "vp_configure", "vp_configure_config", "vp_get_config", "vp_run",
             "vp_set_timeout", "vp_get_trace", "vp_autotune", "vp_profile", "vp_get_output", "vp_set_params", "vp_config_to_string", "vp_config_from_string",
-            "vp_device_info", "vp_memcpy", "vp_set_flags"]
+            "vp_device_info", "vp_memcpy", "vp_set_flags", "vp_bench_red_min_u64"]
 
 
 class VPError(RuntimeError):
@@ -212,6 +213,15 @@ def device_info(device=0):
     if rc != VP_OK:
         raise VPError(rc, "vp_device_info")
     return n.value, (a.value, b.value)
+
+
+def bench_red_min_u64(slots, n_ops=1 << 30, device=0):
+    """vp_bench_red_min_u64: measured 64-bit atomic-min (RED) rate into a `slots`-entry buffer."""
+    r = C.c_double(0.0)
+    rc = vp_bench_red_min_u64(device, slots, n_ops, C.byref(r))
+    if rc != VP_OK:
+        raise VPError(rc, "vp_bench_red_min_u64")
+    return r.value
 
 
 def make_binding(groups, num_sms, blocks_per_sm=None, batch=None):
