@@ -41,6 +41,7 @@ struct FamilyOps {
   virtual size_t params_bytes() const = 0;
   virtual const void* kernel(int lo, int hi, bool rtc) const = 0;
   virtual size_t smem(int lo, int hi, bool rtc) const = 0;
+  virtual int block_threads(int lo, int hi, bool rtc) const = 0;  // blockDim of kernel [lo, hi]
   virtual cudaError_t launch(int lo, int hi, bool rtc, const Common& c, const GroupArgs& g, const void* params,
                              int grid, bool coop, cudaStream_t st) const = 0;
   virtual cudaError_t init_run(const void* params, cudaStream_t st) const = 0;
@@ -53,13 +54,18 @@ template <class F>
 struct FamilyImpl final : FamilyOps {
   using G = Graph<F>;
   const void* fn[kMaxStages][kMaxStages][2] = {};
+  int nthreads[kMaxStages][kMaxStages][2] = {};
 
   template <int LO, int HI>
   void fill() {
     if constexpr (LO < F::S) {
       if constexpr (HI < F::S) {
         fn[LO][HI][0] = (const void*)&vp_kernel<F, LO, HI, false>;
-        if constexpr (G::rtc_legal(LO, HI)) fn[LO][HI][1] = (const void*)&vp_kernel<F, LO, HI, true>;
+        nthreads[LO][HI][0] = Runner<F, LO, HI, false>::kBlockThreads;
+        if constexpr (G::rtc_legal(LO, HI)) {
+          fn[LO][HI][1] = (const void*)&vp_kernel<F, LO, HI, true>;
+          nthreads[LO][HI][1] = Runner<F, LO, HI, true>::kBlockThreads;
+        }
         fill<LO, HI + 1>();
       } else {
         fill<LO + 1, LO + 1>();
@@ -129,6 +135,10 @@ struct FamilyImpl final : FamilyOps {
   size_t params_bytes() const override { return sizeof(typename F::Params); }
   const void* kernel(int lo, int hi, bool rtc) const override { return fn[lo][hi][rtc ? 1 : 0]; }
   size_t smem(int lo, int hi, bool rtc) const override { return (size_t)smem_of<0, 0>(lo, hi, rtc); }
+  int block_threads(int lo, int hi, bool rtc) const override {
+    const int t = nthreads[lo][hi][rtc ? 1 : 0];
+    return t > 0 ? t : kBlock;
+  }
   cudaError_t launch(int lo, int hi, bool rtc, const Common& c, const GroupArgs& g, const void* params, int grid,
                      bool coop, cudaStream_t st) const override {
     const void* k = kernel(lo, hi, rtc);
@@ -139,8 +149,9 @@ struct FamilyImpl final : FamilyOps {
     a.p = *(const typename F::Params*)params;
     void* args[] = {&a};
     size_t sm = smem(lo, hi, rtc);
-    if (coop) return cudaLaunchCooperativeKernel(k, dim3(grid), dim3(kBlock), args, sm, st);
-    return cudaLaunchKernel(k, dim3(grid), dim3(kBlock), args, sm, st);
+    const dim3 blk(block_threads(lo, hi, rtc));
+    if (coop) return cudaLaunchCooperativeKernel(k, dim3(grid), blk, args, sm, st);
+    return cudaLaunchKernel(k, dim3(grid), blk, args, sm, st);
   }
   cudaError_t init_run(const void* params, cudaStream_t st) const override {
     return F::init_run(*(const typename F::Params*)params, st);

@@ -301,7 +301,7 @@ int occupancy(vp_pipeline_s* p, int lo, int hi, bool rtc) {
   // stop co-resident persistent groups (coarse/fine/hybrid) from ever starting.
   cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, (int)cudaSharedmemCarveoutMaxShared);
   int occ = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kBlock, sm) != cudaSuccess) occ = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, p->fam->block_threads(lo, hi, rtc), sm) != cudaSuccess) occ = 0;
   c = occ;
   return occ;
 }
@@ -388,11 +388,12 @@ struct KRes {
   int regs, smem, threads;
 };
 KRes kernel_res(vp_pipeline_s* p, int lo, int hi, bool rtc) {
-  KRes r{0, 0, kBlock};
+  const int nt = p->fam->block_threads(lo, hi, rtc);
+  KRes r{0, 0, nt};
   cudaFuncAttributes at;
-  if (cudaFuncGetAttributes(&at, p->fam->kernel(lo, hi, rtc)) != cudaSuccess) return KRes{1 << 30, 1 << 30, kBlock};
+  if (cudaFuncGetAttributes(&at, p->fam->kernel(lo, hi, rtc)) != cudaSuccess) return KRes{1 << 30, 1 << 30, nt};
   int per_warp = ((at.numRegs * 32 + 255) / 256) * 256;
-  r.regs = per_warp * (kBlock / 32);
+  r.regs = per_warp * (nt / 32);
   r.smem = (int)(at.sharedSizeBytes + p->fam->smem(lo, hi, rtc)) + 1024;
   return r;
 }

@@ -452,6 +452,8 @@ struct Ctx {
   int ob;  // current out buffer
 
   __device__ Ctx(const KArgs<F>& a_, uint8_t* smem_, BlockShared& sh_) : a(a_), smem(smem_), sh(sh_), ob(0) {}
+  static constexpr int kLo = LO, kHi = HI;  // the kernel's stage range (per-kernel code choices)
+  static constexpr bool kRtc = RTC;
 
   __device__ __forceinline__ const typename F::Params& params() const { return a.p; }
   // layout constants are forced to compile time (nvcc does not always fold the
@@ -1276,6 +1278,10 @@ struct Runner {
   }
   // ... or its warps publish their outputs themselves (direct-publish kernels)
   static constexpr bool sink_group() { return direct_publish<F>(LO, HI, RTC) || no_ring_outputs(); }
+  // A sink group has no publisher warp: its blocks are the 8 worker warps + the fetcher, so
+  // the register file is divided among 9 warps, not 10 (more registers per thread at the
+  // same resident blocks per SM).
+  static constexpr int kBlockThreads = sink_group() ? kThreads + 32 : kBlock;
 
   static __device__ void run_sink(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, uint8_t* smem) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -1344,7 +1350,7 @@ struct Runner {
         }
       }
       if constexpr (scratch_of<F>(LO, HI, RTC) > 0) {
-        for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+        for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += blockDim.x) ((uint32_t*)ctx.scratch())[i] = 0u;
       }
       __syncthreads();
       run_sink(a, ctx, sh, smem);
@@ -1353,7 +1359,7 @@ struct Runner {
       return;
     }
     if constexpr (scratch_of<F>(LO, HI, RTC) > 0) {  // family scratch starts zeroed
-      for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += kBlock) ((uint32_t*)ctx.scratch())[i] = 0u;
+      for (int i = threadIdx.x; i < scratch_of<F>(LO, HI, RTC) / 4; i += blockDim.x) ((uint32_t*)ctx.scratch())[i] = 0u;
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     // prologue: stage the first batch into in[0]
@@ -1388,7 +1394,8 @@ struct Runner {
 };
 
 template <class F, int LO, int HI, bool RTC>
-__global__ void __launch_bounds__(kBlock, F::min_blocks(LO, HI, RTC)) vp_kernel(const __grid_constant__ KArgs<F> a) {
+__global__ void __launch_bounds__(Runner<F, LO, HI, RTC>::kBlockThreads, F::min_blocks(LO, HI, RTC))
+    vp_kernel(const __grid_constant__ KArgs<F> a) {
   Runner<F, LO, HI, RTC>::run(a);
 }
 
