@@ -15,9 +15,9 @@
 #include "../../include/vp.h"
 #include "vp_family.cuh"
 
-#ifndef VP_PYR_PREFETCH  // Gray: load the next tile while converting this one
-#define VP_PYR_PREFETCH 0  // measured: +16% time in the megakernel (register pressure), off
-#endif
+#ifndef VP_PYR_PREFETCH  // Gray: load the next tile while converting this one, in every kernel
+#define VP_PYR_PREFETCH 0  // measured: +16% time in the megakernel (register pressure), off;
+#endif                     // a Gray-only kernel (KBK, or Gray as its own group) always prefetches
 #ifndef VP_PYR_MINB
 #define VP_PYR_MINB 3
 #endif
@@ -80,8 +80,13 @@ struct PyramidF {
   using Params = vp_pyramid_params;
   static constexpr int stride(int) { return 16; }
   static constexpr int threads_per_item(int) { return 256; }
-  static constexpr int max_batch(int s) { return s == GRAY ? 8 : s == CDF ? 1 : s == MAP ? 4 : 8; }
+  static constexpr int max_batch(int s) { return s == GRAY ? 16 : s == CDF ? 1 : s == MAP ? 4 : 8; }
   static constexpr int default_batch(int s) { return max_batch(s); }
+  // Gray takes 16 tiles per claim only in its own kernel (the tile loads are pipelined
+  // there, see gray_batch); kernels that also run later stages keep batches of 8
+  static constexpr int kernel_max_batch(int lo, int hi, bool, int s) {
+    return (s == GRAY && !(lo == GRAY && hi == GRAY)) ? 8 : max_batch(s);
+  }
   static constexpr int fanout(int s, int t) {
     return (s == GRAY && t == CDF) ? 1 : (s == CDF && t == MAP) ? kMaxMap : (s == MAP && t == RESIZE) ? 4
                                                                         : (s == RESIZE && t == RESIZE) ? 1 : 0;
@@ -146,12 +151,13 @@ struct PyramidF {
       }
     };
     uint4 vn[3];
-    if (VP_PYR_PREFETCH && n > 0) load(0, vn);
+    constexpr bool kPrefetch = VP_PYR_PREFETCH || (Ctx::kLo == GRAY && Ctx::kHi == GRAY);
+    if (kPrefetch && n > 0) load(0, vn);
     int k0 = 0;
     for (int k = 0; k < n; ++k) {
       const PyrItem it = items[k];
       uint4 v[3];
-      if (VP_PYR_PREFETCH) {
+      if (kPrefetch) {
 #pragma unroll
         for (int q = 0; q < 3; ++q) v[q] = vn[q];
         if (k + 1 < n) load(k + 1, vn);

@@ -97,6 +97,9 @@ struct RasterF {
   using Params = vp_raster_params;
   static constexpr int stride(int s) { return s == FRAGMENT ? 8 : 4; }
   static constexpr int threads_per_item(int s) { return s == RASTER ? 32 : s == FRAGMENT ? 64 : 1; }
+  // (Vertex / Clip batches of 1024 were tried in round 2: no change for Vertex, Clip 20 ->
+  // 18% of HBM under KBK, and the megakernel 3.2 -> 4.3 ms; a KBK wave of these stages is
+  // a ~0.1 ms kernel of 2-10 rounds per block, so its ramp-up and tail bound it)
   static constexpr int max_batch(int s) { return s <= CLIP ? 256 : s == RASTER ? 32 : 32; }
   static constexpr int default_batch(int s) { return max_batch(s); }
   static constexpr int fanout(int s, int t) {

@@ -561,20 +561,37 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
         lo[g] = std::min(lo[g], s);
         hi[g] = std::max(hi[g], s);
       }
-      uint32_t used[kMaskWords] = {};
-      for (int g = 0; g < G && rc == VP_OK; ++g) {
+      // Groups normally own disjoint SMs (coarse pipelining between groups, L27).  Groups may
+      // share SMs -- a fine pipeline between groups (Fig. 5's per-SM block quotas, applied to
+      // group kernels) -- when every group on a shared SM is a MEGA or RTC group with an
+      // explicit block quota and the quotas of all groups on that SM fit it together.
+      for (int g = 0; g < G; ++g) {
         if (hi[g] < 0) return fail(p, VP_ERR_INVALID, "group %d is empty", g);
+        if (mask_count(b->group_sm_mask[g], N) == 0) return fail(p, VP_ERR_INVALID, "group %d has no SM in its mask", g);
+      }
+      for (int sm = 0; sm < N; ++sm) {
+        int on[kMaxStages], non = 0;
+        for (int g = 0; g < G; ++g)
+          if ((b->group_sm_mask[g][sm >> 5] >> (sm & 31)) & 1u) on[non++] = g;
+        if (non < 2) continue;
+        KRes res[kMaxStages];
+        int qs[kMaxStages];
+        for (int i = 0; i < non; ++i) {
+          const int g = on[i], gm = b->group_model[g], q = b->blocks_per_sm[lo[g]];
+          if ((gm != VP_GROUP_MEGA && gm != VP_GROUP_RTC) || q <= 0)
+            return fail(p, VP_ERR_INVALID, "SM masks of groups overlap (SM %d): only MEGA/RTC groups with explicit "
+                                           "blocks_per_sm quotas may share SMs (coarse pipelining between groups, L27)", sm);
+          if (gm == VP_GROUP_RTC && !p->fam->rtc_legal(lo[g], hi[g]))
+            return fail(p, VP_ERR_UNSUPPORTED, "RTC group [%d,%d] has recursion, a loop or a latch", lo[g], hi[g]);
+          res[i] = kernel_res(p, lo[g], hi[g], gm == VP_GROUP_RTC);
+          qs[i] = q;
+        }
+        if (!fits_sm(p, res, qs, non))
+          return fail(p, VP_ERR_INVALID, "groups sharing SM %d: their block quotas do not fit one SM together", sm);
+      }
+      for (int g = 0; g < G && rc == VP_OK; ++g) {
         int gm = b->group_model[g];
         const uint32_t* m = b->group_sm_mask[g];
-        {
-          // KBK groups reserve their SMs too: wave kernels need resources the persistent
-          // groups do not hold (otherwise the host-launched waves could never start)
-          if (mask_count(m, N) == 0) return fail(p, VP_ERR_INVALID, "group %d has no SM in its mask", g);
-          for (int w = 0; w < kMaskWords; ++w) {
-            if (used[w] & m[w]) return fail(p, VP_ERR_INVALID, "SM masks of groups overlap (coarse pipelining between groups, L27)");
-            used[w] |= m[w];
-          }
-        }
         if (gm == VP_GROUP_RTC) {
           if (!p->fam->rtc_legal(lo[g], hi[g]))
             return fail(p, VP_ERR_UNSUPPORTED, "RTC group [%d,%d] has recursion, a loop or a latch", lo[g], hi[g]);

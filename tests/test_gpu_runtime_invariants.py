@@ -179,3 +179,30 @@ def test_online_adaptation_repeated(vpm, orc):
         rp.run()
         key, _ = rp.keys()
         assert np.array_equal(key, ref["key"])
+
+
+def test_groups_sharing_sms_fine_pipeline(vpm, orc):
+    """Groups that share SMs (a fine pipeline between groups: Fig. 5's per-SM block quotas
+    applied to group kernels): [Bound,Split] 1 block and [Dice,Shade] 2 blocks on every SM;
+    every task ran on an SM of its kernel's mask, at most `quota` blocks per (kernel, SM),
+    and the image equals the oracle's.  Quotas that cannot share an SM are rejected."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    scene = inputs.reyes_config5(n_frames=8, n_side=16)
+    rp = ReyesPipeline(scene, flags=vp.FLAG_TRACE, trace_capacity=1 << 22)
+    b = vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm), (2, 3, vp.GROUP_RTC, 0, nsm)], nsm, blocks_per_sm=[1, 0, 2, 0])
+    rp.configure(vp.HYBRID, b)
+    st = rp.run()
+    assert st["model_rerun"] == 0
+    tr = rp.p.trace(st)
+    check_trace_binding(vp, tr, st, {0: mask_sms(b, 0, nsm), 1: mask_sms(b, 1, nsm)}, nsm)
+    ref = orc.reyes_pipeline(scene)
+    key, _ = rp.keys()
+    assert np.array_equal(key, ref["key"]) and np.array_equal(rp.colours(), ref["colour"])
+    with pytest.raises(vp.VPError) as e:  # 3 + 3 blocks of ~70 KB cannot share an SM
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm), (2, 3, vp.GROUP_RTC, 0, nsm)], nsm,
+                                                blocks_per_sm=[3, 0, 3, 0]))
+    assert e.value.status == vp.VP_ERR_INVALID
+    with pytest.raises(vp.VPError):      # overlap without explicit quotas stays a coarse-pipeline error
+        rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm), (2, 3, vp.GROUP_RTC, 0, nsm)], nsm))

@@ -42,6 +42,10 @@ def cfgs(name):
         s = int(s)
         batch = [int(x) for x in bat.split("_")] if bat else None
         return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, s), (2, 3, vp.GROUP_RTC, s, nsm)], nsm, batch=batch)
+    if name.startswith("s") and len(name) == 3:  # both groups on every SM: quotas [Bound,Split] / [Dice,Shade]
+        q0, q1 = int(name[1]), int(name[2])
+        return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm), (2, 3, vp.GROUP_RTC, 0, nsm)], nsm,
+                                          blocks_per_sm=[q0, 0, q1, 0])
     if name.startswith("fine_h"):
         return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_FINE, 0, 40), (2, 3, vp.GROUP_RTC, 40, nsm)], nsm)
     raise ValueError(name)
