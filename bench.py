@@ -63,6 +63,7 @@ def parse():
     ap.add_argument("--e2e-chunk", type=int, default=64, help="frames per chunk of the streamed e2e render")
     ap.add_argument("--no-baselines", action="store_true")
     ap.add_argument("--no-suite", action="store_true", help="skip the configs 1-4 secondary measurements")
+    ap.add_argument("--no-qbench", action="store_true", help="skip the queue microbenchmark (d0)")
     ap.add_argument("--suite-tune-seconds", type=float, default=8.0)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     return ap.parse_args()
@@ -762,6 +763,7 @@ def main():
             suite = workload_suite(torch, vp, stream, args.suite_tune_seconds, pk.get("hbm_gbs", 6548.5))
         except Exception as ex:  # secondary numbers must never lose the headline line
             suite = {"error": repr(ex)}
+    if world == 1 and not args.no_qbench:
         try:
             qbench = queue_microbench(torch, vp, stream)
         except Exception as ex:

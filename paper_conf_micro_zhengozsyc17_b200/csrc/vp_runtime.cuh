@@ -409,7 +409,45 @@ struct Graph {
   static constexpr int in_base(int lo, int hi, bool rtc, int b) { return b * in_region(lo, hi, rtc); }
   static constexpr int out_base(int lo, int hi, bool rtc, int b) { return 2 * in_region(lo, hi, rtc) + b * out_region(lo, hi, rtc); }
   static constexpr int scratch_offset(int lo, int hi, bool rtc) { return out_base(lo, hi, rtc, 2); }
-  static constexpr int smem_bytes(int lo, int hi, bool rtc) { return scratch_offset(lo, hi, rtc) + scratch_of<F>(lo, hi, rtc); }
+  // Block-local queues ("distributed queues"): in a
+  // persistent, non-RTC kernel every self-recursive stage t (t -> t) gets a single-producer
+  // (publisher warp) single-consumer (fetcher warp) ring in shared memory; children of t
+  // stay in the producing block up to one batch, the rest goes to the global ring.
+  static constexpr int pow2ceil(int v) {
+    int p = 1;
+    while (p < v) p <<= 1;
+    return p;
+  }
+  // one default batch per queue (a larger configured batch just keeps fewer children
+  // local); none at all if the queues would cost the kernel a resident block per SM
+  // (shared memory: 228 KB per SM, ~1 KB reserved + ~2 KB static per block)
+  static constexpr int lq_want(int lo, int hi, bool rtc, int t) {
+    return (!rtc && !local_recursion<F>(lo, hi, rtc) && !direct_publish<F>(lo, hi, rtc) && lo <= t && t <= hi &&
+            fan(t, t) > 0)
+               ? pow2ceil(F::default_batch(t) < mb(lo, hi, false, t) ? F::default_batch(t) : mb(lo, hi, false, t))
+               : 0;
+  }
+  static constexpr int smem_blocks(int dyn) { return (228 * 1024) / (dyn + 3 * 1024); }
+  static constexpr bool lq_fits(int lo, int hi, bool rtc) {
+    const int base = scratch_offset(lo, hi, rtc) + scratch_of<F>(lo, hi, rtc);
+    int b = align128(base);
+    for (int u = 0; u < S; ++u) b += align128(lq_want(lo, hi, rtc, u) * F::stride(u));
+    return b <= 224 * 1024 && smem_blocks(b) >= smem_blocks(base);
+  }
+  static constexpr int lq_cap(int lo, int hi, bool rtc, int t) { return lq_fits(lo, hi, rtc) ? lq_want(lo, hi, rtc, t) : 0; }
+  static constexpr int lq_off(int lo, int hi, bool rtc, int t) {
+    int off = align128(scratch_offset(lo, hi, rtc) + scratch_of<F>(lo, hi, rtc));
+    for (int u = 0; u < t; ++u) off += align128(lq_cap(lo, hi, rtc, u) * F::stride(u));
+    return off;
+  }
+  static constexpr bool any_lq(int lo, int hi, bool rtc) {
+    for (int t = 0; t < S; ++t)
+      if (lq_cap(lo, hi, rtc, t) > 0) return true;
+    return false;
+  }
+  static constexpr int smem_bytes(int lo, int hi, bool rtc) {
+    return any_lq(lo, hi, rtc) ? lq_off(lo, hi, rtc, S) : scratch_offset(lo, hi, rtc) + scratch_of<F>(lo, hi, rtc);
+  }
 };
 
 // ------------------------------------------------------------------ per-block context
@@ -432,6 +470,7 @@ struct BlockShared {
   // sink groups (no ring outputs): buffer hand-over without the round barrier
   unsigned long long full[2], empty[2];  // mbarriers: fetcher -> workers, workers -> fetcher
   int bn[2], bstage[2];                // items (-1: stop) and stage of each in buffer
+  int lq_head[kMaxStages], lq_tail[kMaxStages];  // block-local queues (publisher -> fetcher)
 };
 
 // queue helpers defined below, used by Ctx::publish_warp
@@ -790,6 +829,25 @@ struct Runner {
     return smem + CtxT::kOutBase0 + b * CtxT::kOutRegion + CtxT::template OutT<T>::off;
   }
 
+  template <int T>
+  static constexpr int kLQ = G::lq_cap(LO, HI, RTC, T);
+  template <int T>
+  __device__ static __forceinline__ uint8_t* lq_buf(uint8_t* smem) { return smem + G::lq_off(LO, HI, RTC, T); }
+  // warp copy of n items between a contiguous smem batch and a block-local ring (wrap-aware)
+  template <int T, bool kToRing>
+  __device__ static __forceinline__ void lq_copy(uint8_t* smem, uint8_t* batch, int first, int n, int lane) {
+    using V = typename Chunk<F::stride(T)>::T;  // 16-B vectors when the stride allows
+    constexpr int W = Chunk<F::stride(T)>::per_item;
+    V* q = (V*)lq_buf<T>(smem);
+    V* b = (V*)batch;
+    for (int i = lane; i < n * W; i += 32) {
+      const int k = i / W, w = i - k * W;
+      const int slot = (first + k) & (kLQ<T> - 1);
+      if (kToRing) q[slot * W + w] = b[i];
+      else b[i] = q[slot * W + w];
+    }
+  }
+
   // ---------------- publisher warp: push out buffer `pb` (outputs of a batch of
   // `completed` items of stage ps) to the target rings, then retire the batch.
   // Lane T handles target T's reservation, so every L2 round trip of a publish is taken
@@ -844,10 +902,37 @@ struct Runner {
       if (a.g.group >= 0 && dg != 0) red_add(&c->gpend[a.g.group].v, dg);
       sh.acc_neg = 0;
     }
+    // block-local queues first (self-recursive targets): lane T keeps up to one batch of
+    // its children in the block, the rest (myg) goes to the global ring
+    int myloc = 0;
+    if (a.g.mode == MODE_PERSISTENT) {
+      static_for<0, S>([&](auto T_) {
+        constexpr int T = decltype(T_)::value;
+        if constexpr (kLQ<T> > 0) {
+          if (lane == T && myn > 0) {
+            const int occ = sh.lq_tail[T] - *(volatile int*)&sh.lq_head[T];
+            const int lim = a.g.batch[T] < kLQ<T> ? a.g.batch[T] : kLQ<T>;
+            myloc = lim - occ < myn ? lim - occ : myn;
+            if (myloc < 0) myloc = 0;
+          }
+          const int nl = __shfl_sync(0xffffffffu, myloc, T);
+          if (nl > 0) {
+            __threadfence_block();  // the consumer's reads of these slots came before its head update
+            lq_copy<T, true>(smem, out_buf<T>(smem, pb), sh.lq_tail[T], nl, lane);
+            __syncwarp();
+            if (lane == T) {
+              __threadfence_block();  // items before the tail that publishes them
+              *(volatile int*)&sh.lq_tail[T] = sh.lq_tail[T] + nl;
+            }
+          }
+        }
+      });
+    }
+    if (myn > 0) sh.enq[lane] += myn;
+    myn -= myloc;  // from here on: the items for the global ring, out buffer offset myloc
     unsigned long long mybase = 0;
     if (myn > 0) {
       mybase = atom_add(&c->tail[lane].v, myn);
-      sh.enq[lane] += myn;
       if (a.c.flags & FLAG_DEPTH) {
         const unsigned long long h = ld_relaxed(&c->head[lane].v);
         const unsigned long long dd = mybase + myn - h;
@@ -885,14 +970,15 @@ struct Runner {
         const int n = __shfl_sync(0xffffffffu, myn, T);
         const unsigned long long base = __shfl_sync(0xffffffffu, mybase, T);
         if (n > 0) {
+          const uint8_t* src = out_buf<T>(smem, pb) + (size_t)__shfl_sync(0xffffffffu, myloc, T) * F::stride(T);
           if constexpr (F::stride(T) % 16 == 0) {
             if (lane == 0) {
               fence_proxy_async_global();
-              bulk_out<F::stride(T)>(a.c.q[T].slots, out_buf<T>(smem, pb), base, n, a.c.q[T].cap_log2);
+              bulk_out<F::stride(T)>(a.c.q[T].slots, src, base, n, a.c.q[T].cap_log2);
             }
             bulk_used = true;
           } else {
-            copy_out<F::stride(T)>(a.c.q[T].slots, out_buf<T>(smem, pb), base, n, a.c.q[T].cap_log2, lane);
+            copy_out<F::stride(T)>(a.c.q[T].slots, src, base, n, a.c.q[T].cap_log2, lane);
           }
         }
       }
@@ -971,6 +1057,17 @@ struct Runner {
         // the pipeline, bounds live items), rings before seeds.
         static_for<0, NS>([&](auto L_) {
           constexpr int l = decltype(L_)::value, s = HI - l;
+          if constexpr (kLQ<s> > 0) {  // this block's own children of s come first
+            if (!got) {
+              const int occ = *(volatile int*)&sh.lq_tail[s] - sh.lq_head[s];
+              if (occ > 0) {
+                got = occ < a.g.batch[s] ? occ : a.g.batch[s];
+                st = s;
+                fs = 2;
+                base = (unsigned long long)sh.lq_head[s];
+              }
+            }
+          }
           if (!got && av[l] > 0) {
             got = claim_ring_avail(c, s, a.g.batch[s], av[l], base);
             if (got) { st = s; fs = 0; }
@@ -1028,7 +1125,17 @@ struct Runner {
       if (s == SS) {
         const QueueDesc& q = a.c.q[SS];
         if (kBulk) fence_proxy_async_smem();  // earlier generic writes of this buffer -> bulk writes
-        if (sh.nx_seed) {
+        if (kLQ<SS> > 0 && sh.nx_seed == 2) {  // from the block-local queue
+          if constexpr (kLQ<SS> > 0) {
+            __threadfence_block();  // the items the observed tail published
+            lq_copy<SS, false>(smem, dst, (int)base, n, lane);
+            __syncwarp();
+            if (lane == 0) {
+              __threadfence_block();  // reads of the slots before the head frees them
+              *(volatile int*)&sh.lq_head[SS] = sh.lq_head[SS] + n;
+            }
+          }
+        } else if (sh.nx_seed) {
           if constexpr (kBulk) {
             if (lane == 0) {
               mbar_arrive_expect_tx(mb, (uint32_t)(n * F::stride(SS)));
@@ -1202,6 +1309,7 @@ struct Runner {
       sh.work[0] = sh.work[1] = 0;
       sh.nx_n = 0;
       sh.nx_stage = -1;
+      for (int t = 0; t < kMaxStages; ++t) sh.lq_head[t] = sh.lq_tail[t] = 0;
       if (g.mode == MODE_WAVE) {
         long long wn = g.wave_n, wc = g.wave_chunk;
         if (g.wave_n_dev) {
