@@ -37,6 +37,7 @@ MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
 # per grid point 3 coords x 7 + M.p 28 + screen 9 (3 div, 6 mul/add) + Q8 snap 2 = 5616
 FLOP_DICE = 36 * 3 * 7 + 81 * (3 * 7 + 28 + 9 + 2)
 FLOP_SHADE = 64 * 41                 # edges, cross, |n|, n.L, sqrt/div, shade, zq, Q8 snap = 2624
+FLOP_SHADE_MP = 41                   # per micropolygon actually shaded (box holds a pixel centre)
 FLOP_BOUND = 16 * (28 + 9) + 40      # 16 projections + split metric = 632
 FLOP_SPLIT = 3 * 4 * 12              # de Casteljau, 3 coords x 4 curves = 144
 
@@ -655,13 +656,18 @@ def main():
     nk = st["num_kernels"]
     kmean = np.mean(np.array(kms), axis=0) if nk else np.array([ms_per_step])
     d = st["dequeued"]
-    per_stage_flop = [FLOP_BOUND, FLOP_SPLIT, FLOP_DICE, FLOP_SHADE]
+    units = st.get("work_units", [0] * 8)
+    # Shade flops are counted per micropolygon the fused chain actually shades (those whose
+    # box holds a pixel centre, vp_run_stats.work_units) -- 64 per grid only if Shade ran
+    # unfused and no count exists
+    shade_flop = units[3] * FLOP_SHADE_MP if units[3] else d[3] * FLOP_SHADE
+    stage_flop = [d[0] * FLOP_BOUND, d[1] * FLOP_SPLIT, d[2] * FLOP_DICE, shade_flop]
     # persistent groups co-run for the whole step, so the dominant kernel is the one
     # with the most algorithmic work; its time is its own CUDA-event duration
-    kflop = [sum(d[s] * per_stage_flop[s] for s in range(k[0], k[1] + 1)) for k in st["kernels"]] if nk else [0]
+    kflop = [sum(stage_flop[s] for s in range(k[0], k[1] + 1)) for k in st["kernels"]] if nk else [0]
     dom = int(np.argmax(kflop)) if nk else 0
     lo, hi, _ = st["kernels"][dom] if nk else (0, 3, 0)
-    dom_flop = sum(d[s] * per_stage_flop[s] for s in range(lo, hi + 1))
+    dom_flop = sum(stage_flop[s] for s in range(lo, hi + 1))
     pk = peaks()
     sm_max = pk.get("sm_max_mhz", 1965.0)
     # fp32 non-FMA issue peak: 148 SMs x 128 lanes x 1 op/clk (FMA contraction is disabled
@@ -673,15 +679,27 @@ def main():
     # traffic: dram bytes per leaf from the committed ncu --set full capture of this kernel
     # (profiles/r1_rtc_leaf_traffic.json), times the leaves this launch processed
     traffic = None
-    try:
-        tr = json.load(open(os.path.join(ROOT, "profiles", "r1_rtc_leaf_traffic.json")))
-        if (lo, hi) == (2, 3):
-            traffic = tr["bytes_per_leaf"] * d[2]
+    traffic_src = None
+    for name in ("r2_rtc_leaf_traffic.json", "r1_rtc_leaf_traffic.json"):
+        try:
+            tr = json.load(open(os.path.join(ROOT, "profiles", name)))
+            if (lo, hi) == (2, 3):
+                traffic = tr["bytes_per_leaf"] * d[2]
+                traffic_src = f"ncu dram__bytes_read+write per leaf (profiles/{name}) x leaves"
+            break
+        except Exception:
+            continue
+    issue = None
+    try:  # issue-slot view of the same kernels (the bound that actually binds), from committed captures
+        issue = json.load(open(os.path.join(ROOT, "profiles", "r2_reyes_kernels.json")))
     except Exception:
         pass
     roofline = {"bound": "alu", "achieved": achieved, "peak": alu_peak, "unit": "TFLOP/s",
                 "frac": achieved / alu_peak, "traffic": traffic,
-                "traffic_source": "ncu dram__bytes_read+write per leaf (profiles/r1_rtc_leaf_traffic.json) x leaves",
+                "flop_count": {"shaded_micropolygons": int(units[3]), "dice_leaves": int(d[2]),
+                               "shade_flop_per_mp": FLOP_SHADE_MP, "dice_flop_per_leaf": FLOP_DICE},
+                "issue_bound": issue,
+                "traffic_source": traffic_src,
                 "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if is_rtc else 'MEGA'}>",
                 "peak_source": "derived: SMs x 128 fp32 lanes x clocks.max.sm (MEASURED_PEAKS sm_max_mhz), non-FMA",
                 "kernel_ms": float(kmean[dom]), "kernel_share_of_step": float(kmean[dom] / ms_per_step)}

@@ -208,6 +208,9 @@ typedef struct vp_run_stats {
   /* 1: the planned groups were not co-resident (ABORT_NOT_CORESIDENT), so the run was
    * repeated from its seeds as one cooperative megakernel; device_ms covers both attempts */
   int model_rerun;
+  /* family-defined work units per stage (Reyes: micropolygons shaded by the fused
+   * [Dice, Shade] chain, i.e. those whose box holds a pixel centre; 0 elsewhere) */
+  uint64_t work_units[VP_MAX_STAGES];
 } vp_run_stats;
 
 typedef struct vp_autotune_opts {

@@ -1139,6 +1139,7 @@ struct ReyesF {
         tot += c0 + __popc(m1);
       }
       __syncwarp();
+      if (lane == 0) ctx.template note_units<SHADE>(tot);
       for (int t = lane; t < tot; t += 32) {
         const int e = list[t];
         shade_mp(p, (e >> 6) ? g1 : g0, e & 63);

@@ -78,6 +78,9 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
     c->idle_ns[t] = 0;
     c->rounds[t] = 0;
   }
+  if (t < kMaxStages) {
+    c->units[t] = 0;
+  }
   if (t < kMaxKernels) {
     c->arrivals[t].v = 0;
     c->admitted[t].v = 0;
@@ -1390,6 +1393,7 @@ static vp_status run_once(vp_pipeline_s* p, cudaStream_t st, vp_run_stats* stats
     }
     stats->pending = (int64_t)hc.pending.v;
     stats->dispatch_timeouts = dispatch_timeouts;
+    for (int s = 0; s < S; ++s) stats->work_units[s] = hc.units[s];
     stats->model_rerun = 0;
   }
   if (hc.abort.v != ABORT_NONE) {

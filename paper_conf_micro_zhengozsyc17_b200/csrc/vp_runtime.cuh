@@ -70,6 +70,7 @@ struct Ctrl {
   unsigned long long flush_ns[kMaxStages];  // FLAG_TIMERS: publish (queue overhead) per stage
   unsigned long long idle_ns[kMaxKernels];  // FLAG_TIMERS: blocks finding no work, per kernel
   unsigned long long rounds[kMaxKernels];   // persistent-loop rounds, summed over blocks, per kernel
+  unsigned long long units[kMaxStages];     // family-defined work units per stage (vp_run_stats.work_units)
   Line gpend[kMaxKernels];                  // online adaptation: items alive in each group's stages
   unsigned long long retired[kMaxKernels];  // online adaptation: group drained for good, its blocks exit
   unsigned long long exits[kMaxKernels];    // admitted blocks of each kernel slot that have exited
@@ -461,6 +462,7 @@ struct BlockShared {
   unsigned long long idle_since;       // %globaltimer when the fetcher last started idling (0: busy)
   unsigned long long deq[kMaxStages];
   unsigned long long enq[kMaxStages];
+  uint32_t units32[kMaxStages];        // family-defined work units (Ctx::note_units)
   uint32_t deq32[kMaxStages], enq32[kMaxStages];  // counts added by several warps at once (native
                                                   // 32-bit shared atomics; 64-bit ones are CAS loops)
   unsigned long long t_exec[kMaxStages], t_flush[kMaxStages], t_idle, rounds;
@@ -601,6 +603,12 @@ struct Ctx {
         a.c.trace[idx].block = blockIdx.x;
       }
     }
+  }
+  // Family-defined work units of stage T (vp_run_stats.work_units; e.g. Reyes: the
+  // micropolygons Shade actually shades), from any number of threads at once.
+  template <int T>
+  __device__ __forceinline__ void note_units(int n) {
+    if (n) atomicAdd(&sh.units32[T], (uint32_t)n);
   }
   // ... or given the task's item id directly (items that live only in registers).
   template <int T>
@@ -1294,7 +1302,7 @@ struct Runner {
       for (int s = 0; s < kMaxStages; ++s) {
         sh.out_cnt[0][s] = sh.out_cnt[1][s] = 0;
         sh.deq[s] = sh.enq[s] = 0;
-        sh.deq32[s] = sh.enq32[s] = 0;
+        sh.deq32[s] = sh.enq32[s] = sh.units32[s] = 0;
         sh.t_exec[s] = sh.t_flush[s] = 0;
       }
       sh.t_idle = 0;
@@ -1342,6 +1350,7 @@ struct Runner {
         const unsigned long long dq = sh.deq[s] + sh.deq32[s], eq = sh.enq[s] + sh.enq32[s];
         if (dq) atomicAdd(&c->deq[s], dq);
         if (eq) atomicAdd(&c->enq[s], eq);
+        if (sh.units32[s]) atomicAdd(&c->units[s], (unsigned long long)sh.units32[s]);
         if (sh.t_exec[s]) atomicAdd(&c->exec_ns[s], sh.t_exec[s]);
         if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
       }
@@ -1386,10 +1395,12 @@ struct Runner {
   }
   // ... or its warps publish their outputs themselves (direct-publish kernels)
   static constexpr bool sink_group() { return direct_publish<F>(LO, HI, RTC) || no_ring_outputs(); }
-  // A sink group has no publisher warp: its blocks are the 8 worker warps + the fetcher, so
-  // the register file is divided among 9 warps, not 10 (more registers per thread at the
-  // same resident blocks per SM).
-  static constexpr int kBlockThreads = sink_group() ? kThreads + 32 : kBlock;
+  // A direct-publish kernel has no publisher warp at all: its blocks are the 8 worker
+  // warps + the fetcher, so the register file is divided among 9 warps, not 10 (72
+  // registers at 3 blocks/SM instead of 64: the Reyes [Bound, Split] kernel loses its
+  // spills).  Measured A/B for the other sink groups (the fused [Dice, Shade] kernel):
+  // 288 threads at 72 registers was 7% slower than 320 at 64, so they keep 320.
+  static constexpr int kBlockThreads = direct_publish<F>(LO, HI, RTC) ? kThreads + 32 : kBlock;
 
   static __device__ void run_sink(const KArgs<F>& a, CtxT& ctx, BlockShared& sh, uint8_t* smem) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;

@@ -79,7 +79,8 @@ class RunStats(C.Structure):
                 ("kernel_idle_ns", C.c_uint64 * 16), ("ring_tail", C.c_uint64 * MAX_STAGES),
                 ("ring_head", C.c_uint64 * MAX_STAGES), ("ring_count", C.c_int64 * MAX_STAGES),
                 ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16),
-                ("stage_wave_ms", C.c_float * MAX_STAGES), ("dispatch_timeouts", C.c_int), ("model_rerun", C.c_int)]
+                ("stage_wave_ms", C.c_float * MAX_STAGES), ("dispatch_timeouts", C.c_int), ("model_rerun", C.c_int),
+                ("work_units", C.c_uint64 * MAX_STAGES)]
 
 
 class AutotuneOpts(C.Structure):
@@ -381,7 +382,7 @@ def stats_dict(st: RunStats):
                 ring_head=list(st.ring_head), ring_count=list(st.ring_count), seed_head=list(st.seed_head),
                 pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]),
                 stage_wave_ms=list(st.stage_wave_ms), dispatch_timeouts=st.dispatch_timeouts,
-                model_rerun=st.model_rerun)
+                model_rerun=st.model_rerun, work_units=list(st.work_units))
 
 
 def config_to_string(cfg: Config) -> str:
