@@ -205,7 +205,7 @@ __device__ void raster_tri(const vp_reyes_params& p, FbRec* fb, long long ax, lo
 
 // Scratch of the fused [Dice, Shade] chain.
 struct ChainScratch {
-  float4 M[kWarpsW][4];        // per-warp copy of the patch's frame matrix (rows)
+  float4 M[kWarpsW][2][4];     // per-warp copies of the pair's frame matrices (rows)
   float B[kWarpsW][36];        // per-warp Bernstein table B_b(j/8), [9][4]
   uint8_t list[kWarpsW][128];  // per-warp compacted list of pixel-covering micropolygons (q | grid << 6)
 };
@@ -849,33 +849,41 @@ struct ReyesF {
   // Ms: the frame matrix rows in shared memory (fused chain), else read from p.M.
   // Bt (fused chain): the Bernstein weights B_b(j/8) as a [9][4] shared-memory table,
   // computed by bernstein() itself (bit-identical to evaluating it per point).
-  template <bool kSmemM = false>
+  // the u-curve point C_a(v_j), e = 9a + j, of patch P into out's rows 3..5 (one lane)
+  template <bool kSmemM>
+  static __device__ __forceinline__ void dice_c(const RPatch* P, RGrid* out, int e, const float* Bt) {
+    const int a = e / kNG, j = e - a * kNG;
+    float Bv[4];
+    if constexpr (kSmemM) {
+#pragma unroll
+      for (int b = 0; b < 4; ++b) Bv[b] = Bt[4 * j + b];
+    } else {
+      bernstein((float)j * 0.125f, Bv);
+    }
+    float cx = 0.0f, cy = 0.0f, cz = 0.0f;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const float4 cp = P->cp[4 * a + b];
+      cx = cx + Bv[b] * cp.x;
+      cy = cy + Bv[b] * cp.y;
+      cz = cz + Bv[b] * cp.z;
+    }
+    out->g[3][e] = cx;
+    out->g[4][e] = cy;
+    out->g[5][e] = cz;
+  }
+
+  // kHaveC: the caller already computed the u-curve points (the fused chain does both
+  // patches of a pair in one loop: 72 points in 3 warp passes instead of 2 x 2)
+  template <bool kSmemM = false, bool kHaveC = false>
   static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
                                                     const float4* Ms = nullptr, const float* Bt = nullptr) {
     const uint32_t frame = frame_of(p, P->id);
     const float* M = p.M + 16 * (size_t)frame;
-    for (int e = lane; e < 4 * kNG; e += 32) {  // C_a(v_j), e = 9a + j
-      const int a = e / kNG, j = e - a * kNG;
-      float Bv[4];
-      if constexpr (kSmemM) {
-#pragma unroll
-        for (int b = 0; b < 4; ++b) Bv[b] = Bt[4 * j + b];
-      } else {
-        bernstein((float)j * 0.125f, Bv);
-      }
-      float cx = 0.0f, cy = 0.0f, cz = 0.0f;
-#pragma unroll
-      for (int b = 0; b < 4; ++b) {
-        const float4 cp = P->cp[4 * a + b];
-        cx = cx + Bv[b] * cp.x;
-        cy = cy + Bv[b] * cp.y;
-        cz = cz + Bv[b] * cp.z;
-      }
-      out->g[3][e] = cx;
-      out->g[4][e] = cy;
-      out->g[5][e] = cz;
+    if constexpr (!kHaveC) {
+      for (int e = lane; e < 4 * kNG; e += 32) dice_c<kSmemM>(P, out, e, Bt);  // C_a(v_j), e = 9a + j
+      __syncwarp();
     }
-    __syncwarp();
     // S(u_i, v_j): object-space rows 0..2 are written at once (the C rows 3..5 are still
     // being read by other lanes, so the screen rows wait for the next __syncwarp)
 #pragma unroll
@@ -1117,17 +1125,26 @@ struct ReyesF {
       k = __shfl_sync(0xffffffffu, k, 0);
       if (k >= n) break;
       const int np = min(2, n - k);
+      const RPatch* P0 = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
+      const RPatch* P1 = P0 + (np > 1 ? 1 : 0);
+      // both frame matrices (lanes 0..15: patch 0, 16..31: patch 1) and the u-curve points
+      // of both patches (72 points, 3 passes)
+      if ((lane >> 4) < np) {
+        const RPatch* P = (lane >> 4) ? P1 : P0;
+        ((float*)cs.M[warp][lane >> 4])[lane & 15] = __ldg(p.M + 16 * (size_t)frame_of(p, P->id) + (lane & 15));
+      }
+      for (int e2 = lane; e2 < 36 * np; e2 += 32) {
+        const bool second = e2 >= 36;
+        dice_c<true>(second ? P1 : P0, second ? g1 : g0, e2 - (second ? 36 : 0), Bt);
+      }
+      __syncwarp();
       int tot = 0;
 #pragma unroll
       for (int j = 0; j < 2; ++j) {
         if (j >= np) break;
         RGrid* g = j ? g1 : g0;
-        const RPatch* P = (const RPatch*)(items + (size_t)(k + j) * sizeof(RPatch));
-        const uint32_t frame = frame_of(p, P->id);
-        __syncwarp();  // the previous patch's dice is done with the matrix
-        if (lane < 16) ((float*)cs.M[warp])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
-        __syncwarp();
-        dice_patch<true>(p, P, g, lane, cs.M[warp], Bt);
+        const RPatch* P = j ? P1 : P0;
+        dice_patch<true, true>(p, P, g, lane, cs.M[warp][j], Bt);
         __syncwarp();
         if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
         const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
