@@ -197,7 +197,9 @@ struct KernelPlan {
   int group = -1;        // = kslot of the group's primary kernel
   bool can_retire = false;
   uint32_t feeders = 0;  // groups emitting into this kernel's stages
-  int refill = -1;       // kernel whose group gets this kernel's SMs when it retires
+  int refill = -1;       // kernel whose group gets this kernel's SMs when it retires (if no
+                         // candidate has stalled work at that moment)
+  uint32_t refill_cands = 0;  // persistent groups downstream of this one (refill candidates)
 };
 
 struct Plan {
@@ -236,6 +238,8 @@ struct vp_pipeline_s {
   uint32_t* d_arrive = nullptr;
   volatile uint32_t* h_retire = nullptr;  // mapped pinned: per-kernel "retired, SMs free" flags
   uint32_t* d_retire = nullptr;
+  volatile long long* h_gpend = nullptr;  // mapped pinned: group alive counts at each retirement
+  long long* d_gpend = nullptr;
   uint32_t epoch = 0;
   cudaStream_t streams[kMaxKernels] = {};
   cudaEvent_t ev_fork = nullptr, ev_start = nullptr, ev_end = nullptr, ev_join[kMaxKernels] = {};
@@ -245,6 +249,7 @@ struct vp_pipeline_s {
   double timeout_ms = 30000;
   // device-driven KBK: instantiated graph and the launch arguments it was captured with
   int refill_lo[kMaxKernels] = {}, refill_hi[kMaxKernels] = {}, refill_quota[kMaxKernels] = {};
+  int refill_pick[kMaxKernels] = {};  // kernel whose group each retired kernel's SMs went to
   bool launched[kMaxKernels] = {};  // planned kernels launched by the last vp_run
   // host-driven KBK: per-wave event pairs (pooled) and the stage of each wave of the last run
   std::vector<cudaEvent_t> wave_ev;
@@ -380,6 +385,7 @@ Common make_common(vp_pipeline_s* p) {
   c.n_stages = (int)p->st.size();
   c.host_arrive = p->d_arrive;
   c.host_retire = p->d_retire;
+  c.host_gpend = p->d_gpend;
   c.epoch = p->epoch;
   for (int s = 0; s < kMaxStages; ++s) c.stage_group[s] = p->plan.online ? p->plan.stage_group[s] : (int8_t)-1;
   return c;
@@ -688,7 +694,10 @@ vp_status build_plan(vp_pipeline_s* p, int model, const vp_sm_binding* b, int ba
       }
       int best = -1;
       for (const KernelPlan& j : pl.kernels)
-        if (j.lo > k.hi && !j.coop && (best < 0 || j.lo < pl.kernels[best].lo)) best = j.kslot;
+        if (j.lo > k.hi && !j.coop) {
+          k.refill_cands |= 1u << j.kslot;
+          if (best < 0 || j.lo < pl.kernels[best].lo) best = j.kslot;
+        }
       k.refill = best;
     }
   }
@@ -961,6 +970,7 @@ static void free_pipeline(vp_pipeline_s* p) {
   if (p->h_blk) cudaFreeHost(p->h_blk);
   if (p->h_arrive) cudaFreeHost((void*)p->h_arrive);
   if (p->h_retire) cudaFreeHost((void*)p->h_retire);
+  if (p->h_gpend) cudaFreeHost((void*)p->h_gpend);
   for (int i = 0; i < kMaxKernels; ++i) {
     if (p->streams[i]) cudaStreamDestroy(p->streams[i]);
     if (p->ev_join[i]) cudaEventDestroy(p->ev_join[i]);
@@ -1013,6 +1023,11 @@ vp_status vp_pipeline_create(int device, const vp_pipeline_desc* d, void** out) 
     memset(hr, 0, sizeof(uint32_t) * kMaxKernels);
     p->h_retire = (volatile uint32_t*)hr;
     if (bad(cudaHostGetDevicePointer((void**)&p->d_retire, hr, 0))) return VP_ERR_CUDA;
+    void* hg = nullptr;
+    if (bad(cudaHostAlloc(&hg, sizeof(long long) * kMaxKernels * kMaxKernels, cudaHostAllocMapped))) return VP_ERR_OOM;
+    memset(hg, 0, sizeof(long long) * kMaxKernels * kMaxKernels);
+    p->h_gpend = (volatile long long*)hg;
+    if (bad(cudaHostGetDevicePointer((void**)&p->d_gpend, hg, 0))) return VP_ERR_CUDA;
   }
   if (p->desc.flags & VP_FLAG_TRACE)
     if (bad(cudaMalloc(&p->trace, sizeof(TraceRec) * (size_t)p->desc.trace_capacity))) return VP_ERR_OOM;
@@ -1302,7 +1317,21 @@ static vp_status run_once(vp_pipeline_s* p, cudaStream_t st, vp_run_stats* stats
         const KernelPlan& k = pl.kernels[i];
         if (handled[i] || k.refill < 0 || p->h_retire[i] != p->epoch || nk_total >= kMaxKernels) continue;
         handled[i] = true;
-        const KernelPlan& t = pl.kernels[k.refill];
+        // the freed SMs go to the group that has the most stalled items at
+        // that moment (the retiring block's snapshot of every group's alive count); the
+        // first downstream group when none has any
+        int pick = k.refill;
+        long long most = 0;
+        for (uint32_t m = k.refill_cands; m; m &= m - 1) {
+          const int j = __builtin_ctz(m);
+          const long long alive = p->h_gpend[i * kMaxKernels + pl.kernels[j].group];
+          if (alive > most) {
+            most = alive;
+            pick = j;
+          }
+        }
+        p->refill_pick[i] = pick;
+        const KernelPlan& t = pl.kernels[pick];
         const int slot = nk_total++;
         GroupArgs g;
         memset(&g, 0, sizeof(g));

@@ -106,6 +106,8 @@ struct Common {
   volatile uint32_t* host_arrive;  // mapped pinned host words: grid of kernel k fully dispatched;
                                    // [kMaxKernels]: the run aborted as not co-resident
   volatile uint32_t* host_retire;  // mapped pinned host words: every block of kernel k exited on retirement
+  volatile long long* host_gpend;  // mapped pinned [kMaxKernels][kMaxKernels]: every group's alive count,
+                                   // snapshotted when kernel k retires (the host's refill choice)
   uint32_t epoch;                  // run counter written into host_arrive / host_retire
   int8_t stage_group[kMaxStages];  // online adaptation: group of each stage (-1: none / KBK)
   uint32_t peer_mask;              // planned persistent kernel slots of this run: a block stalled
@@ -1292,8 +1294,7 @@ struct Runner {
         if (!good && t == (unsigned long long)gridDim.x - 1 && g.group >= 0 && a.c.host_retire &&
             *(volatile unsigned long long*)&c->retired[g.group] &&
             *(volatile unsigned long long*)&c->exits[g.kslot] == ld_relaxed(&c->admitted[g.kslot].v)) {
-          a.c.host_retire[g.kslot] = a.c.epoch;
-          __threadfence_system();
+          signal_retired(a, g.kslot);
         }
       } else if (sm < (uint32_t)kMaxSM) {
         atomicAdd(&a.c.blk[g.kslot * kMaxSM + sm], 1u);
@@ -1340,6 +1341,18 @@ struct Runner {
     return ok != 0;
   }
 
+  // Tell the host that kernel k's SMs are free (online adaptation), with a snapshot of every
+  // group's alive count so the host can give them to the group with the most stalled work.
+  static __device__ void signal_retired(const KArgs<F>& a, int kslot) {
+    if (a.c.host_gpend) {
+      for (int g = 0; g < kMaxKernels; ++g)
+        a.c.host_gpend[kslot * kMaxKernels + g] = (long long)ld_relaxed(&a.c.ctrl->gpend[g].v);
+      __threadfence_system();
+    }
+    a.c.host_retire[kslot] = a.c.epoch;
+    __threadfence_system();
+  }
+
   static __device__ void flush_stats(const KArgs<F>& a, BlockShared& sh) {
     if (threadIdx.x == 0) {
       Ctrl* c = a.c.ctrl;
@@ -1365,8 +1378,7 @@ struct Runner {
         if (*(volatile unsigned long long*)&c->retired[a.g.group] &&
             ld_relaxed(&c->arrivals[a.g.kslot].v) == (unsigned long long)gridDim.x &&
             e == ld_relaxed(&c->admitted[a.g.kslot].v)) {
-          a.c.host_retire[a.g.kslot] = a.c.epoch;
-          __threadfence_system();
+          signal_retired(a, a.g.kslot);
         }
       }
     }

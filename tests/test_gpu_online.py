@@ -107,3 +107,25 @@ def test_reyes_l2_persist_parity(vpm, orc, model):
         rp.configure({"megakernel": vp.MEGAKERNEL, "kbk_graph": vp.KBK_GRAPH}[model])
     for _ in range(2):
         check_against_oracle(orc, scene, rp, rp.run())
+
+
+def test_refill_goes_to_the_most_stalled_group(vpm, orc):
+    """the freed SMs go to the group with stalled work.  Raster with
+    [Vertex,Clip] (retires first), [Raster] and a deliberately small [Fragment] group: at
+    the retirement Fragment holds far more live items than Raster, so the refill grid runs
+    Fragment, not the first group downstream; the frame stays bit-exact."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import RasterPipeline
+    vp = vpm
+    nsm, _ = vp.device_info(0)
+    scene = inputs.raster_scene(200_000, W=1920, H=1080)
+    rp = RasterPipeline(scene, flags=vp.FLAG_ONLINE)
+    rp.configure(vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_RTC, 0, 40), (2, 2, vp.GROUP_MEGA, 40, 124),
+                                             (3, 3, vp.GROUP_MEGA, 124, nsm)], nsm))
+    ref = orc.raster_pipeline(scene)
+    picked = []
+    for _ in range(3):
+        st = rp.run()
+        assert np.array_equal(rp.keys(), ref["key"]) and np.array_equal(rp.colours(), ref["colour"])
+        picked += [tuple(k[:2]) for k in st["kernels"][3:]]
+    assert picked, "the [Vertex,Clip] group never retired before the end"
+    assert all(k == (3, 3) for k in picked), picked
