@@ -25,12 +25,6 @@ namespace vp {
 #ifndef VP_BS_MINB          // resident blocks/SM the block-local [Bound, Split] kernel is built for
 #define VP_BS_MINB 3
 #endif
-#ifndef VP_BS_STACK         // its shared-memory work stack (patches) = its Bound dump capacity
-#define VP_BS_STACK 48
-#endif
-#ifndef VP_BS_DICE          // its Dice out-buffer capacity per round
-#define VP_BS_DICE 48
-#endif
 
 struct RPatch {           // 272 B
   float4 cp[16];          // P[a][b] at cp[4a+b]; a = u index, b = v index
@@ -218,12 +212,14 @@ struct ReyesF {
   static constexpr int stride(int s) { return s == SHADE ? (int)sizeof(RGrid) : (int)sizeof(RPatch); }
   static constexpr int threads_per_item(int s) { return s == BOUND ? 16 : s == SPLIT ? 16 : s == DICE ? 32 : 64; }
   static constexpr int max_batch(int s) { return s == BOUND ? 32 : s == SPLIT ? 16 : s == DICE ? 64 : 4; }
-  // Dice batches above 8 only in the fused RTC [Dice, Shade] kernel, whose grids stay in
-  // one block-local slot per warp; elsewhere every diced grid needs an out-buffer slot.
+  // Dice batches above 8 only where the fused [Dice, Shade] chain runs them (grids in one
+  // block-local slot per warp): the RTC kernel (64) and a megakernel with depth-first
+  // [Bound, Split] (32: the in buffers stay at the Bound batch's size); elsewhere every
+  // diced grid needs an out-buffer slot.
   static constexpr int kernel_max_batch(int lo, int hi, bool rtc, int s) {
-    // block-local [Bound, Split]: the first stack pass takes the whole claimed batch
-    if (!rtc && lo == BOUND && hi == SPLIT && (s == BOUND || s == SPLIT)) return s == BOUND ? 32 : 16;  // DFS kernel
-    if (!rtc && lo == BOUND && hi >= SPLIT && (s == BOUND || s == SPLIT)) return 16;
+    // depth-first [Bound, Split] (exec_dfs): 32 seeds per claim, two per 16-thread group
+    if (!rtc && lo == BOUND && hi >= SPLIT && (s == BOUND || s == SPLIT)) return s == BOUND ? 32 : 16;  // DFS kernels
+    if (s == DICE && !rtc && lo == BOUND && hi == SHADE) return 32;
     return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
   }
   static constexpr int fused_local_cap(int, int, int) { return kThreads / 32; }
@@ -239,9 +235,8 @@ struct ReyesF {
   // non-RTC ones (a megakernel [Bound..Shade] must not pay for the chain's scratch: it sits
   // at the edge of 2 blocks per SM)
   static constexpr int scratch_bytes_k(int lo, int hi, bool rtc) {
-    return ((rtc && lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
-           ((!rtc && lo == BOUND && hi == SPLIT) ? (int)((sizeof(DfsScratch) + 127) / 128 * 128) : 0) +
-           ((!rtc && lo == BOUND && hi > SPLIT) ? (int)((sizeof(LocalStack) + 127) / 128 * 128) : 0);
+    return (((rtc || local_recursion(lo, hi)) && lo <= DICE && hi == SHADE) ? (int)sizeof(ChainScratch) : 0) +
+           ((!rtc && lo == BOUND && hi >= SPLIT) ? (int)((sizeof(DfsScratch) + 127) / 128 * 128) : 0);
   }
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
@@ -530,24 +525,11 @@ struct ReyesF {
     }
   }
 
-  // -------------------------------------------------------------- [Bound, Split] locally
-  // Block-local recursion (the paper fuses Bound into Split, L55): a batch
-  // of Bound (or Split) items is worked off from a shared-memory stack.  Each pass pops up
-  // to 16 patches (16 threads each), bounds them, culls, appends diceable ones to the Dice
-  // out buffer and splits the others in place, pushing both children back.  Only what is
-  // left when the stack or the Dice buffer would overflow goes back to the Bound ring, so
-  // Split items never travel through a ring.  Same arithmetic as bound() / split().
-  static constexpr int kStack = VP_BS_STACK, kLocalDice = VP_BS_DICE;
-  struct LocalStack {
-    RPatch st[kStack];
-    float4 M[4];        // the batch's frame matrix rows
-    int nchild[2], nsplit, dump;
-    uint32_t mframe;
-  };
   static constexpr bool local_recursion(int lo, int hi) { return lo == BOUND && hi >= SPLIT; }
-  static constexpr int local_out_cap(int, int hi, int t) {
-    return t == BOUND ? kStack : t == DICE ? kLocalDice : (t == SHADE && hi >= DICE) ? 8 : 0;
-  }
+  // out buffers of a local-recursion kernel: none for Bound / Split / Dice (split nodes stay
+  // in the warp, Dice items are published by the warps); a megakernel's Dice batches still
+  // hand their grids to Shade through the out buffer
+  static constexpr int local_out_cap(int, int hi, int t) { return (t == SHADE && hi >= DICE) ? 8 : 0; }
 
   // -------------------------------------------------------------- [Bound, Split] DFS
   // The [Bound, Split] group's own kernel (hi == Split): each warp works
@@ -729,117 +711,13 @@ struct ReyesF {
     }
   }
 
+  // Block-local recursion (the paper fuses Bound into Split, L55): a kernel that runs Bound
+  // and Split -- the [Bound, Split] group's own kernel or a megakernel -- works their
+  // batches depth first (exec_dfs); a megakernel's later stages run as usual.
   template <int SS, int LO, int HI, class Ctx>
   static __device__ void exec_local(Ctx& ctx, const uint8_t* items, int n) {
-    if constexpr (SS == DICE || SS == SHADE) {  // a megakernel's later stages run as usual
-      exec<SS>(ctx, items, n);
-      return;
-    } else if constexpr (HI == SPLIT) {
-      exec_dfs<SS>(ctx, items, n);
-      return;
-    }
-
-    const Params& p = ctx.params();
-    LocalStack& ls = *(LocalStack*)ctx.scratch();
-    const int lane = threadIdx.x & 15, grp = threadIdx.x >> 4;
-    if constexpr (SS == BOUND) {
-      for (int e = threadIdx.x; e < n * 17; e += kThreads) ((uint4*)ls.st)[e] = ((const uint4*)items)[e];
-    } else {
-      for (int r0 = 0; r0 < n; r0 += kThreads / 16) {  // Split items: their Bound already chose the direction
-        const int k = r0 + grp;
-        if (k < n) {
-          const RPatch* P = (const RPatch*)(items + (size_t)k * sizeof(RPatch));
-          const uint32_t depth = P->depth;
-          const int dir = (int)((P->dirs >> depth) & 1u);
-          float4 L, R;
-          int my;
-          split_cp(P, dir, lane, L, R, my);
-          ls.st[2 * k].cp[my] = L;
-          ls.st[2 * k + 1].cp[my] = R;
-          if (lane == 0) split_headers(&ls.st[2 * k], &ls.st[2 * k + 1], P->id, P->path, P->dirs, depth, dir);
-        }
-      }
-    }
-    if (threadIdx.x == 0) ls.nchild[0] = ls.nchild[1] = ls.nsplit = 0;
-    {
-      uint32_t frame = frame_of(p, ((const RPatch*)items)->id);
-      if (threadIdx.x < 16) ((float*)ls.M)[threadIdx.x] = __ldg(p.M + 16 * (size_t)frame + threadIdx.x);
-      if (threadIdx.x == 0) ls.mframe = frame;
-    }
-    worker_sync();
-    int top = (SS == BOUND) ? n : 2 * n, nbound = 0;
-    bool first = SS == BOUND;  // the first pass pops exactly the claimed Bound items (n <= 16)
-    for (int pass = 0;; ++pass) {
-      const int dice_room = Ctx::template cap<DICE>() - ctx.sh.out_cnt[ctx.ob][DICE];
-      const int m = min(min(kThreads / 16, top), min(kStack - top, dice_room));
-      if (m <= 0) break;
-      const int base = top - m;
-      const bool mine = grp < m;
-      const RPatch* P = &ls.st[base + (mine ? grp : 0)];
-      int dir;
-      float4 q;
-      const int cls = bound_patch(p, P, lane, mine, dir, q, ls.M, ls.mframe);
-      const uint32_t id = P->id, path = P->path, dirs = P->dirs, depth = P->depth;
-      float4 L, R;
-      int my = 0;
-      if (cls == 1) split_cp(P, dir, lane, L, R, my);
-      if (lane == 0 && mine) {
-        if (!first) ctx.template trace_local<BOUND>((const uint8_t*)P);
-        if (cls == 1) ctx.template trace_local<SPLIT>((const uint8_t*)P);
-      }
-      const unsigned gm = 0xFFFFu << (threadIdx.x & 16);
-      if (cls == 2) {
-        int slot = 0;
-        if (lane == 0) slot = ctx.template reserve<DICE>();
-        slot = __shfl_sync(gm, slot, threadIdx.x & 16, 32);
-        if (slot >= 0) {
-          RPatch* out = (RPatch*)ctx.template out_ptr<DICE>(slot);
-          out->cp[lane] = q;
-          if (lane == 0) {
-            out->id = id;
-            out->path = path;
-            out->dirs = dirs;
-            out->depth = depth;
-          }
-        }
-      }
-      worker_sync();  // every read of the popped patches is done
-      int* nchild = &ls.nchild[pass & 1];
-      if (cls == 1) {
-        int c = 0;
-        if (lane == 0) {
-          c = atomicAdd(nchild, 2);
-          atomicAdd(&ls.nsplit, 1);
-        }
-        c = __shfl_sync(gm, c, threadIdx.x & 16, 32);
-        RPatch* l = &ls.st[base + c];
-        RPatch* r = &ls.st[base + c + 1];
-        l->cp[my] = L;
-        r->cp[my] = R;
-        if (lane == 0) split_headers(l, r, id, path, dirs, depth, dir);
-      }
-      worker_sync();  // children written, nchild final
-      top = base + *nchild;
-      // the other counter was last read before this pass's first barrier
-      if (threadIdx.x == 0) ls.nchild[(pass + 1) & 1] = 0;
-      if (!first) nbound += m;
-      first = false;
-    }
-    // what is left goes back to the Bound ring (unbounded children: no work is repeated)
-    const int left = top;
-    if (left > 0) {
-      if (threadIdx.x == 0) ls.dump = ctx.template reserve<BOUND>(left);
-      worker_sync();
-      const int d = ls.dump;
-      if (d >= 0) {
-        uint4* dst = (uint4*)ctx.template out_ptr<BOUND>(d);
-        for (int e = threadIdx.x; e < left * 17; e += kThreads) dst[e] = ((const uint4*)ls.st)[e];
-      }
-    }
-    if (threadIdx.x == 0) {
-      ctx.template note_local_count<BOUND>(nbound);
-      ctx.template note_local_count<SPLIT>(ls.nsplit);
-    }
+    if constexpr (SS == DICE || SS == SHADE) exec<SS>(ctx, items, n);
+    else exec_dfs<SS>(ctx, items, n);
   }
 
   // -------------------------------------------------------------- Dice (warp/patch)

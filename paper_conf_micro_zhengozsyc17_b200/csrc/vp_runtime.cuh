@@ -1223,7 +1223,9 @@ struct Runner {
       if (s == SS) {
         record_trace(a, SS, items, n);
         if (threadIdx.x == 0) atomicAdd(&sh.deq32[SS], (uint32_t)n);  // direct-publish warps add too
-        if constexpr (RTC && SS < HI && fused_chain<F>(SS, HI)) {
+        // a fused chain runs in RTC kernels, and in local-recursion kernels (a megakernel
+        // whose Bound / Split batches never use the out buffers) for the chain's stages
+        if constexpr ((RTC || local_recursion<F>(LO, HI, RTC)) && SS < HI && fused_chain<F>(SS, HI)) {
           FusedChain<F>::template run<SS, HI>(ctx, items, n);
         } else if constexpr (local_recursion<F>(LO, HI, RTC)) {
           LocalRec<F>::template run<SS, LO, HI>(ctx, items, n);
