@@ -68,7 +68,8 @@ class ReyesOutC(C.Structure):
                 ("depth_hist", C.c_uint64 * 16), ("culled_depth_hist", C.c_uint64 * 16),
                 ("leaf_ids", P), ("leaf_cap", C.c_size_t), ("n_leaves", C.c_size_t),
                 ("leaf_grids", P),
-                ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t)]
+                ("trace", P), ("trace_cap", C.c_size_t), ("trace_n", C.c_size_t),
+                ("n_mp_covering", C.c_uint64)]
 
 
 def _declare(L):
@@ -221,7 +222,7 @@ def _reyes_run(fn, scene, seeds=None, leaf_cap=0, want_grids=False, trace_cap=0)
     res = dict(key=key.reshape(shp), s=s.reshape(shp), colour=colour.reshape(shp + (4,)),
                n_bound=o.n_bound, n_split=o.n_split, n_dice=o.n_dice, n_shade=o.n_shade,
                n_culled=o.n_culled, depth_hist=list(o.depth_hist),
-               culled_depth_hist=list(o.culled_depth_hist), n_leaves=o.n_leaves)
+               culled_depth_hist=list(o.culled_depth_hist), n_leaves=o.n_leaves, n_mp_covering=o.n_mp_covering)
     if leaf_cap:
         assert o.n_leaves <= leaf_cap, "leaf_cap too small"
         res["leaf_ids"] = leaf_ids[: o.n_leaves].copy()

@@ -114,6 +114,9 @@ typedef struct orc_reyes_out {
   float* leaf_grids;  /* [leaf_cap][6][81]: x, y, z, sx, sy, zs (SoA per leaf)        */
   /* optional per-stage trace (pipeline oracle only) */
   orc_trace_rec* trace; size_t trace_cap, trace_n;
+  /* micropolygons whose Q8 bounding box (clamped to the screen) holds a pixel centre:
+   * the ones Shade has to rasterise (the GPU reports the same count, vp_run_stats.work_units) */
+  uint64_t n_mp_covering;
 } orc_reyes_out;
 
 enum { ORC_REYES_CULL = 0, ORC_REYES_SPLIT = 1, ORC_REYES_DICE = 2 };

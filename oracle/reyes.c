@@ -265,7 +265,7 @@ static void raster_tri(const orc_reyes_scene* sc, uint64_t* fbkey, float* fbs, c
 
 /* Shade one diced grid into the frame's key/s buffers (Fig. 1 "Shade" -> "Image"). */
 static void shade_grid(const orc_reyes_scene* sc, uint32_t id, uint32_t path, uint32_t depth, const float grid[6][81],
-                       uint64_t* key_all, float* s_all) {
+                       uint64_t* key_all, float* s_all, uint64_t* n_covering) {
   size_t frame = id >> 12;
   uint32_t patch = id & 0xFFFu;
   uint64_t* fbkey = key_all + frame * (size_t)sc->W * sc->H;
@@ -298,6 +298,22 @@ static void shade_grid(const orc_reyes_scene* sc, uint32_t id, uint32_t path, ui
         }
       }
       if (!ok) continue;
+      {  /* does the quad's box hold a pixel centre (px + 0.5, py + 0.5) on the screen? */
+        int64_t xmin = v[0][0], xmax = v[0][0], ymin = v[0][1], ymax = v[0][1];
+        for (int k = 1; k < 4; ++k) {
+          if (v[k][0] < xmin) xmin = v[k][0];
+          if (v[k][0] > xmax) xmax = v[k][0];
+          if (v[k][1] < ymin) ymin = v[k][1];
+          if (v[k][1] > ymax) ymax = v[k][1];
+        }
+        int64_t px0 = ceil_div256(xmin - 128), px1 = floor_div256(xmax - 128);
+        int64_t py0 = ceil_div256(ymin - 128), py1 = floor_div256(ymax - 128);
+        if (px0 < 0) px0 = 0;
+        if (py0 < 0) py0 = 0;
+        if (px1 > sc->W - 1) px1 = sc->W - 1;
+        if (py1 > sc->H - 1) py1 = sc->H - 1;
+        if (px0 <= px1 && py0 <= py1) ++*n_covering;
+      }
       raster_tri(sc, fbkey, fbs, v[0], v[1], v[2], key, s);
       raster_tri(sc, fbkey, fbs, v[0], v[2], v[3], key, s);
     }
@@ -310,6 +326,7 @@ static void reyes_out_reset(const orc_reyes_scene* sc, orc_reyes_out* out) {
     out->s[i] = 0.0f;
   }
   out->n_bound = out->n_split = out->n_dice = out->n_shade = out->n_culled = 0;
+  out->n_mp_covering = 0;
   memset(out->depth_hist, 0, sizeof(out->depth_hist));
   memset(out->culled_depth_hist, 0, sizeof(out->culled_depth_hist));
   out->n_leaves = 0;
@@ -362,7 +379,7 @@ static void visit(const orc_reyes_scene* sc, const orc_patch* p, orc_reyes_out* 
     out->depth_hist[p->depth & 15]++;
     orc_reyes_dice(sc, p, grid);
     record_leaf(out, p, grid);
-    shade_grid(sc, p->id, p->path, p->depth, (const float(*)[81])grid, out->key, out->s);
+    shade_grid(sc, p->id, p->path, p->depth, (const float(*)[81])grid, out->key, out->s, &out->n_mp_covering);
   } else {
     orc_patch l, r;
     out->n_split++;
@@ -430,7 +447,8 @@ static void reyes_exec(orc_engine* e, int stage, const void* item) {
   } else { /* Shade */
     const reyes_grid_item* gi = (const reyes_grid_item*)item;
     orc_record(e, 3, ((uint64_t)gi->id << 12) | ((uint64_t)(gi->depth & 0xF) << 8) | (gi->path & 0xFF));
-    shade_grid(u->sc, gi->id, gi->path, gi->depth, (const float(*)[81])gi->grid, u->out->key, u->out->s);
+    shade_grid(u->sc, gi->id, gi->path, gi->depth, (const float(*)[81])gi->grid, u->out->key, u->out->s,
+               &u->out->n_mp_covering);
   }
 }
 

@@ -225,3 +225,17 @@ def test_reyes_stream_host_buffers(vpm, orc, model):
     for f in (0, 9):
         ref = orc.reyes_pipeline(inputs.reyes_config5(n_frames=1, n_side=16, frame0=f))
         assert np.array_equal(got[f], ref["colour"][0])
+
+
+@pytest.mark.parametrize("model", ["hybrid_mega_rtc", "megakernel"])
+def test_shade_work_units_match_oracle(vpm, orc, model):
+    """The micropolygons the fused [Dice, Shade] chain reports shading
+    (vp_run_stats.work_units[Shade], the count bench.py's roofline uses) equal the oracle's
+    count of micropolygons whose screen box holds a pixel centre."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesPipeline
+    for scene in (inputs.reyes_config1(), inputs.reyes_config5(n_frames=8, n_side=16)):
+        rp = ReyesPipeline(scene)
+        configure(vpm, rp, model)
+        st = rp.run()
+        ref = orc.reyes_pipeline(scene)
+        assert st["work_units"][3] == ref["n_mp_covering"] > 0

@@ -265,3 +265,25 @@ def test_planar_fill_rule_on_pixel_centres(orc):
     exp = np.zeros((64, 64), bool)
     exp[9:9 + int(S), 9:9 + int(S)] = True
     assert np.array_equal(cov, exp)
+
+
+@pytest.mark.parametrize("S,x0,W,max_depth", [(48.0, 8.0, 64, 8), (40.0, 8.5, 64, 8), (6.0, 8.0, 64, 8),
+                                               (200.0, 8.0, 256, 4), (48.0, 40.0, 64, 8)])
+def test_planar_covering_micropolygon_count(orc, S, x0, W, max_depth):
+    """The count of micropolygons whose (screen-clamped) box holds a pixel centre (what the
+    GPU reports as Shade's work units) against a closed-form enumeration: the planar patch
+    spans [x0, x0 + S]^2 px and is diced into a uniform (8 L) x (8 L) lattice of squares
+    of side h = S / (8 L), L leaves per side; square k covers [x0 + k h, x0 + (k + 1) h] in
+    x, and holds a column centre iff some integer c in [0, W) has c + 1/2 in that interval.
+    The last case runs off the right / bottom edge (clamping)."""
+    sc = inputs.reyes_planar(S, W=W, H=W, x0=x0, y0=x0, max_depth=max_depth)
+    r = orc.reyes_definition(sc, leaf_cap=4096)
+    d = [i for i, c in enumerate(r["depth_hist"]) if c]
+    assert len(d) == 1 and d[0] % 2 == 0   # alternating u / v splits: every leaf at one depth
+    per_side = 8 << (d[0] // 2)            # leaves wholly off screen are culled, and hold no centre
+    h = S / per_side
+    k = np.arange(per_side)
+    lo, hi = x0 + k * h, x0 + (k + 1) * h
+    has = np.array([any(a <= c + 0.5 <= b for c in range(W)) for a, b in zip(lo, hi)])
+    assert r["n_mp_covering"] == int(has.sum()) ** 2
+    assert orc.reyes_pipeline(sc)["n_mp_covering"] == r["n_mp_covering"]
