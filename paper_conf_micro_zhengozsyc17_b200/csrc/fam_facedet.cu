@@ -132,8 +132,93 @@ struct FaceDetF {
     }
   }
 
+  // Scan (round 2): the windows of all the batch's rows are spread over the block's
+  // threads in one flat loop (thread t takes windows t, t + 256, ... of the concatenated
+  // rows), with no barrier: early-exiting windows do not wait for the slowest thread of a
+  // row.  The cascade is read through the read-only path (it is a kernel parameter
+  // array), the LBP codes with plain L1-cacheable loads -- they were written in this run,
+  // but every Scan item reached its block through a ring slot acquired with
+  // ld.acquire.gpu after the producer's release (DESIGN.md §4.9 coherence argument).
+  template <class Ctx>
+  static __device__ void scan_batch(Ctx& ctx, const FdItem* items, int n) {
+    const Params& p = ctx.params();
+    const FdGeo g(p.W, p.H);
+    const int t = threadIdx.x;
+    int rowlen[4], start[5];
+    start[0] = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      int len = 0;
+      if (k < n) {
+        const FdItem it = items[k];
+        if (it.frame < (uint32_t)p.n_frames && (int)it.level < g.L) len = g.W[it.level] - kWin + 1;
+      }
+      rowlen[k] = len;
+      start[k + 1] = start[k] + len;
+    }
+    unsigned long long surv[16];
+#pragma unroll
+    for (int q = 0; q < 16; ++q) surv[q] = 0;
+    unsigned long long nwin = 0;
+    for (int i0 = 0; i0 < start[4]; i0 += kThreads) {
+      const int i = i0 + t;
+      const bool valid = i < start[4];
+      int k = 0;
+#pragma unroll
+      for (int q = 1; q < 4; ++q) k += i >= start[q] ? 1 : 0;
+      const FdItem it = items[valid ? k : 0];
+      const int l = (int)it.level, y = (int)it.a, x = i - start[k];
+      const uint32_t f = it.frame;
+      bool alive = valid;
+      if (valid) {
+        ++nwin;
+        const int W = g.W[l];
+        const uint8_t* lb = p.lbp + (size_t)f * g.off[g.L] + g.off[l];
+        const int32_t* wk = p.weak;
+        for (int st = 0; st < p.n_stages && alive; ++st) {
+          int32_t sum = 0;
+          for (int w = 0; w < p.n_weak[st]; ++w, wk += 12) {
+            const uint32_t code = lb[(size_t)(y + __ldg(wk + 1)) * W + x + __ldg(wk)];
+            const uint32_t bit = ((uint32_t)__ldg(wk + 2 + (code >> 5)) >> (code & 31u)) & 1u;
+            sum += bit ? __ldg(wk + 10) : __ldg(wk + 11);
+          }
+          if (sum < p.thr[st]) alive = false;
+          else surv[st]++;
+        }
+      }
+      // detections: warp-aggregated append
+      const unsigned m = __ballot_sync(0xffffffffu, valid && alive);
+      if (m) {
+        const int lane = t & 31, leader = __ffs(m) - 1;
+        unsigned long long base = 0;
+        if (lane == leader) base = atomicAdd(p.det_count, (unsigned long long)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (valid && alive) {
+          const unsigned long long di = base + __popc(m & ((1u << lane) - 1u));
+          if (di < p.det_cap) *(uint4*)(p.det + 4 * di) = make_uint4(f, (uint32_t)l, (uint32_t)x, (uint32_t)y);
+        }
+      }
+    }
+    (void)rowlen;
+    // per-stage survivor counts: warp reduce, one atomic per warp per stage
+    for (int st = 0; st < p.n_stages; ++st) {
+      unsigned long long v = surv[st];
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+      if ((t & 31) == 0 && v) atomicAdd(p.survivors + st, v);
+    }
+    unsigned long long v = nwin;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((t & 31) == 0 && v) atomicAdd(p.windows, v);
+  }
+
   template <int s, class Ctx>
   static __device__ void exec(Ctx& ctx, const uint8_t* items, int n) {
+    if constexpr (s == SCAN) {
+      scan_batch(ctx, (const FdItem*)items, n);
+      return;
+    }
     const Params& p = ctx.params();
     const FdGeo g(p.W, p.H);
     const size_t npx = (size_t)p.W * p.H;
@@ -236,64 +321,6 @@ struct FaceDetF {
             }
           }
         }
-      } else {  // SCAN: one row of windows
-        const int l = (int)it.level;
-        if (l >= g.L) continue;
-        int32_t* cas = (int32_t*)ctx.scratch();  // the cascade in shared memory
-        const int nw_total = p.n_weak_total;
-        for (int i = t; i < nw_total * 12; i += kThreads) cas[i] = __ldg(p.weak + i);
-        worker_sync();
-        const uint8_t* lb = lbp + g.off[l];
-        const int W = g.W[l], y = (int)it.a;
-        unsigned long long surv[16];
-#pragma unroll
-        for (int q = 0; q < 16; ++q) surv[q] = 0;
-        unsigned long long nwin = 0;
-        for (int xb = 0; xb < W - kWin + 1; xb += kThreads) {
-          const int x = xb + t;
-          const bool valid = x <= W - kWin;
-          bool alive = valid;
-          if (valid) {
-            ++nwin;
-            const int32_t* wk = cas;
-            for (int st = 0; st < p.n_stages && alive; ++st) {
-              int32_t sum = 0;
-              for (int w = 0; w < p.n_weak[st]; ++w, wk += 12) {
-                const uint32_t code = __ldcg(lb + (size_t)(y + wk[1]) * W + x + wk[0]);
-                const uint32_t bit = ((uint32_t)wk[2 + (code >> 5)] >> (code & 31u)) & 1u;
-                sum += bit ? wk[10] : wk[11];
-              }
-              if (sum < p.thr[st]) alive = false;
-              else surv[st]++;
-            }
-          }
-          // detections: warp-aggregated append
-          const unsigned m = __ballot_sync(0xffffffffu, valid && alive);
-          if (m) {
-            const int lane = t & 31, leader = __ffs(m) - 1;
-            unsigned long long base = 0;
-            if (lane == leader) base = atomicAdd(p.det_count, (unsigned long long)__popc(m));
-            base = __shfl_sync(0xffffffffu, base, leader);
-            if (valid && alive) {
-              const unsigned long long i = base + __popc(m & ((1u << lane) - 1u));
-              if (i < p.det_cap) {
-                uint4 d = make_uint4(f, (uint32_t)l, (uint32_t)x, (uint32_t)y);
-                *(uint4*)(p.det + 4 * i) = d;
-              }
-            }
-          }
-        }
-        // per-stage survivor counts: warp reduce, one atomic per warp per stage
-        for (int st = 0; st < p.n_stages; ++st) {
-          unsigned long long v = surv[st];
-#pragma unroll
-          for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-          if ((t & 31) == 0 && v) atomicAdd(p.survivors + st, v);
-        }
-        unsigned long long v = nwin;
-#pragma unroll
-        for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-        if ((t & 31) == 0 && v) atomicAdd(p.windows, v);
       }
       worker_sync();
     }

@@ -8,7 +8,7 @@ M=gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_secto
 for wl in reyes1x face8 pyr cfd raster raster_near ldpc qb4 qb16 qb272; do
   for m in kbk mega; do
     extra=""
-    [ "$wl" = "pyr" ] && extra="--imgs 8"
+    [ "$wl" = "pyr" ] && extra="--imgs 32"
     timeout 600 ncu --metrics $M --clock-control none -c 600 --csv --log-file gpurun_out/suite/${wl}_${m}.csv \
       python tools/ncu_wl.py $wl $m $extra > gpurun_out/suite/${wl}_${m}.log 2>&1
   done
