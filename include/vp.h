@@ -346,7 +346,7 @@ typedef struct vp_cfd_params {
 } vp_cfd_params;
 
 typedef struct vp_facedet_params {
-  int32_t W, H;              /* level-0 frame size (H <= 2048)                             */
+  int32_t W, H;              /* level-0 frame size (24 <= W <= 8192, 24 <= H <= 2048)      */
   int32_t n_frames;          /* Gray items are {frame, 0, band, 0}, bands of 32 rows        */
   int32_t n_stages;          /* cascade stages K <= 16                                     */
   int32_t n_weak[16];        /* weak classifiers per stage                                 */

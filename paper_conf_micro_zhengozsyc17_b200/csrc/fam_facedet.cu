@@ -78,7 +78,7 @@ struct FaceDetF {
   using Params = vp_facedet_params;
   static constexpr int stride(int) { return 16; }
   static constexpr int threads_per_item(int) { return 256; }
-  static constexpr int max_batch(int s) { return s == CDF ? 1 : s == SCAN ? 4 : 2; }
+  static constexpr int max_batch(int s) { return s == CDF ? 1 : s == SCAN ? 8 : 2; }
   static constexpr int default_batch(int s) { return max_batch(s); }
   static constexpr int fanout(int s, int t) {
     return (s == GRAY && t == CDF)       ? 1
@@ -91,7 +91,7 @@ struct FaceDetF {
                                          : 0;
   }
   static constexpr bool rtc_ok(int lo, int hi) { return !(lo < CDF && hi >= CDF); }
-  static constexpr int scratch_bytes(int, int) { return 6144; }
+  static constexpr int scratch_bytes(int, int hi) { return hi >= SCAN ? kScanScratch : 6144; }
   static constexpr int default_cap_log2(int s) { return s == SCAN ? 15 : 13; }
   static constexpr int min_blocks(int, int, bool) { return VP_FD_MINB; }
 
@@ -132,85 +132,151 @@ struct FaceDetF {
     }
   }
 
-  // Scan (round 2): the windows of all the batch's rows are spread over the block's
-  // threads in one flat loop (thread t takes windows t, t + 256, ... of the concatenated
-  // rows), with no barrier: early-exiting windows do not wait for the slowest thread of a
-  // row.  The cascade is read through the read-only path (it is a kernel parameter
-  // array), the LBP codes with plain L1-cacheable loads -- they were written in this run,
-  // but every Scan item reached its block through a ring slot acquired with
-  // ld.acquire.gpu after the producer's release (DESIGN.md §4.9 coherence argument).
+  // Scan (round 2): per-warp cascade-stage lists.  A warp that runs 32 windows through
+  // the cascade in lockstep pays for its deepest window: with ~30% of windows passing
+  // stage 0 and a few near every face reaching stage 11, a warp almost always ran all 12
+  // stages (~90 weak classifiers) while the mean window needs ~5.  Block-wide stage passes
+  // (one barrier per stage) fixed the divergence but left most warps waiting at the
+  // barriers of the sparse late stages (ncu: 58% of stall samples).  So each worker warp
+  // owns a contiguous range of the batch's windows (the rows concatenated) and, in shared
+  // memory, one list per stage s >= 1 of windows that passed stage s-1.  Every step
+  // evaluates ONE stage for 32 windows: the deepest list holding >= 32 entries, else the
+  // next 32 windows of the range (stage 0), else (range exhausted) the shallowest
+  // non-empty list, partially.  A step adds <= 32 entries to the next list, which is then
+  // the deepest full one and is drained next, so no list exceeds 63 entries.  No block
+  // barrier, the weak classifiers of a step are warp-uniform (broadcast loads), and the
+  // lanes idle only in the final partial steps.  List counts live lane-distributed in
+  // registers (lane s: list s), as do the per-stage survivor counts.  The cascade is read
+  // through the read-only path (a kernel parameter array), the LBP codes with plain
+  // L1-cacheable loads -- they were written in this run, but every Scan item reached its
+  // block through a ring slot acquired with ld.acquire.gpu after the producer's release
+  // (DESIGN.md §4.9 coherence argument).  Entries are (row << 13) | x, hence W <= 8192.
+  static constexpr int kListCap = 64, kListsPerWarp = 15;  // stages 1 .. 15
+  static constexpr int kScanScratch = kThreads / 32 * kListsPerWarp * kListCap * 2;
+
+  // one weak classifier of a window (win = its top-left LBP code, W = the row pitch):
+  // the window's LBP code at (cx, cy) picks a bit of the 256-bit mask
+  static __device__ __forceinline__ int32_t weak_vote(const int32_t* wk, const uint8_t* win, int W) {
+    const uint32_t code = win[__ldg(wk + 1) * W + __ldg(wk)];
+    const uint32_t bit = ((uint32_t)__ldg(wk + 2 + (code >> 5)) >> (code & 31u)) & 1u;
+    return bit ? __ldg(wk + 10) : __ldg(wk + 11);
+  }
+
   template <class Ctx>
   static __device__ void scan_batch(Ctx& ctx, const FdItem* items, int n) {
     const Params& p = ctx.params();
     const FdGeo g(p.W, p.H);
-    const int t = threadIdx.x;
-    int rowlen[4], start[5];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    uint16_t* lists = (uint16_t*)ctx.scratch() + wid * kListsPerWarp * kListCap - kListCap;  // list s at s * kListCap
+    // lane k < n: batch row k (its first window's LBP row, pitch, window count)
+    const uint8_t* myrow = p.lbp;
+    int myW = 0, mylen = 0;
+    if (lane < n) {
+      const FdItem it = items[lane];
+      if (it.frame < (uint32_t)p.n_frames && (int)it.level < g.L) {
+        myW = g.W[it.level];
+        mylen = myW - kWin + 1;
+        myrow = p.lbp + (size_t)it.frame * g.off[g.L] + g.off[it.level] + (size_t)it.a * myW;
+      }
+    }
+    int incl = mylen;
+#pragma unroll
+    for (int o = 1; o < 8; o <<= 1) {
+      const int v = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += v;
+    }
+    int start[9];  // start[k] = first window of row k (rows of the batch concatenated)
     start[0] = 0;
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      int len = 0;
-      if (k < n) {
-        const FdItem it = items[k];
-        if (it.frame < (uint32_t)p.n_frames && (int)it.level < g.L) len = g.W[it.level] - kWin + 1;
-      }
-      rowlen[k] = len;
-      start[k + 1] = start[k] + len;
+    for (int k = 0; k < 8; ++k) start[k + 1] = __shfl_sync(0xffffffffu, incl, k);
+    const int total = start[8], K = p.n_stages;
+    const int lo = (int)((long long)total * wid / (kThreads / 32));
+    const int hi = (int)((long long)total * (wid + 1) / (kThreads / 32));
+    // lane s < K: stage s's weak-classifier offset, count and threshold
+    int woff = 0, nw = 0, thr = 0;
+    if (lane < K) {
+      for (int q = 0; q < lane; ++q) woff += p.n_weak[q];
+      nw = p.n_weak[lane];
+      thr = p.thr[lane];
     }
-    unsigned long long surv[16];
+    int cnt = 0;                   // lane s in [1, K): entries in list s
+    unsigned long long surv = 0;   // lane s < K: windows that passed stage s
+    int next = lo;
+    const bool list_lane = lane >= 1 && lane < K;
+    for (;;) {
+      int s, take;
+      const unsigned full = __ballot_sync(0xffffffffu, list_lane && cnt >= 32);
+      if (full) {
+        s = 31 - __clz(full);
+        take = 32;
+      } else if (next < hi) {
+        s = 0;
+        take = min(32, hi - next);
+      } else {
+        const unsigned any = __ballot_sync(0xffffffffu, list_lane && cnt > 0);
+        if (!any) break;
+        s = __ffs(any) - 1;
+        take = __shfl_sync(0xffffffffu, cnt, s);
+      }
+      const bool v = lane < take;
+      int k = 0, x = 0;
+      if (s == 0) {
+        const int i = next + lane;
 #pragma unroll
-    for (int q = 0; q < 16; ++q) surv[q] = 0;
-    unsigned long long nwin = 0;
-    for (int i0 = 0; i0 < start[4]; i0 += kThreads) {
-      const int i = i0 + t;
-      const bool valid = i < start[4];
-      int k = 0;
-#pragma unroll
-      for (int q = 1; q < 4; ++q) k += i >= start[q] ? 1 : 0;
-      const FdItem it = items[valid ? k : 0];
-      const int l = (int)it.level, y = (int)it.a, x = i - start[k];
-      const uint32_t f = it.frame;
-      bool alive = valid;
-      if (valid) {
-        ++nwin;
-        const int W = g.W[l];
-        const uint8_t* lb = p.lbp + (size_t)f * g.off[g.L] + g.off[l];
-        const int32_t* wk = p.weak;
-        for (int st = 0; st < p.n_stages && alive; ++st) {
-          int32_t sum = 0;
-          for (int w = 0; w < p.n_weak[st]; ++w, wk += 12) {
-            const uint32_t code = lb[(size_t)(y + __ldg(wk + 1)) * W + x + __ldg(wk)];
-            const uint32_t bit = ((uint32_t)__ldg(wk + 2 + (code >> 5)) >> (code & 31u)) & 1u;
-            sum += bit ? __ldg(wk + 10) : __ldg(wk + 11);
-          }
-          if (sum < p.thr[st]) alive = false;
-          else surv[st]++;
+        for (int q = 1; q < 8; ++q) k += i >= start[q] ? 1 : 0;
+        x = i - start[k];
+        next += take;
+      } else {
+        const int c = __shfl_sync(0xffffffffu, cnt, s);
+        if (v) {
+          const uint32_t e = lists[s * kListCap + c - take + lane];
+          k = (int)(e >> 13);
+          x = (int)(e & 0x1fffu);
+        }
+        if (lane == s) cnt -= take;
+      }
+      if (!v) k = 0, x = 0;
+      const unsigned long long rb = (unsigned long long)__shfl_sync(0xffffffffu, (unsigned long long)myrow, k);
+      const int W = __shfl_sync(0xffffffffu, myW, k);
+      const int so = __shfl_sync(0xffffffffu, woff, s), sn = __shfl_sync(0xffffffffu, nw, s);
+      const int st = __shfl_sync(0xffffffffu, thr, s);
+      int32_t sum = 0;
+      if (v) {
+        const uint8_t* win = (const uint8_t*)rb + x;
+        const int32_t* wk = p.weak + 12 * so;
+#pragma unroll 4
+        for (int w = 0; w < sn; ++w, wk += 12) sum += weak_vote(wk, win, W);
+      }
+      const bool pass = v && sum >= st;
+      const unsigned bm = __ballot_sync(0xffffffffu, pass);
+      if (lane == s) surv += (unsigned long long)__popc(bm);
+      if (bm) {
+        if (s + 1 == K) {
+          emit_dets(p, items, bm, pass, k, x);
+        } else {
+          const int c = __shfl_sync(0xffffffffu, cnt, s + 1);
+          if (pass) lists[(s + 1) * kListCap + c + __popc(bm & lt)] = (uint16_t)((k << 13) | x);
+          if (lane == s + 1) cnt += __popc(bm);
         }
       }
-      // detections: warp-aggregated append
-      const unsigned m = __ballot_sync(0xffffffffu, valid && alive);
-      if (m) {
-        const int lane = t & 31, leader = __ffs(m) - 1;
-        unsigned long long base = 0;
-        if (lane == leader) base = atomicAdd(p.det_count, (unsigned long long)__popc(m));
-        base = __shfl_sync(0xffffffffu, base, leader);
-        if (valid && alive) {
-          const unsigned long long di = base + __popc(m & ((1u << lane) - 1u));
-          if (di < p.det_cap) *(uint4*)(p.det + 4 * di) = make_uint4(f, (uint32_t)l, (uint32_t)x, (uint32_t)y);
-        }
-      }
+      __syncwarp();
     }
-    (void)rowlen;
-    // per-stage survivor counts: warp reduce, one atomic per warp per stage
-    for (int st = 0; st < p.n_stages; ++st) {
-      unsigned long long v = surv[st];
-#pragma unroll
-      for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-      if ((t & 31) == 0 && v) atomicAdd(p.survivors + st, v);
+    if (lane < K && surv) atomicAdd(p.survivors + lane, surv);
+    if (threadIdx.x == 0 && total) atomicAdd(p.windows, (unsigned long long)total);
+  }
+
+  // detections of the warp's passing lanes (mask bm): warp-aggregated append
+  static __device__ __forceinline__ void emit_dets(const Params& p, const FdItem* items, unsigned bm, bool pass, int k, int x) {
+    const int lane = threadIdx.x & 31, leader = __ffs(bm) - 1;
+    unsigned long long base = 0;
+    if (lane == leader) base = atomicAdd(p.det_count, (unsigned long long)__popc(bm));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (pass) {
+      const FdItem it = items[k];
+      const unsigned long long di = base + __popc(bm & ((1u << lane) - 1u));
+      if (di < p.det_cap) *(uint4*)(p.det + 4 * di) = make_uint4(it.frame, it.level, (uint32_t)x, it.a);
     }
-    unsigned long long v = nwin;
-#pragma unroll
-    for (int o = 16; o >= 1; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-    if ((t & 31) == 0 && v) atomicAdd(p.windows, v);
   }
 
   template <int s, class Ctx>
@@ -334,7 +400,8 @@ struct FaceDetF {
     return false;
   }
   static const char* validate(const Params& p) {
-    if (p.W < kWin || p.H < kWin || p.H > kMaxBands0 * kBand) return "vp_facedet_params: W, H >= 24 and H <= 2048";
+    if (p.W < kWin || p.H < kWin || p.H > kMaxBands0 * kBand || p.W > 8192)
+      return "vp_facedet_params: 24 <= W <= 8192, 24 <= H <= 2048";
     if (p.n_frames <= 0 || p.n_stages <= 0 || p.n_stages > 16) return "vp_facedet_params: bad n_frames / n_stages";
     int tot = 0;
     for (int k = 0; k < p.n_stages; ++k) tot += p.n_weak[k];
