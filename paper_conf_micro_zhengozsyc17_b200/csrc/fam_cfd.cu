@@ -87,6 +87,8 @@ __device__ __forceinline__ bool cfd_latch_arrive(int* latch) {
   return false;
 }
 
+__device__ __forceinline__ float f4_at(const float4& v, int i) { return i == 0 ? v.x : i == 1 ? v.y : i == 2 ? v.z : v.w; }
+
 struct CfdF {
   static constexpr int S = 4;
   static constexpr int COPY = 0, STEP = 1, FLUX = 2, TIME = 3;
@@ -138,27 +140,32 @@ struct CfdF {
   static constexpr int kShare = 20;        // d mx my mz e | speed c p | fmx[3] fmy[3] fmz[3] fe[3]
   static constexpr int kHalo = 8;          // left/right halo cell per chunk, <= 4 chunks per item
   static constexpr int kLd = kThreads + kHalo;
-  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= FLUX && FLUX <= hi) ? kShare * kLd * 4 : 0; }
+  // two chunk buffers (chunk parity) + the halo records: one barrier per chunk
+  static constexpr int scratch_bytes(int lo, int hi) { return (lo <= FLUX && FLUX <= hi) ? kShare * (kLd + kThreads) * 4 : 0; }
 
-  static __device__ __forceinline__ void share_put(float* sh, int col, const CCell& c, const CPrim& q, float speed) {
-    const float v[kShare] = {c.d, c.mx, c.my, c.mz, c.e, speed, q.c, q.p, q.fmx[0], q.fmx[1], q.fmx[2],
-                             q.fmy[0], q.fmy[1], q.fmy[2], q.fmz[0], q.fmz[1], q.fmz[2], q.fe[0], q.fe[1], q.fe[2]};
-#pragma unroll
-    for (int f = 0; f < kShare; ++f) sh[f * kLd + col] = v[f];
+  // Records are 20-float structures (five float4, 80 B apart: the 8 lanes of each
+  // 128-bit shared-memory phase hit 8 distinct 4-bank groups, conflict-free).
+  //   [d mx my mz] [e speed c p] [fmx0 fmx1 fmx2 fmy0] [fmy1 fmy2 fmz0 fmz1] [fmz2 fe0 fe1 fe2]
+  static __device__ __forceinline__ void share_put(float4* sh, int col, const CCell& c, const CPrim& q, float speed) {
+    float4* r = sh + 5 * col;
+    r[0] = make_float4(c.d, c.mx, c.my, c.mz);
+    r[1] = make_float4(c.e, speed, q.c, q.p);
+    r[2] = make_float4(q.fmx[0], q.fmx[1], q.fmx[2], q.fmy[0]);
+    r[3] = make_float4(q.fmy[1], q.fmy[2], q.fmz[0], q.fmz[1]);
+    r[4] = make_float4(q.fmz[2], q.fe[0], q.fe[1], q.fe[2]);
   }
   struct NbRec {
     float d, mx, my, mz, e, speed, c, fmx[3], fmy[3], fmz[3], fe[3];
   };
-  static __device__ __forceinline__ void share_get(const float* sh, int col, NbRec& r) {
-    r.d = sh[0 * kLd + col]; r.mx = sh[1 * kLd + col]; r.my = sh[2 * kLd + col]; r.mz = sh[3 * kLd + col];
-    r.e = sh[4 * kLd + col]; r.speed = sh[5 * kLd + col]; r.c = sh[6 * kLd + col];
-#pragma unroll
-    for (int a = 0; a < 3; ++a) {
-      r.fmx[a] = sh[(8 + a) * kLd + col];
-      r.fmy[a] = sh[(11 + a) * kLd + col];
-      r.fmz[a] = sh[(14 + a) * kLd + col];
-      r.fe[a] = sh[(17 + a) * kLd + col];
-    }
+  static __device__ __forceinline__ void share_get(const float4* sh, int col, NbRec& r) {
+    const float4* q = sh + 5 * col;
+    const float4 a = q[0], b = q[1], f2 = q[2], f3 = q[3], f4 = q[4];
+    r.d = a.x; r.mx = a.y; r.my = a.z; r.mz = a.w;
+    r.e = b.x; r.speed = b.y; r.c = b.z;
+    r.fmx[0] = f2.x; r.fmx[1] = f2.y; r.fmx[2] = f2.z;
+    r.fmy[0] = f2.w; r.fmy[1] = f3.x; r.fmy[2] = f3.y;
+    r.fmz[0] = f3.z; r.fmz[1] = f3.w; r.fmz[2] = f4.x;
+    r.fe[0] = f4.y; r.fe[1] = f4.z; r.fe[2] = f4.w;
   }
   // offsets are 32-bit: validate() bounds 16 * N < 2^31
   static __device__ __forceinline__ void gather(const float* cur, uint32_t N, uint32_t nb, NbRec& r) {
@@ -183,7 +190,7 @@ struct CfdF {
     const size_t N = (size_t)p.G * p.G;
     const float* cur = p.vars + (size_t)(ci.k & 1u) * 5 * N;
     const size_t i0 = (size_t)ci.tile * p.T;
-    float* sh = (float*)ctx.scratch();
+    float4* sh = (float4*)ctx.scratch();
     const int t = threadIdx.x, nchunks = (p.T + kThreads - 1) / kThreads;
     const CCell ffc{p.ff[0], p.ff[1], p.ff[2], p.ff[3], p.ff[4]};
     // halo records: chunk h/2's left (h even) or right (h odd) neighbour cell, one per warp
@@ -208,6 +215,7 @@ struct CfdF {
       const int nch = min(kThreads, p.T - c0), chunk = c0 / kThreads;
       const long long lo = (long long)i0 + c0, hi = lo + nch;
       const bool act = t < nch;
+      const int buf = (chunk & 1) ? kLd : 0;  // this chunk's record columns
       const uint32_t c = (uint32_t)lo + (act ? t : 0);
       // this cell's faces: neighbour ids and normals are loaded before the barrier, so
       // their latency overlaps the primitive-variable computation
@@ -223,14 +231,14 @@ struct CfdF {
         }
         CPrim qi;
         cfd_prim(ic, qi);
-        share_put(sh, t, ic, qi, sqrtf(qi.sq));
+        share_put(sh, buf + t, ic, qi, sqrtf(qi.sq));
       }
       worker_sync();
       if (act) {
         // this cell's record is read back from shared memory where it is used (registers
         // are the limit here: 3 resident blocks of 320 threads)
-        const float* me = sh + t;
-#define ME(f) me[(f) * kLd]
+        const float4* me = sh + 5 * (buf + t);
+#define ME(f) f4_at(me[(f) >> 2], (f) & 3)
         float fd = 0.0f, fe = 0.0f, fx = 0.0f, fy = 0.0f, fz = 0.0f;
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
@@ -241,7 +249,7 @@ struct CfdF {
           const float nn[3] = {nx, ny, nz};
           if (nb >= 0) {
             int col = -1;
-            if ((long long)nb >= lo && (long long)nb < hi) col = (int)((long long)nb - lo);
+            if ((long long)nb >= lo && (long long)nb < hi) col = buf + (int)((long long)nb - lo);
             else if ((long long)nb == lo - 1) col = kThreads + 2 * chunk;
             else if ((long long)nb == hi) col = kThreads + 2 * chunk + 1;
             NbRec r;
@@ -289,8 +297,10 @@ struct CfdF {
         __stcg(p.flux + (3 * N32 + c), fz);
         __stcg(p.flux + (4 * N32 + c), fe);
       }
-      worker_sync();  // the chunk's records are rewritten next
+      // no second barrier: chunk + 1 writes the other buffer, and chunk + 2's barrier
+      // orders this chunk's reads before its buffer is rewritten
     }
+    worker_sync();  // the next item rewrites the halo records and buffer 0
   }
 
   template <int s, class Ctx>
