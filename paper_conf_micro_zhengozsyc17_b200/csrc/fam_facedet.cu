@@ -162,8 +162,16 @@ struct FaceDetF {
     return bit ? __ldg(wk + 10) : __ldg(wk + 11);
   }
 
+  // A batch may exceed max_batch(SCAN): an RTC [.., Scan] chain runs all the block-local
+  // Scan items of its LBP batch at once.  Rows are taken 8 at a time (every list drains
+  // before the next group).
   template <class Ctx>
   static __device__ void scan_batch(Ctx& ctx, const FdItem* items, int n) {
+    for (int r0 = 0; r0 < n; r0 += 8) scan_rows(ctx, items + r0, min(8, n - r0));
+  }
+
+  template <class Ctx>
+  static __device__ void scan_rows(Ctx& ctx, const FdItem* items, int n) {
     const Params& p = ctx.params();
     const FdGeo g(p.W, p.H);
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;

@@ -28,6 +28,8 @@ def configure(vp, fp, model):
     elif model == "hybrid_kbk":  # [Gray] mega | [CDF] KBK | [Map..Scan] mega
         fp.configure(vp.HYBRID, vp.make_binding([(0, 0, vp.GROUP_MEGA, 0, 30), (1, 1, vp.GROUP_KBK, 30, 40),
                                                  (2, 5, vp.GROUP_MEGA, 40, nsm)], nsm))
+    elif model == "hybrid_rtc":  # [Gray..Resize] mega | [LBP, Scan] RTC: Scan runs LBP's 64-row local batches
+        fp.configure(vp.HYBRID, vp.make_binding([(0, 3, vp.GROUP_MEGA, 0, 40), (4, 5, vp.GROUP_RTC, 40, nsm)], nsm))
     else:
         raise ValueError(model)
 
@@ -45,7 +47,8 @@ def check(orc, sc, fp, st):
     assert st["dequeued"][:6] == ref["deq"]
 
 
-@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk"])
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "megakernel", "coarse", "fine", "hybrid", "hybrid_kbk",
+                                   "hybrid_rtc"])
 def test_facedet_reduced(vpm, orc, model):
     """480x270 frame (SURVEY §8(d) reduced size), 2 frames."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import FaceDetPipeline
@@ -56,12 +59,14 @@ def test_facedet_reduced(vpm, orc, model):
         check(orc, sc, fp, fp.run())
 
 
-def test_facedet_full_frame(vpm, orc):
-    """Config 2: 1920x1080, 8 levels, 5 306 934 windows, in the megakernel configuration."""
+@pytest.mark.parametrize("model", ["megakernel", "hybrid_rtc"])
+def test_facedet_full_frame(vpm, orc, model):
+    """Config 2: 1920x1080, 8 levels, 5 306 934 windows, in the megakernel configuration
+    and with an RTC [LBP, Scan] group (Scan batches of up to 128 block-local rows)."""
     from paper_conf_micro_zhengozsyc17_b200.workloads import FaceDetPipeline
     sc = inputs.face_scene()
     fp = FaceDetPipeline(sc)
-    configure(vpm, fp, "megakernel")
+    configure(vpm, fp, model)
     st = fp.run()
     check(orc, sc, fp, st)
     assert fp.results()["windows"] == 5_306_934
