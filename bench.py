@@ -629,7 +629,7 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
 
-    # ---- timed region: inputs resident in HBM (seeds 4096 x 272 B per frame > L2)
+    # ---- timed region: inputs resident in HBM (seeds 4096 x 208 B per frame > L2)
     barrier()
     clk = Clocks(local)
     clk.wait_ready()
@@ -706,7 +706,7 @@ def main():
     hbm = pk.get("hbm_gbs", 6548.5)
     # HBM bytes per step that must move: seeds read + fb clear/CAS/resolve + colour write
     npix = scene.n_frames * scene.W * scene.H
-    bytes_step = scene.seeds.nbytes + npix * (16 + 16 + 16 + 16)
+    bytes_step = scene.seeds.size * inputs.GPU_PATCH_DTYPE.itemsize + npix * (16 + 16 + 16 + 16)
 
     # ---- baselines on the same shard: KBK (one launch per stage per wave) + megakernel
     extra = {}
@@ -738,7 +738,7 @@ def main():
         from paper_conf_micro_zhengozsyc17_b200.workloads import ReyesStream
         rs = ReyesStream(scene, chunk=args.e2e_chunk)
         rs.configure_config(main_cfg)
-        host_seeds = torch.from_numpy(scene.seeds.view(np.uint8).reshape(-1).copy()).pin_memory()
+        host_seeds = ReyesStream.host_seeds(scene)
         host_M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).pin_memory()
         host_out = torch.empty((scene.n_frames, scene.H, scene.W, 4), dtype=torch.float32).pin_memory()
         e_steps = max(1, min(args.steps, 5))
@@ -807,7 +807,7 @@ def main():
                    "patches_per_frame": 4096, "image": "256x256", "max_depth": 8, "model": args.model,
                    "parallelism": f"frames sharded over {world} GPU(s)",
                    "l2": "inputs larger than L2 (seeds %.0f MB/GPU, frame buffers %.0f MB/GPU)" % (
-                       scene.seeds.nbytes / 1e6, npix * 32 / 1e6)},
+                       scene.seeds.size * inputs.GPU_PATCH_DTYPE.itemsize / 1e6, npix * 32 / 1e6)},
         "items_per_sec": ips, "items_per_step": items_all,
         "stage_counts": [int(x) for x in d[:4]],
         "roofline": roofline,

@@ -74,7 +74,12 @@ typedef enum vp_stage_kind {
   VP_TOY_S1 = 1, VP_TOY_S2 = 2, VP_TOY_S3 = 3,
   /* Collatz queue stress (not in the paper): step (recursive), sink */
   VP_COLLATZ_STEP = 10, VP_COLLATZ_SINK = 11,
-  /* Reyes (Fig. 1, L3; L55): Bound, Split (recursive via Bound), Dice, Shade */
+  /* Reyes (Fig. 1, L3; L55): Bound, Split (recursive via Bound), Dice, Shade.  Bound,
+   * Split and Dice items (and the seeds vp_insert takes for Bound) are 208-B patches:
+   * float x[16], y[16], z[16] (control point P[a][b] at 4a + b, affine: w = 1), then
+   * uint32 id = frame << 12 | patch, path, dirs, depth -- the paper's 272-B float4 item
+   * (Table 2) without its constant w (reading R-S10).  Shade items are
+   * 1968-B grids.  Register each stage with exactly these strides. */
   VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23,
   /* Rasterization (Fig. 16, L59): Vertex + Clip (the paper's Clip), Raster (its
    * Interpolate: triangle -> 8x8 tiles), Fragment (its Shade: coverage + z-buffer) */

@@ -26,11 +26,25 @@ namespace vp {
 #define VP_BS_MINB 3
 #endif
 
-struct RPatch {           // 272 B
-  float4 cp[16];          // P[a][b] at cp[4a+b]; a = u index, b = v index
+// Patch item as queued, 208 B (reading R-S10): the paper's 272-B item (Table 2:
+// float4 control points) carries w = 1 in every point -- the patches are polynomial
+// (affine control points) and de Casteljau keeps w = (1 + 1) / 2 = 1 exactly -- so the
+// queues carry x, y, z only, as three 16-float planes (§8.5: "methods that
+// reduce data item size in the queues could also be beneficial").  P[a][b] is point
+// 4a + b (a = u index, b = v index).
+struct RPatch {
+  float x[16], y[16], z[16];
   uint32_t id, path, dirs, depth;
 };
-static_assert(sizeof(RPatch) == 272, "patch item is 272 B (Table 2)");
+static_assert(sizeof(RPatch) == 208, "queued patch item is 208 B");
+
+// control point k as (x, y, z, w = 1) / its x, y, z into a patch
+__device__ __forceinline__ float4 cp_get(const RPatch* P, int k) { return make_float4(P->x[k], P->y[k], P->z[k], 1.0f); }
+__device__ __forceinline__ void cp_put(RPatch* P, int k, const float4 v) {
+  P->x[k] = v.x;
+  P->y[k] = v.y;
+  P->z[k] = v.z;
+}
 
 constexpr int kG = 8, kNG = 9, kNP = 81;
 struct RGrid {            // Dice -> Shade item: header + SoA grid (x,y,z object; sx,sy,zs screen)
@@ -273,7 +287,7 @@ struct ReyesF {
   static __device__ __forceinline__ int bound_patch(const Params& p, const RPatch* P, int lane, bool valid, int& dir,
                                                     float4& q, const float4* Mc = nullptr, uint32_t mframe = ~0u) {
     uint32_t frame = frame_of(p, P->id);
-    q = P->cp[lane];
+    q = cp_get(P, lane);
     return bound_q(p, q, P->depth, frame, lane, valid, dir, Mc, mframe);
   }
   // local frame index of an item id (frame << 12 | patch) in this run's matrices
@@ -457,7 +471,7 @@ struct ReyesF {
       slot = __shfl_sync(0xffffffffu, slot, 0, 16);
       if (cls != 0 && slot >= 0) {
         RPatch* out = (RPatch*)(cls == 1 ? ctx.template out_ptr<SPLIT>(slot) : ctx.template out_ptr<DICE>(slot));
-        out->cp[lane] = q;
+        cp_put(out, lane, q);
         if (lane == 0) {
           out->id = P->id;
           out->path = P->path;
@@ -476,7 +490,8 @@ struct ReyesF {
     // control point u of this thread's curve: (u, line) for a u-split, (line, u) for v
     const int base = dir == 0 ? line : 4 * line, step = dir == 0 ? 4 : 1;
     my = base + step * t;
-    float4 a = P->cp[base], b = P->cp[base + step], c = P->cp[base + 2 * step], d = P->cp[base + 3 * step];
+    const float4 a = cp_get(P, base), b = cp_get(P, base + step), c = cp_get(P, base + 2 * step),
+                 d = cp_get(P, base + 3 * step);
     // per component, exactly this order
 #define VP_CASTELJAU(comp)                                                   \
   {                                                                          \
@@ -487,8 +502,9 @@ struct ReyesF {
     L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
     R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
   }
-    VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+    VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z)  // w stays 1 (R-S10)
 #undef VP_CASTELJAU
+    L.w = R.w = 1.0f;
   }
   // children headers (split tree: path bit `depth` = 0 left / 1 right, dirs bit = direction)
   static __device__ __forceinline__ void split_headers(RPatch* l, RPatch* r, uint32_t id, uint32_t path, uint32_t dirs,
@@ -518,8 +534,8 @@ struct ReyesF {
       if (valid && slot >= 0) {
         RPatch* l = (RPatch*)ctx.template out_ptr<BOUND>(slot);
         RPatch* r = (RPatch*)ctx.template out_ptr<BOUND>(slot + 1);
-        l->cp[my] = L;
-        r->cp[my] = R;
+        cp_put(l, my, L);
+        cp_put(r, my, R);
         if (lane == 0) split_headers(l, r, P->id, P->path, P->dirs, depth, dir);
       }
     }
@@ -553,9 +569,9 @@ struct ReyesF {
   static constexpr bool direct_publish(int lo, int hi, bool rtc) { return !rtc && lo == BOUND && hi == SPLIT; }
   static constexpr int direct_out_cap(int, int, int t) { return t == DICE ? kWarpsW * kDfsStage : 0; }
 
+  // a control point from another lane of the 16-thread group (w = 1 is not shuffled)
   static __device__ __forceinline__ float4 shfl4(unsigned m, float4 v, int src) {
-    return make_float4(__shfl_sync(m, v.x, src, 16), __shfl_sync(m, v.y, src, 16), __shfl_sync(m, v.z, src, 16),
-                       __shfl_sync(m, v.w, src, 16));
+    return make_float4(__shfl_sync(m, v.x, src, 16), __shfl_sync(m, v.y, src, 16), __shfl_sync(m, v.z, src, 16), 1.0f);
   }
 
   template <int SS, class Ctx>
@@ -595,7 +611,7 @@ struct ReyesF {
             claimed = true;
           }
           if (src) {
-            q = src->cp[lane];
+            q = cp_get(src, lane);
             id = src->id;
             path = src->path;
             dirs = src->dirs;
@@ -636,7 +652,7 @@ struct ReyesF {
       const unsigned lb = __ballot_sync(0xffffffffu, leaf && lane == 0);
       if (leaf) {
         RPatch* out = &stage[wcnt + ((half && (lb & 1u)) ? 1 : 0)];
-        out->cp[lane] = q;
+        cp_put(out, lane, q);
         if (lane == 0) {
           out->id = id;
           out->path = path;
@@ -664,8 +680,9 @@ struct ReyesF {
     L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
     R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
   }
-        VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z) VP_CASTELJAU(w)
+        VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z)  // w stays 1 (R-S10)
 #undef VP_CASTELJAU
+        L.w = R.w = 1.0f;
         if (split) {
           const int slot = wsp + ((half && (sb & 1u)) ? 1 : 0);
           if (slot >= kDfsStack) {  // deeper than max_depth allows (cannot happen for valid seeds)
@@ -678,7 +695,7 @@ struct ReyesF {
             }
             const uint32_t ndirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
             RPatch* r = &stk[slot];
-            r->cp[lane] = R;
+            cp_put(r, lane, R);
             if (lane == 0) {
               r->id = id;
               r->path = path | (1u << depth);
@@ -738,13 +755,15 @@ struct ReyesF {
     } else {
       bernstein((float)j * 0.125f, Bv);
     }
+    // P[a][0..3] of each coordinate plane: one 16-B load each
+    const float4 X = *(const float4*)&P->x[4 * a], Y = *(const float4*)&P->y[4 * a], Z = *(const float4*)&P->z[4 * a];
+    const float px[4] = {X.x, X.y, X.z, X.w}, py[4] = {Y.x, Y.y, Y.z, Y.w}, pz[4] = {Z.x, Z.y, Z.z, Z.w};
     float cx = 0.0f, cy = 0.0f, cz = 0.0f;
 #pragma unroll
     for (int b = 0; b < 4; ++b) {
-      const float4 cp = P->cp[4 * a + b];
-      cx = cx + Bv[b] * cp.x;
-      cy = cy + Bv[b] * cp.y;
-      cz = cz + Bv[b] * cp.z;
+      cx = cx + Bv[b] * px[b];
+      cy = cy + Bv[b] * py[b];
+      cz = cz + Bv[b] * pz[b];
     }
     out->g[3][e] = cx;
     out->g[4][e] = cy;

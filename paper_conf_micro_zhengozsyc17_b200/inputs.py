@@ -85,6 +85,25 @@ PATCH_DTYPE = np.dtype([("cp", "<f4", (16, 4)), ("id", "<u4"), ("path", "<u4"),
                         ("dirs", "<u4"), ("depth", "<u4")])
 assert PATCH_DTYPE.itemsize == 272
 
+# The queued patch item of the CUDA path, 208 B (reading R-S10): the same
+# records with the constant w = 1 dropped and x, y, z as three 16-float planes.
+GPU_PATCH_DTYPE = np.dtype([("x", "<f4", (16,)), ("y", "<f4", (16,)), ("z", "<f4", (16,)), ("id", "<u4"),
+                            ("path", "<u4"), ("dirs", "<u4"), ("depth", "<u4")])
+assert GPU_PATCH_DTYPE.itemsize == 208
+
+
+def gpu_patch_items(items: np.ndarray) -> np.ndarray:
+    """PATCH_DTYPE records -> GPU_PATCH_DTYPE (a repack: no arithmetic).  Every control
+    point must be affine (w == 1), which the generators guarantee."""
+    if items.size and not np.all(items["cp"][..., 3] == np.float32(1.0)):
+        raise ValueError("the queued Reyes patch item carries affine control points (w == 1)")
+    out = np.zeros(items.shape, GPU_PATCH_DTYPE)
+    for c, name in enumerate("xyz"):
+        out[name] = items["cp"][..., c]
+    for name in ("id", "path", "dirs", "depth"):
+        out[name] = items[name]
+    return out
+
 
 @dataclass
 class ReyesScene:

@@ -323,7 +323,7 @@ class FaceDetPipeline:
 
 
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
-REYES_STRIDES = (272, 272, 272, 1968)
+REYES_STRIDES = (inputs.GPU_PATCH_DTYPE.itemsize,) * 3 + (1968,)  # 208-B patches (R-S10), grids
 
 
 class ReyesPipeline:
@@ -350,7 +350,8 @@ class ReyesPipeline:
         caps = queue_caps or [0, 0, 0, 0]
         for kind, stride, cap in zip(REYES_STAGES, REYES_STRIDES, caps):
             self.p.register(kind, stride, self.prm, queue_capacity=cap)
-        seeds = np.ascontiguousarray(scene.seeds)
+        seeds = scene.seeds if scene.seeds.dtype == inputs.GPU_PATCH_DTYPE else inputs.gpu_patch_items(scene.seeds)
+        seeds = np.ascontiguousarray(seeds)
         if seeds_on_device:
             self.seeds_dev = torch.from_numpy(seeds.view(np.uint8).reshape(-1)).to(dev)
             self.p.insert(0, self.seeds_dev, n=seeds.size)
@@ -396,7 +397,7 @@ class ReyesStream:
         if config is not None:
             for rp in self.pipes:
                 rp.p.configure_config(config)
-        self.seed_bytes = chunk * ppf * scene.seeds.dtype.itemsize
+        self.seed_bytes = chunk * ppf * inputs.GPU_PATCH_DTYPE.itemsize
         self.M_dev = torch.empty((2, F, 16), dtype=torch.float32, device=dev)  # per pass parity
         self.staging = [torch.empty(self.seed_bytes, dtype=torch.uint8, device=dev) for _ in range(2)]
         self.s_in, self.s_out = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
@@ -404,6 +405,12 @@ class ReyesStream:
         self.ev_used = [torch.cuda.Event() for _ in range(2)]    # staging[b] copied into pipeline b
         self.ev_out = [torch.cuda.Event() for _ in range(2)]     # pipeline b's colours downloaded
         self.ev_M = [torch.cuda.Event() for _ in range(2)]   # a pass's last chunk has rendered
+
+    @staticmethod
+    def host_seeds(scene: inputs.ReyesScene) -> torch.Tensor:
+        """The batch's seed items as the queues carry them (208-B records), in pinned host
+        memory: the `host_seeds` argument of render()."""
+        return torch.from_numpy(inputs.gpu_patch_items(scene.seeds).view(np.uint8).reshape(-1).copy()).pin_memory()
 
     def configure(self, model, binding=None, batch=0):
         for rp in self.pipes:
@@ -422,7 +429,8 @@ class ReyesStream:
 
     def render(self, host_seeds: torch.Tensor, host_M: torch.Tensor, host_out: torch.Tensor, stream=None,
                steps: int = 1):
-        """`steps` passes over the batch: host_seeds (pinned uint8, every frame's seed items),
+        """`steps` passes over the batch: host_seeds (pinned uint8, every frame's 208-B seed
+        items, see host_seeds()),
         host_M (pinned [F, 16] float32) -> host_out (pinned [F, H, W, 4] float32).  Copies of
         consecutive passes overlap too.  Returns the last run's stats."""
         st = stream or torch.cuda.current_stream(self.dev)
@@ -451,7 +459,7 @@ class ReyesStream:
             st.wait_event(self.ev_in[b])     # seeds (and matrices) of chunk c are on the device
             st.wait_event(self.ev_out[b])    # pipeline b's previous colours are downloaded
             self._params(b, c, k)
-            rp.p.insert(0, self.staging[b], n=self.seed_bytes // self.scene.seeds.dtype.itemsize, replace=True,
+            rp.p.insert(0, self.staging[b], n=self.seed_bytes // inputs.GPU_PATCH_DTYPE.itemsize, replace=True,
                         stream=st)
             self.ev_used[b].record(st)
             st_last = rp.run(st)             # vp_run returns when the chunk is rendered

@@ -215,7 +215,7 @@ def test_reyes_stream_host_buffers(vpm, orc, model):
     rs = ReyesStream(scene, chunk=4)
     for p in rs.pipes:
         configure(vpm, p, model)
-    host_seeds = torch.from_numpy(scene.seeds.view(np.uint8).reshape(-1).copy()).pin_memory()
+    host_seeds = ReyesStream.host_seeds(scene)
     host_M = torch.from_numpy(np.ascontiguousarray(scene.M, np.float32)).pin_memory()
     host_out = torch.full((16, scene.H, scene.W, 4), -1.0).pin_memory()
     rs.render(host_seeds, host_M, host_out, steps=2)
