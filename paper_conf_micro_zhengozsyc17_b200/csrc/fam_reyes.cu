@@ -23,7 +23,7 @@ namespace vp {
 #define VP_REYES_MINB 3
 #endif
 #ifndef VP_BS_MINB          // resident blocks/SM the block-local [Bound, Split] kernel is built for
-#define VP_BS_MINB 3
+#define VP_BS_MINB 4
 #endif
 
 // Patch item as queued, 208 B (reading R-S10): the paper's 272-B item (Table 2:

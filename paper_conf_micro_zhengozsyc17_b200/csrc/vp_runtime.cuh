@@ -1410,9 +1410,9 @@ struct Runner {
   // ... or its warps publish their outputs themselves (direct-publish kernels)
   static constexpr bool sink_group() { return direct_publish<F>(LO, HI, RTC) || no_ring_outputs(); }
   // A direct-publish kernel has no publisher warp at all: its blocks are the 8 worker
-  // warps + the fetcher, so the register file is divided among 9 warps, not 10 (72
-  // registers at 3 blocks/SM instead of 64: the Reyes [Bound, Split] kernel loses its
-  // spills).  Measured A/B for the other sink groups (the fused [Dice, Shade] kernel):
+  // warps + the fetcher, so the register file is divided among 9 warps, not 10 (the
+  // Reyes [Bound, Split] kernel: 56 registers at 4 blocks/SM, no spills; DESIGN.md
+  // §4.3).  Measured A/B for the other sink groups (the fused [Dice, Shade] kernel):
   // 288 threads at 72 registers was 7% slower than 320 at 64, so they keep 320.
   static constexpr int kBlockThreads = direct_publish<F>(LO, HI, RTC) ? kThreads + 32 : kBlock;
 

@@ -70,7 +70,7 @@ elif args.target == "rtc_leaf":
     import numpy as np
     sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
     import reyes_leaves
-    lv = np.ascontiguousarray(reyes_leaves.leaves(scene, args.frames))
+    lv = np.ascontiguousarray(inputs.gpu_patch_items(reyes_leaves.leaves(scene, args.frames)))  # 208-B items
     leaves_dev = torch.from_numpy(lv.view(np.uint8).reshape(-1)).cuda()
     rp.p.insert(0, rp.seeds_dev, n=0, replace=True)
     rp.p.insert(2, leaves_dev, n=lv.size)
