@@ -22,6 +22,12 @@ namespace vp {
 #ifndef VP_REYES_MINB
 #define VP_REYES_MINB 3
 #endif
+#ifndef VP_DS_MINB          // resident blocks/SM the RTC [Dice, Shade] kernel is built for
+#define VP_DS_MINB 3
+#endif
+#ifndef VP_DS_BATCH         // its Dice batch (staging: 2 x batch x 208 B per block)
+#define VP_DS_BATCH 64
+#endif
 #ifndef VP_BS_MINB          // resident blocks/SM the block-local [Bound, Split] kernel is built for
 #define VP_BS_MINB 4
 #endif
@@ -234,6 +240,7 @@ struct ReyesF {
     // depth-first [Bound, Split] (exec_dfs): 32 seeds per claim, two per 16-thread group
     if (!rtc && lo == BOUND && hi >= SPLIT && (s == BOUND || s == SPLIT)) return s == BOUND ? 32 : 16;  // DFS kernels
     if (s == DICE && !rtc && lo == BOUND && hi == SHADE) return 32;
+    if (s == DICE && rtc && lo == DICE && hi == SHADE) return VP_DS_BATCH;
     return (s == DICE && !(rtc && lo == DICE && hi == SHADE)) ? 8 : max_batch(s);
   }
   static constexpr int fused_local_cap(int, int, int) { return kThreads / 32; }
@@ -255,7 +262,7 @@ struct ReyesF {
   static constexpr int default_cap_log2(int s) { return s == BOUND ? 20 : s == SHADE ? 17 : 19; }
   // register budget: kernels containing Shade are held to 3 resident blocks per SM
   static constexpr int min_blocks(int lo, int hi, bool rtc) {
-    return (!rtc && lo == BOUND && hi == SPLIT) ? VP_BS_MINB : VP_REYES_MINB;
+    return (!rtc && lo == BOUND && hi == SPLIT) ? VP_BS_MINB : (rtc && lo == DICE && hi == SHADE) ? VP_DS_MINB : VP_REYES_MINB;
   }
 
   template <int s>
