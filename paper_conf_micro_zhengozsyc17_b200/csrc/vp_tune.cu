@@ -306,8 +306,7 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best_out, v
     double best_ms = 1e30;
     for (const Cand& k : fastest) {
       bool to = false;
-      const double t = timeoutexec(p, k.c, 2.0 * k.ms, std::max(3, reps), &to, &fatal);
-      R.candidates_run++;
+      const double t = timeoutexec(p, k.c, 2.0 * k.ms, std::max(3, reps), &to, &fatal);  // (not a new candidate)
       if (fatal != VP_OK) break;
       if (t > 0 && t < best_ms) {
         best_ms = t;
