@@ -79,7 +79,8 @@ typedef enum vp_stage_kind {
    * float x[16], y[16], z[16] (control point P[a][b] at 4a + b, affine: w = 1), then
    * uint32 id = frame << 12 | patch, path, dirs, depth -- the paper's 272-B float4 item
    * (Table 2) without its constant w (reading R-S10).  Shade items are
-   * 1968-B grids.  Register each stage with exactly these strides. */
+   * 1968-B grids (vp_stage_kind_info reports every kind's stride).  Register each stage
+   * with exactly these strides. */
   VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23,
   /* Rasterization (Fig. 16, L59): Vertex + Clip (the paper's Clip), Raster (its
    * Interpolate: triangle -> 8x8 tiles), Fragment (its Shade: coverage + z-buffer) */
@@ -443,6 +444,11 @@ vp_status vp_config_from_string(const char* s, vp_config* out);
  * `slots` x 8-B device buffer; *ops_per_s = n_ops / best-of-3 CUDA-event time.
  * Diagnostics only; it does not touch any pipeline. */
 vp_status vp_bench_red_min_u64(int device, unsigned long long slots, unsigned long long n_ops, double* ops_per_s);
+
+/* Item stride (bytes) a built-in stage kind must be registered with (vp_stage_desc.
+ * item_bytes), and its threads per item.  VP_ERR_INVALID for an unknown kind.  Host-only:
+ * no device is touched. */
+vp_status vp_stage_kind_info(int kind, int* item_bytes, int* threads_per_item);
 
 /* Device properties the binding layer needs (no torch types cross the ABI). */
 vp_status vp_device_info(int device, int* num_sms, int* cc_major, int* cc_minor);

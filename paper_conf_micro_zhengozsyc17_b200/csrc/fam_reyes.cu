@@ -53,12 +53,19 @@ __device__ __forceinline__ void cp_put(RPatch* P, int k, const float4 v) {
 }
 
 constexpr int kG = 8, kNG = 9, kNP = 81;
-struct RGrid {            // Dice -> Shade item: header + SoA grid (x,y,z object; sx,sy,zs screen)
+// Dice -> Shade item (1968 B).  o[g] = object-space point (x, y, z) with its screen depth zs
+// in .w, so Shade's normal and depth take 4 16-B loads; s[g] = the Q8 fixed-point snap of
+// (sx, sy) (reading R-R9; INT_MIN where it does not fit).  While Dice runs, s[] stages the
+// 36 u-curve points C_a(v_j) as float4.  (Round 2: carrying each point's pixel-centre
+// index range as well -- a 2608-B grid -- made the box test cheaper but pushed the fused
+// kernel's shared memory past the 196-KB carve-out step, and it ran 5% slower.)
+struct RGrid {
   uint32_t id, path, depth, dirs;
-  float g[6][kNP];
-  uint32_t pad[2];
+  float4 o[kNP];
+  int2 s[kNP];
 };
 static_assert(sizeof(RGrid) == 1968, "grid item stride");
+static_assert(sizeof(int2) * kNP >= sizeof(float4) * 4 * kNG, "u-curve staging fits in s[]");
 
 struct __align__(16) FbRec {
   unsigned long long key;
@@ -751,14 +758,14 @@ struct ReyesF {
   // Ms: the frame matrix rows in shared memory (fused chain), else read from p.M.
   // Bt (fused chain): the Bernstein weights B_b(j/8) as a [9][4] shared-memory table,
   // computed by bernstein() itself (bit-identical to evaluating it per point).
-  // the u-curve point C_a(v_j), e = 9a + j, of patch P into out's rows 3..5 (one lane)
+  // the u-curve point C_a(v_j), e = 9a + j, of patch P into the staging area (one lane)
   template <bool kSmemM>
   static __device__ __forceinline__ void dice_c(const RPatch* P, RGrid* out, int e, const float* Bt) {
     const int a = e / kNG, j = e - a * kNG;
     float Bv[4];
     if constexpr (kSmemM) {
-#pragma unroll
-      for (int b = 0; b < 4; ++b) Bv[b] = Bt[4 * j + b];
+      const float4 b4 = *(const float4*)&Bt[4 * j];
+      Bv[0] = b4.x; Bv[1] = b4.y; Bv[2] = b4.z; Bv[3] = b4.w;
     } else {
       bernstein((float)j * 0.125f, Bv);
     }
@@ -772,15 +779,14 @@ struct ReyesF {
       cy = cy + Bv[b] * py[b];
       cz = cz + Bv[b] * pz[b];
     }
-    out->g[3][e] = cx;
-    out->g[4][e] = cy;
-    out->g[5][e] = cz;
+    ((float4*)out->s)[e] = make_float4(cx, cy, cz, 0.0f);
   }
 
   // kHaveC: the caller already computed the u-curve points (the fused chain does both
-  // patches of a pair in one loop: 72 points in 3 warp passes instead of 2 x 2)
+  // patches of a pair in one loop: 72 points in 3 warp passes instead of 2 x 2).
+  // Returns (warp-uniform) whether every grid point was snappable.
   template <bool kSmemM = false, bool kHaveC = false>
-  static __device__ __forceinline__ void dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
+  static __device__ __forceinline__ bool dice_patch(const Params& p, const RPatch* P, RGrid* out, int lane,
                                                     const float4* Ms = nullptr, const float* Bt = nullptr) {
     const uint32_t frame = frame_of(p, P->id);
     const float* M = p.M + 16 * (size_t)frame;
@@ -788,8 +794,9 @@ struct ReyesF {
       for (int e = lane; e < 4 * kNG; e += 32) dice_c<kSmemM>(P, out, e, Bt);  // C_a(v_j), e = 9a + j
       __syncwarp();
     }
-    // S(u_i, v_j): object-space rows 0..2 are written at once (the C rows 3..5 are still
-    // being read by other lanes, so the screen rows wait for the next __syncwarp)
+    const float4* C = (const float4*)out->s;
+    // S(u_i, v_j) into o[g].xyz at once (the staged C in s[] is still being read by other
+    // lanes, so s[] is written after the next __syncwarp)
 #pragma unroll
     for (int r = 0; r < 3; ++r) {
       const int g = lane + 32 * r;
@@ -797,29 +804,30 @@ struct ReyesF {
         const int i = g / kNG, j = g - i * kNG;
         float Bu[4];
         if constexpr (kSmemM) {
-#pragma unroll
-          for (int a = 0; a < 4; ++a) Bu[a] = Bt[4 * i + a];
+          const float4 b4 = *(const float4*)&Bt[4 * i];
+          Bu[0] = b4.x; Bu[1] = b4.y; Bu[2] = b4.z; Bu[3] = b4.w;
         } else {
           bernstein((float)i * 0.125f, Bu);
         }
         float x = 0.0f, y = 0.0f, z = 0.0f;
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
-          x = x + Bu[a] * out->g[3][a * kNG + j];
-          y = y + Bu[a] * out->g[4][a * kNG + j];
-          z = z + Bu[a] * out->g[5][a * kNG + j];
+          const float4 c = C[a * kNG + j];
+          x = x + Bu[a] * c.x;
+          y = y + Bu[a] * c.y;
+          z = z + Bu[a] * c.z;
         }
-        out->g[0][g] = x;
-        out->g[1][g] = y;
-        out->g[2][g] = z;
+        out->o[g] = make_float4(x, y, z, 0.0f);
       }
     }
-    __syncwarp();  // every C read before the screen rows are written
+    __syncwarp();  // every C read before s[] is written
+    bool ok_all = true;
 #pragma unroll
     for (int r = 0; r < 3; ++r) {
       const int g = lane + 32 * r;
       if (g < kNP) {
-        const float x = out->g[0][g], y = out->g[1][g], z = out->g[2][g];  // this lane's own writes
+        const float4 ov = out->o[g];  // this lane's own write
+        const float x = ov.x, y = ov.y, z = ov.z;
         float4 c;
         if constexpr (kSmemM) {
           float cc[4];
@@ -841,9 +849,10 @@ struct ReyesF {
         // Shade only uses the Q8 fixed-point snap of (sx, sy): store it (reading R-R9)
         const float X = sx * 256.0f, Y = sy * 256.0f;
         const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
-        out->g[3][g] = __int_as_float(ok ? __float2int_rn(X) : INT_MIN);
-        out->g[4][g] = __int_as_float(ok ? __float2int_rn(Y) : INT_MIN);
-        out->g[5][g] = zs;
+        const int Xi = ok ? __float2int_rn(X) : INT_MIN, Yi = ok ? __float2int_rn(Y) : INT_MIN;
+        out->o[g].w = zs;
+        out->s[g] = make_int2(Xi, Yi);
+        ok_all = ok_all && ok;
       }
     }
     if (lane == 0) {
@@ -852,6 +861,7 @@ struct ReyesF {
       out->depth = P->depth;
       out->dirs = P->dirs;
     }
+    return __all_sync(0xffffffffu, ok_all);
   }
 
   template <class Ctx>
@@ -886,8 +896,9 @@ struct ReyesF {
     bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
-      vx[v] = __float_as_int(Gd->g[3][gi[v]]);
-      vy[v] = __float_as_int(Gd->g[4][gi[v]]);
+      const int2 sv = Gd->s[gi[v]];
+      vx[v] = sv.x;
+      vy[v] = sv.y;
       if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
     }
     if (!ok) return;
@@ -901,12 +912,9 @@ struct ReyesF {
     px1 = min(px1, p.W - 1);
     py1 = min(py1, p.H - 1);
     if (px0 > px1 || py0 > py1) return;
-    float e1[3], e2[3];
-#pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      e1[c] = Gd->g[c][g10] - Gd->g[c][g00];
-      e2[c] = Gd->g[c][g01] - Gd->g[c][g00];
-    }
+    const float4 o00 = Gd->o[g00], o10 = Gd->o[g10], o01 = Gd->o[g01], o11 = Gd->o[g11];
+    const float e1[3] = {o10.x - o00.x, o10.y - o00.y, o10.z - o00.z};
+    const float e2[3] = {o01.x - o00.x, o01.y - o00.y, o01.z - o00.z};
     float nx = e1[1] * e2[2] - e1[2] * e2[1];
     float ny = e1[2] * e2[0] - e1[0] * e2[2];
     float nz = e1[0] * e2[1] - e1[1] * e2[0];
@@ -922,7 +930,7 @@ struct ReyesF {
       if (!(t > 0.0f)) t = 0.0f;
       s = 0.1f + 0.9f * t;
     }
-    const float zq = ((Gd->g[5][g00] + Gd->g[5][g10]) + (Gd->g[5][g11] + Gd->g[5][g01])) * 0.25f;
+    const float zq = ((o00.w + o10.w) + (o11.w + o01.w)) * 0.25f;
     const uint32_t mp = (patch << 18) | ((Gd->path & 0xFFu) << 10) | ((Gd->depth & 0xFu) << 6) | (uint32_t)q;
     const unsigned long long key = ((unsigned long long)zkey(zq) << 32) | mp;
     FbRec* fb = (FbRec*)p.fb + (size_t)frame * p.W * p.H;
@@ -978,17 +986,19 @@ struct ReyesF {
   // holds a pixel centre (~1 in 4 at config 5) are shaded, compacted onto the warp's lanes.
   static constexpr bool fused_rtc(int s, int hi) { return s == DICE && hi == SHADE; }
 
-  // shade_mp's early exit alone: does micropolygon q's box hold a pixel centre?
+  // shade_mp's early exit alone: does micropolygon q's box hold a pixel centre?  (any grid)
+  template <bool kFrame = true>
   static __device__ __forceinline__ bool mp_box(const Params& p, const RGrid* Gd, int q) {
-    if ((Gd->id >> 12) - (uint32_t)p.frame_base >= (uint32_t)p.n_frames) return false;
+    if (kFrame && (Gd->id >> 12) - (uint32_t)p.frame_base >= (uint32_t)p.n_frames) return false;
     const int i = q >> 3, j = q & 7;
     const int gi[4] = {i * kNG + j, (i + 1) * kNG + j, (i + 1) * kNG + j + 1, i * kNG + j + 1};
     int vx[4], vy[4];
     bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
-      vx[v] = __float_as_int(Gd->g[3][gi[v]]);
-      vy[v] = __float_as_int(Gd->g[4][gi[v]]);
+      const int2 sv = Gd->s[gi[v]];
+      vx[v] = sv.x;
+      vy[v] = sv.y;
       if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
     }
     const int xmin = min(min(vx[0], vx[1]), min(vx[2], vx[3])), xmax = max(max(vx[0], vx[1]), max(vx[2], vx[3]));
@@ -997,7 +1007,6 @@ struct ReyesF {
     const int py0 = max(-((128 - ymin) >> 8), 0), py1 = min((ymax - 128) >> 8, p.H - 1);
     return ok && px0 <= px1 && py0 <= py1;
   }
-
   template <int S0, int HI, class Ctx>
   static __device__ void exec_rtc_chain(Ctx& ctx, const uint8_t* items, int n) {
     static_assert(S0 == DICE && HI == SHADE, "only the [Dice, Shade] chain is fused");
@@ -1051,7 +1060,8 @@ struct ReyesF {
         dice_patch<true, true>(p, P, g, lane, cs.M[warp][j], Bt);
         __syncwarp();
         if (lane == 0) ctx.template trace_local<SHADE>((const uint8_t*)g);
-        const bool a0 = mp_box(p, g, lane), a1 = mp_box(p, g, lane + 32);
+        const bool fv = (P->id >> 12) - (uint32_t)p.frame_base < (uint32_t)p.n_frames;  // per patch
+        const bool a0 = fv && mp_box<false>(p, g, lane), a1 = fv && mp_box<false>(p, g, lane + 32);
         const unsigned m0 = __ballot_sync(0xffffffffu, a0), m1 = __ballot_sync(0xffffffffu, a1);
         const unsigned lt = (1u << lane) - 1u;
         const int c0 = __popc(m0);
@@ -1079,7 +1089,7 @@ struct ReyesF {
     return false;
   }
   static const char* validate(const Params& p) {
-    if (p.W <= 0 || p.H <= 0 || p.W > 32768 || p.H > 32768) return "vp_reyes_params: bad W/H";
+    if (p.W <= 0 || p.H <= 0 || p.W > 32767 || p.H > 32767) return "vp_reyes_params: bad W/H (int16 pixel ranges)";
     if (p.n_frames <= 0 || p.n_frames > (1 << 20)) return "vp_reyes_params: bad n_frames";
     if (p.patches_per_frame <= 0 || p.patches_per_frame > 4096) return "vp_reyes_params: patches_per_frame must be in [1, 4096]";
     if (p.max_depth < 0 || p.max_depth > 8) return "vp_reyes_params: max_depth must be in [0, 8] (8-bit path)";

@@ -1051,6 +1051,15 @@ vp_status vp_pipeline_destroy(void* h) {
   return VP_OK;
 }
 
+vp_status vp_stage_kind_info(int kind, int* item_bytes, int* threads_per_item) {
+  int pos = -1;
+  const FamilyOps* f = family_of_kind(kind, &pos);
+  if (!f) return VP_ERR_INVALID;
+  if (item_bytes) *item_bytes = f->stride(pos);
+  if (threads_per_item) *threads_per_item = f->threads_per_item(pos);
+  return VP_OK;
+}
+
 vp_status vp_stage_register(void* h, const vp_stage_desc* s, int* stage_id) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;
   if (!p || !s) return VP_ERR_INVALID;

@@ -171,6 +171,7 @@ vp_get_output = _decl("vp_get_output", [P, C.c_int, C.POINTER(P), C.POINTER(C.c_
 vp_set_params = _decl("vp_set_params", [P, P, C.c_size_t])
 vp_config_to_string = _decl("vp_config_to_string", [C.POINTER(Config), C.c_char_p, C.c_size_t])
 vp_config_from_string = _decl("vp_config_from_string", [C.c_char_p, C.POINTER(Config)])
+vp_stage_kind_info = _decl("vp_stage_kind_info", [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int)])
 vp_device_info = _decl("vp_device_info", [C.c_int, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_int)])
 vp_memcpy = _decl("vp_memcpy", [P, P, C.c_size_t, C.c_int, P])
 vp_set_flags = _decl("vp_set_flags", [P, C.c_uint32, C.POINTER(C.c_uint32)])
@@ -179,7 +180,7 @@ vp_bench_red_min_u64 = _decl("vp_bench_red_min_u64", [C.c_int, C.c_ulonglong, C.
 EXPORTED = ["vp_status_string", "vp_last_error", "vp_pipeline_create", "vp_pipeline_destroy", "vp_stage_register",
             "vp_insert", "vp_insert_async", "vp_configure", "vp_configure_config", "vp_get_config", "vp_run",
             "vp_set_timeout", "vp_get_trace", "vp_autotune", "vp_profile", "vp_get_output", "vp_set_params", "vp_config_to_string", "vp_config_from_string",
-            "vp_device_info", "vp_memcpy", "vp_set_flags", "vp_bench_red_min_u64"]
+            "vp_device_info", "vp_memcpy", "vp_set_flags", "vp_bench_red_min_u64", "vp_stage_kind_info"]
 
 
 class VPError(RuntimeError):
@@ -206,6 +207,15 @@ def _stream_handle(stream):
     if hasattr(stream, "cuda_stream"):
         return C.c_void_p(stream.cuda_stream)
     return C.c_void_p(int(stream))
+
+
+def stage_kind_info(kind):
+    """vp_stage_kind_info: (item_bytes, threads_per_item) a built-in stage kind is registered with."""
+    b, t = C.c_int(), C.c_int()
+    rc = vp_stage_kind_info(kind, C.byref(b), C.byref(t))
+    if rc != VP_OK:
+        raise VPError(rc, f"vp_stage_kind_info({kind})")
+    return b.value, t.value
 
 
 def device_info(device=0):

@@ -323,7 +323,9 @@ class FaceDetPipeline:
 
 
 REYES_STAGES = (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)
-REYES_STRIDES = (inputs.GPU_PATCH_DTYPE.itemsize,) * 3 + (1968,)  # 208-B patches (R-S10), grids
+# 208-B patches (R-S10) for Bound / Split / Dice; Shade's grid item as the library defines it
+REYES_STRIDES = tuple(vp.stage_kind_info(k)[0] for k in REYES_STAGES)
+assert REYES_STRIDES[:3] == (inputs.GPU_PATCH_DTYPE.itemsize,) * 3
 
 
 class ReyesPipeline:

@@ -91,3 +91,16 @@ def test_config_string_roundtrip():
     assert vp.config_to_string(c2) == s
     with pytest.raises(vp.VPError):
         vp.config_from_string("garbage")
+
+
+def test_stage_kind_info_host_only():
+    """vp_stage_kind_info needs no device: the strides every built-in kind is registered with
+    (include/vp.h: 208-B patches for Reyes Bound/Split/Dice, reading R-S10; 1968-B grids)."""
+    from paper_conf_micro_zhengozsyc17_b200 import vp
+    assert [vp.stage_kind_info(k)[0] for k in (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)] == [
+        208, 208, 208, 1968]
+    assert [vp.stage_kind_info(k)[1] for k in (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)] == [
+        16, 16, 32, 64]
+    assert vp.stage_kind_info(vp.TOY_S1) == (4, 1)
+    with pytest.raises(vp.VPError):
+        vp.stage_kind_info(9999)
