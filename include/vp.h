@@ -79,7 +79,7 @@ typedef enum vp_stage_kind {
    * float x[16], y[16], z[16] (control point P[a][b] at 4a + b, affine: w = 1), then
    * uint32 id = frame << 12 | patch, path, dirs, depth -- the paper's 272-B float4 item
    * (Table 2) without its constant w (reading R-S10).  Shade items are
-   * 1968-B grids (vp_stage_kind_info reports every kind's stride).  Register each stage
+   * 2032-B grids (vp_stage_kind_info reports every kind's stride).  Register each stage
    * with exactly these strides. */
   VP_REYES_BOUND = 20, VP_REYES_SPLIT = 21, VP_REYES_DICE = 22, VP_REYES_SHADE = 23,
   /* Rasterization (Fig. 16, L59): Vertex + Clip (the paper's Clip), Raster (its

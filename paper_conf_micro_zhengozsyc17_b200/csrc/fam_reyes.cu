@@ -53,18 +53,27 @@ __device__ __forceinline__ void cp_put(RPatch* P, int k, const float4 v) {
 }
 
 constexpr int kG = 8, kNG = 9, kNP = 81;
-// Dice -> Shade item (1968 B).  o[g] = object-space point (x, y, z) with its screen depth zs
-// in .w, so Shade's normal and depth take 4 16-B loads; s[g] = the Q8 fixed-point snap of
-// (sx, sy) (reading R-R9; INT_MIN where it does not fit).  While Dice runs, s[] stages the
+// Dice -> Shade item (2032 B).  Grid point (i, j) = S(i/8, j/8) is o[9j + i] (v-major: Dice's
+// lanes then take consecutive points of one u-curve row, so the 4 u-curve points each reads
+// are the same for 9 lanes -- shared-memory broadcasts instead of bank conflicts) and
+// s[10j + i] (a padded row: the 16 lanes of a 64-bit load phase of the box test, (i, j) and
+// (i + 1, j) for j = 0..7, then hit 16 distinct bank pairs).  o = object-space point
+// (x, y, z) with its screen depth zs in .w, so Shade's normal and depth take 4 16-B loads;
+// s = the Q8 fixed-point snap of (sx, sy) (reading R-R9; INT_MIN where it does not fit).  While Dice runs, s[] stages the
 // 36 u-curve points C_a(v_j) as float4.  (Round 2: carrying each point's pixel-centre
 // index range as well -- a 2608-B grid -- made the box test cheaper but pushed the fused
 // kernel's shared memory past the 196-KB carve-out step, and it ran 5% slower.)
+#ifndef VP_SROW
+#define VP_SROW 10
+#endif
+constexpr int kSR = VP_SROW;  // row stride of RGrid::s (9: unpadded)
+__device__ __forceinline__ int sidx(int i, int j) { return j * kSR + i; }
 struct RGrid {
   uint32_t id, path, depth, dirs;
   float4 o[kNP];
-  int2 s[kNP];
+  int2 s[kSR * kG + kNG];
 };
-static_assert(sizeof(RGrid) == 1968, "grid item stride");
+static_assert(sizeof(RGrid) == (kSR == 10 ? 2032 : 1968), "grid item stride");
 static_assert(sizeof(int2) * kNP >= sizeof(float4) * 4 * kNG, "u-curve staging fits in s[]");
 
 struct __align__(16) FbRec {
@@ -801,7 +810,7 @@ struct ReyesF {
     for (int r = 0; r < 3; ++r) {
       const int g = lane + 32 * r;
       if (g < kNP) {
-        const int i = g / kNG, j = g - i * kNG;
+        const int j = g / kNG, i = g - j * kNG;  // point (i, j) is stored at 9j + i (RGrid)
         float Bu[4];
         if constexpr (kSmemM) {
           const float4 b4 = *(const float4*)&Bt[4 * i];
@@ -851,7 +860,7 @@ struct ReyesF {
         const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
         const int Xi = ok ? __float2int_rn(X) : INT_MIN, Yi = ok ? __float2int_rn(Y) : INT_MIN;
         out->o[g].w = zs;
-        out->s[g] = make_int2(Xi, Yi);
+        out->s[g + (kSR - kNG) * (g / kNG)] = make_int2(Xi, Yi);  // sidx(i, j), g = 9j + i
         ok_all = ok_all && ok;
       }
     }
@@ -886,17 +895,17 @@ struct ReyesF {
     const uint32_t frame = (Gd->id >> 12) - (uint32_t)p.frame_base, patch = Gd->id & 0xFFFu;
     if (frame >= (uint32_t)p.n_frames) return;
     const int i = q >> 3, j = q & 7;
-    const int g00 = i * kNG + j, g10 = (i + 1) * kNG + j, g01 = i * kNG + j + 1, g11 = (i + 1) * kNG + j + 1;
+    const int g00 = j * kNG + i, g10 = j * kNG + i + 1, g01 = (j + 1) * kNG + i, g11 = (j + 1) * kNG + i + 1;
     // Coverage first: the two triangles cover exactly the pixel centres inside either
     // one, all within the quad's box; a micropolygon whose box holds no pixel centre
     // (most of them at config 5: ~0.25 px^2 each) writes nothing, so its shading is
     // never computed.
-    const int gi[4] = {g00, g10, g11, g01};
+    const int si[4] = {sidx(i, j), sidx(i + 1, j), sidx(i + 1, j + 1), sidx(i, j + 1)};
     int vx[4], vy[4];
     bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
-      const int2 sv = Gd->s[gi[v]];
+      const int2 sv = Gd->s[si[v]];
       vx[v] = sv.x;
       vy[v] = sv.y;
       if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
@@ -991,12 +1000,12 @@ struct ReyesF {
   static __device__ __forceinline__ bool mp_box(const Params& p, const RGrid* Gd, int q) {
     if (kFrame && (Gd->id >> 12) - (uint32_t)p.frame_base >= (uint32_t)p.n_frames) return false;
     const int i = q >> 3, j = q & 7;
-    const int gi[4] = {i * kNG + j, (i + 1) * kNG + j, (i + 1) * kNG + j + 1, i * kNG + j + 1};
+    const int si[4] = {sidx(i, j), sidx(i + 1, j), sidx(i + 1, j + 1), sidx(i, j + 1)};
     int vx[4], vy[4];
     bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
-      const int2 sv = Gd->s[gi[v]];
+      const int2 sv = Gd->s[si[v]];
       vx[v] = sv.x;
       vy[v] = sv.y;
       if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;

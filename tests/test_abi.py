@@ -98,7 +98,7 @@ def test_stage_kind_info_host_only():
     (include/vp.h: 208-B patches for Reyes Bound/Split/Dice, reading R-S10; 1968-B grids)."""
     from paper_conf_micro_zhengozsyc17_b200 import vp
     assert [vp.stage_kind_info(k)[0] for k in (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)] == [
-        208, 208, 208, 1968]
+        208, 208, 208, 2032]
     assert [vp.stage_kind_info(k)[1] for k in (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)] == [
         16, 16, 32, 64]
     assert vp.stage_kind_info(vp.TOY_S1) == (4, 1)
