@@ -63,6 +63,9 @@ constexpr int kG = 8, kNG = 9, kNP = 81;
 // 36 u-curve points C_a(v_j) as float4.  (Round 2: carrying each point's pixel-centre
 // index range as well -- a 2608-B grid -- made the box test cheaper but pushed the fused
 // kernel's shared memory past the 196-KB carve-out step, and it ran 5% slower.)
+#ifndef VP_MS_REG  // 1: Dice keeps the frame matrix rows in registers for a lane's 3 points
+#define VP_MS_REG 1
+#endif
 #ifndef VP_SROW
 #define VP_SROW 10
 #endif
@@ -804,13 +807,19 @@ struct ReyesF {
       __syncwarp();
     }
     const float4* C = (const float4*)out->s;
-    // S(u_i, v_j) into o[g].xyz at once (the staged C in s[] is still being read by other
-    // lanes, so s[] is written after the next __syncwarp)
+    // Lanes 0..26: grid row j = lane / 3 (its u-curve points C_a(v_j) loaded once), points
+    // i = i0 .. i0 + 2, i0 = 3 (lane % 3); g = 9j + i.  S(u_i, v_j) goes into o[g].xyz at once
+    // (the staged C in s[] is still being read by other lanes, so s[] is written after the
+    // next __syncwarp).
+    const bool lw = lane < 3 * kNG;
+    const int j = lane / 3, i0 = 3 * (lane - 3 * j), g0 = j * kNG + i0;
+    if (lw) {
+      float4 Cj[4];
 #pragma unroll
-    for (int r = 0; r < 3; ++r) {
-      const int g = lane + 32 * r;
-      if (g < kNP) {
-        const int j = g / kNG, i = g - j * kNG;  // point (i, j) is stored at 9j + i (RGrid)
+      for (int a = 0; a < 4; ++a) Cj[a] = C[a * kNG + j];
+#pragma unroll
+      for (int r = 0; r < 3; ++r) {
+        const int i = i0 + r;
         float Bu[4];
         if constexpr (kSmemM) {
           const float4 b4 = *(const float4*)&Bt[4 * i];
@@ -821,20 +830,26 @@ struct ReyesF {
         float x = 0.0f, y = 0.0f, z = 0.0f;
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
-          const float4 c = C[a * kNG + j];
-          x = x + Bu[a] * c.x;
-          y = y + Bu[a] * c.y;
-          z = z + Bu[a] * c.z;
+          x = x + Bu[a] * Cj[a].x;
+          y = y + Bu[a] * Cj[a].y;
+          z = z + Bu[a] * Cj[a].z;
         }
-        out->o[g] = make_float4(x, y, z, 0.0f);
+        out->o[g0 + r] = make_float4(x, y, z, 0.0f);
       }
     }
     __syncwarp();  // every C read before s[] is written
     bool ok_all = true;
+    if (lw) {
+#if VP_MS_REG
+      float4 Mr[4];
+      if constexpr (kSmemM) {
 #pragma unroll
-    for (int r = 0; r < 3; ++r) {
-      const int g = lane + 32 * r;
-      if (g < kNP) {
+        for (int q = 0; q < 4; ++q) Mr[q] = Ms[q];
+      }
+#endif
+#pragma unroll
+      for (int r = 0; r < 3; ++r) {
+        const int g = g0 + r;
         const float4 ov = out->o[g];  // this lane's own write
         const float x = ov.x, y = ov.y, z = ov.z;
         float4 c;
@@ -842,7 +857,11 @@ struct ReyesF {
           float cc[4];
 #pragma unroll
           for (int q = 0; q < 4; ++q) {
+#if VP_MS_REG
+            const float4 m = Mr[q];
+#else
             const float4 m = Ms[q];
+#endif
             float acc = m.x * x;
             acc = acc + m.y * y;
             acc = acc + m.z * z;
@@ -860,7 +879,7 @@ struct ReyesF {
         const bool ok = fabsf(X) < 1073741824.0f && fabsf(Y) < 1073741824.0f;
         const int Xi = ok ? __float2int_rn(X) : INT_MIN, Yi = ok ? __float2int_rn(Y) : INT_MIN;
         out->o[g].w = zs;
-        out->s[g + (kSR - kNG) * (g / kNG)] = make_int2(Xi, Yi);  // sidx(i, j), g = 9j + i
+        out->s[sidx(i0 + r, j)] = make_int2(Xi, Yi);
         ok_all = ok_all && ok;
       }
     }
