@@ -590,7 +590,6 @@ struct ReyesF {
     RPatch stack[kWarpsW][kDfsStack];
     RPatch stage[kWarpsW][kDfsStage];
     float4 M[2 * kWarpsW][4];            // each group's current frame matrix (rows)
-    uint32_t mframe[2 * kWarpsW];        // its frame + 1 (0: none; scratch starts zeroed)
   };
   static constexpr bool direct_publish(int lo, int hi, bool rtc) { return !rtc && lo == BOUND && hi == SPLIT; }
   static constexpr int direct_out_cap(int, int, int t) { return t == DICE ? kWarpsW * kDfsStage : 0; }
@@ -611,6 +610,7 @@ struct ReyesF {
     RPatch* const stage = ds.stage[warp];
     int wsp = 0, wcnt = 0, nb = 0, nsp = 0;  // wsp, wcnt: warp-uniform
     bool have = false, first = false, presplit = false, drained = false;
+    uint32_t mtag = 0;  // frame + 1 of the rows in ds.M[hw] (0: none), the same in every lane of the group
     float4 q = make_float4(0.f, 0.f, 0.f, 0.f);
     uint32_t id = 0, path = 0, dirs = 0, depth = 0;
     for (;;) {
@@ -653,12 +653,12 @@ struct ReyesF {
       }
       if (!__any_sync(0xffffffffu, have)) break;
       const uint32_t frame = frame_of(p, id);
-      const bool reload = have && ds.mframe[hw] != frame + 1;
+      const bool reload = have && mtag != frame + 1;
       if (__any_sync(0xffffffffu, reload)) {
-        __syncwarp();  // every read of the old rows and tags is done
+        __syncwarp();  // every read of the old rows is done
         if (reload) {
           ((float*)ds.M[hw])[lane] = __ldg(p.M + 16 * (size_t)frame + lane);
-          if (lane == 0) ds.mframe[hw] = frame + 1;
+          mtag = frame + 1;
         }
         __syncwarp();
       }
@@ -671,7 +671,7 @@ struct ReyesF {
       const unsigned long long node = ((unsigned long long)id << 12) | ((unsigned long long)(depth & 15u) << 8) | (path & 0xFFu);
       if (have && !presplit && !first) {  // a Bound task that never went through a ring
         ++nb;
-        if (lane == 0) ctx.template trace_local_id<BOUND>(node);
+        if (ctx.tracing() && lane == 0) ctx.template trace_local_id<BOUND>(node);
       }
       // Dice: stage the leaf in the warp's buffer (both groups may add one this step)
       const bool leaf = have && cls == 2;
@@ -717,7 +717,7 @@ struct ReyesF {
           } else {
             if (!(first && presplit)) {  // a claimed Split item was counted when it was claimed
               ++nsp;
-              if (lane == 0) ctx.template trace_local_id<SPLIT>(node);
+              if (ctx.tracing() && lane == 0) ctx.template trace_local_id<SPLIT>(node);
             }
             const uint32_t ndirs = (dirs & ~(1u << depth)) | ((uint32_t)dir << depth);
             RPatch* r = &stk[slot];

@@ -209,12 +209,17 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* m, uint32_t parity
 // time hint) instead of re-issuing try_wait, so idle workers leave the issue slots to the
 // warps that still execute.
 // The suspend hint alone returns often (round 2 profile: the retry loop was 5.4% of the
-// fused [Dice, Shade] kernel's executed instructions).  VP_MBAR_NS > 0 adds an exponential
-// __nanosleep back-off after a failed try_wait; measured on config 5 it did not pay
-// (256 / 1024 ns: within +-0.5% of none), so the default is none.
+// fused [Dice, Shade] kernel's executed instructions).  kMaxNs > 0 adds an exponential
+// __nanosleep back-off after a failed try_wait (capped at kMaxNs).  Measured on config 5:
+// no gain for the fused [Dice, Shade] kernel (256 / 1024 ns: within +-0.5%), so only the
+// direct-publish kernels ([Bound, Split]) use it, VP_BS_BACKOFF_NS.
 #ifndef VP_MBAR_NS
 #define VP_MBAR_NS 0
 #endif
+#ifndef VP_BS_BACKOFF_NS
+#define VP_BS_BACKOFF_NS 0
+#endif
+template <int kMaxNs = VP_MBAR_NS>
 __device__ __forceinline__ void mbar_wait_sleep(unsigned long long* m, uint32_t parity) {
   uint32_t done = 0;
   uint32_t ns = 32;
@@ -227,9 +232,9 @@ __device__ __forceinline__ void mbar_wait_sleep(unsigned long long* m, uint32_t 
         : "r"(smem_u32(m)), "r"(parity), "r"(20000u)
         : "memory");
     if (done) break;
-    if (VP_MBAR_NS > 0) {
+    if (kMaxNs > 0) {
       __nanosleep(ns);
-      ns = ns * 2 < (uint32_t)VP_MBAR_NS ? ns * 2 : (uint32_t)VP_MBAR_NS;
+      ns = ns * 2 < (uint32_t)kMaxNs ? ns * 2 : (uint32_t)kMaxNs;
     }
   }
 }
@@ -625,6 +630,7 @@ struct Ctx {
   __device__ __forceinline__ void note_units(int n) {
     if (n) atomicAdd(&sh.units32[T], (uint32_t)n);
   }
+  __device__ __forceinline__ bool tracing() const { return (a.c.flags & FLAG_TRACE) != 0; }
   // ... or given the task's item id directly (items that live only in registers).
   template <int T>
   __device__ __forceinline__ void trace_local_id(unsigned long long id) {
@@ -1434,7 +1440,7 @@ struct Runner {
     if (warp < kWarpsW) {
       for (int it = 0;; ++it) {
         const int b = it & 1;
-        mbar_wait_sleep(&sh.full[b], (uint32_t)((it >> 1) & 1));
+        mbar_wait_sleep<direct_publish<F>(LO, HI, RTC) ? VP_BS_BACKOFF_NS : VP_MBAR_NS>(&sh.full[b], (uint32_t)((it >> 1) & 1));
         const int n = sh.bn[b];
         if (n < 0) break;
         ctx.ob = b;
