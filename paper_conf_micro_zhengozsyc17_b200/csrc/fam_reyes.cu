@@ -1021,19 +1021,21 @@ struct ReyesF {
     const int i = q >> 3, j = q & 7;
     const int si[4] = {sidx(i, j), sidx(i + 1, j), sidx(i + 1, j + 1), sidx(i, j + 1)};
     int vx[4], vy[4];
-    bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
       const int2 sv = Gd->s[si[v]];
       vx[v] = sv.x;
       vy[v] = sv.y;
-      if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
     }
     const int xmin = min(min(vx[0], vx[1]), min(vx[2], vx[3])), xmax = max(max(vx[0], vx[1]), max(vx[2], vx[3]));
     const int ymin = min(min(vy[0], vy[1]), min(vy[2], vy[3])), ymax = max(max(vy[0], vy[1]), max(vy[2], vy[3]));
-    const int px0 = max(-((128 - xmin) >> 8), 0), px1 = min((xmax - 128) >> 8, p.W - 1);
-    const int py0 = max(-((128 - ymin) >> 8), 0), py1 = min((ymax - 128) >> 8, p.H - 1);
-    return ok && px0 <= px1 && py0 <= py1;
+    // shade_mp's test max(c, 0) <= min(f, W - 1), c = ceil((xmin - 128) / 256), f = floor((xmax
+    // - 128) / 256), restated without the divisions: c <= f <=> 256 f + 128 >= xmin, c <= W - 1
+    // <=> xmin <= 256 (W - 1) + 128, 0 <= f <=> xmax >= 128 (same for y).  An unsnappable
+    // corner is INT_MIN in both coordinates, so it is the minimum: xmin != INT_MIN.
+    const bool inx = xmin != INT_MIN && xmax >= 128 && xmin <= p.W * 256 - 128 && ((xmax - 128) & ~255) + 128 >= xmin;
+    const bool iny = ymax >= 128 && ymin <= p.H * 256 - 128 && ((ymax - 128) & ~255) + 128 >= ymin;
+    return inx && iny;
   }
   template <int S0, int HI, class Ctx>
   static __device__ void exec_rtc_chain(Ctx& ctx, const uint8_t* items, int n) {
