@@ -910,9 +910,12 @@ struct ReyesF {
   // -------------------------------------------------------------- Shade (per micropolygon)
   // Micropolygon q = 8i + j of grid Gd: the quad (i,j)..(i+1,j+1), split into the
   // triangles (v0,v1,v2), (v0,v2,v3) (reading R-R8..R-R10).
+  // kBoxed: the caller already established mp_box (valid frame, snappable corners, a pixel
+  // centre in the box), so those early exits are skipped
+  template <bool kBoxed = false>
   static __device__ __forceinline__ void shade_mp(const Params& p, const RGrid* Gd, int q) {
     const uint32_t frame = (Gd->id >> 12) - (uint32_t)p.frame_base, patch = Gd->id & 0xFFFu;
-    if (frame >= (uint32_t)p.n_frames) return;
+    if (!kBoxed && frame >= (uint32_t)p.n_frames) return;
     const int i = q >> 3, j = q & 7;
     const int g00 = j * kNG + i, g10 = j * kNG + i + 1, g01 = (j + 1) * kNG + i, g11 = (j + 1) * kNG + i + 1;
     // Coverage first: the two triangles cover exactly the pixel centres inside either
@@ -921,17 +924,16 @@ struct ReyesF {
     // never computed.
     const int si[4] = {sidx(i, j), sidx(i + 1, j), sidx(i + 1, j + 1), sidx(i, j + 1)};
     int vx[4], vy[4];
-    bool ok = true;
 #pragma unroll
     for (int v = 0; v < 4; ++v) {
       const int2 sv = Gd->s[si[v]];
       vx[v] = sv.x;
       vy[v] = sv.y;
-      if (vx[v] == INT_MIN || vy[v] == INT_MIN) ok = false;
     }
-    if (!ok) return;
     const int xmin = min(min(vx[0], vx[1]), min(vx[2], vx[3])), xmax = max(max(vx[0], vx[1]), max(vx[2], vx[3]));
     const int ymin = min(min(vy[0], vy[1]), min(vy[2], vy[3])), ymax = max(max(vy[0], vy[1]), max(vy[2], vy[3]));
+    // an unsnappable corner is INT_MIN in both coordinates, hence the minimum
+    if (!kBoxed && xmin == INT_MIN) return;
     // |coords| < 2^30: these int expressions cannot overflow
     int px0 = -((128 - xmin) >> 8), px1 = (xmax - 128) >> 8;  // ceil / floor of (v - 128) / 256
     int py0 = -((128 - ymin) >> 8), py1 = (ymax - 128) >> 8;
@@ -939,7 +941,7 @@ struct ReyesF {
     py0 = max(py0, 0);
     px1 = min(px1, p.W - 1);
     py1 = min(py1, p.H - 1);
-    if (px0 > px1 || py0 > py1) return;
+    if (!kBoxed && (px0 > px1 || py0 > py1)) return;
     const float4 o00 = Gd->o[g00], o10 = Gd->o[g10], o01 = Gd->o[g01], o11 = Gd->o[g11];
     const float e1[3] = {o10.x - o00.x, o10.y - o00.y, o10.z - o00.z};
     const float e2[3] = {o01.x - o00.x, o01.y - o00.y, o01.z - o00.z};
@@ -1103,7 +1105,7 @@ struct ReyesF {
       if (lane == 0) ctx.template note_units<SHADE>(tot);
       for (int t = lane; t < tot; t += 32) {
         const int e = list[t];
-        shade_mp(p, (e >> 6) ? g1 : g0, e & 63);
+        shade_mp<true>(p, (e >> 6) ? g1 : g0, e & 63);
       }
       __syncwarp();  // the slots, the matrix and the list are rewritten next
     }
