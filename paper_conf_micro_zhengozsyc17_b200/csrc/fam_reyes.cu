@@ -334,7 +334,7 @@ struct ReyesF {
         float acc = m.x * q.x;
         acc = acc + m.y * q.y;
         acc = acc + m.z * q.z;
-        acc = acc + m.w * q.w;
+        acc = acc + m.w;  // m.w * q.w with q.w = 1 exactly (R-S10): x * 1 = x in IEEE arithmetic
         cc[r] = acc;
       }
       c = make_float4(cc[0], cc[1], cc[2], cc[3]);
@@ -415,7 +415,7 @@ struct ReyesF {
       float acc = m.x * q.x;
       acc = acc + m.y * q.y;
       acc = acc + m.z * q.z;
-      acc = acc + m.w * q.w;
+      acc = acc + m.w;  // m.w * q.w with q.w = 1 exactly (R-S10): x * 1 = x in IEEE arithmetic
       cc[r] = acc;
     }
     const float4 c = make_float4(cc[0], cc[1], cc[2], cc[3]);
@@ -865,7 +865,7 @@ struct ReyesF {
             float acc = m.x * x;
             acc = acc + m.y * y;
             acc = acc + m.z * z;
-            acc = acc + m.w * 1.0f;
+            acc = acc + m.w;  // m.w * 1: exact, so the multiply is dropped
             cc[q] = acc;
           }
           c = make_float4(cc[0], cc[1], cc[2], cc[3]);

@@ -46,6 +46,19 @@ def cfgs(name):
         q0, q1 = int(name[1]), int(name[2])
         return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, nsm), (2, 3, vp.GROUP_RTC, 0, nsm)], nsm,
                                           blocks_per_sm=[q0, 0, q1, 0])
+    if name[0] in "xe" and name[1].isdigit():
+        # x{s}: [Bound,Split] on SMs [0, s/2) and [nsm/2, nsm/2 + s/2) (both halves of the
+        # SM-id range); e{s}: on s evenly spaced SMs; [Dice,Shade] on the rest
+        s = int(name[1:])
+        if name[0] == "x":
+            bs = set(range(s // 2)) | set(range(nsm // 2, nsm // 2 + s - s // 2))
+        else:
+            bs = {(k * nsm) // s for k in range(s)}
+        b = vp.make_binding([(0, 1, vp.GROUP_MEGA, 0, 0), (2, 3, vp.GROUP_RTC, 0, 0)], nsm)
+        for sm in range(nsm):
+            g = 0 if sm in bs else 1
+            b.group_sm_mask[g][sm >> 5] |= 1 << (sm & 31)
+        return vp.HYBRID, b
     if name.startswith("fine_h"):
         return vp.HYBRID, vp.make_binding([(0, 1, vp.GROUP_FINE, 0, 40), (2, 3, vp.GROUP_RTC, 40, nsm)], nsm)
     raise ValueError(name)
