@@ -34,12 +34,14 @@ MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
 # Algorithmic fp32 operations per task (counted from the stage
 # definitions, excluding per-point constant Bernstein tables and integer coverage work):
 # Dice (reading R-R7, separable form): 36 u-curve points x 3 coords x (4 mul + 3 add), then
-# per grid point 3 coords x 7 + M.p 28 + screen 9 (3 div, 6 mul/add) + Q8 snap 2 = 5616
-FLOP_DICE = 36 * 3 * 7 + 81 * (3 * 7 + 28 + 9 + 2)
+# per grid point 3 coords x 7 + M.p 24 (4 rows x (3 mul + 3 add): w = 1, R-S10, so the 4th
+# product is no work and the kernel does not execute it) + screen 9 (3 div, 6 mul/add) +
+# Q8 snap 2 = 5292
+FLOP_DICE = 36 * 3 * 7 + 81 * (3 * 7 + 24 + 9 + 2)
 FLOP_SHADE = 64 * 41                 # edges, cross, |n|, n.L, sqrt/div, shade, zq, Q8 snap = 2624
 FLOP_SHADE_MP = 41                   # per micropolygon actually shaded (box holds a pixel centre)
-FLOP_BOUND = 16 * (28 + 9) + 40      # 16 projections + split metric = 632
-FLOP_SPLIT = 3 * 4 * 12              # de Casteljau, 3 coords x 4 curves = 144
+FLOP_BOUND = 16 * (24 + 6) + 40      # 16 affine projections, sx / sy (2 div + 4), split metric = 520
+FLOP_SPLIT = 3 * 4 * 12              # de Casteljau, 3 coords (w = 1) x 4 curves x 12 = 144
 
 
 def env_int(k, d):
