@@ -447,12 +447,14 @@ struct ReyesF {
       const float sx3 = __shfl_down_sync(0xffffffffu, sx, 3, 16), sy3 = __shfl_down_sync(0xffffffffu, sy, 3, 16);
       float lu = (lane < 4) ? fabsf(sx12 - sx) + fabsf(sy12 - sy) : 0.0f;
       float lv = ((lane & 3) == 0) ? fabsf(sx3 - sx) + fabsf(sy3 - sy) : 0.0f;
-#pragma unroll
-      for (int o = 8; o >= 1; o >>= 1) {
-        lu = fmaxf(lu, __shfl_xor_sync(0xffffffffu, lu, o, 16));
-        lv = fmaxf(lv, __shfl_xor_sync(0xffffffffu, lv, o, 16));
-      }
-      if (!straddle) dir = (lu >= lv) ? 0 : 1;
+      // lu lives on the group's lanes 0..3, lv on lanes 0, 4, 8, 12: two levels each bring
+      // both maxima to the group's lane 0, which decides for the group
+      lu = fmaxf(lu, __shfl_xor_sync(0xffffffffu, lu, 1, 16));
+      lu = fmaxf(lu, __shfl_xor_sync(0xffffffffu, lu, 2, 16));
+      lv = fmaxf(lv, __shfl_xor_sync(0xffffffffu, lv, 4, 16));
+      lv = fmaxf(lv, __shfl_xor_sync(0xffffffffu, lv, 8, 16));
+      const int d0 = __shfl_sync(0xffffffffu, (lu >= lv) ? 0 : 1, 0, 16);
+      if (!straddle) dir = d0;
     }
     if (__any_sync(0xffffffffu, cls == 1 && straddle)) {  // object-space metric (near-plane straddle, R-R4)
       const float ox12 = __shfl_sync(0xffffffffu, q.x, (lane & 3) + 12, 16);
@@ -469,12 +471,12 @@ struct ReyesF {
         olv = fabsf(ox3 - q.x) + fabsf(oy3 - q.y);
         olv = olv + fabsf(oz3 - q.z);
       }
-#pragma unroll
-      for (int o = 8; o >= 1; o >>= 1) {
-        olu = fmaxf(olu, __shfl_xor_sync(0xffffffffu, olu, o, 16));
-        olv = fmaxf(olv, __shfl_xor_sync(0xffffffffu, olv, o, 16));
-      }
-      if (straddle) dir = (olu >= olv) ? 0 : 1;
+      olu = fmaxf(olu, __shfl_xor_sync(0xffffffffu, olu, 1, 16));
+      olu = fmaxf(olu, __shfl_xor_sync(0xffffffffu, olu, 2, 16));
+      olv = fmaxf(olv, __shfl_xor_sync(0xffffffffu, olv, 4, 16));
+      olv = fmaxf(olv, __shfl_xor_sync(0xffffffffu, olv, 8, 16));
+      const int d0 = __shfl_sync(0xffffffffu, (olu >= olv) ? 0 : 1, 0, 16);
+      if (straddle) dir = d0;
     }
     return cls;
   }
@@ -594,11 +596,6 @@ struct ReyesF {
   static constexpr bool direct_publish(int lo, int hi, bool rtc) { return !rtc && lo == BOUND && hi == SPLIT; }
   static constexpr int direct_out_cap(int, int, int t) { return t == DICE ? kWarpsW * kDfsStage : 0; }
 
-  // a control point from another lane of the 16-thread group (w = 1 is not shuffled)
-  static __device__ __forceinline__ float4 shfl4(unsigned m, float4 v, int src) {
-    return make_float4(__shfl_sync(m, v.x, src, 16), __shfl_sync(m, v.y, src, 16), __shfl_sync(m, v.z, src, 16), 1.0f);
-  }
-
   template <int SS, class Ctx>
   static __device__ void exec_dfs(Ctx& ctx, const uint8_t* items, int n) {
     const Params& p = ctx.params();
@@ -692,19 +689,26 @@ struct ReyesF {
       if (sb) {  // warp-uniform: the shuffles below run converged
         // de Casteljau at 1/2 (reading R-R6) of the curve through this lane's control point
         // along the split direction; same operations as split_cp, points from shuffles
+        // Lane t of a curve (points a b c d) computes the de Casteljau levels at its own
+        // position, h1 = (p_t + p_t+1) / 2, h2 = (h1_t + h1_t+1) / 2, h3 likewise, from the
+        // next lane's value (lanes past the curve's end compute values nobody uses): h1 at
+        // t = 0, 1, 2 is ab, bc, cd; h2 at t = 0, 1 is abc, bcd; h3 at t = 0 is m -- the same
+        // operations in the same order as split_cp.  Right child point t is level 3 - t of
+        // lane t itself, left child point t is level t of the curve's first lane.
         const int base = dir == 0 ? (lane & 3) : (lane & ~3), step = dir == 0 ? 4 : 1;
         const int t = dir == 0 ? (lane >> 2) : (lane & 3);
-        const float4 a = shfl4(0xffffffffu, q, base), b = shfl4(0xffffffffu, q, base + step);
-        const float4 c = shfl4(0xffffffffu, q, base + 2 * step), d = shfl4(0xffffffffu, q, base + 3 * step);
         float4 L, R;
-#define VP_CASTELJAU(comp)                                                   \
-  {                                                                          \
-    float ab = (a.comp + b.comp) * 0.5f, bc = (b.comp + c.comp) * 0.5f;      \
-    float cd = (c.comp + d.comp) * 0.5f;                                     \
-    float abc = (ab + bc) * 0.5f, bcd = (bc + cd) * 0.5f;                    \
-    float m = (abc + bcd) * 0.5f;                                            \
-    L.comp = t == 0 ? a.comp : t == 1 ? ab : t == 2 ? abc : m;              \
-    R.comp = t == 0 ? m : t == 1 ? bcd : t == 2 ? cd : d.comp;              \
+#define VP_CASTELJAU(comp)                                                          \
+  {                                                                                 \
+    const float v = q.comp;                                                         \
+    const float h1 = (v + __shfl_down_sync(0xffffffffu, v, step, 16)) * 0.5f;       \
+    const float h2 = (h1 + __shfl_down_sync(0xffffffffu, h1, step, 16)) * 0.5f;     \
+    const float h3 = (h2 + __shfl_down_sync(0xffffffffu, h2, step, 16)) * 0.5f;     \
+    const float g1 = __shfl_sync(0xffffffffu, h1, base, 16);                        \
+    const float g2 = __shfl_sync(0xffffffffu, h2, base, 16);                        \
+    const float g3 = __shfl_sync(0xffffffffu, h3, base, 16);                        \
+    L.comp = t == 0 ? v : t == 1 ? g1 : t == 2 ? g2 : g3;                           \
+    R.comp = t == 0 ? h3 : t == 1 ? h2 : t == 2 ? h1 : v;                           \
   }
         VP_CASTELJAU(x) VP_CASTELJAU(y) VP_CASTELJAU(z)  // w stays 1 (R-S10)
 #undef VP_CASTELJAU
