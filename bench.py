@@ -614,7 +614,7 @@ def main():
         # the paper's offline auto-tuner (L41-L45, Fig. 10) picks {grouping, models, SM
         # split, batch} on this shard before anything is timed
         t_tune = time.perf_counter()
-        best_cfg, rep = rp.p.autotune(time_budget_s=args.tune_seconds, sm_granularity=2, batch_choices=(1, 2))
+        best_cfg, rep = rp.p.autotune(time_budget_s=args.tune_seconds, sm_granularity=1, batch_choices=(1, 2))
         tune = {"seconds": round(time.perf_counter() - t_tune, 2), "candidates_run": rep.candidates_run,
                 "candidates_total": rep.candidates_total, "timed_out": rep.candidates_timed_out,
                 "best_ms": rep.best_ms, "kbk_ms": rep.baseline_kbk_ms, "megakernel_ms": rep.baseline_mega_ms,

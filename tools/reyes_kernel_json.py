@@ -55,16 +55,21 @@ kern = {"source": f"ncu --set full, profiles/{tag}_rtc_leaf.txt and profiles/{ta
                              "warp_instructions_per_leaf": f(r, "smsp__inst_executed.sum") / leaves,
                              "dram_bytes_per_leaf": (rd + wr) / leaves,
                              "registers": int(f(r, "launch__registers_per_thread")),
-                             "duration_us_64_frames_alone": f(r, "gpu__time_duration.sum") / 1e3},
+                             "duration_us_64_frames_alone": f(r, "gpu__time_duration.sum") / 1e3,
+                             # the second limit: the L1/shared-memory data pipe
+                             "smem_wavefronts_per_leaf": f(r, "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum") / leaves,
+                             "smem_pipe_pct_of_peak": f(r, "l1tex__data_pipe_lsu_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed"),
+                             "l1tex_throughput_pct": f(r, "l1tex__throughput.avg.pct_of_peak_sustained_active")},
         "bound_split_dfs": {"kernel": "vp_kernel<ReyesF,0,1,MEGA> (depth-first, direct publish)",
                             "issue_active_pct": f(b, "smsp__issue_active.avg.pct_of_peak_sustained_active"),
                             "warps_active_pct": f(b, "sm__warps_active.avg.pct_of_peak_sustained_active"),
                             "warp_instructions_per_bound_task": f(b, "smsp__inst_executed.sum") / bound_tasks,
                             "registers": int(f(b, "launch__registers_per_thread")),
                             "blocks_per_sm": int(f(b, "launch__occupancy_limit_registers"))},
-        "note": "both kernels are issue-bound (IEEE div/sqrt, integer coverage, shuffles, 128-bit CAS), so the "
-                "fp32 fraction understates how busy they are; issue_active is the fraction of issue slots used on "
-                "the SMs the kernel ran on"}
+        "note": "both kernels are issue-bound (IEEE div/sqrt, integer coverage, shuffles, 128-bit CAS), and the "
+                "fused Dice+Shade kernel also keeps the L1/shared-memory pipe busy (its grids live in shared memory), "
+                "so the fp32 fraction understates how busy they are; issue_active is the fraction of issue slots "
+                "used on the SMs the kernel ran on"}
 json.dump(traffic, open(f"profiles/{tag}_rtc_leaf_traffic.json", "w"), indent=1)
 json.dump(kern, open(f"profiles/{tag}_reyes_kernels.json", "w"), indent=1)
 print(json.dumps(kern, indent=1))
