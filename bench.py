@@ -273,8 +273,12 @@ def queue_microbench(torch, vp, stream):
             n = (1 << 20 if ib < 272 else 1 << 18) if fan == 1 else (1 << 7 if ib < 272 else 1 << 4)
             qb = QBenchPipeline(n, ib, fan, depth)
             r = {}
-            for name, model in (("megakernel", vp.MEGAKERNEL), ("kbk", vp.KBK), ("kbk_graph", vp.KBK_GRAPH)):
-                qb.configure(model)
+            # the megakernel at the default batch and at the largest one its kernel allows (the
+            # batch is one of the tuner's parameters, L41; trees publish 2 children per task,
+            # and larger batches amortise the publisher warp's per-round work)
+            for name, model, bat in (("megakernel", vp.MEGAKERNEL, 0), ("megakernel_max_batch", vp.MEGAKERNEL, 64 if ib == 272 else 1024),
+                                     ("kbk", vp.KBK, 0), ("kbk_graph", vp.KBK_GRAPH, 0)):
+                qb.configure(model, None, bat)
                 qb.run(stream)
                 ts = []
                 for _ in range(3):
@@ -282,7 +286,7 @@ def queue_microbench(torch, vp, stream):
                     assert res["bad"] == 0 and st["dequeued"][qb.stage] == qb.tasks()
                     ts.append(st["device_ms"])
                 ms = min(ts)
-                r[name] = {"ms": ms, "mtasks_per_s": qb.tasks() / ms / 1e3,
+                r[name] = {"ms": ms, "mtasks_per_s": qb.tasks() / ms / 1e3, "batch": bat or "default",
                            # every task reads its item once; every non-seed item was written once
                            "ring_gbs": (2 * qb.tasks() - n) * ib / ms / 1e6}
             out[f"item{ib}_fan{fan}"] = {"tasks": qb.tasks(), **r}
