@@ -94,9 +94,10 @@ typedef enum vp_stage_kind {
   /* LBP face detection (Fig. 14, L55): Grayscale, HistEq as CDF + Map, Resize
    * (recursive), Feature Extraction (LBP), Scanning (rows of 24x24 windows) */
   VP_FD_GRAY = 60, VP_FD_CDF = 61, VP_FD_MAP = 62, VP_FD_RESIZE = 63, VP_FD_LBP = 64, VP_FD_SCAN = 65,
-  /* Queue microbenchmark (not a paper workload): three independent
-   * self-recursive stages with 4-, 16- and 272-B items (Fig. 9's int; Table 2's window /
-   * tile items; the Reyes patch, L61 §8.5).  See vp_qbench_params. */
+  /* Queue microbenchmark (not a paper workload): a self-recursive stage
+   * with 4-, 16- or 272-B items (Fig. 9's int; Table 2's window / tile items; the Reyes
+   * patch, L61 §8.5), each kind a single-stage pipeline of its own: register one of them.
+   * See vp_qbench_params (counters indexed by item size: 0 = 4 B, 1 = 16 B, 2 = 272 B). */
   VP_QB_ITEM4 = 70, VP_QB_ITEM16 = 71, VP_QB_ITEM272 = 72,
   /* LDPC decoder (Fig. 17, L59): Initialize, C2V, V2C, ProbVar (loops back to C2V for the
    * next of n_iter iterations); items {frame, iteration}; see vp_ldpc_params */

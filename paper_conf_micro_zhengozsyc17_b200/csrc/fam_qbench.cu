@@ -14,14 +14,19 @@
 
 namespace vp {
 
+// One single-stage family per item size (round 2): a family's kernels reserve shared
+// memory for every stage they cover, so three sizes in one family gave its megakernel the
+// buffers of all three (1 block/SM) while a KBK wave kernel held one stage's (2 blocks/SM).
+// K: 0 = 4 B, 1 = 16 B, 2 = 272 B; also the counter slot in vp_qbench_params.
+template <int K>
 struct QBenchF {
-  static constexpr int S = 3;
-  static constexpr int kinds[S] = {VP_QB_ITEM4, VP_QB_ITEM16, VP_QB_ITEM272};
+  static constexpr int S = 1;
+  static constexpr int kinds[S] = {K == 0 ? VP_QB_ITEM4 : K == 1 ? VP_QB_ITEM16 : VP_QB_ITEM272};
   using Params = vp_qbench_params;
-  static constexpr int stride(int s) { return s == 0 ? 4 : s == 1 ? 16 : 272; }
+  static constexpr int stride(int) { return K == 0 ? 4 : K == 1 ? 16 : 272; }
   static constexpr int threads_per_item(int) { return 1; }
-  static constexpr int max_batch(int s) { return s == 2 ? 64 : 1024; }
-  static constexpr int default_batch(int s) { return s == 2 ? 32 : 256; }
+  static constexpr int max_batch(int) { return K == 2 ? 64 : 1024; }
+  static constexpr int default_batch(int) { return K == 2 ? 32 : 256; }
   static constexpr int fanout(int s, int t) { return s == t ? 2 : 0; }
   static constexpr bool rtc_ok(int, int) { return true; }
   static constexpr int kMaxBatch = 1024;
@@ -76,8 +81,8 @@ struct QBenchF {
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) ids += __shfl_xor_sync(0xffffffffu, ids, o);
       if (lane == 0 && lm) {
-        atomicAdd(&p.leaves[s], (unsigned long long)__popc(lm));
-        atomicAdd(&p.idsum[s], ids);
+        atomicAdd(&p.leaves[K], (unsigned long long)__popc(lm));
+        atomicAdd(&p.idsum[K], ids);
       }
     }
     worker_sync();
@@ -102,7 +107,7 @@ struct QBenchF {
     for (int base = 0; base < n; base += kThreads) {
       const int k = base + threadIdx.x;
       const unsigned bm = __ballot_sync(0xffffffffu, k < n && badf[k] != 0);
-      if (lane == 0 && bm) atomicAdd(&p.bad[s], (unsigned long long)__popc(bm));
+      if (lane == 0 && bm) atomicAdd(&p.bad[K], (unsigned long long)__popc(bm));
     }
   }
   static cudaError_t init_run(const Params& p, cudaStream_t st) {
@@ -127,8 +132,16 @@ struct QBenchF {
   }
 };
 
-const FamilyOps* family_qbench() {
-  static FamilyImpl<QBenchF> f("qbench");
+const FamilyOps* family_qbench4() {
+  static FamilyImpl<QBenchF<0>> f("qbench4");
+  return &f;
+}
+const FamilyOps* family_qbench16() {
+  static FamilyImpl<QBenchF<1>> f("qbench16");
+  return &f;
+}
+const FamilyOps* family_qbench272() {
+  static FamilyImpl<QBenchF<2>> f("qbench272");
   return &f;
 }
 

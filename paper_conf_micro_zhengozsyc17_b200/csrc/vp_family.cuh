@@ -173,7 +173,9 @@ const FamilyOps* family_raster();
 const FamilyOps* family_pyramid();
 const FamilyOps* family_cfd();
 const FamilyOps* family_facedet();
-const FamilyOps* family_qbench();
+const FamilyOps* family_qbench4();
+const FamilyOps* family_qbench16();
+const FamilyOps* family_qbench272();
 const FamilyOps* family_ldpc();
 
 }  // namespace vp

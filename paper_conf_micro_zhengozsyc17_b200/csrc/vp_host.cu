@@ -21,11 +21,13 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
     all_families[8] = family_ldpc();
-    all_families[7] = family_qbench();
+    all_families[7] = family_qbench4();
+    all_families[9] = family_qbench16();
+    all_families[10] = family_qbench272();
     all_families[5] = family_cfd();
     all_families[6] = family_facedet();
     all_families[0] = family_toy();

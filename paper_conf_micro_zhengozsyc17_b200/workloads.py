@@ -46,7 +46,8 @@ class QBenchPipeline:
     SIZES = (4, 16, 272)
 
     def __init__(self, n: int, item_bytes: int, fanout: int, depth: int, device: int = 0, **kw):
-        self.stage = self.SIZES.index(item_bytes)
+        self.slot = self.SIZES.index(item_bytes)  # counter slot (vp_qbench_params arrays)
+        self.stage = 0                            # one single-stage family per item size
         self.n, self.item_bytes, self.fanout, self.depth = n, item_bytes, fanout, depth
         self.cnt = torch.zeros(9, dtype=torch.int64, device=_dev(device))
         ptr = self.cnt.data_ptr()
@@ -54,10 +55,10 @@ class QBenchPipeline:
         # full rings: a breadth-first fan-out-2 tree's frontier is a whole tree level
         kw["flags"] = kw.get("flags", 0) | vp.FLAG_FULL_RINGS
         self.p = vp.Pipeline(device, **kw)
-        # only the seeded stage gets a large ring (a whole tree level must fit for KBK waves)
+        # the ring holds a whole tree level (KBK waves) or chain frontier
         big = 1 << (21 if item_bytes == 272 else 24)
-        for kind, sz in zip((vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272), self.SIZES):
-            self.p.register(kind, sz, self.prm, queue_capacity=big if sz == item_bytes else 1 << 12)
+        kind = (vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272)[self.slot]
+        self.p.register(kind, item_bytes, self.prm, queue_capacity=big)
         self.seeds = inputs.qbench_seeds(n, item_bytes, depth)
         self.p.insert(self.stage, self.seeds, n=n)
 
@@ -71,7 +72,7 @@ class QBenchPipeline:
     def run(self, stream=None):
         st = self.p.run(stream)
         c = self.cnt.cpu().numpy().astype(np.uint64)
-        return {"leaves": int(c[self.stage]), "idsum": int(c[3 + self.stage]), "bad": int(c[6 + self.stage])}, st
+        return {"leaves": int(c[self.slot]), "idsum": int(c[3 + self.slot]), "bad": int(c[6 + self.slot])}, st
 
 
 class LdpcPipeline:

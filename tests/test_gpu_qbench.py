@@ -49,7 +49,7 @@ def test_qbench_batch_sizes(vpm, orc, batch):
     lv, ids, _, deq = orc.qbench_pipeline(qb.seeds, 16, 1)
     qb.configure(vp.MEGAKERNEL, None, batch)
     r, st = qb.run()
-    assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["dequeued"][1] == deq
+    assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["dequeued"][qb.stage] == deq
 
 
 def test_qbench_graph_kbk_launch_count(vpm):
@@ -61,5 +61,5 @@ def test_qbench_graph_kbk_launch_count(vpm):
     r1, st1 = qb.run()
     r2, st2 = qb.run()
     assert r1 == r2 and r1["leaves"] == 1000
-    # one chain level per iteration at least: >= depth + 1 iterations x 3 stages
-    assert st1["kbk_launches"] >= 3 * 21 and st1["kbk_launches"] % 3 == 0
+    # one chain level per iteration at least: >= depth + 1 iterations of the single stage
+    assert st1["kbk_launches"] >= 21 and st1["kbk_launches"] == st2["kbk_launches"]
