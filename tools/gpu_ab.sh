@@ -14,3 +14,9 @@ for lib in ${VP_AB_LIBS:-libvp.so}; do
   fi
 done
 done
+# optional: a full ncu capture of the fused [Dice,Shade] kernel of the default build
+if [ -n "$VP_AB_NCU_TAG" ]; then
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:vp_kernel -c 1 -o gpurun_out/rtc_leaf$VP_AB_NCU_TAG python tools/ncu_targets.py rtc_leaf --frames 64 --runs 1 > gpurun_out/ncu_full$VP_AB_NCU_TAG.log 2>&1
+  ncu -i gpurun_out/rtc_leaf$VP_AB_NCU_TAG.ncu-rep --page source --csv --print-source cuda,sass > gpurun_out/rtc_leaf_src$VP_AB_NCU_TAG.csv 2>&1
+  python tools/ncu_summary.py gpurun_out/rtc_leaf$VP_AB_NCU_TAG.ncu-rep 40 > gpurun_out/rtc_leaf_sum$VP_AB_NCU_TAG.txt 2>&1
+fi

@@ -1,6 +1,6 @@
 """Dev tool: write profiles/<tag>_rtc_leaf_traffic.json and profiles/<tag>_reyes_kernels.json
 (the figures bench.py's roofline.traffic / roofline.issue_bound carry) from the two ncu
-captures of tools/gpu_prof_reyes.sh and the task counts ncu_targets.py printed.
+captures of tools/gpu_evidence.sh and the task counts ncu_targets.py printed.
 
 usage: python tools/reyes_kernel_json.py TAG RTC_REP RTC_LOG BS_REP BS_LOG"""
 import csv
