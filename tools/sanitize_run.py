@@ -73,7 +73,7 @@ def raster(model):
 def pyramid(model):
     rgb = inputs.pyramid_images(2, 256)
     p = W.PyramidPipeline(rgb, **KW)
-    conf(p, model, [(0, 0, vp.GROUP_MEGA, 0, 40), (1, 3, vp.GROUP_MEGA, 40, nsm)])
+    conf(p, model, [(0, 1, vp.GROUP_MEGA, 0, 40), (2, 3, vp.GROUP_MEGA, 40, nsm)])
     p.run()
     return np.array_equal(p.pyramid(), oracle.pyr_pipeline(rgb)["pyr"])
 
@@ -104,8 +104,20 @@ def ldpc(model):
 
 
 ok_all = True
+def qbench(model):
+    # single-stage family: "hybrid" runs it as KBK waves (one group, nothing to bind)
+    ok = True
+    for ib in (4, 16, 272):
+        p = W.QBenchPipeline(64, ib, 2, 6, **KW)
+        p.configure(vp.MEGAKERNEL if model == "mega" else vp.KBK)
+        lv, ids, _, deq = oracle.qbench_pipeline(p.seeds, ib, 2)
+        r, st = p.run()
+        ok &= (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["dequeued"][p.stage] == deq
+    return ok
+
+
 for name, fn in (("toy", toy), ("collatz", collatz), ("reyes", reyes), ("raster", raster), ("pyramid", pyramid),
-                 ("cfd", cfd), ("facedet", facedet), ("ldpc", ldpc)):
+                 ("cfd", cfd), ("facedet", facedet), ("ldpc", ldpc), ("qbench", qbench)):
     if args.only and name not in args.only.split(","):
         continue
     for m in args.models.split(","):
