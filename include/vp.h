@@ -99,6 +99,9 @@ typedef enum vp_stage_kind {
    * patch, L61 §8.5), each kind a single-stage pipeline of its own: register one of them.
    * See vp_qbench_params (counters indexed by item size: 0 = 4 B, 1 = 16 B, 2 = 272 B). */
   VP_QB_ITEM4 = 70, VP_QB_ITEM16 = 71, VP_QB_ITEM272 = 72,
+  /* the same 4- and 16-B stages built with cluster work stealing (VP_FLAG_CLUSTER_STEAL;
+   * SURVEY §8(f-2)): separate kernels, so the plain ones are unchanged */
+  VP_QB_ITEM4_CS = 73, VP_QB_ITEM16_CS = 74,
   /* LDPC decoder (Fig. 17, L59): Initialize, C2V, V2C, ProbVar (loops back to C2V for the
    * next of n_iter iterations); items {frame, iteration}; see vp_ldpc_params */
   VP_LDPC_INIT = 80, VP_LDPC_C2V = 81, VP_LDPC_V2C = 82, VP_LDPC_PROBVAR = 83
@@ -130,6 +133,12 @@ typedef enum vp_stage_kind {
                                       /* with no resident block), vp_run returns                 */
                                       /* VP_ERR_UNSUPPORTED instead of repeating the run as one  */
                                       /* cooperative megakernel (vp_run_stats.model_rerun)        */
+#define VP_FLAG_CLUSTER_STEAL 0x200u  /* a cooperative megakernel of a family   */
+                                      /* that allows it (the queue microbenchmark) runs as      */
+                                      /* clusters of 2 CTAs, and a CTA with nothing to claim    */
+                                      /* takes up to half of its sibling's block-local queue    */
+                                      /* over distributed shared memory                         */
+                                      /* (vp_run_stats.stolen)                 */
 #define VP_FLAG_FULL_RINGS 0x10u    /* persistent plans keep every ring at its registered     */
                                     /* capacity instead of shrinking it to what the producer  */
                                     /* blocks can hold (needed when a recursive stage's live   */
@@ -218,6 +227,8 @@ typedef struct vp_run_stats {
   /* family-defined work units per stage (Reyes: micropolygons shaded by the fused
    * [Dice, Shade] chain, i.e. those whose box holds a pixel centre; 0 elsewhere) */
   uint64_t work_units[VP_MAX_STAGES];
+  /* VP_FLAG_CLUSTER_STEAL: items taken from a cluster sibling's block-local queue */
+  uint64_t stolen[VP_MAX_STAGES];
 } vp_run_stats;
 
 typedef struct vp_autotune_opts {
@@ -419,7 +430,7 @@ vp_status vp_autotune(void* p, const vp_autotune_opts* o, vp_config* best, vp_tu
 vp_status vp_profile(void* p, int* max_blocks_per_sm, int* regs_per_thread, int* smem_per_block);
 
 /* Change the run-time flags of a pipeline (VP_FLAG_QUEUE_DEPTH, VP_FLAG_STRICT_BINDING,
- * VP_FLAG_TIMERS, VP_FLAG_SERIALIZE_GROUPS, VP_FLAG_NO_RERUN; the others are fixed at create
+ * VP_FLAG_TIMERS, VP_FLAG_SERIALIZE_GROUPS, VP_FLAG_NO_RERUN, VP_FLAG_CLUSTER_STEAL; the others are fixed at create
  * and rejected with VP_ERR_INVALID).  old_flags (optional) receives all flags before the change. */
 vp_status vp_set_flags(void* p, uint32_t flags, uint32_t* old_flags);
 

@@ -18,10 +18,13 @@ namespace vp {
 // memory for every stage they cover, so three sizes in one family gave its megakernel the
 // buffers of all three (1 block/SM) while a KBK wave kernel held one stage's (2 blocks/SM).
 // K: 0 = 4 B, 1 = 16 B, 2 = 272 B; also the counter slot in vp_qbench_params.
-template <int K>
+// kSteal: the cluster-work-stealing variant (kinds VP_QB_ITEM{4,16}_CS) --
+// a separate instantiation, so the plain kernels are not changed by the stealing code.
+template <int K, bool kSteal = false>
 struct QBenchF {
   static constexpr int S = 1;
-  static constexpr int kinds[S] = {K == 0 ? VP_QB_ITEM4 : K == 1 ? VP_QB_ITEM16 : VP_QB_ITEM272};
+  static constexpr int kinds[S] = {kSteal ? (K == 0 ? VP_QB_ITEM4_CS : VP_QB_ITEM16_CS)
+                                          : (K == 0 ? VP_QB_ITEM4 : K == 1 ? VP_QB_ITEM16 : VP_QB_ITEM272)};
   using Params = vp_qbench_params;
   static constexpr int stride(int) { return K == 0 ? 4 : K == 1 ? 16 : 272; }
   static constexpr int threads_per_item(int) { return 1; }
@@ -33,6 +36,9 @@ struct QBenchF {
   static constexpr int scratch_bytes(int, int) { return 2 * kMaxBatch * 4; }
   static constexpr int default_cap_log2(int) { return 16; }  // callers size the seeded ring
   static constexpr int min_blocks(int, int, bool) { return 2; }
+  // the two CTAs of a cluster may take items from each other's block-local queue (DSMEM;
+  // with VP_FLAG_CLUSTER_STEAL)
+  static constexpr bool kClusterSteal = kSteal;
 
   // word 0: id (low 24 bits) | remaining depth << 24; words 1..: payload(id, k)
   static __device__ __forceinline__ uint32_t payload(uint32_t id, int k) { return id * 2654435761u + (uint32_t)k * 40503u; }
@@ -142,6 +148,14 @@ const FamilyOps* family_qbench16() {
 }
 const FamilyOps* family_qbench272() {
   static FamilyImpl<QBenchF<2>> f("qbench272");
+  return &f;
+}
+const FamilyOps* family_qbench4_cs() {
+  static FamilyImpl<QBenchF<0, true>> f("qbench4_cs");
+  return &f;
+}
+const FamilyOps* family_qbench16_cs() {
+  static FamilyImpl<QBenchF<1, true>> f("qbench16_cs");
   return &f;
 }
 

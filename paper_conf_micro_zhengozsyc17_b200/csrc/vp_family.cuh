@@ -150,6 +150,29 @@ struct FamilyImpl final : FamilyOps {
     void* args[] = {&a};
     size_t sm = smem(lo, hi, rtc);
     const dim3 blk(block_threads(lo, hi, rtc));
+    if constexpr (HasClusterSteal<F>::value) {
+      // cluster work stealing (VP_FLAG_CLUSTER_STEAL): the cooperative megakernel as
+      // clusters of 2 CTAs; if the driver refuses, the plain cooperative launch (the kernel
+      // then sees a cluster of 1 and does not steal)
+      if (coop && (c.flags & FLAG_STEAL) && grid % 2 == 0) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid);
+        cfg.blockDim = blk;
+        cfg.dynamicSmemBytes = sm;
+        cfg.stream = st;
+        cudaLaunchAttribute at[2];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = 2;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        at[1].id = cudaLaunchAttributeCooperative;
+        at[1].val.cooperative = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 2;
+        if (cudaLaunchKernelExC(&cfg, k, args) == cudaSuccess) return cudaSuccess;
+        (void)cudaGetLastError();
+      }
+    }
     if (coop) return cudaLaunchCooperativeKernel(k, dim3(grid), blk, args, sm, st);
     return cudaLaunchKernel(k, dim3(grid), blk, args, sm, st);
   }
@@ -176,6 +199,8 @@ const FamilyOps* family_facedet();
 const FamilyOps* family_qbench4();
 const FamilyOps* family_qbench16();
 const FamilyOps* family_qbench272();
+const FamilyOps* family_qbench4_cs();
+const FamilyOps* family_qbench16_cs();
 const FamilyOps* family_ldpc();
 
 }  // namespace vp

@@ -21,13 +21,15 @@ using namespace vp;
 
 namespace {
 
-const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+const FamilyOps* all_families[] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
 void init_families() {
   if (!all_families[0]) {
     all_families[8] = family_ldpc();
     all_families[7] = family_qbench4();
     all_families[9] = family_qbench16();
     all_families[10] = family_qbench272();
+    all_families[11] = family_qbench4_cs();
+    all_families[12] = family_qbench16_cs();
     all_families[5] = family_cfd();
     all_families[6] = family_facedet();
     all_families[0] = family_toy();
@@ -82,6 +84,7 @@ __global__ void k_run_init(Ctrl* c, uint32_t* blk, RunInit ri) {
   }
   if (t < kMaxStages) {
     c->units[t] = 0;
+    c->stolen[t] = 0;
   }
   if (t < kMaxKernels) {
     c->arrivals[t].v = 0;
@@ -383,7 +386,7 @@ Common make_common(vp_pipeline_s* p) {
   c.trace = p->trace;
   c.trace_cap = (p->desc.flags & VP_FLAG_TRACE) ? (unsigned long long)p->desc.trace_capacity : 0ull;
   c.flags = ((p->desc.flags & VP_FLAG_TRACE) ? FLAG_TRACE : 0u) | ((p->desc.flags & VP_FLAG_QUEUE_DEPTH) ? FLAG_DEPTH : 0u) |
-            ((p->desc.flags & VP_FLAG_TIMERS) ? FLAG_TIMERS : 0u);
+            ((p->desc.flags & VP_FLAG_TIMERS) ? FLAG_TIMERS : 0u) | ((p->desc.flags & VP_FLAG_CLUSTER_STEAL) ? FLAG_STEAL : 0u);
   c.n_stages = (int)p->st.size();
   c.host_arrive = p->d_arrive;
   c.host_retire = p->d_retire;
@@ -1434,6 +1437,7 @@ static vp_status run_once(vp_pipeline_s* p, cudaStream_t st, vp_run_stats* stats
     stats->pending = (int64_t)hc.pending.v;
     stats->dispatch_timeouts = dispatch_timeouts;
     for (int s = 0; s < S; ++s) stats->work_units[s] = hc.units[s];
+    for (int s = 0; s < S; ++s) stats->stolen[s] = hc.stolen[s];
     stats->model_rerun = 0;
   }
   if (hc.abort.v != ABORT_NONE) {
@@ -1517,9 +1521,11 @@ vp_status vp_set_flags(void* h, uint32_t flags, uint32_t* old_flags) {
   vp_pipeline_s* p = (vp_pipeline_s*)h;
   if (!p) return VP_ERR_INVALID;
   const uint32_t mutable_bits =
-      VP_FLAG_QUEUE_DEPTH | VP_FLAG_STRICT_BINDING | VP_FLAG_TIMERS | VP_FLAG_SERIALIZE_GROUPS | VP_FLAG_NO_RERUN;
+      VP_FLAG_QUEUE_DEPTH | VP_FLAG_STRICT_BINDING | VP_FLAG_TIMERS | VP_FLAG_SERIALIZE_GROUPS | VP_FLAG_NO_RERUN |
+      VP_FLAG_CLUSTER_STEAL;
   if (flags & ~mutable_bits)
-    return fail(p, VP_ERR_INVALID, "vp_set_flags: only QUEUE_DEPTH, STRICT_BINDING, TIMERS, SERIALIZE_GROUPS, NO_RERUN change after create");
+    return fail(p, VP_ERR_INVALID,
+                "vp_set_flags: only QUEUE_DEPTH, STRICT_BINDING, TIMERS, SERIALIZE_GROUPS, NO_RERUN, CLUSTER_STEAL change after create");
   if (old_flags) *old_flags = p->desc.flags;
   p->desc.flags = (p->desc.flags & ~mutable_bits) | flags;
   return VP_OK;

@@ -76,6 +76,7 @@ struct Ctrl {
   unsigned long long exits[kMaxKernels];    // admitted blocks of each kernel slot that have exited
   unsigned long long graph_iters;           // device-driven KBK: iterations of the graph's while loop
   long long wave_n[kMaxStages];             // device-driven KBK: size of each stage's current wave
+  unsigned long long stolen[kMaxStages];    // cluster work stealing: items taken from a sibling's queue
 };
 
 struct QueueDesc {
@@ -93,7 +94,73 @@ struct TraceRec {
   uint32_t kslot, block;  // kernel slot and blockIdx.x of the executing block (binding checks)
 };
 
-enum : uint32_t { FLAG_TRACE = 1u, FLAG_DEPTH = 2u, FLAG_TIMERS = 4u };
+enum : uint32_t { FLAG_TRACE = 1u, FLAG_DEPTH = 2u, FLAG_TIMERS = 4u, FLAG_STEAL = 8u };
+
+// ------------------------------------------------------------------ thread-block clusters
+// (cluster-local queues over distributed shared memory)
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t cluster_nctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(r));
+  return r;
+}
+// shared::cluster address of `p` (this CTA's shared memory) in the CTA of cluster rank `rank`
+__device__ __forceinline__ uint32_t dsmem_addr(const void* p, uint32_t rank) {
+  const uint32_t a = (uint32_t)__cvta_generic_to_shared(p);
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ bool dsmem_trylock(uint32_t addr) {
+  uint32_t old;
+  asm volatile("atom.acquire.cluster.shared::cluster.cas.b32 %0, [%1], 0, 1;" : "=r"(old) : "r"(addr) : "memory");
+  return old == 0;
+}
+__device__ __forceinline__ void dsmem_st_release(uint32_t addr, int v) {
+  asm volatile("st.release.cluster.shared::cluster.b32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+__device__ __forceinline__ int dsmem_ld_acquire(uint32_t addr) {
+  int v;
+  asm volatile("ld.acquire.cluster.shared::cluster.b32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ int dsmem_ld_relaxed(uint32_t addr) {
+  int v;
+  asm volatile("ld.relaxed.cluster.shared::cluster.b32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint4 dsmem_ld_v4(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared::cluster.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t dsmem_ld_u32(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ void fence_acq_rel_cluster() { asm volatile("fence.acq_rel.cluster;" ::: "memory"); }
+template <class V>
+__device__ __forceinline__ V dsmem_ld(uint32_t addr) {
+  if constexpr (sizeof(V) == 16) {
+    const uint4 v = dsmem_ld_v4(addr);
+    return *(const V*)&v;
+  } else if constexpr (sizeof(V) == 8) {
+    uint2 v;
+    asm volatile("ld.shared::cluster.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(addr) : "memory");
+    return *(const V*)&v;
+  } else {
+    const uint32_t v = dsmem_ld_u32(addr);
+    return *(const V*)&v;
+  }
+}
 
 struct Common {
   QueueDesc q[kMaxStages];
@@ -316,6 +383,15 @@ constexpr int scratch_of(int lo, int hi, bool rtc) {
   else return F::scratch_bytes(lo, hi);
 }
 
+// A family may let the two CTAs of a thread-block cluster take items from each other's
+// block-local queues over distributed shared memory (F::kClusterSteal).
+// Active only when the kernel was launched as clusters of 2 (the host does that for a
+// cooperative megakernel with VP_FLAG_CLUSTER_STEAL).
+template <class F, class = void>
+struct HasClusterSteal : std::false_type {};
+template <class F>
+struct HasClusterSteal<F, std::void_t<decltype(F::kClusterSteal)>> : std::bool_constant<F::kClusterSteal> {};
+
 template <class F>
 constexpr int fused_local_cap(int lo, int hi, int t) {
   if constexpr (HasFusedRtc<F>::value) return F::fused_local_cap(lo, hi, t);
@@ -493,6 +569,14 @@ struct BlockShared {
   unsigned long long full[2], empty[2];  // mbarriers: fetcher -> workers, workers -> fetcher
   int bn[2], bstage[2];                // items (-1: stop) and stage of each in buffer
   int lq_head[kMaxStages], lq_tail[kMaxStages];  // block-local queues (publisher -> fetcher)
+  // cluster work stealing (F::kClusterSteal, cluster launch): the consumer side of each
+  // block-local queue is taken under lq_lock by the owner's fetcher or the sibling's
+  int lq_lock[kMaxStages];
+  int steal_s;                         // stage of the batch being consumed under a lock (-1 none)
+  uint32_t stolen32[kMaxStages];       // items this block took from its sibling's queues
+  int alive;                           // admitted (the sibling may steal from this block)
+  int sib_alive;                       // the cluster sibling was admitted (steals from it allowed)
+  int steal_on;                        // this launch steals (Runner::steal_active)
 };
 
 // queue helpers defined below, used by Ctx::publish_warp
@@ -850,6 +934,11 @@ struct Runner {
   using CtxT = Ctx<F, LO, HI, RTC>;
   static constexpr int S = F::S;
   static constexpr int W_FETCH = kWarpsW, W_PUBLISH = kWarpsW + 1;
+  static constexpr bool kSteal = HasClusterSteal<F>::value && !RTC && G::any_lq(LO, HI, RTC);
+  // this launch steals: a persistent kernel with the flag, launched as clusters of 2
+  static __device__ __forceinline__ bool steal_active(const KArgs<F>& a) {
+    return kSteal && (a.c.flags & FLAG_STEAL) && a.g.mode == MODE_PERSISTENT && cluster_nctarank() == 2;
+  }
 
   static constexpr int kInRegion = G::in_region(LO, HI, RTC);
   __device__ static __forceinline__ uint8_t* in_buf(uint8_t* smem, int b) { return smem + b * kInRegion; }
@@ -950,7 +1039,9 @@ struct Runner {
             lq_copy<T, true>(smem, out_buf<T>(smem, pb), sh.lq_tail[T], nl, lane);
             __syncwarp();
             if (lane == T) {
-              __threadfence_block();  // items before the tail that publishes them
+              // items before the tail that publishes them (to the sibling too, when it may steal)
+              if (kSteal && sh.steal_on) fence_acq_rel_cluster();
+              else __threadfence_block();
               *(volatile int*)&sh.lq_tail[T] = sh.lq_tail[T] + nl;
             }
           }
@@ -1036,6 +1127,41 @@ struct Runner {
 
   // ---------------- fetcher warp: claim the next batch (task scheduler) and stage it
   // into in buffer nb.  quiescent: this block holds no batch and flushes nothing now.
+  // Thief side of the cluster work stealing (fetcher lane 0): take up to half of the
+  // sibling's block-local queue of the most downstream stage that has >= 2 items.  The
+  // victim's consumer lock is held until the items are copied (fetch, nx_seed == 3).
+  static __device__ __noinline__ int steal_claim(const KArgs<F>& a, BlockShared& sh, int& st, int& fs,
+                                                 unsigned long long& base) {
+    constexpr int NS = HI - LO + 1;
+    const uint32_t sib = cluster_ctarank() ^ 1u;
+    int got = 0;
+    static_for<0, NS>([&](auto L_) {
+      constexpr int l = decltype(L_)::value, s = HI - l;
+      if constexpr (kLQ<s> > 0) {
+        if (!got) {
+          const uint32_t rh = dsmem_addr(&sh.lq_head[s], sib), rt = dsmem_addr(&sh.lq_tail[s], sib);
+          if (dsmem_ld_relaxed(rt) - dsmem_ld_relaxed(rh) >= 2) {
+            const uint32_t rl = dsmem_addr(&sh.lq_lock[s], sib);
+            if (dsmem_trylock(rl)) {
+              const int h = dsmem_ld_relaxed(rh), t = dsmem_ld_acquire(rt);
+              const int k = min((t - h + 1) / 2, a.g.batch[s]);
+              if (k > 0) {
+                got = k;
+                st = s;
+                fs = 3;
+                base = (unsigned long long)h;
+                sh.steal_s = s;
+              } else {
+                dsmem_st_release(rl, 0);
+              }
+            }
+          }
+        }
+      }
+    });
+    return got;
+  }
+
   static __device__ void fetch(const KArgs<F>& a, BlockShared& sh, uint8_t* smem, int nb, bool quiescent, int lane) {
     Ctrl* c = a.c.ctrl;
     const bool timers = a.c.flags & FLAG_TIMERS;
@@ -1088,12 +1214,25 @@ struct Runner {
           constexpr int l = decltype(L_)::value, s = HI - l;
           if constexpr (kLQ<s> > 0) {  // this block's own children of s come first
             if (!got) {
-              const int occ = *(volatile int*)&sh.lq_tail[s] - sh.lq_head[s];
+              int occ = *(volatile int*)&sh.lq_tail[s] - sh.lq_head[s];
+              if constexpr (kSteal) {
+                // the consumer side is shared with the sibling: take it under the lock
+                // and re-read head (a thief may have advanced it)
+                if (occ > 0 && sh.steal_on) {
+                  if (dsmem_trylock(dsmem_addr(&sh.lq_lock[s], cluster_ctarank()))) {
+                    occ = *(volatile int*)&sh.lq_tail[s] - *(volatile int*)&sh.lq_head[s];
+                    if (occ > 0) sh.steal_s = s;
+                    else dsmem_st_release(dsmem_addr(&sh.lq_lock[s], cluster_ctarank()), 0);
+                  } else {
+                    occ = 0;  // a thief is copying from it; try the rings
+                  }
+                }
+              }
               if (occ > 0) {
                 got = occ < a.g.batch[s] ? occ : a.g.batch[s];
                 st = s;
                 fs = 2;
-                base = (unsigned long long)sh.lq_head[s];
+                base = (unsigned long long)(kSteal ? *(volatile int*)&sh.lq_head[s] : sh.lq_head[s]);
               }
             }
           }
@@ -1109,6 +1248,12 @@ struct Runner {
             if (got) { st = s; fs = 1; }
           }
         });
+        if constexpr (kSteal) {
+          // nothing in this block's queues, the rings or the seeds: take up to half of the
+          // cluster sibling's block-local queue over DSMEM (a separate, non-inlined path:
+          // the plain fetch stays as it was)
+          if (!got && sh.steal_on && sh.sib_alive) got = steal_claim(a, sh, st, fs, base);
+        }
         if (!got && quiescent) {
           // idle: retire deferred completions first, then test for termination
           if (sh.acc_neg != 0) {
@@ -1161,7 +1306,34 @@ struct Runner {
             __syncwarp();
             if (lane == 0) {
               __threadfence_block();  // reads of the slots before the head frees them
-              *(volatile int*)&sh.lq_head[SS] = sh.lq_head[SS] + n;
+              *(volatile int*)&sh.lq_head[SS] = (int)base + n;
+              if constexpr (kSteal) {
+                if (sh.steal_s >= 0) {  // taken under the queue's lock
+                  dsmem_st_release(dsmem_addr(&sh.lq_lock[SS], cluster_ctarank()), 0);
+                  sh.steal_s = -1;
+                }
+              }
+            }
+          }
+        } else if (kSteal && kLQ<SS> > 0 && sh.nx_seed == 3) {  // from the sibling's queue
+          if constexpr (kSteal && kLQ<SS> > 0) {
+            using V = typename Chunk<F::stride(SS)>::T;
+            constexpr int W = Chunk<F::stride(SS)>::per_item;
+            const uint32_t sib = cluster_ctarank() ^ 1u;
+            const uint32_t rq = dsmem_addr(lq_buf<SS>(smem), sib);  // same offset in the sibling
+            V* bdst = (V*)dst;
+            for (int i = lane; i < n * W; i += 32) {
+              const int k = i / W, w = i - k * W;
+              const int slot = ((int)base + k) & (kLQ<SS> - 1);
+              bdst[i] = dsmem_ld<V>(rq + (uint32_t)((slot * W + w) * (int)sizeof(V)));
+            }
+            __syncwarp();
+            if (lane == 0) {
+              // the slots are read before the head that frees them, then the lock
+              dsmem_st_release(dsmem_addr(&sh.lq_head[SS], sib), (int)base + n);
+              dsmem_st_release(dsmem_addr(&sh.lq_lock[SS], sib), 0);
+              sh.steal_s = -1;
+              sh.stolen32[SS] += (uint32_t)n;
             }
           }
         } else if (sh.nx_seed) {
@@ -1339,7 +1511,15 @@ struct Runner {
       sh.work[0] = sh.work[1] = 0;
       sh.nx_n = 0;
       sh.nx_stage = -1;
-      for (int t = 0; t < kMaxStages; ++t) sh.lq_head[t] = sh.lq_tail[t] = 0;
+      for (int t = 0; t < kMaxStages; ++t) {
+        sh.lq_head[t] = sh.lq_tail[t] = 0;
+        sh.lq_lock[t] = 0;
+        sh.stolen32[t] = 0;
+      }
+      sh.steal_s = -1;
+      sh.alive = 1;
+      sh.sib_alive = 0;
+      sh.steal_on = steal_active(a) ? 1 : 0;
       if (g.mode == MODE_WAVE) {
         long long wn = g.wave_n, wc = g.wave_chunk;
         if (g.wave_n_dev) {
@@ -1385,6 +1565,7 @@ struct Runner {
         if (dq) atomicAdd(&c->deq[s], dq);
         if (eq) atomicAdd(&c->enq[s], eq);
         if (sh.units32[s]) atomicAdd(&c->units[s], (unsigned long long)sh.units32[s]);
+        if (sh.stolen32[s]) atomicAdd(&c->stolen[s], (unsigned long long)sh.stolen32[s]);
         if (sh.t_exec[s]) atomicAdd(&c->exec_ns[s], sh.t_exec[s]);
         if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
       }
@@ -1492,7 +1673,21 @@ struct Runner {
   static __device__ void run(const KArgs<F>& a) {
     extern __shared__ __align__(128) uint8_t smem[];
     __shared__ BlockShared sh;
-    if (!admit(a, sh)) return;
+    const bool admitted = admit(a, sh);
+    // cluster launch (work stealing): both CTAs learn whether the other was admitted, and
+    // neither leaves before the other is done with its shared memory (final barrier)
+    const bool clustered = kSteal && cluster_nctarank() == 2;
+    if (clustered) {
+      if (threadIdx.x == 0) sh.alive = admitted ? 1 : 0;
+      cluster_sync_all();
+      if (threadIdx.x == 0) sh.sib_alive = dsmem_ld_relaxed(dsmem_addr(&sh.alive, cluster_ctarank() ^ 1u));
+      __syncthreads();
+      if (!admitted) {
+        cluster_sync_all();
+        return;
+      }
+    }
+    if (!admitted) return;
     CtxT ctx(a, smem, sh);
     if constexpr (sink_group()) {
       if (threadIdx.x == 0) {
@@ -1542,6 +1737,7 @@ struct Runner {
       b ^= 1;
     }
     flush_stats(a, sh);
+    if (clustered) cluster_sync_all();
   }
 };
 

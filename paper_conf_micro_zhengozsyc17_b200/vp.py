@@ -38,10 +38,11 @@ PYR_GRAY, PYR_CDF, PYR_MAP, PYR_RESIZE = 40, 41, 42, 43
 CFD_COPY, CFD_STEP_FACTOR, CFD_FLUX, CFD_TIME_STEP = 50, 51, 52, 53
 FD_GRAY, FD_CDF, FD_MAP, FD_RESIZE, FD_LBP, FD_SCAN = 60, 61, 62, 63, 64, 65
 QB_ITEM4, QB_ITEM16, QB_ITEM272 = 70, 71, 72
+QB_ITEM4_CS, QB_ITEM16_CS = 73, 74
 LDPC_INIT, LDPC_C2V, LDPC_V2C, LDPC_PROBVAR = 80, 81, 82, 83
 FLAG_TRACE, FLAG_QUEUE_DEPTH, FLAG_STRICT_BINDING, FLAG_TIMERS, FLAG_FULL_RINGS, FLAG_ONLINE, FLAG_L2_PERSIST = (
     1, 2, 4, 8, 16, 32, 64)
-FLAG_SERIALIZE_GROUPS, FLAG_NO_RERUN = 0x80, 0x100
+FLAG_SERIALIZE_GROUPS, FLAG_NO_RERUN, FLAG_CLUSTER_STEAL = 0x80, 0x100, 0x200
 INSERT_DEVICE, INSERT_REPLACE = 1, 2
 
 P = C.c_void_p
@@ -80,7 +81,7 @@ class RunStats(C.Structure):
                 ("ring_head", C.c_uint64 * MAX_STAGES), ("ring_count", C.c_int64 * MAX_STAGES),
                 ("seed_head", C.c_uint64 * MAX_STAGES), ("pending", C.c_int64), ("kernel_rounds", C.c_uint64 * 16),
                 ("stage_wave_ms", C.c_float * MAX_STAGES), ("dispatch_timeouts", C.c_int), ("model_rerun", C.c_int),
-                ("work_units", C.c_uint64 * MAX_STAGES)]
+                ("work_units", C.c_uint64 * MAX_STAGES), ("stolen", C.c_uint64 * MAX_STAGES)]
 
 
 class AutotuneOpts(C.Structure):
@@ -392,7 +393,7 @@ def stats_dict(st: RunStats):
                 ring_head=list(st.ring_head), ring_count=list(st.ring_count), seed_head=list(st.seed_head),
                 pending=st.pending, kernel_rounds=list(st.kernel_rounds[:max(nk, 1)]),
                 stage_wave_ms=list(st.stage_wave_ms), dispatch_timeouts=st.dispatch_timeouts,
-                model_rerun=st.model_rerun, work_units=list(st.work_units))
+                model_rerun=st.model_rerun, work_units=list(st.work_units), stolen=list(st.stolen))
 
 
 def config_to_string(cfg: Config) -> str:

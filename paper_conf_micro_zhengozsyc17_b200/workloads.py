@@ -45,7 +45,9 @@ class QBenchPipeline:
 
     SIZES = (4, 16, 272)
 
-    def __init__(self, n: int, item_bytes: int, fanout: int, depth: int, device: int = 0, **kw):
+    def __init__(self, n: int, item_bytes: int, fanout: int, depth: int, device: int = 0, steal: bool = False, **kw):
+        """steal: the cluster-work-stealing build of the 4- / 16-B stage (VP_QB_ITEM*_CS with
+        VP_FLAG_CLUSTER_STEAL)."""
         self.slot = self.SIZES.index(item_bytes)  # counter slot (vp_qbench_params arrays)
         self.stage = 0                            # one single-stage family per item size
         self.n, self.item_bytes, self.fanout, self.depth = n, item_bytes, fanout, depth
@@ -53,11 +55,13 @@ class QBenchPipeline:
         ptr = self.cnt.data_ptr()
         self.prm = vp.QBenchParams(fanout=fanout, depth=depth, leaves=ptr, idsum=ptr + 24, bad=ptr + 48)
         # full rings: a breadth-first fan-out-2 tree's frontier is a whole tree level
-        kw["flags"] = kw.get("flags", 0) | vp.FLAG_FULL_RINGS
+        kw["flags"] = kw.get("flags", 0) | vp.FLAG_FULL_RINGS | (vp.FLAG_CLUSTER_STEAL if steal else 0)
         self.p = vp.Pipeline(device, **kw)
         # the ring holds a whole tree level (KBK waves) or chain frontier
         big = 1 << (21 if item_bytes == 272 else 24)
-        kind = (vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272)[self.slot]
+        if steal and item_bytes == 272:
+            raise ValueError("no stealing build of the 272-B stage (it has no block-local queue)")
+        kind = ((vp.QB_ITEM4_CS, vp.QB_ITEM16_CS) if steal else (vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272))[self.slot]
         self.p.register(kind, item_bytes, self.prm, queue_capacity=big)
         self.seeds = inputs.qbench_seeds(n, item_bytes, depth)
         self.p.insert(self.stage, self.seeds, n=n)

@@ -63,3 +63,30 @@ def test_qbench_graph_kbk_launch_count(vpm):
     assert r1 == r2 and r1["leaves"] == 1000
     # one chain level per iteration at least: >= depth + 1 iterations of the single stage
     assert st1["kbk_launches"] >= 21 and st1["kbk_launches"] == st2["kbk_launches"]
+
+
+@pytest.mark.parametrize("item_bytes", [4, 16])
+@pytest.mark.parametrize("fanout,depth,n", [(2, 12, 8), (1, 30, 3000), (2, 6, 500)])
+def test_qbench_cluster_steal(vpm, orc, item_bytes, fanout, depth, n):
+    """the cooperative megakernel as clusters of 2 CTAs that take items from
+    each other's block-local queue over DSMEM (VP_FLAG_CLUSTER_STEAL): same leaves, leaf-id
+    sum and payloads as the oracle, every item dequeued exactly once, on repeated runs; and
+    stealing happens (a tree grown from a few seeds starts in one CTA's local queue)."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import QBenchPipeline
+    vp = vpm
+    qb = QBenchPipeline(n, item_bytes, fanout, depth, steal=True)
+    lv, ids, bad, deq = orc.qbench_pipeline(qb.seeds, item_bytes, fanout)
+    qb.configure(vp.MEGAKERNEL)
+    stolen = 0
+    for _ in range(3):
+        r, st = qb.run()
+        assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0)
+        assert st["dequeued"][qb.stage] == deq and st["enqueued"][qb.stage] == deq
+        assert st["abort_reason"] == 0 and st["pending"] == 0
+        stolen += st["stolen"][qb.stage]
+    if fanout == 2 and n == 8:
+        assert stolen > 0
+    # the flag is a run-time one: off again, nothing is stolen
+    qb.p.set_flags(0)
+    r, st = qb.run()
+    assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["stolen"][qb.stage] == 0
