@@ -1511,14 +1511,16 @@ struct Runner {
       sh.work[0] = sh.work[1] = 0;
       sh.nx_n = 0;
       sh.nx_stage = -1;
-      for (int t = 0; t < kMaxStages; ++t) {
-        sh.lq_head[t] = sh.lq_tail[t] = 0;
-        sh.lq_lock[t] = 0;
-        sh.stolen32[t] = 0;
+      for (int t = 0; t < kMaxStages; ++t) sh.lq_head[t] = sh.lq_tail[t] = 0;
+      if constexpr (kSteal) {
+        for (int t = 0; t < kMaxStages; ++t) {
+          sh.lq_lock[t] = 0;
+          sh.stolen32[t] = 0;
+        }
+        sh.steal_s = -1;
+        sh.alive = 1;
+        sh.sib_alive = 0;
       }
-      sh.steal_s = -1;
-      sh.alive = 1;
-      sh.sib_alive = 0;
       sh.steal_on = steal_active(a) ? 1 : 0;
       if (g.mode == MODE_WAVE) {
         long long wn = g.wave_n, wc = g.wave_chunk;
@@ -1565,7 +1567,9 @@ struct Runner {
         if (dq) atomicAdd(&c->deq[s], dq);
         if (eq) atomicAdd(&c->enq[s], eq);
         if (sh.units32[s]) atomicAdd(&c->units[s], (unsigned long long)sh.units32[s]);
-        if (sh.stolen32[s]) atomicAdd(&c->stolen[s], (unsigned long long)sh.stolen32[s]);
+        if constexpr (kSteal) {
+          if (sh.stolen32[s]) atomicAdd(&c->stolen[s], (unsigned long long)sh.stolen32[s]);
+        }
         if (sh.t_exec[s]) atomicAdd(&c->exec_ns[s], sh.t_exec[s]);
         if (sh.t_flush[s]) atomicAdd(&c->flush_ns[s], sh.t_flush[s]);
       }
