@@ -66,9 +66,6 @@ constexpr int kG = 8, kNG = 9, kNP = 81;
 #ifndef VP_MS_REG  // 1: Dice keeps the frame matrix rows in registers for a lane's 3 points
 #define VP_MS_REG 1
 #endif
-#ifndef VP_BS_MINMAX  // 1: bound_warp's box as two min/max shuffle trees instead of four
-#define VP_BS_MINMAX 1
-#endif
 #ifndef VP_SROW
 #define VP_SROW 10
 #endif
@@ -113,19 +110,6 @@ __device__ __forceinline__ float red16_max(float v) {
 #pragma unroll
   for (int o = 8; o >= 1; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o, 16));
   return v;
-}
-// min and max of v over a 16-lane group in one shuffle tree: after the xor-8 level the
-// group's lanes 0..7 carry min(v_l, v_l+8) and lanes 8..15 carry -max(v_l, v_l-8), so the
-// next three levels are minima in both halves (-max(a, b) = min(-a, -b) exactly); lane 0
-// then holds the minimum (the same fminf tree as red16_min) and lane 8 minus the maximum.
-// Called by all 32 lanes, converged.
-__device__ __forceinline__ void red16_minmax(float v, float& mn, float& mx) {
-  const float o = __shfl_xor_sync(0xffffffffu, v, 8, 16);
-  float m = (threadIdx.x & 8) ? -fmaxf(v, o) : fminf(v, o);
-#pragma unroll
-  for (int k = 4; k >= 1; k >>= 1) m = fminf(m, __shfl_xor_sync(0xffffffffu, m, k, 16));
-  mn = __shfl_sync(0xffffffffu, m, 0, 16);
-  mx = -__shfl_sync(0xffffffffu, m, 8, 16);
 }
 __device__ __forceinline__ float red16_min(float v) {
 #pragma unroll
@@ -440,13 +424,7 @@ struct ReyesF {
     const int nbehind = __popc((bal >> (threadIdx.x & 16)) & 0xFFFFu);
     float sx, sy, zs;
     screen(p, c, sx, sy, zs);
-    float xmin, xmax, ymin, ymax;
-#if VP_BS_MINMAX
-    red16_minmax(sx, xmin, xmax);
-    red16_minmax(sy, ymin, ymax);
-#else
-    xmin = red16_min(sx); xmax = red16_max(sx); ymin = red16_min(sy); ymax = red16_max(sy);
-#endif
+    const float xmin = red16_min(sx), xmax = red16_max(sx), ymin = red16_min(sy), ymax = red16_max(sy);
     const bool deep = (int)depth >= p.max_depth;
     int cls;  // 0 cull, 1 split, 2 dice
     if (!valid || nbehind == 16) {
