@@ -102,5 +102,8 @@ def test_stage_kind_info_host_only():
     assert [vp.stage_kind_info(k)[1] for k in (vp.REYES_BOUND, vp.REYES_SPLIT, vp.REYES_DICE, vp.REYES_SHADE)] == [
         16, 16, 32, 64]
     assert vp.stage_kind_info(vp.TOY_S1) == (4, 1)
+    # queue microbenchmark: plain and cluster-stealing kinds share their item layouts
+    assert [vp.stage_kind_info(k)[0] for k in (vp.QB_ITEM4, vp.QB_ITEM16, vp.QB_ITEM272, vp.QB_ITEM4_CS,
+                                                vp.QB_ITEM16_CS)] == [4, 16, 272, 4, 16]
     with pytest.raises(vp.VPError):
         vp.stage_kind_info(9999)
