@@ -529,8 +529,18 @@ def workload_suite(torch, vp, stream, tune_s, hbm_gbs):
         # SURVEY §8(f-4), DESIGN R-S9: config-4 triangles with per-vertex z ~ U(-0.6, 0.95),
         # so about half straddle the near plane and Clip fans out 0..2 sub-triangles
         rs = inputs.raster_near_scene(n=1 << 20, W=1920, H=1080, area_range=(0.5, 512.0))
-        out["raster_near_clip"] = measure(RasterPipeline(rs), 1)
-        out["raster_near_clip"]["triangles_per_s"] = rs.n_tris / (out["raster_near_clip"]["ms"] / 1e3)
+        rp = RasterPipeline(rs)
+        r = measure(rp, 1)
+        r["triangles_per_s"] = rs.n_tris / (r["ms"] / 1e3)
+        t0 = time.perf_counter()
+        ref = oracle_mod().raster_pipeline(rs)
+        secs = time.perf_counter() - t0
+        r["cpu_baseline"] = cpu_rec(1, "frames/s", secs, 1, "the full 1M-triangle 1920x1080 near-clip frame, single-threaded")
+        key = rp.keys()
+        col = rp.colours()
+        r["parity"] = {"pass": bool(np.array_equal(key, ref["key"]) and np.array_equal(col, ref["colour"])),
+                       "keys_differing": int(np.count_nonzero(key != ref["key"]))}
+        out["raster_near_clip"] = r
 
     def w_pyr_fig13():
         # PAPER.md Fig. 13 (L53-L55): the pyramid at 1..32 images under KBK, KBK with
