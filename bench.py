@@ -719,6 +719,22 @@ def main():
                 "kernel": f"vp_kernel<ReyesF,{lo},{hi},{'RTC' if is_rtc else 'MEGA'}>",
                 "peak_source": "derived: SMs x 128 fp32 lanes x clocks.max.sm (MEASURED_PEAKS sm_max_mhz), non-FMA",
                 "kernel_ms": float(kmean[dom]), "kernel_share_of_step": float(kmean[dom] / ms_per_step)}
+    # the other persistent group(s) of the step (VERDICT r1 named the [Bound, Split] group
+    # as the kernel furthest below its roofline): the same ALU view, against the fp32 peak
+    # of the SMs the group is bound to
+    others = []
+    for i, (klo, khi, _) in enumerate(st["kernels"] if nk else []):
+        if i == dom:
+            continue
+        g = b.group_of_stage[klo] if main_cfg.has_binding else 0
+        sms = sum(bin(w).count("1") for w in b.group_sm_mask[g]) if main_cfg.has_binding else nsm
+        kf = sum(stage_flop[s] for s in range(klo, khi + 1))
+        ka = kf / (kmean[i] / 1e3) / 1e12
+        kpeak = sms * 128 * sm_max * 1e6 / 1e12
+        others.append({"kernel": f"vp_kernel<ReyesF,{klo},{khi}>", "sms": sms, "achieved": ka, "peak": kpeak,
+                       "unit": "TFLOP/s", "frac": ka / kpeak if kpeak else None, "kernel_ms": float(kmean[i]),
+                       "flop_per_task": {"bound": FLOP_BOUND, "split": FLOP_SPLIT}})
+    roofline["other_groups"] = others
     hbm = pk.get("hbm_gbs", 6548.5)
     # HBM bytes per step that must move: seeds read + fb clear/CAS/resolve + colour write
     npix = scene.n_frames * scene.W * scene.H
