@@ -769,8 +769,9 @@ struct ReyesF {
 
   // -------------------------------------------------------------- Dice (warp/patch)
   // One warp evaluates the 9x9 grid of patch P into `out` (readings R-R7, R-R9): the
-  // separable Bernstein form, the 36 u-curve points C_a(v_j) staged in the (not yet
-  // written) screen rows of `out`, then the 81 surface points, projection and Q8 snap.
+  // separable Bernstein form, the 36 u-curve points C_a(v_j) staged as float4 in the (not
+  // yet written) Q8-snap array s[] of `out`, then the 81 surface points (one lane per grid
+  // row and 3 points), projection and Q8 snap.
   // Ms: the frame matrix rows in shared memory (fused chain), else read from p.M.
   // Bt (fused chain): the Bernstein weights B_b(j/8) as a [9][4] shared-memory table,
   // computed by bernstein() itself (bit-identical to evaluating it per point).
