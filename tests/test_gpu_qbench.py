@@ -90,3 +90,18 @@ def test_qbench_cluster_steal(vpm, orc, item_bytes, fanout, depth, n):
     qb.p.set_flags(0)
     r, st = qb.run()
     assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["stolen"][qb.stage] == 0
+
+
+@pytest.mark.parametrize("model", ["kbk", "kbk_graph", "fine"])
+def test_qbench_cluster_steal_kinds_other_models(vpm, orc, model):
+    """The stealing kinds under the other execution models: no cluster launch, so nothing is
+    stolen and the results are those of the plain kinds."""
+    from paper_conf_micro_zhengozsyc17_b200.workloads import QBenchPipeline
+    vp = vpm
+    for item_bytes in (4, 16):
+        qb = QBenchPipeline(500, item_bytes, 2, 6, steal=True)
+        lv, ids, _, deq = orc.qbench_pipeline(qb.seeds, item_bytes, 2)
+        qb.configure(model_of(vp, model))
+        r, st = qb.run()
+        assert (r["leaves"], r["idsum"], r["bad"]) == (lv, ids, 0) and st["dequeued"][qb.stage] == deq
+        assert st["stolen"][qb.stage] == 0 and st["pending"] == 0
